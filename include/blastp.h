@@ -1,0 +1,185 @@
+/*
+ * blastp.h -- C-ABI of libblastp.so, the B200-native (sm_100a) hot path of
+ * cuBLASTP (Zhang, Wang, Feng; IPDPS'14 / TCBB'15): BLASTP hit detection,
+ * two-hit filtering on diagonals and X-drop ungapped extension.
+ *
+ * Citations "P:L<n>" are lines of the paper text;
+ * "R<k>" are the readings of SURVEY.md section 8(c), restated in DESIGN.md.
+ *
+ * Conventions (all entry points):
+ *  - Every function returns an int status: BLASTP_OK (0) or a negative
+ *    BLASTP_E_* code.  Nothing throws or aborts.  blastp_last_error() gives a
+ *    thread-local, human-readable detail of the last failure.
+ *  - Plain pointers and sizes only.  "host" pointers are ordinary (ideally
+ *    pinned) CPU memory; "device" pointers are CUDA global memory on the
+ *    device the handle was created on (e.g. a torch.cuda tensor's data_ptr()).
+ *  - `cuda_stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  All device work of a call is enqueued on it.
+ *  - Inputs are copied; the caller keeps ownership.  Handles and library-
+ *    allocated host arrays are owned by the library until the matching
+ *    *_free call.
+ *  - A database handle owns scratch counters: do not run two searches on
+ *    the same blastp_db concurrently on different streams.
+ *
+ * Residue encoding (R1): 24 letters in NCBI order "ARNDCQEGHILKMFPSTWYVBZX*"
+ * -> codes 0..23; lowercase is upper-cased; U, O and J map to X; any other
+ * byte is BLASTP_E_BAD_RESIDUE.  Scoring is BLOSUM62 (R2).
+ */
+#ifndef BLASTP_H
+#define BLASTP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define BLASTP_OK 0
+#define BLASTP_E_INVALID_ARG (-1) /* NULL pointer, bad size or parameter   */
+#define BLASTP_E_BAD_RESIDUE (-2) /* character outside R1's alphabet       */
+#define BLASTP_E_TOO_LONG (-3)    /* query > BLASTP_MAX_QUERY_LEN, subject > BLASTP_MAX_SUBJECT_LEN */
+#define BLASTP_E_NOMEM (-4)       /* host or device allocation failed      */
+#define BLASTP_E_CUDA (-5)        /* CUDA runtime error (detail in last_error) */
+#define BLASTP_E_CAPACITY (-6)    /* caller buffer too small (see below)   */
+
+#define BLASTP_MAX_QUERY_LEN 16000
+#define BLASTP_MAX_SUBJECT_LEN (1 << 30)
+#define BLASTP_FILTER_LEFT 0   /* R6 default: W <= h - p < A              */
+#define BLASTP_FILTER_EITHER 1 /* Fig. 7 reading: W <= |h - p| < A        */
+
+/* Search parameters.  Defaults (blastp_params_default) are the BASELINE.json
+ * configuration: w = 3, T = 11, A = 40, X = 7 bits -> 16 raw, cutoff 41. */
+typedef struct {
+  int32_t word_len;    /* word length W; only 3 is supported     */
+  int32_t threshold;   /* T: word v neighbours query word iff score >= T (R3) */
+  int32_t window;      /* A: two-hit window (R6), 1..4096       */
+  int32_t min_gap;     /* non-overlap distance (R6), 1..8; default = word_len */
+  int32_t xdrop;       /* X: stop when best - run >= X (Fig. 8, R8), 1..127   */
+  int32_t cutoff;      /* emit an extension iff score >= cutoff (R10)         */
+  int32_t filter_mode; /* BLASTP_FILTER_LEFT or BLASTP_FILTER_EITHER          */
+} blastp_params;
+
+/* One ungapped extension ("start and end position of this extension with
+ * the highest score").  28 bytes; it is also the hand-off
+ * record to a gapped-extension stage (out of scope here).
+ * diagonal = s_start - q_start; the segment is
+ * [q_start, q_start+length) x [s_start, s_start+length), score = sum of
+ * BLOSUM62 over it.  subject_id is GLOBAL (shard base + local index). */
+typedef struct {
+  int32_t query_id, subject_id, diagonal, q_start, s_start, length, score;
+} blastp_hsp;
+
+/* Debug record of a hit / passing hit (subject-local coordinates). */
+typedef struct {
+  int32_t query_id, subject_id, q, s;
+} blastp_hit;
+
+typedef struct blastp_query_table blastp_query_table; /* opaque */
+typedef struct blastp_db blastp_db;                   /* opaque: one shard */
+
+void blastp_params_default(blastp_params *p);
+const char *blastp_strerror(int status);
+const char *blastp_last_error(void);
+const char *blastp_version(void);
+
+/* Query lookup table (R3): for every query position
+ * q in [0, len-3] the list of all 24^3 words v with
+ * sum_i BLOSUM62[query[q+i]][v_i] >= p->threshold, stored as a CSR table
+ * word -> ascending query positions (the function of the paper's DFA),
+ * plus the query codes.  Built on the host, copied to `device` on
+ * `cuda_stream`; the call returns after the copies complete.
+ * query_ascii: host, `len` bytes (3 <= len <= BLASTP_MAX_QUERY_LEN).
+ * Errors: INVALID_ARG (NULL, len < 3, word_len != 3), BAD_RESIDUE,
+ * TOO_LONG, NOMEM, CUDA. */
+int blastp_build_query_table(const char *query_ascii, int32_t len,
+                             const blastp_params *p, int device,
+                             void *cuda_stream, blastp_query_table **out);
+
+/* Same for `nq` queries; query_id of results = index in `queries`. */
+int blastp_build_query_batch(const char *const *queries, const int32_t *lens,
+                             int32_t nq, const blastp_params *p, int device,
+                             void *cuda_stream, blastp_query_table **out);
+
+/* Database pack + shard (coalesced residue access).
+ * residues_ascii: host, all subjects concatenated; subject i is
+ * residues_ascii[offsets[i] .. offsets[i+1]) (offsets: host, nseq+1 entries,
+ * non-decreasing, offsets[0] may be non-zero).  The subjects are split into
+ * num_shards contiguous ranges balanced by residues (blastp_shard_range) and
+ * only range `shard_index` is packed: its bytes are copied host->device on
+ * `cuda_stream` and encoded on the GPU into a sentinel-separated code stream
+ * (1 byte per residue).  Returns after the device work completes.
+ * Errors: INVALID_ARG, BAD_RESIDUE, TOO_LONG (a subject > MAX_SUBJECT_LEN),
+ * NOMEM, CUDA. */
+int blastp_pack_db(const char *residues_ascii, const int64_t *offsets,
+                   int64_t nseq, int32_t shard_index, int32_t num_shards,
+                   int device, void *cuda_stream, blastp_db **out);
+
+/* Subject range [*lo, *hi) of shard `shard_index` (host-only helper, no GPU):
+ * the first subject of shard k is the first i with
+ * offsets[i] - offsets[0] >= total * k / num_shards. */
+int blastp_shard_range(const int64_t *offsets, int64_t nseq,
+                       int32_t shard_index, int32_t num_shards, int64_t *lo,
+                       int64_t *hi);
+
+/* Shard description: number of subjects, residues, global id of its first
+ * subject (shard base), packed stream bytes.  Any pointer may be NULL. */
+int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues,
+                   int64_t *subject_base, int64_t *stream_bytes,
+                   int64_t *num_chunks);
+int blastp_query_table_info(const blastp_query_table *q, int32_t *num_queries,
+                            int64_t *table_entries);
+
+/* Ungapped search (Alg. 1-5; R4-R10): every hit of every query against
+ * every subject of the shard, the two-hit filter per (subject, diagonal),
+ * X-drop extension of passing hits not covered by a previous extension of
+ * the same diagonal, and every extension with score >= cutoff returned.
+ * HOST variant: *out_host (library-malloc'd, free with blastp_hsp_free) gets
+ * *out_count HSPs in canonical order (R11: lexicographic on all 7 fields).
+ * Synchronous on cuda_stream.  `p` must equal the params of the table for
+ * word_len/threshold (they shaped the table); the others may differ. */
+int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
+                           const blastp_params *p, void *cuda_stream,
+                           blastp_hsp **out_host, int64_t *out_count);
+
+/* DEVICE variant, asynchronous: HSPs are appended (unordered) to d_out
+ * (device, `capacity` records); d_count (device, one int64) receives the
+ * number of HSPs found, which may exceed capacity -- then only `capacity`
+ * records were written and the caller should retry with a larger buffer.
+ * Nothing is read back; no host synchronisation. */
+int blastp_search_ungapped_device(const blastp_query_table *q,
+                                  const blastp_db *db, const blastp_params *p,
+                                  void *cuda_stream, blastp_hsp *d_out,
+                                  int64_t capacity, int64_t *d_count);
+
+/* Canonical order (R11) of n device HSPs, in place, on the GPU. */
+int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream);
+
+/* Debug / parity entry points (synchronous, host buffers).  They run the
+ * same kernel as the search with tracing enabled and return:
+ *  hits:    every hit (R4) as (query_id, subject_id, q, s), unordered;
+ *  passing: every hit passing the two-hit filter (R6), unordered;
+ *  exts:    every extension performed (R10), emitted or not, unordered.
+ * Counts are written even when they exceed the capacities (then only the
+ * first `cap` records are filled and BLASTP_E_CAPACITY is returned).
+ * Any buffer may be NULL (with cap 0) to skip that list. */
+int blastp_debug_trace(const blastp_query_table *q, const blastp_db *db,
+                       const blastp_params *p, void *cuda_stream,
+                       blastp_hit *hits, int64_t hits_cap, int64_t *n_hits,
+                       blastp_hit *passing, int64_t passing_cap,
+                       int64_t *n_passing, blastp_hsp *exts, int64_t exts_cap,
+                       int64_t *n_exts);
+int blastp_debug_hits(const blastp_query_table *q, const blastp_db *db,
+                      const blastp_params *p, void *cuda_stream,
+                      blastp_hit *hits, int64_t cap, int64_t *n);
+int blastp_debug_passing(const blastp_query_table *q, const blastp_db *db,
+                         const blastp_params *p, void *cuda_stream,
+                         blastp_hit *passing, int64_t cap, int64_t *n);
+
+void blastp_hsp_free(blastp_hsp *h);
+void blastp_query_table_free(blastp_query_table *q);
+void blastp_db_free(blastp_db *db);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* BLASTP_H */

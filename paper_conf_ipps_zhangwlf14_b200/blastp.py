@@ -1,0 +1,307 @@
+"""Thin ctypes binding of libblastp.so (include/blastp.h), same names as the C-ABI.
+
+Argument marshalling only: every step of the search runs in the library's
+CUDA kernels.  There is no CPU fallback -- if libblastp.so is missing the
+import fails (build it with ``python -m paper_conf_ipps_zhangwlf14_b200.build``
+or ``__graft_entry__.build()``).
+
+PyTorch is used only for what the C-ABI leaves to the caller: device memory
+for the device-side output (``search_ungapped_device``) and CUDA streams.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libblastp.so")
+
+OK, E_INVALID_ARG, E_BAD_RESIDUE, E_TOO_LONG, E_NOMEM, E_CUDA, E_CAPACITY = 0, -1, -2, -3, -4, -5, -6
+FILTER_LEFT, FILTER_EITHER = 0, 1
+
+HSP_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("diagonal", "<i4"),
+                      ("q_start", "<i4"), ("s_start", "<i4"), ("length", "<i4"),
+                      ("score", "<i4")])
+HIT_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("q", "<i4"), ("s", "<i4")])
+HSP_BYTES = 28
+
+
+class BlastpError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        super().__init__(f"{where}: {detail} (status {status})")
+        self.status = status
+
+
+class _CParams(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in
+                ("word_len", "threshold", "window", "min_gap", "xdrop", "cutoff", "filter_mode")]
+
+
+@dataclass
+class Params:
+    """blastp_params; defaults = BASELINE.json (w=3, T=11, A=40, X=16 raw, cutoff 41)."""
+    word_len: int = 3
+    threshold: int = 11
+    window: int = 40
+    min_gap: int = 3
+    xdrop: int = 16
+    cutoff: int = 41
+    filter_mode: int = FILTER_LEFT
+
+    def c(self) -> _CParams:
+        return _CParams(self.word_len, self.threshold, self.window, self.min_gap, self.xdrop,
+                        self.cutoff, self.filter_mode)
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build the CUDA library first "
+                          "(python -m paper_conf_ipps_zhangwlf14_b200.build)")
+    L = ctypes.CDLL(LIB_PATH)
+    vp, i32, i64, P = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.POINTER
+    L.blastp_params_default.argtypes = [P(_CParams)]
+    L.blastp_params_default.restype = None
+    L.blastp_strerror.argtypes = [ctypes.c_int]
+    L.blastp_strerror.restype = ctypes.c_char_p
+    L.blastp_last_error.argtypes = []
+    L.blastp_last_error.restype = ctypes.c_char_p
+    L.blastp_version.argtypes = []
+    L.blastp_version.restype = ctypes.c_char_p
+    L.blastp_build_query_table.argtypes = [ctypes.c_char_p, i32, P(_CParams), ctypes.c_int, vp, P(vp)]
+    L.blastp_build_query_batch.argtypes = [P(ctypes.c_char_p), P(i32), i32, P(_CParams),
+                                           ctypes.c_int, vp, P(vp)]
+    L.blastp_pack_db.argtypes = [vp, vp, i64, i32, i32, ctypes.c_int, vp, P(vp)]
+    L.blastp_shard_range.argtypes = [vp, i64, i32, i32, P(i64), P(i64)]
+    L.blastp_db_info.argtypes = [vp, P(i64), P(i64), P(i64), P(i64), P(i64)]
+    L.blastp_query_table_info.argtypes = [vp, P(i32), P(i64)]
+    L.blastp_search_ungapped.argtypes = [vp, vp, P(_CParams), vp, P(vp), P(i64)]
+    L.blastp_search_ungapped_device.argtypes = [vp, vp, P(_CParams), vp, vp, i64, vp]
+    L.blastp_sort_hsps_device.argtypes = [vp, i64, vp]
+    L.blastp_debug_trace.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64), vp, i64, P(i64),
+                                     vp, i64, P(i64)]
+    L.blastp_debug_hits.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
+    L.blastp_debug_passing.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
+    for f in ("blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"):
+        getattr(L, f).argtypes = [vp]
+        getattr(L, f).restype = None
+    return L
+
+
+lib = _load()
+
+EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "blastp_version",
+            "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
+            "blastp_shard_range", "blastp_db_info", "blastp_query_table_info",
+            "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_sort_hsps_device",
+            "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing",
+            "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
+
+
+def _check(rc: int, where: str):
+    if rc != OK:
+        raise BlastpError(rc, where, lib.blastp_last_error().decode(errors="replace") or
+                          lib.blastp_strerror(rc).decode())
+
+
+def _stream_handle(stream) -> int | None:
+    if stream is None:
+        try:
+            import torch
+            if torch.cuda.is_available():
+                return torch.cuda.current_stream().cuda_stream or None
+        except ImportError:
+            pass
+        return None
+    if isinstance(stream, int):
+        return stream or None
+    return getattr(stream, "cuda_stream", None) or None
+
+
+def version() -> str:
+    return lib.blastp_version().decode()
+
+
+def params_default() -> Params:
+    c = _CParams()
+    lib.blastp_params_default(ctypes.byref(c))
+    return Params(*(getattr(c, f) for f, _ in _CParams._fields_))
+
+
+def _as_bytes(q) -> bytes:
+    return q.encode() if isinstance(q, str) else bytes(q)
+
+
+class QueryTable:
+    """blastp_query_table handle (one or more queries, query_id = index)."""
+
+    def __init__(self, queries, params: Params | None = None, device: int = 0, stream=None):
+        self.params = params or Params()
+        qs = [queries] if isinstance(queries, (str, bytes, bytearray)) else list(queries)
+        bufs = [_as_bytes(q) for q in qs]
+        arr = (ctypes.c_char_p * len(bufs))(*bufs)
+        lens = (ctypes.c_int32 * len(bufs))(*[len(b) for b in bufs])
+        h = ctypes.c_void_p()
+        c = self.params.c()
+        _check(lib.blastp_build_query_batch(arr, lens, len(bufs), ctypes.byref(c), device,
+                                            _stream_handle(stream), ctypes.byref(h)),
+               "blastp_build_query_batch")
+        self.handle = h
+        self.device = device
+        self.lengths = [len(b) for b in bufs]
+
+    @property
+    def num_queries(self) -> int:
+        n = ctypes.c_int32()
+        e = ctypes.c_int64()
+        _check(lib.blastp_query_table_info(self.handle, ctypes.byref(n), ctypes.byref(e)),
+               "blastp_query_table_info")
+        return n.value
+
+    @property
+    def entries(self) -> int:
+        n = ctypes.c_int32()
+        e = ctypes.c_int64()
+        _check(lib.blastp_query_table_info(self.handle, ctypes.byref(n), ctypes.byref(e)),
+               "blastp_query_table_info")
+        return e.value
+
+    def free(self):
+        if getattr(self, "handle", None):
+            lib.blastp_query_table_free(self.handle)
+            self.handle = None
+
+    __del__ = free
+
+
+def build_query_table(query, params: Params | None = None, device: int = 0, stream=None):
+    return QueryTable(query, params, device, stream)
+
+
+def build_query_batch(queries, params: Params | None = None, device: int = 0, stream=None):
+    return QueryTable(list(queries), params, device, stream)
+
+
+def shard_range(offsets: np.ndarray, shard_index: int, num_shards: int) -> tuple[int, int]:
+    """Host-only: residue-balanced contiguous subject range of a shard."""
+    off = np.ascontiguousarray(offsets, dtype=np.int64)
+    lo, hi = ctypes.c_int64(), ctypes.c_int64()
+    _check(lib.blastp_shard_range(off.ctypes.data, len(off) - 1, shard_index, num_shards,
+                                  ctypes.byref(lo), ctypes.byref(hi)), "blastp_shard_range")
+    return lo.value, hi.value
+
+
+class Database:
+    """blastp_db handle: one shard of a database, packed on the GPU."""
+
+    def __init__(self, residues: np.ndarray | bytes, offsets: np.ndarray, shard_index: int = 0,
+                 num_shards: int = 1, device: int = 0, stream=None):
+        if isinstance(residues, (bytes, bytearray)):
+            residues = np.frombuffer(residues, dtype=np.uint8)
+        res = residues if residues.flags["C_CONTIGUOUS"] else np.ascontiguousarray(residues)
+        off = np.ascontiguousarray(offsets, dtype=np.int64)
+        h = ctypes.c_void_p()
+        ptr = res.ctypes.data if hasattr(res, "ctypes") else res.data_ptr()
+        _check(lib.blastp_pack_db(ptr, off.ctypes.data, len(off) - 1, shard_index, num_shards,
+                                  device, _stream_handle(stream), ctypes.byref(h)),
+               "blastp_pack_db")
+        self.handle = h
+        self.device = device
+        vals = [ctypes.c_int64() for _ in range(5)]
+        _check(lib.blastp_db_info(h, *[ctypes.byref(v) for v in vals]), "blastp_db_info")
+        self.nseq, self.residues, self.subject_base, self.stream_bytes, self.num_chunks = \
+            (v.value for v in vals)
+
+    @classmethod
+    def from_pinned(cls, residues_ptr: int, offsets: np.ndarray, shard_index=0, num_shards=1,
+                    device=0, stream=None):
+        """Pack from a raw host pointer (e.g. a pinned torch tensor's data_ptr())."""
+        self = cls.__new__(cls)
+        off = np.ascontiguousarray(offsets, dtype=np.int64)
+        h = ctypes.c_void_p()
+        _check(lib.blastp_pack_db(residues_ptr, off.ctypes.data, len(off) - 1, shard_index,
+                                  num_shards, device, _stream_handle(stream), ctypes.byref(h)),
+               "blastp_pack_db")
+        self.handle = h
+        self.device = device
+        vals = [ctypes.c_int64() for _ in range(5)]
+        _check(lib.blastp_db_info(h, *[ctypes.byref(v) for v in vals]), "blastp_db_info")
+        self.nseq, self.residues, self.subject_base, self.stream_bytes, self.num_chunks = \
+            (v.value for v in vals)
+        return self
+
+    def free(self):
+        if getattr(self, "handle", None):
+            lib.blastp_db_free(self.handle)
+            self.handle = None
+
+    __del__ = free
+
+
+def pack_db(residues, offsets, shard_index=0, num_shards=1, device=0, stream=None) -> Database:
+    return Database(residues, offsets, shard_index, num_shards, device, stream)
+
+
+def search_ungapped(table: QueryTable, db: Database, params: Params | None = None,
+                    stream=None) -> np.ndarray:
+    """Host variant: canonical-order HSP array (HSP_DTYPE)."""
+    c = (params or table.params).c()
+    out = ctypes.c_void_p()
+    n = ctypes.c_int64()
+    _check(lib.blastp_search_ungapped(table.handle, db.handle, ctypes.byref(c),
+                                      _stream_handle(stream), ctypes.byref(out), ctypes.byref(n)),
+           "blastp_search_ungapped")
+    try:
+        if n.value == 0:
+            return np.zeros(0, dtype=HSP_DTYPE)
+        buf = (ctypes.c_char * (n.value * HSP_BYTES)).from_address(out.value)
+        return np.frombuffer(bytes(buf), dtype=HSP_DTYPE).copy()
+    finally:
+        lib.blastp_hsp_free(out)
+
+
+def search_ungapped_device(table: QueryTable, db: Database, out_ptr: int, capacity: int,
+                           count_ptr: int, params: Params | None = None, stream=None):
+    """Device variant (async): HSPs appended to device memory at out_ptr
+    (capacity records of 28 B), total count written to the int64 at count_ptr."""
+    c = (params or table.params).c()
+    _check(lib.blastp_search_ungapped_device(table.handle, db.handle, ctypes.byref(c),
+                                             _stream_handle(stream), out_ptr, capacity,
+                                             count_ptr), "blastp_search_ungapped_device")
+
+
+def sort_hsps_device(ptr: int, n: int, stream=None):
+    _check(lib.blastp_sort_hsps_device(ptr, n, _stream_handle(stream)), "blastp_sort_hsps_device")
+
+
+@dataclass
+class Trace:
+    hits: np.ndarray
+    passing: np.ndarray
+    extensions: np.ndarray
+
+
+def debug_trace(table: QueryTable, db: Database, params: Params | None = None, stream=None,
+                hits_cap: int = 1 << 20, passing_cap: int = 1 << 18,
+                exts_cap: int = 1 << 18) -> Trace:
+    """Every hit, passing hit and extension of a search (unordered)."""
+    c = (params or table.params).c()
+    for _ in range(3):
+        hb = np.zeros(max(hits_cap, 1), dtype=HIT_DTYPE)
+        pb = np.zeros(max(passing_cap, 1), dtype=HIT_DTYPE)
+        eb = np.zeros(max(exts_cap, 1), dtype=HSP_DTYPE)
+        nh, np_, ne = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        rc = lib.blastp_debug_trace(table.handle, db.handle, ctypes.byref(c),
+                                    _stream_handle(stream), hb.ctypes.data, hits_cap,
+                                    ctypes.byref(nh), pb.ctypes.data, passing_cap,
+                                    ctypes.byref(np_), eb.ctypes.data, exts_cap, ctypes.byref(ne))
+        if rc == E_CAPACITY:
+            hits_cap = max(hits_cap, nh.value)
+            passing_cap = max(passing_cap, np_.value)
+            exts_cap = max(exts_cap, ne.value)
+            continue
+        _check(rc, "blastp_debug_trace")
+        return Trace(hb[:nh.value].copy(), pb[:np_.value].copy(), eb[:ne.value].copy())
+    raise BlastpError(E_CAPACITY, "blastp_debug_trace", "capacity retries exhausted")

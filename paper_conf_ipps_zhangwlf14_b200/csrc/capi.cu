@@ -1,0 +1,652 @@
+// capi.cu -- the extern "C" boundary of libblastp.so (include/blastp.h).
+//
+// Host logic only: argument validation, the query lookup-table builder (R3),
+// the database packer / sharder, launch drivers and result marshalling.
+// Every step of the search itself runs in the kernels of search.cu.
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+using namespace blastp;
+
+// ------------------------------------------------------------------ errors
+
+namespace {
+
+thread_local std::string g_last_error;
+
+int fail(int code, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return code;
+}
+
+#define CUDA_TRY(expr)                                                                    \
+  do {                                                                                    \
+    cudaError_t _e = (expr);                                                              \
+    if (_e != cudaSuccess)                                                                \
+      return fail(BLASTP_E_CUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(_e), \
+                  __FILE__, __LINE__);                                                    \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  cudaError_t err = cudaSuccess;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) err = cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+// R1 encoding (host side, for queries)
+int encode_char(unsigned char c) {
+  if (c >= 'a' && c <= 'z') c = static_cast<unsigned char>(c - 'a' + 'A');
+  if (c == 'U' || c == 'O' || c == 'J') c = 'X';
+  for (int k = 0; k < kNumLetters; ++k)
+    if (static_cast<unsigned char>(kAlphabet[k]) == c) return k;
+  return -1;
+}
+
+int validate_params(const blastp_params *p) {
+  if (!p) return fail(BLASTP_E_INVALID_ARG, "params is NULL");
+  if (p->word_len != 3) return fail(BLASTP_E_INVALID_ARG, "word_len %d unsupported (3 only)", p->word_len);
+  if (p->min_gap < 1 || p->min_gap > 8)
+    return fail(BLASTP_E_INVALID_ARG, "min_gap %d outside [1, 8]", p->min_gap);
+  if (p->window < 1 || p->window > 1024)
+    return fail(BLASTP_E_INVALID_ARG, "window %d outside [1, 1024]", p->window);
+  if (p->xdrop < 1 || p->xdrop > 127)
+    return fail(BLASTP_E_INVALID_ARG, "xdrop %d outside [1, 127]", p->xdrop);
+  if (p->threshold < -100 || p->threshold > 100)
+    return fail(BLASTP_E_INVALID_ARG, "threshold %d outside [-100, 100]", p->threshold);
+  if (p->filter_mode != BLASTP_FILTER_LEFT && p->filter_mode != BLASTP_FILTER_EITHER)
+    return fail(BLASTP_E_INVALID_ARG, "filter_mode %d unknown", p->filter_mode);
+  return BLASTP_OK;
+}
+
+int num_sms(int device) {
+  int sms = 0;
+  if (cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess ||
+      sms <= 0)
+    sms = 148;
+  return sms;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ handles
+
+struct QueryDev {
+  uint32_t *woff = nullptr;
+  uint16_t *qpos = nullptr;
+  uint8_t *qcodes = nullptr;
+  int32_t lq = 0;
+  int64_t entries = 0;
+};
+
+struct blastp_query_table {
+  int device = 0;
+  blastp_params p{};
+  std::vector<QueryDev> q;
+  int64_t entries = 0;
+};
+
+struct blastp_db {
+  int device = 0;
+  int sms = 148;
+  int64_t nseq = 0, residues = 0, subject_base = 0, stream_len = 0;
+  uint8_t *stream = nullptr;
+  int64_t *sstart = nullptr;
+  Chunk *chunks = nullptr;
+  int32_t nchunks = 0;
+  std::vector<int64_t> h_sstart;
+  unsigned long long *counters = nullptr;  // [0] hsp count, [1] chunk cursor, [2..4] trace
+  blastp_hsp *out = nullptr;               // scratch for the host-array search
+  int64_t out_cap = 0;
+};
+
+static void free_query_dev(QueryDev &d) {
+  cudaFree(d.woff);
+  cudaFree(d.qpos);
+  cudaFree(d.qcodes);
+  d = QueryDev{};
+}
+
+extern "C" {
+
+void blastp_params_default(blastp_params *p) {
+  if (!p) return;
+  p->word_len = 3;
+  p->threshold = 11;
+  p->window = 40;
+  p->min_gap = 3;
+  p->xdrop = 16;
+  p->cutoff = 41;
+  p->filter_mode = BLASTP_FILTER_LEFT;
+}
+
+const char *blastp_strerror(int status) {
+  switch (status) {
+    case BLASTP_OK: return "ok";
+    case BLASTP_E_INVALID_ARG: return "invalid argument";
+    case BLASTP_E_BAD_RESIDUE: return "invalid residue character";
+    case BLASTP_E_TOO_LONG: return "sequence too long";
+    case BLASTP_E_NOMEM: return "out of memory";
+    case BLASTP_E_CUDA: return "CUDA error";
+    case BLASTP_E_CAPACITY: return "output capacity exceeded";
+    default: return "unknown status";
+  }
+}
+
+const char *blastp_last_error(void) { return g_last_error.c_str(); }
+
+const char *blastp_version(void) { return "blastp-b200 0.1 (sm_100a)"; }
+
+// ------------------------------------------------------- query table (R3)
+
+static int build_one_query(const char *ascii, int32_t len, const blastp_params *p, QueryDev &out,
+                           cudaStream_t s) {
+  if (!ascii) return fail(BLASTP_E_INVALID_ARG, "query is NULL");
+  if (len < 3) return fail(BLASTP_E_INVALID_ARG, "query length %d < 3", len);
+  if (len > BLASTP_MAX_QUERY_LEN)
+    return fail(BLASTP_E_TOO_LONG, "query length %d > %d", len, BLASTP_MAX_QUERY_LEN);
+  std::vector<uint8_t> Q(static_cast<size_t>(len));
+  for (int32_t i = 0; i < len; ++i) {
+    const int c = encode_char(static_cast<unsigned char>(ascii[i]));
+    if (c < 0) return fail(BLASTP_E_BAD_RESIDUE, "query byte %d (0x%02x) is not a residue", i,
+                           static_cast<unsigned char>(ascii[i]));
+    Q[static_cast<size_t>(i)] = static_cast<uint8_t>(c);
+  }
+  // Neighbourhood words by pruned enumeration: for each query word, walk the
+  // 24^3 words letter by letter and cut a branch as soon as even the best
+  // remaining letters cannot reach T.  Same set as the brute-force
+  // definition (R3); lists come out with q ascending.
+  int rowmax[kNumLetters];
+  for (int a = 0; a < kNumLetters; ++a) {
+    int m = -1000;
+    for (int b = 0; b < kNumLetters; ++b) m = std::max(m, int(kBlosum62[a][b]));
+    rowmax[a] = m;
+  }
+  const int T = p->threshold;
+  std::vector<uint32_t> count(kWords + 1, 0);
+  auto enumerate = [&](auto &&emit) {
+    for (int32_t q = 0; q + 3 <= len; ++q) {
+      const int a0 = Q[q], a1 = Q[q + 1], a2 = Q[q + 2];
+      for (int x = 0; x < kNumLetters; ++x) {
+        const int s1 = kBlosum62[a0][x];
+        if (s1 + rowmax[a1] + rowmax[a2] < T) continue;
+        for (int y = 0; y < kNumLetters; ++y) {
+          const int s2 = s1 + kBlosum62[a1][y];
+          if (s2 + rowmax[a2] < T) continue;
+          for (int z = 0; z < kNumLetters; ++z)
+            if (s2 + kBlosum62[a2][z] >= T) emit((x * kNumLetters + y) * kNumLetters + z, q);
+        }
+      }
+    }
+  };
+  enumerate([&](int w, int) { count[static_cast<size_t>(w) + 1]++; });
+  for (int w = 0; w < kWords; ++w) count[static_cast<size_t>(w) + 1] += count[static_cast<size_t>(w)];
+  const int64_t total = count[kWords];
+  std::vector<uint16_t> pos(static_cast<size_t>(std::max<int64_t>(total, 1)));
+  std::vector<uint32_t> cur(count.begin(), count.end() - 1);
+  enumerate([&](int w, int q) { pos[cur[static_cast<size_t>(w)]++] = static_cast<uint16_t>(q); });
+
+  out.lq = len;
+  out.entries = total;
+  if (cudaMalloc(&out.woff, sizeof(uint32_t) * (kWords + 1)) != cudaSuccess ||
+      cudaMalloc(&out.qpos, sizeof(uint16_t) * pos.size()) != cudaSuccess ||
+      cudaMalloc(&out.qcodes, static_cast<size_t>(len) + 16) != cudaSuccess) {
+    free_query_dev(out);
+    return fail(BLASTP_E_NOMEM, "device allocation for the query table failed");
+  }
+  CUDA_TRY(cudaMemcpyAsync(out.woff, count.data(), sizeof(uint32_t) * (kWords + 1),
+                           cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(out.qpos, pos.data(), sizeof(uint16_t) * pos.size(),
+                           cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(out.qcodes, Q.data(), Q.size(), cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaStreamSynchronize(s));  // host vectors die here
+  return BLASTP_OK;
+}
+
+int blastp_build_query_batch(const char *const *queries, const int32_t *lens, int32_t nq,
+                             const blastp_params *p, int device, void *cuda_stream,
+                             blastp_query_table **out) {
+  if (!out) return fail(BLASTP_E_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (!queries || !lens || nq < 1) return fail(BLASTP_E_INVALID_ARG, "no queries");
+  int rc = validate_params(p);
+  if (rc) return rc;
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
+  auto *t = new (std::nothrow) blastp_query_table;
+  if (!t) return fail(BLASTP_E_NOMEM, "host allocation failed");
+  t->device = device;
+  t->p = *p;
+  t->q.resize(static_cast<size_t>(nq));
+  for (int32_t i = 0; i < nq; ++i) {
+    rc = build_one_query(queries[i], lens[i], p, t->q[static_cast<size_t>(i)],
+                         static_cast<cudaStream_t>(cuda_stream));
+    if (rc) {
+      blastp_query_table_free(t);
+      return rc;
+    }
+    t->entries += t->q[static_cast<size_t>(i)].entries;
+  }
+  *out = t;
+  return BLASTP_OK;
+}
+
+int blastp_build_query_table(const char *query_ascii, int32_t len, const blastp_params *p,
+                             int device, void *cuda_stream, blastp_query_table **out) {
+  const char *qs[1] = {query_ascii};
+  int32_t ls[1] = {len};
+  return blastp_build_query_batch(qs, ls, 1, p, device, cuda_stream, out);
+}
+
+int blastp_query_table_info(const blastp_query_table *q, int32_t *num_queries,
+                            int64_t *table_entries) {
+  if (!q) return fail(BLASTP_E_INVALID_ARG, "table is NULL");
+  if (num_queries) *num_queries = static_cast<int32_t>(q->q.size());
+  if (table_entries) *table_entries = q->entries;
+  return BLASTP_OK;
+}
+
+void blastp_query_table_free(blastp_query_table *q) {
+  if (!q) return;
+  DeviceGuard g(q->device);
+  for (auto &d : q->q) free_query_dev(d);
+  delete q;
+}
+
+// --------------------------------------------------------- database / shards
+
+int blastp_shard_range(const int64_t *offsets, int64_t nseq, int32_t shard_index,
+                       int32_t num_shards, int64_t *lo, int64_t *hi) {
+  if (!offsets || !lo || !hi || nseq < 0 || num_shards < 1 || shard_index < 0 ||
+      shard_index >= num_shards)
+    return fail(BLASTP_E_INVALID_ARG, "bad shard arguments (shard %d of %d, nseq %lld)",
+                shard_index, num_shards, static_cast<long long>(nseq));
+  const int64_t total = offsets[nseq] - offsets[0];
+  auto first_at = [&](int32_t k) -> int64_t {
+    if (k <= 0) return 0;
+    if (k >= num_shards) return nseq;
+    // first i with offsets[i] - offsets[0] >= total * k / num_shards
+    const __int128 num = static_cast<__int128>(total) * k;
+    const int64_t target = static_cast<int64_t>(num / num_shards);
+    int64_t a = 0, b = nseq;
+    while (a < b) {
+      const int64_t m = (a + b) / 2;
+      if (offsets[m] - offsets[0] >= target) b = m; else a = m + 1;
+    }
+    return a;
+  };
+  *lo = first_at(shard_index);
+  *hi = first_at(shard_index + 1);
+  if (*hi < *lo) *hi = *lo;
+  return BLASTP_OK;
+}
+
+int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t nseq,
+                   int32_t shard_index, int32_t num_shards, int device, void *cuda_stream,
+                   blastp_db **out) {
+  if (!out) return fail(BLASTP_E_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (!offsets || nseq < 0) return fail(BLASTP_E_INVALID_ARG, "offsets NULL or nseq < 0");
+  int64_t lo = 0, hi = 0;
+  int rc = blastp_shard_range(offsets, nseq, shard_index, num_shards, &lo, &hi);
+  if (rc) return rc;
+  for (int64_t i = 0; i < nseq; ++i) {
+    const int64_t L = offsets[i + 1] - offsets[i];
+    if (L < 0) return fail(BLASTP_E_INVALID_ARG, "offsets decrease at subject %lld", static_cast<long long>(i));
+    if (i >= lo && i < hi && L > BLASTP_MAX_SUBJECT_LEN)
+      return fail(BLASTP_E_TOO_LONG, "subject %lld has %lld residues", static_cast<long long>(i),
+                  static_cast<long long>(L));
+  }
+  const int64_t n = hi - lo;
+  const int64_t nres = offsets[hi] - offsets[lo];
+  if (nres > 0 && !residues_ascii) return fail(BLASTP_E_INVALID_ARG, "residues is NULL");
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+
+  auto *db = new (std::nothrow) blastp_db;
+  if (!db) return fail(BLASTP_E_NOMEM, "host allocation failed");
+  db->device = device;
+  db->sms = num_sms(device);
+  db->nseq = n;
+  db->residues = nres;
+  db->subject_base = lo;
+  // Stream layout: kStreamPadFront sentinels, then subject i at
+  // sstart[i] = pad + (offsets[lo+i] - offsets[lo]) + i, each followed by
+  // one sentinel; kStreamPadBack trailing sentinels; 16-byte multiple.
+  db->h_sstart.resize(static_cast<size_t>(n));
+  for (int64_t i = 0; i < n; ++i)
+    db->h_sstart[static_cast<size_t>(i)] = kStreamPadFront + (offsets[lo + i] - offsets[lo]) + i;
+  db->stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 15) & ~int64_t(15);
+
+  // Chunks of whole subjects, ~C residues each (>= 4 chunks per warp at
+  // 16 warps/SM), the long ones first so they start early.
+  int64_t C = nres / (int64_t(db->sms) * 16 * 4);
+  C = std::min<int64_t>(std::max<int64_t>(C, 1024), 16384);
+  std::vector<Chunk> chunks;
+  for (int64_t i = 0; i < n;) {
+    const int64_t first = i;
+    int64_t acc = 0;
+    while (i < n) {
+      const int64_t L = offsets[lo + i + 1] - offsets[lo + i];
+      if (i != first && acc + L > C) break;
+      acc += L;
+      ++i;
+    }
+    Chunk c;
+    c.start = db->h_sstart[static_cast<size_t>(first)];
+    c.end = db->h_sstart[static_cast<size_t>(i - 1)] + (offsets[lo + i] - offsets[lo + i - 1]);
+    c.first_subj = first;
+    c.last_subj = i;
+    chunks.push_back(c);
+  }
+  std::stable_partition(chunks.begin(), chunks.end(),
+                        [&](const Chunk &c) { return c.end - c.start > 2 * C; });
+  db->nchunks = static_cast<int32_t>(chunks.size());
+
+  uint8_t *d_ascii = nullptr;
+  int64_t *d_off = nullptr;
+  int *d_err = nullptr;
+  auto cleanup = [&](int code) {
+    cudaFree(d_ascii);
+    cudaFree(d_off);
+    cudaFree(d_err);
+    if (code != BLASTP_OK) blastp_db_free(db);
+    return code;
+  };
+  if (cudaMalloc(&db->stream, static_cast<size_t>(db->stream_len)) != cudaSuccess ||
+      cudaMalloc(&db->sstart, sizeof(int64_t) * static_cast<size_t>(std::max<int64_t>(n, 1))) != cudaSuccess ||
+      cudaMalloc(&db->chunks, sizeof(Chunk) * std::max<size_t>(chunks.size(), 1)) != cudaSuccess ||
+      cudaMalloc(&db->counters, sizeof(unsigned long long) * 8) != cudaSuccess ||
+      cudaMalloc(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1))) != cudaSuccess ||
+      cudaMalloc(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1)) != cudaSuccess ||
+      cudaMalloc(&d_err, sizeof(int)) != cudaSuccess) {
+    cudaGetLastError();
+    return cleanup(fail(BLASTP_E_NOMEM, "device allocation for the database failed"));
+  }
+  upload_encode_table();
+  cudaError_t e = cudaMemsetAsync(db->stream, kSentinel, static_cast<size_t>(db->stream_len), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(d_err, 0, sizeof(int), s);
+  if (e == cudaSuccess && nres > 0)
+    e = cudaMemcpyAsync(d_ascii, residues_ascii + offsets[lo], static_cast<size_t>(nres),
+                        cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d_off, offsets + lo, sizeof(int64_t) * static_cast<size_t>(n + 1),
+                        cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess && n > 0)
+    e = cudaMemcpyAsync(db->sstart, db->h_sstart.data(), sizeof(int64_t) * static_cast<size_t>(n),
+                        cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess && !chunks.empty())
+    e = cudaMemcpyAsync(db->chunks, chunks.data(), sizeof(Chunk) * chunks.size(),
+                        cudaMemcpyHostToDevice, s);
+  if (e == cudaSuccess) e = launch_pack(d_ascii, d_off, n, db->sstart, db->stream, d_err, s);
+  int h_err = 0;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&h_err, d_err, sizeof(int), cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess)
+    return cleanup(fail(BLASTP_E_CUDA, "packing the database failed: %s", cudaGetErrorString(e)));
+  if (h_err) {
+    // find the offending byte on the host for a precise message
+    for (int64_t k = offsets[lo]; k < offsets[hi]; ++k)
+      if (encode_char(static_cast<unsigned char>(residues_ascii[k])) < 0)
+        return cleanup(fail(BLASTP_E_BAD_RESIDUE, "database byte %lld (0x%02x) is not a residue",
+                            static_cast<long long>(k), static_cast<unsigned char>(residues_ascii[k])));
+    return cleanup(fail(BLASTP_E_BAD_RESIDUE, "database holds an invalid residue"));
+  }
+  *out = db;
+  return cleanup(BLASTP_OK);
+}
+
+int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues, int64_t *subject_base,
+                   int64_t *stream_bytes, int64_t *num_chunks) {
+  if (!db) return fail(BLASTP_E_INVALID_ARG, "db is NULL");
+  if (nseq) *nseq = db->nseq;
+  if (residues) *residues = db->residues;
+  if (subject_base) *subject_base = db->subject_base;
+  if (stream_bytes) *stream_bytes = db->stream_len;
+  if (num_chunks) *num_chunks = db->nchunks;
+  return BLASTP_OK;
+}
+
+void blastp_db_free(blastp_db *db) {
+  if (!db) return;
+  DeviceGuard g(db->device);
+  cudaFree(db->stream);
+  cudaFree(db->sstart);
+  cudaFree(db->chunks);
+  cudaFree(db->counters);
+  cudaFree(db->out);
+  delete db;
+}
+
+void blastp_hsp_free(blastp_hsp *h) { free(h); }
+
+// ------------------------------------------------------------------ search
+
+static int check_pair(const blastp_query_table *q, const blastp_db *db, const blastp_params *p) {
+  if (!q || !db) return fail(BLASTP_E_INVALID_ARG, "table or db is NULL");
+  int rc = validate_params(p);
+  if (rc) return rc;
+  if (q->device != db->device)
+    return fail(BLASTP_E_INVALID_ARG, "table on device %d, db on device %d", q->device, db->device);
+  if (p->threshold != q->p.threshold || p->word_len != q->p.word_len)
+    return fail(BLASTP_E_INVALID_ARG, "threshold/word_len differ from the table's (%d/%d)",
+                q->p.threshold, q->p.word_len);
+  return BLASTP_OK;
+}
+
+// Enqueue the search of every query of `q` against `db`: HSPs appended to
+// out (capacity cap) with the count in *count (device).  trace: optional.
+static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
+                          const blastp_params *p, cudaStream_t s, blastp_hsp *out, int64_t cap,
+                          unsigned long long *count, TraceRec *const trace[3],
+                          const int64_t trace_cap[3], unsigned long long *trace_count) {
+  CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
+  if (trace_count) CUDA_TRY(cudaMemsetAsync(trace_count, 0, 3 * sizeof(unsigned long long), s));
+  if (db->nchunks == 0) return BLASTP_OK;
+  for (const QueryDev &qd : q->q) {
+    SearchArgs a{};
+    a.stream = db->stream;
+    a.sstart = db->sstart;
+    a.subject_base = db->subject_base;
+    a.chunks = db->chunks;
+    a.nchunks = db->nchunks;
+    a.qv.woff = qd.woff;
+    a.qv.qpos = qd.qpos;
+    a.qv.qcodes = qd.qcodes;
+    a.qv.lq = qd.lq;
+    a.qv.query_id = static_cast<int32_t>(&qd - q->q.data());
+    a.word_len = p->word_len;
+    a.threshold = p->threshold;
+    a.window = p->window;
+    a.min_gap = p->min_gap;
+    a.xdrop = p->xdrop;
+    a.cutoff = p->cutoff;
+    a.filter_mode = p->filter_mode;
+    a.ring = search_ring_slots(qd.lq, p->window);
+    a.hitbuf = search_hitbuf(qd.lq);
+    a.out = out;
+    a.out_cap = cap;
+    a.hsp_count = count;
+    a.chunk_cursor = db->counters + 1;
+    for (int k = 0; k < 3; ++k) {
+      a.trace[k] = trace ? trace[k] : nullptr;
+      a.trace_cap[k] = trace ? trace_cap[k] : 0;
+    }
+    a.trace_count = trace_count;
+    CUDA_TRY(cudaMemsetAsync(db->counters + 1, 0, sizeof(unsigned long long), s));
+    CUDA_TRY(launch_search(a, db->sms, s));
+  }
+  return BLASTP_OK;
+}
+
+int blastp_search_ungapped_device(const blastp_query_table *q, const blastp_db *db,
+                                  const blastp_params *p, void *cuda_stream, blastp_hsp *d_out,
+                                  int64_t capacity, int64_t *d_count) {
+  int rc = check_pair(q, db, p);
+  if (rc) return rc;
+  if (!d_count || capacity < 0 || (capacity > 0 && !d_out))
+    return fail(BLASTP_E_INVALID_ARG, "bad output buffer");
+  DeviceGuard g(db->device);
+  return enqueue_search(q, db, p, static_cast<cudaStream_t>(cuda_stream), d_out, capacity,
+                        reinterpret_cast<unsigned long long *>(d_count), nullptr, nullptr, nullptr);
+}
+
+int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream) {
+  if (n < 0 || (n > 0 && !d_hsps)) return fail(BLASTP_E_INVALID_ARG, "bad HSP buffer");
+  CUDA_TRY(sort_hsps(d_hsps, n, static_cast<cudaStream_t>(cuda_stream)));
+  return BLASTP_OK;
+}
+
+int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
+                           const blastp_params *p, void *cuda_stream, blastp_hsp **out_host,
+                           int64_t *out_count) {
+  if (!out_host || !out_count) return fail(BLASTP_E_INVALID_ARG, "output pointers are NULL");
+  *out_host = nullptr;
+  *out_count = 0;
+  int rc = check_pair(q, db, p);
+  if (rc) return rc;
+  DeviceGuard g(db->device);
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  auto *mdb = const_cast<blastp_db *>(db);
+  if (mdb->out_cap == 0) {
+    const int64_t want = std::max<int64_t>(4096, (db->residues / 1000 + 1) * int64_t(q->q.size()));
+    if (cudaMalloc(&mdb->out, sizeof(blastp_hsp) * static_cast<size_t>(want)) != cudaSuccess)
+      return fail(BLASTP_E_NOMEM, "device HSP buffer");
+    mdb->out_cap = want;
+  }
+  unsigned long long h_count = 0;
+  for (int attempt = 0; attempt < 2; ++attempt) {
+    rc = enqueue_search(q, db, p, s, mdb->out, mdb->out_cap, mdb->counters, nullptr, nullptr,
+                        nullptr);
+    if (rc) return rc;
+    CUDA_TRY(cudaMemcpyAsync(&h_count, mdb->counters, sizeof(h_count), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    if (static_cast<int64_t>(h_count) <= mdb->out_cap) break;
+    cudaFree(mdb->out);
+    mdb->out = nullptr;
+    mdb->out_cap = 0;
+    const int64_t want = static_cast<int64_t>(h_count) + static_cast<int64_t>(h_count) / 4 + 1024;
+    if (cudaMalloc(&mdb->out, sizeof(blastp_hsp) * static_cast<size_t>(want)) != cudaSuccess)
+      return fail(BLASTP_E_NOMEM, "device HSP buffer (%lld)", static_cast<long long>(want));
+    mdb->out_cap = want;
+  }
+  const int64_t n = static_cast<int64_t>(h_count);
+  CUDA_TRY(sort_hsps(mdb->out, n, s));
+  auto *h = static_cast<blastp_hsp *>(malloc(sizeof(blastp_hsp) * static_cast<size_t>(std::max<int64_t>(n, 1))));
+  if (!h) return fail(BLASTP_E_NOMEM, "host HSP array");
+  if (n > 0) CUDA_TRY(cudaMemcpyAsync(h, mdb->out, sizeof(blastp_hsp) * static_cast<size_t>(n),
+                                      cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  *out_host = h;
+  *out_count = n;
+  return BLASTP_OK;
+}
+
+// ------------------------------------------------------------------- debug
+
+int blastp_debug_trace(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,
+                       void *cuda_stream, blastp_hit *hits, int64_t hits_cap, int64_t *n_hits,
+                       blastp_hit *passing, int64_t passing_cap, int64_t *n_passing,
+                       blastp_hsp *exts, int64_t exts_cap, int64_t *n_exts) {
+  int rc = check_pair(q, db, p);
+  if (rc) return rc;
+  if (hits_cap < 0 || passing_cap < 0 || exts_cap < 0 || (hits_cap && !hits) ||
+      (passing_cap && !passing) || (exts_cap && !exts))
+    return fail(BLASTP_E_INVALID_ARG, "bad trace buffers");
+  DeviceGuard g(db->device);
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  const int64_t caps[3] = {hits_cap, passing_cap, exts_cap};
+  TraceRec *tr[3] = {nullptr, nullptr, nullptr};
+  unsigned long long *tcount = nullptr, *hcount = nullptr;
+  blastp_hsp *dout = nullptr;
+  auto cleanup = [&](int code) {
+    for (auto *t : tr) cudaFree(t);
+    cudaFree(tcount);
+    cudaFree(hcount);
+    cudaFree(dout);
+    return code;
+  };
+  for (int k = 0; k < 3; ++k)
+    if (cudaMalloc(&tr[k], sizeof(TraceRec) * static_cast<size_t>(std::max<int64_t>(caps[k], 1))) != cudaSuccess)
+      return cleanup(fail(BLASTP_E_NOMEM, "trace buffers"));
+  if (cudaMalloc(&tcount, 3 * sizeof(unsigned long long)) != cudaSuccess ||
+      cudaMalloc(&hcount, sizeof(unsigned long long)) != cudaSuccess ||
+      cudaMalloc(&dout, sizeof(blastp_hsp)) != cudaSuccess)
+    return cleanup(fail(BLASTP_E_NOMEM, "trace counters"));
+  rc = enqueue_search(q, db, p, s, dout, 0, hcount, tr, caps, tcount);
+  if (rc) return cleanup(rc);
+  unsigned long long cnt[3] = {0, 0, 0};
+  if (cudaMemcpyAsync(cnt, tcount, sizeof(cnt), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+      cudaStreamSynchronize(s) != cudaSuccess)
+    return cleanup(fail(BLASTP_E_CUDA, "trace readback: %s", cudaGetErrorString(cudaGetLastError())));
+  int64_t *outs[3] = {n_hits, n_passing, n_exts};
+  bool over = false;
+  std::vector<TraceRec> buf;
+  for (int k = 0; k < 3; ++k) {
+    if (outs[k]) *outs[k] = static_cast<int64_t>(cnt[k]);
+    const int64_t m = std::min<int64_t>(static_cast<int64_t>(cnt[k]), caps[k]);
+    if (static_cast<int64_t>(cnt[k]) > caps[k]) over = true;
+    if (m <= 0) continue;
+    buf.resize(static_cast<size_t>(m));
+    if (cudaMemcpy(buf.data(), tr[k], sizeof(TraceRec) * static_cast<size_t>(m),
+                   cudaMemcpyDeviceToHost) != cudaSuccess)
+      return cleanup(fail(BLASTP_E_CUDA, "trace copy"));
+    for (int64_t i = 0; i < m; ++i) {
+      const TraceRec &r = buf[static_cast<size_t>(i)];
+      const auto it = std::upper_bound(db->h_sstart.begin(), db->h_sstart.end(), r.sp);
+      const int64_t subj = (it - db->h_sstart.begin()) - 1;
+      const int32_t sl = static_cast<int32_t>(r.sp - db->h_sstart[static_cast<size_t>(subj)]);
+      const int32_t sid = static_cast<int32_t>(db->subject_base + subj);
+      if (k < 2) {
+        blastp_hit h{r.query_id, sid, r.q, sl};
+        (k == 0 ? hits : passing)[i] = h;
+      } else {
+        blastp_hsp h;
+        h.query_id = r.query_id;
+        h.subject_id = sid;
+        h.q_start = r.q - r.llen;
+        h.s_start = sl - r.llen;
+        h.diagonal = h.s_start - h.q_start;
+        h.length = r.llen + p->word_len + r.rlen;
+        h.score = r.score;
+        exts[i] = h;
+      }
+    }
+  }
+  return cleanup(over ? fail(BLASTP_E_CAPACITY, "trace capacity exceeded") : BLASTP_OK);
+}
+
+int blastp_debug_hits(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,
+                      void *cuda_stream, blastp_hit *hits, int64_t cap, int64_t *n) {
+  return blastp_debug_trace(q, db, p, cuda_stream, hits, cap, n, nullptr, 0, nullptr, nullptr, 0,
+                            nullptr);
+}
+
+int blastp_debug_passing(const blastp_query_table *q, const blastp_db *db,
+                         const blastp_params *p, void *cuda_stream, blastp_hit *passing,
+                         int64_t cap, int64_t *n) {
+  return blastp_debug_trace(q, db, p, cuda_stream, nullptr, 0, nullptr, passing, cap, n, nullptr,
+                            0, nullptr);
+}
+
+}  // extern "C"

@@ -1,0 +1,111 @@
+// common.cuh -- product-side constants and device structs of libblastp.so.
+//
+// This is the CUDA path's own copy of the alphabet (R1) and BLOSUM62 (R2);
+// it shares nothing with oracle/ (the oracle has its own literal).
+#pragma once
+
+#include <cstdint>
+
+#include <cuda_runtime.h>
+
+#include "../../include/blastp.h"
+
+namespace blastp {
+
+// R1 alphabet: NCBI order; code = index.  Code 31 separates subjects in the
+// packed stream ("sentinel"); codes 24..30 are never produced.
+constexpr char kAlphabet[] = "ARNDCQEGHILKMFPSTWYVBZX*";
+constexpr int kNumLetters = 24;
+constexpr int kSentinel = 31;
+constexpr int kWords = kNumLetters * kNumLetters * kNumLetters;  // 13824
+// Scores involving a sentinel (or an unused code).  An extension that steps
+// onto a sentinel drops by >= 128 - 11*2 > X (X <= 127 is validated), so the
+// X-drop stops exactly at a subject boundary (R8 "end of either sequence").
+constexpr int kSentinelScore = -128;
+
+// Leading / trailing sentinel padding of the packed stream (bytes).
+constexpr int64_t kStreamPadFront = 16;
+constexpr int64_t kStreamPadBack = 256;
+
+// NCBI BLOSUM62, order kAlphabet.
+constexpr int8_t kBlosum62[kNumLetters][kNumLetters] = {
+    {4, -1, -2, -2, 0, -1, -1, 0, -2, -1, -1, -1, -1, -2, -1, 1, 0, -3, -2, 0, -2, -1, 0, -4},
+    {-1, 5, 0, -2, -3, 1, 0, -2, 0, -3, -2, 2, -1, -3, -2, -1, -1, -3, -2, -3, -1, 0, -1, -4},
+    {-2, 0, 6, 1, -3, 0, 0, 0, 1, -3, -3, 0, -2, -3, -2, 1, 0, -4, -2, -3, 3, 0, -1, -4},
+    {-2, -2, 1, 6, -3, 0, 2, -1, -1, -3, -4, -1, -3, -3, -1, 0, -1, -4, -3, -3, 4, 1, -1, -4},
+    {0, -3, -3, -3, 9, -3, -4, -3, -3, -1, -1, -3, -1, -2, -3, -1, -1, -2, -2, -1, -3, -3, -2, -4},
+    {-1, 1, 0, 0, -3, 5, 2, -2, 0, -3, -2, 1, 0, -3, -1, 0, -1, -2, -1, -2, 0, 3, -1, -4},
+    {-1, 0, 0, 2, -4, 2, 5, -2, 0, -3, -3, 1, -2, -3, -1, 0, -1, -3, -2, -2, 1, 4, -1, -4},
+    {0, -2, 0, -1, -3, -2, -2, 6, -2, -4, -4, -2, -3, -3, -2, 0, -2, -2, -3, -3, -1, -2, -1, -4},
+    {-2, 0, 1, -1, -3, 0, 0, -2, 8, -3, -3, -1, -2, -1, -2, -1, -2, -2, 2, -3, 0, 0, -1, -4},
+    {-1, -3, -3, -3, -1, -3, -3, -4, -3, 4, 2, -3, 1, 0, -3, -2, -1, -3, -1, 3, -3, -3, -1, -4},
+    {-1, -2, -3, -4, -1, -2, -3, -4, -3, 2, 4, -2, 2, 0, -3, -2, -1, -2, -1, 1, -4, -3, -1, -4},
+    {-1, 2, 0, -1, -3, 1, 1, -2, -1, -3, -2, 5, -1, -3, -1, 0, -1, -3, -2, -2, 0, 1, -1, -4},
+    {-1, -1, -2, -3, -1, 0, -2, -3, -2, 1, 2, -1, 5, 0, -2, -1, -1, -1, -1, 1, -3, -1, -1, -4},
+    {-2, -3, -3, -3, -2, -3, -3, -3, -1, 0, 0, -3, 0, 6, -4, -2, -2, 1, 3, -1, -3, -3, -1, -4},
+    {-1, -2, -2, -1, -3, -1, -1, -2, -2, -3, -3, -1, -2, -4, 7, -1, -1, -4, -3, -2, -2, -1, -2, -4},
+    {1, -1, 1, 0, -1, 0, 0, 0, -1, -2, -2, 0, -1, -2, -1, 4, 1, -3, -2, -2, 0, 0, 0, -4},
+    {0, -1, 0, -1, -1, -1, -1, -2, -2, -1, -1, -1, -1, -2, -1, 1, 5, -2, -2, 0, -1, -1, 0, -4},
+    {-3, -3, -4, -4, -2, -2, -3, -2, -2, -3, -2, -3, -1, 1, -4, -3, -2, 11, 2, -3, -4, -3, -2, -4},
+    {-2, -2, -2, -3, -2, -1, -2, -3, 2, -1, -1, -2, -1, 3, -3, -2, -2, 2, 7, -1, -3, -2, -1, -4},
+    {0, -3, -3, -3, -1, -2, -2, -3, -3, 3, 1, -2, 1, -1, -2, -2, 0, -3, -1, 4, -3, -2, -1, -4},
+    {-2, -1, 3, 4, -3, 0, 1, -1, 0, -3, -4, 0, -3, -3, -2, 0, -1, -4, -3, -3, 4, 1, -1, -4},
+    {-1, 0, 0, 1, -3, 3, 4, -2, 0, -3, -3, 1, -1, -3, -1, 0, -1, -3, -2, -2, 1, 4, -1, -4},
+    {0, -1, -1, -1, -2, -1, -1, -1, -1, -1, -1, -1, -1, -1, -2, 0, 0, -2, -1, -1, -1, -1, -1, -4},
+    {-4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, -4, 1},
+};
+
+// A contiguous range of whole subjects searched by one warp.  Positions are
+// byte offsets in the packed stream; stream[start-1] and stream[end] are
+// sentinels.  Subjects [first_subj, last_subj) (shard-local indices).
+struct Chunk {
+  int64_t start, end;
+  int64_t first_subj, last_subj;
+};
+
+// Trace record (debug entry points only): stream position of the hit /
+// seed, query position, and for extensions llen/rlen/score.
+struct TraceRec {
+  int64_t sp;
+  int32_t q, llen, rlen, score, query_id, pad;
+};
+
+// Per-query device view of a lookup table (R3): CSR word -> query positions.
+struct QueryView {
+  const uint32_t *woff;   // [kWords + 1]
+  const uint16_t *qpos;   // [entries], ascending within a word
+  const uint8_t *qcodes;  // [lq] query codes
+  int32_t lq, query_id;
+};
+
+struct SearchArgs {
+  const uint8_t *stream;
+  const int64_t *sstart;  // [nseq]: stream position of each subject's first residue
+  int64_t subject_base;
+  const Chunk *chunks;
+  int32_t nchunks;
+  QueryView qv;
+  int32_t word_len, threshold, window, min_gap, xdrop, cutoff, filter_mode;
+  int32_t ring;      // M: per-warp diagonal ring slots
+  int32_t hitbuf;    // per-warp flattened hit buffer capacity
+  blastp_hsp *out;
+  int64_t out_cap;
+  unsigned long long *hsp_count;     // one counter
+  unsigned long long *chunk_cursor;  // work-stealing cursor
+  TraceRec *trace[3];                // hits, passing, extensions (or null)
+  int64_t trace_cap[3];
+  unsigned long long *trace_count;   // [3]
+};
+
+// Launch helpers implemented in search.cu / pack.cu / sort.cu.
+size_t search_smem_bytes(int lq, int ring, int hitbuf, int warps);
+int search_ring_slots(int lq, int window);
+int search_hitbuf(int lq);
+cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s);
+cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
+                        const int64_t *sstart, uint8_t *stream, int *err,
+                        cudaStream_t s);
+cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
+void upload_encode_table();
+
+}  // namespace blastp

@@ -1,0 +1,241 @@
+"""GPU parity: the CUDA path through the C-ABI vs the CPU oracle, element by
+element (bit-exact: all arithmetic is integer).  Run with -m gpu on a B200."""
+import os
+
+import numpy as np
+import pytest
+
+from synth import config_workload, gen_db, gen_query
+
+pytestmark = pytest.mark.gpu
+
+ALPHA = "ARNDCQEGHILKMFPSTWYVBZX*"
+
+
+@pytest.fixture(scope="module")
+def bp():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_ipps_zhangwlf14_b200 import build
+    build.build()
+    from paper_conf_ipps_zhangwlf14_b200 import blastp
+    return blastp
+
+
+def tuples(a):
+    return [tuple(int(v) for v in x) for x in a.tolist()]
+
+
+def hit_set(a):
+    return sorted((int(h[0]), int(h[1]), int(h[2]), int(h[3])) for h in a)
+
+
+def oracle_run(orc, q_ascii, ascii, offsets, p, want_hits=False, nthreads=1, query_id=0):
+    P = orc.Params(word_len=p.word_len, threshold=p.threshold, window=p.window,
+                   min_gap=p.min_gap, xdrop=p.xdrop, cutoff=p.cutoff, filter_mode=p.filter_mode)
+    codes = orc.encode(ascii.tobytes() if hasattr(ascii, "tobytes") else ascii)
+    return orc.search(orc.encode(q_ascii), codes, np.asarray(offsets, dtype=np.int64), P,
+                      want_hits=want_hits, nthreads=nthreads, query_id=query_id)
+
+
+def gpu_run(bp, q_ascii, ascii, offsets, p, trace=False):
+    t = bp.build_query_table(q_ascii, p)
+    d = bp.pack_db(ascii, offsets)
+    hsps = bp.search_ungapped(t, d, p)
+    tr = bp.debug_trace(t, d, p) if trace else None
+    return hsps, tr
+
+
+def assert_same(bp, orc, q, ascii, offsets, p, trace=True, nthreads=1):
+    g, tr = gpu_run(bp, q, ascii, offsets, p, trace)
+    r = oracle_run(orc, q, ascii, offsets, p, want_hits=trace, nthreads=nthreads)
+    assert tuples(g) == tuples(r.hsps), (len(g), len(r.hsps))
+    if trace:
+        oh = sorted((0, int(a), int(b), int(c)) for a, b, c in r.hits)
+        op = sorted((0, int(a), int(b), int(c)) for a, b, c in r.passing)
+        assert hit_set(tr.hits) == oh
+        assert hit_set(tr.passing) == op
+        ext = np.sort(tr.extensions, order=list(tr.extensions.dtype.names))
+        assert tuples(ext) == tuples(r.extensions)
+    return g, r
+
+
+# ------------------------------------------------------------------ configs
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_config1_full_trace(bp, orc, mode):
+    """Config 1 (q127 vs 1,000 subjects): hits, passing hits, every extension
+    and the HSP list identical to the oracle, both filter readings."""
+    (q,), db = config_workload(1)
+    p = bp.Params(filter_mode=mode)
+    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, p)
+    assert len(g) > 10
+
+
+def test_config2_full(bp, orc):
+    """Config 2 (q517 vs 20M residues), complete HSP list."""
+    (q,), db = config_workload(2)
+    p = bp.Params()
+    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, p, trace=False,
+                       nthreads=os.cpu_count() or 8)
+    assert len(g) > 1000
+
+
+def test_config3_full_size_sampled(bp, orc):
+    """Config 3 at full size (q1054 vs ~1.2G residues, the bench launch):
+    the oracle re-searches a deterministic sample of subject blocks and the
+    GPU's HSPs restricted to those subjects must be identical; every GPU HSP
+    is re-scored from the sequences."""
+    (q,), db = config_workload(3)
+    p = bp.Params()
+    t = bp.build_query_table(q, p)
+    d = bp.pack_db(db.ascii, db.offsets)
+    g = bp.search_ungapped(t, d, p)
+    assert len(g) > 10000
+    B = orc.blosum62()
+    Q = orc.encode(q)
+    rng = np.random.default_rng(0)
+    for h in g[rng.choice(len(g), size=2000, replace=False)]:
+        a = db.offsets[h["subject_id"]] + h["s_start"]
+        S = orc.encode(db.ascii[a:a + h["length"]].tobytes())
+        assert B[Q[h["q_start"]:h["q_start"] + h["length"]], S].sum() == h["score"]
+    n = db.nseq
+    blocks = [(k, min(k + 3000, n)) for k in range(0, n, n // 12)][:12]
+    blocks.append((n // 2 - 5, n // 2 + 5))  # the 36,805-residue subject
+    for lo, hi in blocks:
+        sub_off = db.offsets[lo:hi + 1]
+        ascii = db.ascii[sub_off[0]:sub_off[-1]]
+        r = oracle_run(orc, q, ascii, sub_off - sub_off[0], p)
+        exp = r.hsps.copy()
+        exp["subject_id"] += lo
+        sel = g[(g["subject_id"] >= lo) & (g["subject_id"] < hi)]
+        assert tuples(sel) == tuples(exp), (lo, hi)
+
+
+# ------------------------------------------------------------------ fuzz
+
+def _rand_db(rng, n, lo, hi, q=None, plant=0.3):
+    subs = []
+    for _ in range(n):
+        L = int(rng.integers(lo, hi + 1))
+        s = rng.choice(list(ALPHA[:20]), size=L)
+        if q is not None and L > 10 and rng.random() < plant:
+            k = int(rng.integers(5, min(L, len(q)) + 1))
+            a = int(rng.integers(0, len(q) - k + 1))
+            b = int(rng.integers(0, L - k + 1))
+            seg = np.array(list(q[a:a + k]))
+            mut = rng.random(k) < 0.25
+            seg[mut] = rng.choice(list(ALPHA[:20]), size=int(mut.sum()))
+            s[b:b + k] = seg
+        subs.append("".join(s))
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    return np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy(), off
+
+
+def test_fuzz_small_random(bp, orc):
+    rng = np.random.default_rng(99)
+    for case in range(120):
+        lq = int(rng.choice([3, 5, 17, 64, 127, 300, 517]))
+        q = "".join(rng.choice(list(ALPHA[:20] if case % 4 else ALPHA), size=lq))
+        ascii, off = _rand_db(rng, int(rng.integers(1, 60)), 0, 400, q)
+        p = bp.Params(threshold=int(rng.choice([11, 11, 9, 13])),
+                      window=int(rng.choice([40, 40, 10, 80, 3])),
+                      min_gap=int(rng.choice([3, 3, 1, 2, 5])),
+                      xdrop=int(rng.choice([16, 16, 5, 30])),
+                      cutoff=int(rng.choice([41, 20, 0])),
+                      filter_mode=int(case % 2))
+        assert_same(bp, orc, q, ascii, off, p, trace=True)
+
+
+def test_adversarial_low_complexity(bp, orc):
+    """Poly-W query vs poly-W subjects: every (q, s) is a hit (the hit-dense
+    slow path), plus runs of mixed low-complexity residues."""
+    q = "W" * 300 + "AAAAQQQQ" * 10 + "W" * 50
+    subs = ["W" * 1000, "A" * 200 + "W" * 40, "WA" * 300, "Q" * 500, "W" * 3]
+    ascii = np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy()
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    for mode in (0, 1):
+        assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=mode), trace=True)
+
+
+def test_edge_cases(bp, orc):
+    q = gen_query(3, 200).decode()
+    # empty subjects, subjects shorter than a word, query itself, long subject
+    long_s = gen_query(4, 36805).decode()
+    long_s = long_s[:20000] + q + long_s[20000 + len(q):]
+    subs = ["", "A", "MK", q, "", q[::-1], long_s, q[:3], q[-5:], ""]
+    ascii = np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy()
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    g, r = assert_same(bp, orc, q, ascii, off, bp.Params(), trace=True)
+    assert any(h[1] == 3 and h[2] == 0 for h in tuples(g))  # the self hit
+    # query of exactly one word
+    assert_same(bp, orc, "WCW", ascii, off, bp.Params(threshold=5), trace=True)
+    # a database with no subjects at all
+    empty = np.zeros(0, dtype=np.uint8)
+    g, _ = gpu_run(bp, q, empty, np.zeros(1, dtype=np.int64), bp.Params())
+    assert len(g) == 0
+
+
+def test_long_query_2000(bp, orc):
+    q = gen_query(2000, 2000)
+    db = gen_db(7, 8, n_subjects=400, mean_len=375.0, queries=[q], plant_frac=0.2)
+    assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(), trace=True)
+
+
+# ------------------------------------------------------------------ API
+
+def test_device_variant_and_sort_match_host_variant(bp, orc):
+    import torch
+    (q,), db = config_workload(1)
+    p = bp.Params()
+    t = bp.build_query_table(q, p)
+    d = bp.pack_db(db.ascii, db.offsets)
+    host = bp.search_ungapped(t, d, p)
+    cap = len(host) + 5
+    out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    bp.search_ungapped_device(t, d, out.data_ptr(), cap, cnt.data_ptr(), p)
+    n = int(cnt.item())
+    assert n == len(host)
+    bp.sort_hsps_device(out.data_ptr(), n)
+    dev = out[: n * 7].view(n, 7).cpu().numpy()
+    assert [tuple(x) for x in dev.tolist()] == tuples(host)
+    # a too-small buffer still reports the full count
+    small = torch.zeros(7 * 3, dtype=torch.int32, device="cuda")
+    bp.search_ungapped_device(t, d, small.data_ptr(), 3, cnt.data_ptr(), p)
+    assert int(cnt.item()) == len(host)
+
+
+def test_query_batch_equals_single_queries(bp, orc):
+    qs = [gen_query(11 + i, L) for i, L in enumerate([100, 350, 900])]
+    db = gen_db(12, 13, n_subjects=500, mean_len=300.0, queries=qs, plant_frac=0.3)
+    p = bp.Params()
+    d = bp.pack_db(db.ascii, db.offsets)
+    batch = bp.search_ungapped(bp.build_query_batch(qs, p), d, p)
+    exp = []
+    for i, q in enumerate(qs):
+        exp += tuples(oracle_run(orc, q, db.ascii, db.offsets, p, query_id=i).hsps)
+    assert tuples(batch) == sorted(exp)
+
+
+def test_sharded_union_equals_whole(bp, orc):
+    (q,), db = config_workload(1)
+    p = bp.Params()
+    t = bp.build_query_table(q, p)
+    whole = tuples(bp.search_ungapped(t, bp.pack_db(db.ascii, db.offsets), p))
+    for n in (2, 3, 8):
+        parts = []
+        for k in range(n):
+            parts += tuples(bp.search_ungapped(t, bp.pack_db(db.ascii, db.offsets, k, n), p))
+        assert parts == whole  # contiguous ranges, canonical order per shard
+
+
+def test_bad_residue_reported(bp):
+    ascii = np.frombuffer(b"MKVLA-GG", dtype=np.uint8).copy()
+    with pytest.raises(bp.BlastpError) as e:
+        bp.pack_db(ascii, np.array([0, 8], dtype=np.int64))
+    assert e.value.status == bp.E_BAD_RESIDUE
+    with pytest.raises(bp.BlastpError) as e:
+        bp.build_query_table("MKV1", bp.Params())
+    assert e.value.status == bp.E_BAD_RESIDUE
