@@ -124,13 +124,14 @@ __device__ bool has_successor(const uint8_t *__restrict__ stream, int64_t sp, in
                               const uint8_t *qc, const int8_t *b62, int lq, int W, int A, int T) {
   const int kmax = min(A - 1, lq - 3 - q);
   if (kmax < W) return false;
-  int s1 = score(b62, qc[q + W], __ldg(stream + sp + W));
-  int s2 = score(b62, qc[q + W + 1], __ldg(stream + sp + W + 1));
-  for (int k = W; k <= kmax; ++k) {
-    const uint32_t c3 = __ldg(stream + sp + k + 2);
-    if (c3 == uint32_t(kSentinel)) return false;  // the subject ends here
-    const int s3 = score(b62, qc[q + k + 2], c3);
-    if (s1 + s2 + s3 >= T) return true;
+  // rolling pair scores at offsets j-2, j-1 (offsets 1, 2 lie in the hit word)
+  int s1 = score(b62, qc[q + 1], __ldg(stream + sp + 1));
+  int s2 = score(b62, qc[q + 2], __ldg(stream + sp + 2));
+  for (int j = 3; j <= kmax + 2; ++j) {
+    const uint32_t c = __ldg(stream + sp + j);
+    if (c == uint32_t(kSentinel)) return false;  // the subject ends: no later word
+    const int s3 = score(b62, qc[q + j], c);
+    if (j - 2 >= W && s1 + s2 + s3 >= T) return true;
     s1 = s2;
     s2 = s3;
   }
