@@ -1,0 +1,373 @@
+#!/usr/bin/env python
+"""bench.py -- database residues/s of the B200 BLASTP hot path (hit detection +
+two-hit filter + X-drop ungapped extension), BASELINE.json's metric.
+
+  python bench.py [--gpus N --steps K --warmup W] [--impl ours|reference]
+  torchrun --nproc-per-node N bench.py --gpus N ...      (N > 1, NCCL)
+
+Workload: BASELINE config 3 -- query length 1054
+against the env_nr-shaped synthetic database (6.0M subjects, ~1.2G residues,
+RR frequencies, 0.5% planted homologs).  At N > 1 the same database is
+sharded by subject range over the ranks (config 4, strong scaling) and the
+HSPs are gathered to rank 0 over NCCL inside every step.
+
+One step = one full search of every query against the (local shard of the)
+database: the fused search kernel(s) plus, at N > 1, the HSP gather.  The
+database (1.2 GB) is larger than L2 (126 MB), so no flush is needed between
+steps.  Device time: CUDA events on the launching stream, barrier +
+synchronize around the timed region, max over ranks.
+
+e2e: the same metric through the C-ABI with HOST buffers: each step packs the
+shard from pinned host memory (H2D inside blastp_pack_db), searches, gathers
+(N > 1) and reads the HSP list back to the host.
+
+--impl reference: the CPU oracle (oracle/, test infrastructure) timed on the
+host cores on a bounded sample of the same workload, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "database residues/sec (hit detect + ungapped ext) at 1/2/4/8 B200; % HBM roofline"
+UNIT = "residues/s"
+CPU_SAMPLE_RESIDUES = 240_000_000  # oracle sample (first subjects of the DB)
+
+
+def parse_args():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", type=int, default=3, choices=[1, 2, 3])
+    ap.add_argument("--query-lens", default="1054",
+                    help="comma list of query lengths searched as one batch (config 4: 127,517,1054)")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--scale", type=float, default=1.0, help="DB scale (tests only)")
+    return ap.parse_args()
+
+
+def env_rank():
+    return (int(os.environ.get("RANK", "0")), int(os.environ.get("LOCAL_RANK", "0")),
+            int(os.environ.get("WORLD_SIZE", "1")))
+
+
+# --------------------------------------------------------------- workload
+
+def workload(args, rank, world):
+    from paper_conf_ipps_zhangwlf14_b200.dist import shard_subjects
+    from synth import CONFIGS, config_offsets, gen_db, gen_query
+    c = CONFIGS[args.config]
+    lens = [int(x) for x in args.query_lens.split(",")] if args.config == 3 else [c["query_len"]]
+    queries = [gen_query(c["query_seed"] if L == c["query_len"] else L, L) for L in lens]
+    full_off = config_offsets(args.config, args.scale)
+    lo, hi = shard_subjects(full_off, rank, world)
+    ns, tr = c["n_subjects"], c["total_residues"]
+    if args.scale != 1.0:
+        ns = None if ns is None else max(1, int(ns * args.scale))
+        tr = None if tr is None else max(1000, int(tr * args.scale))
+    db = gen_db(c["db_seed"], c["plant_seed"], n_subjects=ns, total_residues=tr,
+                mean_len=c["mean_len"], queries=queries, plant_frac=c["plant_frac"],
+                subject_range=(lo, hi))
+    desc = (f"config{args.config}{'/4' if world > 1 else ''}: q{'+'.join(map(str, lens))} vs "
+            f"{c['name'].split('_vs_')[-1]} synthetic DB ({len(full_off) - 1} subjects, "
+            f"{int(full_off[-1])} residues)" + (f", sharded over {world} GPUs" if world > 1 else ""))
+    return queries, db, full_off, (lo, hi), desc
+
+
+# --------------------------------------------------------------- clocks
+
+class ClockSampler:
+    """nvidia-smi sampled every 100 ms while the timed region runs."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.tmp = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"], stdout=self.tmp,
+                stderr=subprocess.DEVNULL)
+        except OSError:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        self.proc.wait()
+        self.tmp.flush()
+        rows = []
+        with open(self.tmp.name) as f:
+            for line in f:
+                parts = [p.strip() for p in line.split(",")]
+                if len(parts) >= 8 and parts[0].replace(".", "").isdigit():
+                    rows.append(parts)
+        os.unlink(self.tmp.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [float(r[0]) for r in rows]
+        mx = max(float(r[1]) for r in rows)
+        loaded = [v for v in sm if v > 0.5 * mx] or sm
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({n for r in rows for n, v in zip(names, r[4:8]) if v == "Active"})
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(rows), "power_w_max": max(float(r[2]) for r in rows
+                                                         if r[2].replace(".", "").isdigit())}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic():
+    """Per-launch DRAM bytes of the search kernel from the committed ncu capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_search_kernel.json")
+    if not os.path.exists(p):
+        return None, None
+    with open(p) as f:
+        d = json.load(f)
+    return d.get("dram_bytes_per_launch"), d.get("source")
+
+
+# --------------------------------------------------------------- reference arm
+
+def run_reference(args):
+    rank, _, world = env_rank()
+    if rank != 0:
+        return  # rank 0 alone runs the CPU arm
+    from oracle import oracle as o
+    queries, db, full_off, (lo, hi), desc = workload(args, 0, 1)
+    Qs = [o.encode(q) for q in queries]
+    tables = [o.neighbourhood(Q, o.blosum62(), 11) for Q in Qs]
+    nsub = int(np.searchsorted(db.offsets, CPU_SAMPLE_RESIDUES // max(1, args.steps + args.warmup)))
+    nsub = max(1, min(nsub, db.nseq))
+    sub_off = db.offsets[: nsub + 1]
+    codes = o.encode(db.ascii[: sub_off[-1]].tobytes())
+    cores = os.cpu_count() or 1
+    times = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        for Q, tab in zip(Qs, tables):
+            o.search(Q, codes, sub_off, table=tab, nthreads=cores, want_extensions=False)
+        if i >= args.warmup:
+            times.append(time.perf_counter() - t0)
+    res = int(sub_off[-1]) * len(Qs)
+    value = res * len(times) / sum(times)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": desc, "sample_subjects": nsub,
+                       "sample_residues": int(sub_off[-1])},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": f"first {nsub} subjects ({int(sub_off[-1])} residues) of "
+                                       f"the workload per step, {cores} pthreads"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------- our arm
+
+def cpu_baseline(queries, db):
+    from oracle import oracle as o
+    Qs = [o.encode(q) for q in queries]
+    tables = [o.neighbourhood(Q, o.blosum62(), 11) for Q in Qs]
+    nsub = max(1, min(int(np.searchsorted(db.offsets, CPU_SAMPLE_RESIDUES)), db.nseq))
+    sub_off = db.offsets[: nsub + 1]
+    codes = o.encode(db.ascii[: sub_off[-1]].tobytes())
+    cores = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    for Q, tab in zip(Qs, tables):
+        o.search(Q, codes, sub_off, table=tab, nthreads=cores, want_extensions=False)
+    dt = time.perf_counter() - t0
+    return {"value": int(sub_off[-1]) * len(Qs) / dt, "unit": UNIT, "cores": cores,
+            "kind": "oracle", "seconds": dt,
+            "sample": f"first {nsub} subjects ({int(sub_off[-1])} residues) of the same DB, "
+                      f"scan+filter+extension only (table prebuilt), {cores} pthreads"}
+
+
+def main():
+    args = parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_zhangwlf14_b200 import blastp as bp
+    from paper_conf_ipps_zhangwlf14_b200.dist import gather_hsps
+
+    rank, local_rank, world = env_rank()
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream()
+
+    queries, db, full_off, (lo, hi), desc = workload(args, rank, world)
+    params = bp.Params()
+    table = bp.build_query_batch(queries, params, device=local_rank, stream=stream)
+    nq = len(queries)
+    # pinned copy of this rank's residues: the e2e input and the pack source
+    pinned = torch.empty(max(1, db.residues), dtype=torch.uint8, pin_memory=True)
+    pinned[: db.residues].copy_(torch.from_numpy(db.ascii))
+    base_ptr = pinned.data_ptr() - int(full_off[lo])
+    gdb = bp.Database.from_pinned(base_ptr, full_off, rank, world, device=local_rank,
+                                  stream=stream)
+    assert gdb.subject_base == lo and gdb.residues == db.residues
+    cap = max(1 << 20, gdb.residues // 500 * nq)
+    out = torch.empty((cap, 7), dtype=torch.int32, device=dev)
+    cnt = torch.zeros(1, dtype=torch.int64, device=dev)
+
+    def search():
+        bp.search_ungapped_device(table, gdb, out.data_ptr(), cap, cnt.data_ptr(), params, stream)
+
+    def step():
+        search()
+        if world > 1:
+            n = int(cnt.item())
+            gather_hsps(out[: min(n, cap)])
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize()
+    n_hsp = int(cnt.item())
+    assert n_hsp <= cap, "HSP buffer too small"
+
+    # ---- timed region -------------------------------------------------------
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for k in range(args.steps):
+        ev[k][0].record(stream)
+        search()
+        ev[k][1].record(stream)
+        if world > 1:
+            gather_hsps(out[: min(int(cnt.item()), cap)])
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    elapsed_ms = t_start.elapsed_time(t_end)
+    kern_ms = [a.elapsed_time(b) for a, b in ev]
+    t = torch.tensor([elapsed_ms, statistics.mean(kern_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    elapsed_ms, kern_avg_ms = float(t[0]), float(t[1])
+    total_residues = int(full_off[-1] - full_off[0])
+    value = total_residues * nq * args.steps / (elapsed_ms / 1e3)
+
+    # ---- roofline of the dominant kernel (search_kernel) --------------------
+    peak, peak_src = peaks()
+    # algorithmic bytes per step on this rank: 1 B per residue per query pass
+    # + the HSP records written
+    alg_bytes = gdb.residues * nq + n_hsp * 28
+    achieved = alg_bytes / (statistics.mean(kern_ms) / 1e3) / 1e9
+    traffic, traffic_src = ncu_traffic()
+
+    # ---- e2e through the C-ABI with host buffers ---------------------------
+    e2e = None
+    if not args.no_e2e and args.e2e_steps > 0:
+        times, h2d, d2h = [], 0, 0
+        for k in range(args.e2e_steps + 1):
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            d = bp.Database.from_pinned(base_ptr, full_off, rank, world, device=local_rank,
+                                        stream=stream)
+            bp.search_ungapped_device(table, d, out.data_ptr(), cap, cnt.data_ptr(), params,
+                                      stream)
+            n = int(cnt.item())
+            res = out[: min(n, cap)]
+            if world > 1:
+                res = gather_hsps(res)
+            host = res.cpu() if res is not None else None
+            torch.cuda.synchronize()
+            dt = time.perf_counter() - t0
+            d.free()
+            tt = torch.tensor([dt], dtype=torch.float64, device=dev)
+            if world > 1:
+                dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            if k > 0:  # first e2e step is a warm-up
+                times.append(float(tt[0]))
+            h2d = db.residues + 8 * (hi - lo + 1)
+            d2h = 8 + (host.numel() * 4 if host is not None else 0)
+        e2e = {"value": total_residues * nq / statistics.mean(times), "unit": UNIT,
+               "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": 1e3 * statistics.mean(times),
+               "path": "blastp_pack_db(pinned host) + blastp_search_ungapped_device + "
+                       + ("NCCL gather + " if world > 1 else "") + "D2H of the HSP list"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(queries, db)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": max(args.warmup, 3),
+            "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": desc, "query_lens": [len(q) for q in queries],
+                       "db_subjects": int(len(full_off) - 1), "db_residues": total_residues,
+                       "shard_residues_rank0": int(gdb.residues),
+                       "params": {"word_len": 3, "T": 11, "A": 40, "X": 16, "cutoff": 41,
+                                  "filter": "LEFT"},
+                       "l2": "inputs larger than L2 (DB shard >> 126 MB), no flush",
+                       "hsps_per_step": n_hsp, "parallelism": f"db-shard{world}"},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "search_kernel", "kernel_ms": kern_avg_ms,
+                         "alg_bytes_per_launch": alg_bytes // nq,
+                         "peak_source": peak_src, "traffic_source": traffic_src},
+            "clocks": clk,
+            "e2e": e2e,
+            "gpu_launches": args.steps * nq,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -207,6 +207,7 @@ typedef struct {
   const int64_t *off;
   const int32_t *pos;
   oracle_hitlist *hits, *passing;
+  int collect_ext; /* keep every extension (else only count them) */
   /* outputs */
   hsp_vec out, ext;
   int err;
@@ -307,7 +308,11 @@ static void search_range(range_job *J) {
         e.length = llen + w + rlen;
         e.score = s0 + bestL + bestR;
         ext_reach = h + w - 1 + rlen; /* HSP subject end, inclusive */
-        if (hsp_push(&J->ext, &e)) { J->err = 1; break; }
+        if (J->collect_ext) {
+          if (hsp_push(&J->ext, &e)) { J->err = 1; break; }
+        } else {
+          J->ext.n++;
+        }
         if (e.score >= p->cutoff && hsp_push(&J->out, &e)) { J->err = 1; break; }
       }
     }
@@ -365,6 +370,7 @@ int64_t oracle_search(const uint8_t *query, int32_t lq, int32_t query_id,
       J->db = db; J->offsets = offsets; J->subject_base = subject_base;
       J->matrix = matrix; J->na = na; J->p = p; J->off = off; J->pos = pos;
       J->hits = hits; J->passing = passing;
+      J->collect_ext = ext_out != NULL;
       J->first = cur;
       int64_t target = offsets[0] + total * (t + 1) / nthreads;
       while (cur < nseq && offsets[cur] < target) ++cur;

@@ -169,7 +169,8 @@ class SearchResult:
 
 def search(query: np.ndarray, db: np.ndarray, offsets: np.ndarray, params: Params | None = None,
            *, query_id: int = 0, subject_base: int = 0, matrix: np.ndarray | None = None,
-           table=None, nthreads: int = 1, want_hits: bool = False) -> SearchResult:
+           table=None, nthreads: int = 1, want_hits: bool = False,
+           want_extensions: bool = True) -> SearchResult:
     """Oracle search of one query (codes) against db codes with offsets[nseq+1]."""
     p = params or Params()
     q = np.ascontiguousarray(query, dtype=np.uint8)
@@ -195,18 +196,19 @@ def search(query: np.ndarray, db: np.ndarray, offsets: np.ndarray, params: Param
         cap = 1 << 12
         for _ in range(8):
             out = np.zeros(cap, dtype=HSP_DTYPE)
-            ext = np.zeros(cap * 8, dtype=HSP_DTYPE)
+            ext = np.zeros(cap * 8 if want_extensions else 1, dtype=HSP_DTYPE)
             ext_n = ctypes.c_int64(0)
             n = lib().oracle_search(_ptr(q), len(q), query_id, _ptr(d), _ptr(off), nseq,
                                     subject_base, _ptr(m), m.shape[0], ctypes.byref(cp),
                                     None if t_off is None else _ptr(t_off),
                                     None if t_pos is None else _ptr(t_pos), nthreads,
-                                    _ptr(out), cap, _ptr(ext), len(ext), ctypes.byref(ext_n),
+                                    _ptr(out), cap, _ptr(ext) if want_extensions else None,
+                                    len(ext) if want_extensions else 0, ctypes.byref(ext_n),
                                     ctypes.byref(hl) if hl is not None else None,
                                     ctypes.byref(ps) if ps is not None else None)
             if n < 0:
                 raise RuntimeError(f"oracle_search failed ({n})")
-            if n <= cap and ext_n.value <= len(ext):
+            if n <= cap and (not want_extensions or ext_n.value <= len(ext)):
                 break
             cap = max(int(n), int(ext_n.value) // 8 + 1, cap) * 2
         if want_hits and (hl.count > cap_h or ps.count > cap_h):
@@ -217,4 +219,5 @@ def search(query: np.ndarray, db: np.ndarray, offsets: np.ndarray, params: Param
     if want_hits:
         hits = np.stack([hbufs[0][:hl.count], hbufs[1][:hl.count], hbufs[2][:hl.count]], axis=1)
         passing = np.stack([hbufs[3][:ps.count], hbufs[4][:ps.count], hbufs[5][:ps.count]], axis=1)
-    return SearchResult(out[:n].copy(), ext[:ext_n.value].copy(), hits, passing)
+    exts = ext[:ext_n.value].copy() if want_extensions else np.zeros(0, dtype=HSP_DTYPE)
+    return SearchResult(out[:n].copy(), exts, hits, passing)

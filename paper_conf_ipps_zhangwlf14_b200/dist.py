@@ -1,0 +1,116 @@
+"""Multi-GPU: one process per GPU, subject-range shards, HSP gather over NCCL.
+
+The database shards by contiguous subject ranges balanced by residues
+(blastp_shard_range); subjects are independent, so each rank
+searches its shard with no data-path communication.  The one exchange is the
+result: every rank's HSP list (int32 x 7 per HSP, device memory) is gathered
+to rank 0 with two collectives -- an all_gather of the counts, then an
+all_gather of the lists padded to the largest count -- and concatenated in
+rank order.  Because shards are contiguous in subject id and each rank's list
+is canonical (R11), the concatenation is already canonical for one query;
+for query batches rank 0 re-sorts (query_id major) on the GPU.
+
+The collective code is backend-agnostic (NCCL on GPUs, gloo in the CPU tests).
+"""
+from __future__ import annotations
+
+from typing import Callable
+
+import numpy as np
+
+HSP_FIELDS = 7
+
+
+def shard_subjects(offsets: np.ndarray, rank: int, world: int) -> tuple[int, int]:
+    """[lo, hi) of this rank's shard (same rule as blastp_shard_range)."""
+    off = np.asarray(offsets, dtype=np.int64)
+    total = int(off[-1] - off[0])
+
+    def first_at(k: int) -> int:
+        if k <= 0:
+            return 0
+        if k >= world:
+            return len(off) - 1
+        target = total * k // world
+        return int(np.searchsorted(off - off[0], target, side="left"))
+
+    lo, hi = first_at(rank), first_at(rank + 1)
+    return lo, max(lo, hi)
+
+
+def gather_hsps(local, group=None, dst: int = 0):
+    """Gather [n_r, 7] int32 HSP tensors of every rank onto rank `dst`.
+
+    Returns the concatenation in rank order on rank dst (None elsewhere).
+    Works for any torch.distributed backend; tensors stay on their device.
+    """
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    dev = local.device
+    n = torch.tensor([local.shape[0]], dtype=torch.int64, device=dev)
+    counts = [torch.zeros_like(n) for _ in range(world)]
+    dist.all_gather(counts, n, group=group)
+    counts = [int(c.item()) for c in counts]
+    maxn = max(counts) if counts else 0
+    if maxn == 0:
+        return local.new_zeros((0, HSP_FIELDS)) if rank == dst else None
+    padded = local.new_zeros((maxn, HSP_FIELDS))
+    if local.shape[0]:
+        padded[: local.shape[0]] = local
+    bufs = [local.new_empty((maxn, HSP_FIELDS)) for _ in range(world)]
+    dist.all_gather(bufs, padded, group=group)
+    if rank != dst:
+        return None
+    return torch.cat([b[:c] for b, c in zip(bufs, counts)], dim=0)
+
+
+def search_sharded(search_fn: Callable[[int, int], "object"], offsets: np.ndarray, group=None,
+                   dst: int = 0):
+    """Run `search_fn(lo, hi)` on this rank's shard and gather the results.
+
+    search_fn returns a [n, 7] int32 tensor of HSPs with GLOBAL subject ids.
+    """
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    lo, hi = shard_subjects(offsets, rank, world)
+    local = search_fn(lo, hi)
+    return gather_hsps(local, group=group, dst=dst)
+
+
+def gpu_shard_search(table, residues_local: np.ndarray, offsets_full: np.ndarray, rank: int,
+                     world: int, params=None, capacity: int | None = None, stream=None):
+    """Pack this rank's shard -- only its bytes need to be resident on the
+    host -- and search it on the current CUDA device.  Returns a device
+    [n, 7] int32 tensor (global subject ids, canonical order)."""
+    import torch
+
+    from . import blastp as bp
+
+    off = np.ascontiguousarray(offsets_full, dtype=np.int64)
+    lo, hi = shard_subjects(off, rank, world)
+    # libblastp reads residues at base + offsets[i] for the shard's subjects
+    # only; hand it a base such that base + offsets[lo] is the local buffer.
+    base = residues_local.ctypes.data - int(off[lo])
+    db = bp.Database.from_pinned(base, off, rank, world, device=torch.cuda.current_device(),
+                                 stream=stream)
+    assert db.subject_base == lo
+    try:
+        cap = capacity or max(4096, db.residues // 1000 * max(1, table.num_queries))
+        while True:
+            out = torch.empty((cap, 7), dtype=torch.int32, device="cuda")
+            cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+            bp.search_ungapped_device(table, db, out.data_ptr(), cap, cnt.data_ptr(), params,
+                                      stream)
+            n = int(cnt.item())
+            if n <= cap:
+                break
+            cap = n + n // 4 + 1024
+        res = out[:n]
+        bp.sort_hsps_device(res.data_ptr(), n, stream)
+        return res
+    finally:
+        db.free()

@@ -195,6 +195,20 @@ CONFIGS = {
 }
 
 
+def config_offsets(cfg: int, scale: float = 1.0) -> np.ndarray:
+    """Full int64 offsets of a config's database (lengths only, no residues),
+    enough to plan shards before generating just one range."""
+    c = CONFIGS[cfg]
+    ns, tr = c["n_subjects"], c["total_residues"]
+    if scale != 1.0:
+        ns = None if ns is None else max(1, int(ns * scale))
+        tr = None if tr is None else max(1000, int(tr * scale))
+    lens = _lengths(c["db_seed"], ns, tr, c["mean_len"])
+    off = np.zeros(len(lens) + 1, dtype=np.int64)
+    np.cumsum(lens, out=off[1:])
+    return off
+
+
 def config_workload(cfg: int, *, subject_range=None, scale: float = 1.0):
     """(queries, db) for a BASELINE.json config.  scale < 1 shrinks the DB
     (same generator, fewer subjects) for quick tests."""

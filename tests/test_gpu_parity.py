@@ -120,7 +120,7 @@ def _rand_db(rng, n, lo, hi, q=None, plant=0.3):
     for _ in range(n):
         L = int(rng.integers(lo, hi + 1))
         s = rng.choice(list(ALPHA[:20]), size=L)
-        if q is not None and L > 10 and rng.random() < plant:
+        if q is not None and L > 10 and len(q) >= 5 and rng.random() < plant:
             k = int(rng.integers(5, min(L, len(q)) + 1))
             a = int(rng.integers(0, len(q) - k + 1))
             b = int(rng.integers(0, L - k + 1))
