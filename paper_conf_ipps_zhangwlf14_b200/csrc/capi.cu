@@ -336,7 +336,7 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   db->h_sstart.resize(static_cast<size_t>(n));
   for (int64_t i = 0; i < n; ++i)
     db->h_sstart[static_cast<size_t>(i)] = kStreamPadFront + (offsets[lo + i] - offsets[lo]) + i;
-  db->stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 15) & ~int64_t(15);
+  db->stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 511) & ~int64_t(511);
 
   // Chunks of whole subjects, ~C residues each (>= 4 chunks per warp at
   // 16 warps/SM), the long ones first so they start early.
@@ -483,7 +483,7 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.cutoff = p->cutoff;
     a.filter_mode = p->filter_mode;
     a.ring = search_ring_slots(qd.lq, p->window);
-    a.hitbuf = search_hitbuf(qd.lq);
+    a.table_entries = qd.entries;
     a.out = out;
     a.out_cap = cap;
     a.hsp_count = count;

@@ -25,7 +25,7 @@ constexpr int kSentinelScore = -128;
 
 // Leading / trailing sentinel padding of the packed stream (bytes).
 constexpr int64_t kStreamPadFront = 16;
-constexpr int64_t kStreamPadBack = 256;
+constexpr int64_t kStreamPadBack = 2048;  // covers the 512-B staging prefetch
 
 // NCBI BLOSUM62, order kAlphabet.
 constexpr int8_t kBlosum62[kNumLetters][kNumLetters] = {
@@ -87,7 +87,7 @@ struct SearchArgs {
   QueryView qv;
   int32_t word_len, threshold, window, min_gap, xdrop, cutoff, filter_mode;
   int32_t ring;      // M: per-warp diagonal ring slots
-  int32_t hitbuf;    // per-warp flattened hit buffer capacity
+  int64_t table_entries;  // CSR entries of the query table (positions)
   blastp_hsp *out;
   int64_t out_cap;
   unsigned long long *hsp_count;     // one counter
@@ -98,9 +98,8 @@ struct SearchArgs {
 };
 
 // Launch helpers implemented in search.cu / pack.cu / sort.cu.
-size_t search_smem_bytes(int lq, int ring, int hitbuf, int warps);
+size_t search_smem_bytes(int lq, int ring, int64_t table_entries, int warps);
 int search_ring_slots(int lq, int window);
-int search_hitbuf(int lq);
 cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s);
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
                         const int64_t *sstart, uint8_t *stream, int *err,

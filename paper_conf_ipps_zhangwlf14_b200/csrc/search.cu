@@ -1,29 +1,33 @@
-// search.cu -- the fused BLASTP ungapped hot path for sm_100a.
+// search.cu -- the fused BLASTP ungapped hot path for sm_100a (v2).
 //
-// One kernel does the whole path of PAPER.md Sec. 3.2-3.4 for a chunk of
-// whole subjects per warp:
+// One kernel does the whole path of PAPER.md Sec. 3.2-3.4.  Each warp owns a
+// chunk of whole subjects at a time (work-stealing over chunks) and walks it
+// in ascending subject position:
 //
-//   hit detection     Alg. 2: lanes = consecutive subject
-//                     words, coalesced byte loads, CSR table lookup (R3/R4)
-//   "binning/sorting" P:L967-1343: replaced by a per-warp diagonal ring in
-//                     shared memory indexed by (s - q) mod M; because the
-//                     warp walks its subjects in ascending s, each diagonal's
-//                     hits arrive already sorted -- the order the paper's
-//                     segmented sort establishes, without materialising bins
-//   two-hit filter    P:L1344-1351 (R6): exists p on the same diagonal with
-//                     W <= h - p < A; in-iteration predecessors via a 32-bit
-//                     lane mask per diagonal, earlier ones via ring.last
+//   hit detection     Alg. 2: a 32-lane window of consecutive
+//                     word positions, residues staged per warp in shared
+//                     memory by cp.async ("coalesced"), lookup
+//                     table (R3) in shared memory (P:L1702-1730 hierarchical
+//                     buffering).  The window advances by just enough
+//                     positions that all their hits fit one 32-lane round.
+//   binning/sorting   P:L967-1343: replaced by a per-warp diagonal ring in
+//                     shared memory indexed by (s - q) mod M.  Positions are
+//                     visited in ascending s, so each diagonal's hits arrive
+//                     in the order the paper's segmented sort establishes.
+//                     Hits of one round on the same diagonal are grouped by
+//                     __match_any_sync and ordered by lane (= s).
+//   two-hit filter    P:L1344-1351 (R6): exists p on the same diagonal and
+//                     subject with W <= h - p < A; the ring keeps, per
+//                     diagonal, the last hit, the last hit <= last - W
+//                     ("far") and a bit mask of the hits in between ("near").
 //   extension         Alg. 3/5 + Fig. 8 (R7-R10): passing hits
 //                     not covered by ext_reach are queued; 32 at a time are
-//                     X-dropped lane-parallel and the ext_reach chain is then
-//                     resolved per diagonal in queue (= s) order
-//   output            P:L1352-1353: one global atomic per emitted HSP
+//                     X-dropped lane-parallel (4 residues per load) and the
+//                     ext_reach chain is resolved per diagonal in queue order.
+//   output            P:L1352-1353: one global atomic per emitted HSP.
 //
-// Per-iteration layout: a warp covers 32 consecutive stream positions
-// s0-CTX .. s0-CTX+31, CTX = min_gap-1 "context" lanes that were already
-// processed by the previous iteration (so that every new hit sees all hits
-// at distance < min_gap in the same lane mask).  Each iteration advances
-// 32-CTX positions.
+// Positions inside a warp are 16-bit "frame" positions (rebased every 32K
+// positions), so a diagonal's state is one 8-byte word.
 #include <cuda_runtime.h>
 
 #include "common.cuh"
@@ -32,39 +36,72 @@ namespace blastp {
 
 namespace {
 
-constexpr int kWarps = 4;       // warps per CTA (each independent)
+constexpr int kMaxWarps = 16;   // warps per CTA (each independent)
 constexpr int kQcap = 64;       // extension queue slots per warp
-constexpr int kNeg = -(1 << 30);
+constexpr int kResShift = 9;    // residue staging block = 512 B (16 B per lane)
+constexpr int kResBlock = 1 << kResShift;
+constexpr int kResBlocks = 4;   // staging ring depth (blocks)
+constexpr int kQPad = 4;        // sentinel codes before the query codes
+constexpr int kFrameMin = 1024;    // first frame position (> window + margin)
+constexpr int kFrameSpan = 32768;  // rebase step
 constexpr unsigned kFull = 0xffffffffu;
 
 __constant__ int8_t c_b62[32 * 32];
 
 __host__ __device__ constexpr size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
 
+// Diagonal state (one per ring slot), frame positions, 0 = none.
+//   bits  0..15 last   most recent hit
+//   bits 16..31 far    largest hit <= last - W
+//   bits 32..47 reach  end (inclusive) of the last extension (R10)
+//   bits 48..55 near   bit j set iff a hit at last - j (1 <= j < W)
+__device__ __forceinline__ uint32_t st_last(uint64_t e) { return uint32_t(e) & 0xffffu; }
+__device__ __forceinline__ uint32_t st_far(uint64_t e) { return uint32_t(e) >> 16; }
+__device__ __forceinline__ uint32_t st_reach(uint64_t e) { return uint32_t(e >> 32) & 0xffffu; }
+__device__ __forceinline__ uint32_t st_near(uint64_t e) { return uint32_t(e >> 48) & 0xffu; }
+__device__ __forceinline__ uint64_t st_make(uint32_t last, uint32_t far, uint32_t reach,
+                                            uint32_t near) {
+  return uint64_t(last | (far << 16)) | (uint64_t(reach | (near << 16)) << 32);
+}
+
+// Append a hit at position p (> last) to (last, far, near); W = min_gap.
+__device__ __forceinline__ void st_append(uint32_t &last, uint32_t &far, uint32_t &near, int p,
+                                          int W, uint32_t nearmask) {
+  if (last != 0) {
+    const int d = p - int(last);
+    if (d >= W) {
+      far = last;
+      near = 0;
+    } else {
+      // near hits that fall out of (p-W, p): the largest becomes `far`
+      const uint32_t gone = (near << d) & ~((1u << W) - 1u);
+      if (gone) far = uint32_t(p - (__ffs(gone) - 1));
+      near = ((near << d) | (1u << d)) & nearmask;
+    }
+  } else {
+    near = 0;
+  }
+  last = uint32_t(p);
+}
+
 struct WarpSmem {
-  int2 *ring;         // [M]: .x = last hit (virtual pos) at <= s0-W, .y = ext_reach
-  uint32_t *imask;    // [M]: lanes of the current iteration with a hit on the slot
-  uint32_t *hbuf;     // [hb]: flattened hits of the iteration, (q << 5) | lane
-  uint32_t *mbuf;     // [hb]: imask value seen by each hit (pass C)
-  int2 *queue;        // [kQcap]: (vpos, slot << 16 | q)
+  uint64_t *ring;   // [M]
+  uint8_t *res;     // [kResBlocks * kResBlock] residue staging ring
+  int2 *queue;      // [kQcap]: x = P | q << 16, y = slot
   int *fs_vp, *fs_end, *fs_acc;  // [32] flush scratch
 };
 
-__host__ __device__ size_t warp_smem_bytes(int ring, int hb) {
-  return align16(size_t(ring) * 8) + align16(size_t(ring) * 4) + 2 * align16(size_t(hb) * 4) +
-         size_t(kQcap) * 8 + 3 * 32 * 4;
+__host__ __device__ size_t warp_smem_bytes(int ring) {
+  return align16(size_t(ring) * 8) + size_t(kResBlocks) * kResBlock + size_t(kQcap) * 8 +
+         3 * 32 * 4;
 }
 
-__device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring, int hb) {
+__device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
   WarpSmem w;
-  w.ring = reinterpret_cast<int2 *>(base);
+  w.ring = reinterpret_cast<uint64_t *>(base);
   base += align16(size_t(ring) * 8);
-  w.imask = reinterpret_cast<uint32_t *>(base);
-  base += align16(size_t(ring) * 4);
-  w.hbuf = reinterpret_cast<uint32_t *>(base);
-  base += align16(size_t(hb) * 4);
-  w.mbuf = reinterpret_cast<uint32_t *>(base);
-  base += align16(size_t(hb) * 4);
+  w.res = base;
+  base += size_t(kResBlocks) * kResBlock;
   w.queue = reinterpret_cast<int2 *>(base);
   base += size_t(kQcap) * 8;
   w.fs_vp = reinterpret_cast<int *>(base);
@@ -74,63 +111,102 @@ __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring, int hb) {
 }
 
 __device__ __forceinline__ unsigned lanemask_lt(int lane) { return (1u << lane) - 1u; }
-// bits lo..hi inclusive (0 <= lo <= hi <= 31)
-__device__ __forceinline__ unsigned bit_range(int lo, int hi) {
-  unsigned upto = (hi >= 31) ? kFull : ((2u << hi) - 1u);
-  return upto & ~((1u << lo) - 1u);
-}
 
 __device__ __forceinline__ int score(const int8_t *b62, uint32_t qcode, uint32_t scode) {
   return b62[(qcode << 5) | scode];
 }
 
-// R7/R8: X-drop extension from the seed word at (q, sp) (sp = stream pos).
-// Subject boundaries are sentinels scoring -128, which stops the walk.
+__device__ __forceinline__ uint32_t ldg32(const uint8_t *p) {
+  return __ldg(reinterpret_cast<const uint32_t *>(p));
+}
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+  const unsigned s = static_cast<unsigned>(__cvta_generic_to_shared(smem));
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n"); }
+__device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_group 1;\n"); }
+
+// R7/R8: X-drop extension from the seed word at (q, sp).  qc is the query
+// with kQPad sentinels before it and >= 4 after it; the stream has sentinels
+// between subjects.  Sentinels score -128, which stops the walk at either
+// sequence end.  Four residues per 32-bit load; the stop rule is applied
+// position by position (predicated) so the result is exactly R8.
 __device__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int q,
-                             const uint8_t *qc, const int8_t *b62, int lq, int wl, int X,
-                             int &total, int &llen, int &rlen) {
-  int seed = 0;
-  for (int i = 0; i < wl; ++i) seed += score(b62, qc[q + i], __ldg(stream + sp + i));
-  // right: from (q+wl, sp+wl)
+                             const uint8_t *qc, const int8_t *b62, int X, int &total, int &llen,
+                             int &rlen) {
+  const uint8_t *qq = qc + kQPad;
+  const int seed = score(b62, qq[q], __ldg(stream + sp)) +
+                   score(b62, qq[q + 1], __ldg(stream + sp + 1)) +
+                   score(b62, qq[q + 2], __ldg(stream + sp + 2));
+  // ---- right, from (q+3, sp+3)
   int run = 0, best = 0, bl = 0;
   {
-    const int qi = q + wl;
-    const int n = lq - qi;
-    const uint8_t *sptr = stream + sp + wl;
-    for (int t = 0; t < n; ++t) {
-      run += score(b62, qc[qi + t], __ldg(sptr + t));
-      if (run > best) { best = run; bl = t + 1; }
-      if (best - run >= X) break;
+    const int64_t a = sp + 3;
+    const uint8_t *base = stream + (a & ~int64_t(3));
+    const uint32_t sh = uint32_t(a & 3) * 8;
+    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
+    const uint8_t *qp = qq + q + 3;
+    bool stop = false;
+    for (int t = 0; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      lo = hi;
+      hi = ldg32(base + t + 8);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int s = score(b62, qp[t + j], (w >> (8 * j)) & 0xffu);
+        if (!stop) {
+          run += s;
+          if (run > best) { best = run; bl = t + j + 1; }
+          stop = best - run >= X;
+        }
+      }
     }
   }
   const int best_r = best;
   rlen = bl;
+  // ---- left, from (q-1, sp-1) downwards
   run = 0; best = 0; bl = 0;
   {
-    const uint8_t *sptr = stream + sp - 1;
-    for (int t = 0; t < q; ++t) {
-      run += score(b62, qc[q - 1 - t], __ldg(sptr - t));
-      if (run > best) { best = run; bl = t + 1; }
-      if (best - run >= X) break;
+    const int64_t a3 = sp - 4;  // bytes a3 .. a3+3 = positions sp-4 .. sp-1
+    const uint8_t *base = stream + (a3 & ~int64_t(3));
+    const uint32_t sh = uint32_t(a3 & 3) * 8;
+    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
+    const uint8_t *qp = qq + q - 1;
+    bool stop = false;
+    for (int t = 0; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      hi = lo;
+      lo = ldg32(base - t - 4);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int s = score(b62, qp[-(t + j)], (w >> (8 * (3 - j))) & 0xffu);
+        if (!stop) {
+          run += s;
+          if (run > best) { best = run; bl = t + j + 1; }
+          stop = best - run >= X;
+        }
+      }
     }
   }
   llen = bl;
   total = seed + best_r + best;
 }
 
-// EITHER mode (R6, Fig. 7 reading): does a hit exist at (q+k, sp+k) for some
-// k in [W, A-1]?  Scored directly along the diagonal (the definition of a hit).
+// EITHER mode (R6, Fig. 7 reading): a hit at (q+k, sp+k) for some k in
+// [W, A-1], scored directly along the diagonal (the definition of a hit).
 __device__ bool has_successor(const uint8_t *__restrict__ stream, int64_t sp, int q,
                               const uint8_t *qc, const int8_t *b62, int lq, int W, int A, int T) {
+  const uint8_t *qq = qc + kQPad;
   const int kmax = min(A - 1, lq - 3 - q);
   if (kmax < W) return false;
-  // rolling pair scores at offsets j-2, j-1 (offsets 1, 2 lie in the hit word)
-  int s1 = score(b62, qc[q + 1], __ldg(stream + sp + 1));
-  int s2 = score(b62, qc[q + 2], __ldg(stream + sp + 2));
+  int s1 = score(b62, qq[q + 1], __ldg(stream + sp + 1));
+  int s2 = score(b62, qq[q + 2], __ldg(stream + sp + 2));
   for (int j = 3; j <= kmax + 2; ++j) {
     const uint32_t c = __ldg(stream + sp + j);
     if (c == uint32_t(kSentinel)) return false;  // the subject ends: no later word
-    const int s3 = score(b62, qc[q + j], c);
+    const int s3 = score(b62, qq[q + j], c);
     if (j - 2 >= W && s1 + s2 + s3 >= T) return true;
     s1 = s2;
     s2 = s3;
@@ -150,53 +226,61 @@ __device__ __forceinline__ void trace_push(const SearchArgs &a, int which, int64
 }
 
 struct WarpState {
-  int64_t voff;        // vpos = stream pos + voff
+  int64_t spbase;  // stream position of frame position 0
   int64_t first_subj, last_subj;
   int qhead, qcount;
 };
 
 // Extend up to 32 queued passing hits lane-parallel, then resolve the
-// ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue order.
+// ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order.
+template <bool kTrace>
 __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &st, int n,
                             const uint8_t *qc, const int8_t *b62, int lane) {
   const bool act = lane < n;
   int2 ent = make_int2(0, 0);
   if (act) ent = w.queue[(st.qhead + lane) & (kQcap - 1)];
-  const int vp = ent.x;
-  const int slot = int(uint32_t(ent.y) >> 16);
-  const int q = int(uint32_t(ent.y) & 0xffffu);
-  const int64_t sp = int64_t(vp) - st.voff;
+  const int P = ent.x & 0xffff;
+  const int q = int(uint32_t(ent.x) >> 16);
+  const int slot = ent.y;
+  const int64_t sp = st.spbase + P;
   int total = 0, llen = 0, rlen = 0;
-  if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.qv.lq, a.word_len, a.xdrop, total, llen, rlen);
-  const int endv = vp + a.word_len - 1 + rlen;  // HSP subject end (inclusive), virtual
+  if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen);
+  const int endp = min(P + 2 + rlen, 0xffff);  // HSP subject end (inclusive), frame
   const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
-  w.fs_vp[lane] = vp;
-  w.fs_end[lane] = endv;
-  __syncwarp();
-  bool acc = false;
   const bool uniq = (grp == (1u << lane));
-  if (act) {
-    if (uniq) {
-      const int r = w.ring[slot].y;
-      acc = vp > r;
-      if (acc) w.ring[slot].y = endv;
-    } else if (lane == __ffs(grp) - 1) {
-      int r = w.ring[slot].y;
-      unsigned g = grp;
-      while (g) {
-        const int j = __ffs(g) - 1;
-        g &= g - 1;
-        const bool aj = w.fs_vp[j] > r;
-        if (aj) r = w.fs_end[j];
-        w.fs_acc[j] = aj;
-      }
-      w.ring[slot].y = r;
+  bool acc = false;
+  uint16_t *reach16 = reinterpret_cast<uint16_t *>(w.ring) + 4 * slot + 2;
+  if (__all_sync(kFull, uniq || !act)) {
+    if (act) {
+      acc = P > int(*reach16);
+      if (acc) *reach16 = uint16_t(endp);
     }
+  } else {
+    w.fs_vp[lane] = P;
+    w.fs_end[lane] = endp;
+    __syncwarp();
+    if (act) {
+      if (uniq) {
+        acc = P > int(*reach16);
+        if (acc) *reach16 = uint16_t(endp);
+      } else if (lane == __ffs(grp) - 1) {
+        int r = *reach16;
+        unsigned g = grp;
+        while (g) {
+          const int j = __ffs(g) - 1;
+          g &= g - 1;
+          const bool aj = w.fs_vp[j] > r;
+          if (aj) r = w.fs_end[j];
+          w.fs_acc[j] = aj;
+        }
+        *reach16 = uint16_t(r);
+      }
+    }
+    __syncwarp();
+    if (act && !uniq) acc = w.fs_acc[lane] != 0;
   }
-  __syncwarp();
-  if (act && !uniq) acc = w.fs_acc[lane] != 0;
   if (acc) {
-    if (a.trace[2]) trace_push(a, 2, sp, q, llen, rlen, total);
+    if (kTrace) trace_push(a, 2, sp, q, llen, rlen, total);
     if (total >= a.cutoff) {
       // subject of the seed: largest i with sstart[i] <= sp
       int64_t lo = st.first_subj, hi = st.last_subj - 1;
@@ -211,7 +295,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
       h.q_start = q - llen;
       h.s_start = int32_t(s_local) - llen;
       h.diagonal = h.s_start - h.q_start;
-      h.length = llen + a.word_len + rlen;
+      h.length = llen + 3 + rlen;
       h.score = total;
       const unsigned long long idx = atomicAdd(a.hsp_count, 1ull);
       if ((long long)idx < a.out_cap) a.out[idx] = h;
@@ -222,72 +306,109 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   st.qcount -= n;
 }
 
-__global__ void __launch_bounds__(kWarps * 32) search_kernel(const SearchArgs a) {
+// OffT: uint16_t (table in shared memory) or uint32_t (table in global memory)
+template <bool kTrace, bool kEither, typename OffT>
+__global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
+  const int lq = a.qv.lq;
   int8_t *b62 = reinterpret_cast<int8_t *>(smem);
   uint8_t *qc = smem + 1024;
-  const int lq = a.qv.lq;
-  for (int i = threadIdx.x; i < 1024; i += blockDim.x) b62[i] = c_b62[i];
-  for (int i = threadIdx.x; i < lq; i += blockDim.x) qc[i] = a.qv.qcodes[i];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int M = a.ring, HB = a.hitbuf;
-  WarpSmem w = carve(smem + 1024 + align16(lq) + size_t(warp) * warp_smem_bytes(M, HB), M, HB);
-  for (int i = lane; i < M; i += 32) {
-    w.ring[i] = make_int2(kNeg, kNeg);
-    w.imask[i] = 0;
+  const size_t qc_bytes = align16(size_t(lq) + 2 * kQPad + 8);
+  uint8_t *after_qc = qc + qc_bytes;
+  const OffT *woff;
+  const uint16_t *qpos;
+  size_t table_bytes = 0;
+  if constexpr (sizeof(OffT) == 2) {
+    // Hierarchical buffering: the whole lookup table in smem.
+    uint16_t *woff_s = reinterpret_cast<uint16_t *>(after_qc);
+    const int nw = kWords + 1;
+    uint16_t *qpos_s = woff_s + ((nw + 7) & ~7);
+    const uint32_t entries = uint32_t(a.table_entries);
+    for (int i = threadIdx.x; i < nw; i += blockDim.x) woff_s[i] = uint16_t(__ldg(a.qv.woff + i));
+    for (uint32_t i = threadIdx.x; i < entries; i += blockDim.x) qpos_s[i] = __ldg(a.qv.qpos + i);
+    woff = reinterpret_cast<const OffT *>(woff_s);
+    qpos = qpos_s;
+    table_bytes = align16(size_t((nw + 7) & ~7) * 2 + size_t(entries) * 2);
+  } else {
+    woff = reinterpret_cast<const OffT *>(a.qv.woff);
+    qpos = a.qv.qpos;
   }
+  for (int i = threadIdx.x; i < 1024; i += blockDim.x) b62[i] = c_b62[i];
+  for (int i = threadIdx.x; i < int(qc_bytes); i += blockDim.x) {
+    const int k = i - kQPad;
+    qc[i] = (k >= 0 && k < lq) ? a.qv.qcodes[k] : uint8_t(kSentinel);
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int M = a.ring;
+  WarpSmem w = carve(after_qc + table_bytes + size_t(warp) * warp_smem_bytes(M), M);
+  for (int i = lane; i < M; i += 32) w.ring[i] = 0;
   __syncthreads();
 
-  const uint32_t *__restrict__ woff = a.qv.woff;
-  const uint16_t *__restrict__ qpos = a.qv.qpos;
   const uint8_t *__restrict__ stream = a.stream;
-  const int W = a.min_gap, A = a.window, CTX = W - 1, step = 32 - CTX;
-  const unsigned lastmask = (CTX == 0) ? kFull : (kFull >> CTX);  // lanes <= 31-CTX
-  const bool either = a.filter_mode == BLASTP_FILTER_EITHER;
-  const bool tracing = a.trace[0] != nullptr;
+  const int W = a.min_gap, A = a.window;
+  const uint32_t nearmask = (1u << W) - 2u;  // bits 1 .. W-1
 
   WarpState st;
-  int vbase = 1 << 20;
+  int frame = kFrameMin;  // frame position of the next chunk's first residue
+  int base_slot = 0;      // ring slot of diagonal (win - q + const) at q = lane = 0
   for (;;) {
     unsigned long long ci = 0;
     if (lane == 0) ci = atomicAdd(a.chunk_cursor, 1ull);
     ci = __shfl_sync(kFull, ci, 0);
     if (ci >= (unsigned long long)a.nchunks) break;
     const Chunk ch = a.chunks[ci];
-    if (vbase > (1 << 30)) {  // re-base the virtual positions (ring ages out)
-      for (int i = lane; i < M; i += 32) w.ring[i] = make_int2(kNeg, kNeg);
-      __syncwarp();
-      vbase = 1 << 20;
-    }
-    st.voff = int64_t(vbase) - ch.start;
     st.first_subj = ch.first_subj;
     st.last_subj = ch.last_subj;
     st.qhead = 0;
     st.qcount = 0;
-    int lastsent = vbase - 1;  // virtual pos of the last sentinel before the iteration
-    int base_slot = int((int64_t(vbase) - CTX + lq) % M);
+    st.spbase = ch.start - frame;
+    int win = frame;                        // frame position of lane 0 of the window
+    int lastsent = frame - 1;               // the sentinel before the chunk
+    int64_t end = ch.end - st.spbase;       // frame position of the chunk end (exclusive)
+    int64_t next_blk = ch.start >> kResShift;  // next staging block to request
+    cp_async_wait_all();
+    __syncwarp();
 
-    for (int64_t s0 = ch.start; s0 < ch.end; s0 += step) {
-      const int64_t p = s0 - CTX + lane;
-      const int vp0 = int(s0 - CTX + st.voff);  // virtual pos of lane 0
-      // residues p, p+1, p+2 (one coalesced byte load + shuffles)
-      const uint32_t r0 = __ldg(stream + p);
-      uint32_t xr = 0;
-      if (lane < 2) xr = __ldg(stream + s0 - CTX + 32 + lane);
-      uint32_t r1 = __shfl_down_sync(kFull, r0, 1);
-      uint32_t r2 = __shfl_down_sync(kFull, r0, 2);
-      const uint32_t x0 = __shfl_sync(kFull, xr, 0), x1 = __shfl_sync(kFull, xr, 1);
-      if (lane == 31) { r1 = x0; r2 = x1; }
-      if (lane == 30) r2 = x0;
-      const bool inrange = (p >= ch.start) && (p < ch.end);
-      const bool valid = inrange && (max(r0, max(r1, r2)) < uint32_t(kNumLetters));
+    while (win < end) {
+      // ---- rebase the frame before positions outgrow 16 bits --------------
+      if (win >= kFrameMin + kFrameSpan) {
+        while (st.qcount > 0) flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane);
+        for (int i = lane; i < M; i += 32) {
+          const uint64_t e = w.ring[i];
+          auto rb = [](uint32_t v) { return v > uint32_t(kFrameSpan) ? v - kFrameSpan : 0u; };
+          w.ring[i] = st_make(rb(st_last(e)), rb(st_far(e)), rb(st_reach(e)), st_near(e));
+        }
+        __syncwarp();
+        win -= kFrameSpan;
+        lastsent -= kFrameSpan;
+        end -= kFrameSpan;
+        st.spbase += kFrameSpan;
+      }
+      const int64_t wsp = st.spbase + win;  // stream position of lane 0
+      // ---- residues: stream[wsp .. wsp+33] staged, one block prefetched ---
+      const int64_t need_blk = (wsp + 33) >> kResShift;
+      if (next_blk <= need_blk + 1) {
+        while (next_blk <= need_blk + 1) {
+          cp_async16(w.res + (next_blk & (kResBlocks - 1)) * kResBlock + lane * 16,
+                     stream + (next_blk << kResShift) + lane * 16);
+          cp_async_commit();
+          ++next_blk;
+        }
+        cp_async_wait_1();  // all but the prefetched block have landed
+        __syncwarp();
+      }
+      const int64_t p = wsp + lane;
+      auto res_at = [&](int64_t x) -> uint32_t {
+        return w.res[((x >> kResShift) & (kResBlocks - 1)) * kResBlock + (x & (kResBlock - 1))];
+      };
+      const uint32_t r0 = res_at(p), r1 = res_at(p + 1), r2 = res_at(p + 2);
+      const bool valid = (win + lane < end) && (max(r0, max(r1, r2)) < uint32_t(kNumLetters));
       const unsigned sm = __ballot_sync(kFull, r0 == uint32_t(kSentinel));
-
       uint32_t o = 0, cnt = 0;
       if (valid) {
         const uint32_t c = (r0 * kNumLetters + r1) * kNumLetters + r2;
-        o = __ldg(woff + c);
-        cnt = __ldg(woff + c + 1) - o;
+        o = woff[c];
+        cnt = uint32_t(woff[c + 1]) - o;
       }
       uint32_t incl = cnt;
 #pragma unroll
@@ -295,137 +416,123 @@ __global__ void __launch_bounds__(kWarps * 32) search_kernel(const SearchArgs a)
         const uint32_t t = __shfl_up_sync(kFull, incl, d);
         if (lane >= d) incl += t;
       }
-      const uint32_t H = __shfl_sync(kFull, incl, 31);
+      const uint32_t excl = incl - cnt;
+      // positions consumed this iteration: all lanes whose hits fit one round
+      int npos = __popc(__ballot_sync(kFull, incl <= 32u));
+      if (npos == 0) npos = 1;  // a single word with > 32 hits: several rounds
+      const uint32_t Hn = __shfl_sync(kFull, incl, npos - 1);
+      // last sentinel at or before each lane (before `win`: lastsent)
+      const unsigned prior = sm & ((lane == 31) ? kFull : ((2u << lane) - 1u));
+      const int ls_lane = prior ? (win + 31 - __clz(prior)) : lastsent;
 
-      if (H != 0) {
-        // per-hit helpers ------------------------------------------------
-        auto slot_of = [&](int l, int q) {
-          int s = base_slot + l - q;
-          s += (s < 0) ? M : 0;
-          s -= (s >= M) ? M : 0;
-          return s;
-        };
-        auto seg_lo_of = [&](int l) {
-          const unsigned prior = sm & ((l == 31) ? kFull : ((2u << l) - 1u));
-          return prior ? (32 - __clz(prior)) : 0;
-        };
-        // pass B body: two-hit test (R6) + coverage pre-check; returns enqueue
-        auto test_hit = [&](int l, int q, int slot, unsigned m, int &vpk) -> bool {
-          if (l < CTX) return false;  // context lane: already tested last iteration
-          const int P = vp0 + l;
-          const int lo_seg = seg_lo_of(l);
-          const int lo = max(lo_seg, l - A + 1), hi = l - W;
-          bool pass = (hi >= lo) && (m & bit_range(lo, hi)) != 0;
-          const int2 rr = w.ring[slot];
-          if (!pass && lo_seg == 0 && rr.x > lastsent && rr.x >= P - A + 1) pass = true;
-          const int64_t sp = s0 - CTX + l;
-          if (!pass && either) pass = has_successor(stream, sp, q, qc, b62, lq, W, A, a.threshold);
-          if (tracing) {
-            trace_push(a, 0, sp, q, 0, 0, 0);
-            if (pass) trace_push(a, 1, sp, q, 0, 0, 0);
-          }
-          vpk = P;
-          return pass && P > rr.y;
-        };
-        auto enqueue_round = [&](bool enq, int vpk, int slot, int q) {
-          const unsigned bal = __ballot_sync(kFull, enq);
-          if (bal) {
-            const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
-            if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = make_int2(vpk, (slot << 16) | q);
-            st.qcount += __popc(bal);
-            __syncwarp();
-            if (st.qcount >= 32) flush_queue(a, w, st, 32, qc, b62, lane);
-          }
-        };
-
-        if (H <= uint32_t(HB)) {
-          // ---- fast path: flatten the iteration's hits into smem -------
-          const uint32_t excl = incl - cnt;
-          for (uint32_t i = 0; i < cnt; ++i)
-            w.hbuf[excl + i] = (uint32_t(__ldg(qpos + o + i)) << 5) | uint32_t(lane);
-          __syncwarp();
-          const int rounds = int((H + 31) >> 5);
-          // pass A: mark the lanes that hit each diagonal slot
-          for (int r = 0; r < rounds; ++r) {
-            const uint32_t k = uint32_t(r * 32 + lane);
-            if (k < H) {
-              const uint32_t e = w.hbuf[k];
-              const int l = int(e & 31), q = int(e >> 5);
-              atomicOr(&w.imask[slot_of(l, q)], 1u << l);
-            }
-          }
-          __syncwarp();
-          // pass B: two-hit test, coverage pre-check, enqueue in s order
-          for (int r = 0; r < rounds; ++r) {
-            const uint32_t k = uint32_t(r * 32 + lane);
-            bool enq = false;
-            int vpk = 0, slot = 0, q = 0;
-            if (k < H) {
-              const uint32_t e = w.hbuf[k];
-              const int l = int(e & 31);
-              q = int(e >> 5);
-              slot = slot_of(l, q);
-              const unsigned m = w.imask[slot];
-              w.mbuf[k] = m;
-              enq = test_hit(l, q, slot, m, vpk);
-            }
-            enqueue_round(enq, vpk, slot, q);
-          }
-          __syncwarp();
-          // pass C: ring.last <- last hit at lanes <= 31-CTX; clear masks
-          for (int r = 0; r < rounds; ++r) {
-            const uint32_t k = uint32_t(r * 32 + lane);
-            if (k < H) {
-              const uint32_t e = w.hbuf[k];
-              const int l = int(e & 31), q = int(e >> 5);
-              const int slot = slot_of(l, q);
-              const unsigned m2 = w.mbuf[k] & lastmask;
-              if (m2 && l == 31 - __clz(m2)) w.ring[slot].x = vp0 + l;
-              w.imask[slot] = 0;
-            }
-          }
-          __syncwarp();
-        } else {
-          // ---- slow path (hit-dense iteration): lane-major cooperative --
-          for (int pass = 0; pass < 4; ++pass) {
-            for (int j = 0; j < 32; ++j) {
-              const uint32_t cj = __shfl_sync(kFull, cnt, j);
-              const uint32_t oj = __shfl_sync(kFull, o, j);
-              for (uint32_t kk = 0; kk < cj; kk += 32) {
-                const uint32_t k = kk + uint32_t(lane);
-                const bool active = k < cj;
-                const int q = active ? int(__ldg(qpos + oj + k)) : 0;
-                const int slot = active ? slot_of(j, q) : 0;
-                if (pass == 0) {
-                  if (active) atomicOr(&w.imask[slot], 1u << j);
-                } else if (pass == 1) {
-                  bool enq = false;
-                  int vpk = 0;
-                  if (active) enq = test_hit(j, q, slot, w.imask[slot], vpk);
-                  enqueue_round(enq, vpk, slot, q);
-                } else if (pass == 2) {
-                  if (active) {
-                    const unsigned m2 = w.imask[slot] & lastmask;
-                    if (m2 && j == 31 - __clz(m2)) w.ring[slot].x = vp0 + j;
-                  }
-                } else {
-                  if (active) w.imask[slot] = 0;
-                }
-              }
-            }
-            __syncwarp();
+      for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
+        const uint32_t k = k0 + uint32_t(lane);
+        const bool act = k < Hn;
+        // owner lane of hit k: number of lanes with incl <= k
+        int own = 0;
+#pragma unroll
+        for (int b = 16; b >= 1; b >>= 1) {
+          const uint32_t v = __shfl_sync(kFull, incl, own + b - 1);
+          if (v <= k) own += b;
+        }
+        const uint32_t o_own = __shfl_sync(kFull, o, own);
+        const uint32_t e_own = __shfl_sync(kFull, excl, own);
+        const int ls = __shfl_sync(kFull, ls_lane, own);
+        int q = 0, slot = 0;
+        const int Ph = win + own;
+        if (act) {
+          q = qpos[o_own + (k - e_own)];
+          slot = base_slot + own - q;
+          slot += (slot < 0) ? M : 0;
+          slot -= (slot >= M) ? M : 0;
+        }
+        const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
+        const unsigned earlier = grp & lanemask_lt(lane);
+        uint64_t e = 0;
+        if (act) e = w.ring[slot];
+        uint32_t last = st_last(e), far = st_far(e), near = st_near(e);
+        // R6 predecessor among stored hits: the largest one <= Ph - W
+        const int hi_ok = Ph - W;
+        const int lo_ok = max(Ph - A + 1, ls + 1);  // within A, same subject
+        int cand = 0;
+        if (last != 0) {
+          if (int(last) <= hi_ok) {
+            cand = int(last);
+          } else {
+            const int jmin = int(last) - hi_ok;  // 1 .. W-1
+            const uint32_t m = near >> jmin;
+            cand = m ? int(last) - (jmin + __ffs(m) - 1) : int(far);
           }
         }
+        // earlier hits of this round on the same diagonal (rare): candidates,
+        // and appended to the state the group's last member writes back
+        const int nearly = __reduce_max_sync(kFull, __popc(earlier));
+        if (nearly) {
+          unsigned rem = earlier;
+          for (int it = 0; it < nearly; ++it) {
+            const int src = rem ? __ffs(rem) - 1 : lane;
+            rem &= rem - 1;
+            const int Pj = __shfl_sync(kFull, Ph, src);
+            if (act && src != lane) {
+              if (Pj <= hi_ok && Pj > cand) cand = Pj;
+              st_append(last, far, near, Pj, W, nearmask);
+            }
+          }
+        }
+        bool pass = act && cand >= lo_ok;
+        const int64_t sph = st.spbase + Ph;
+        if (kEither && act && !pass)
+          pass = has_successor(stream, sph, q, qc, b62, lq, W, A, a.threshold);
+        if (kTrace && act) {
+          trace_push(a, 0, sph, q, 0, 0, 0);
+          if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
+        }
+        // the group's last member writes the diagonal state with its own hit
+        if (act && (grp >> lane) == 1u) {
+          st_append(last, far, near, Ph, W, nearmask);
+          w.ring[slot] = st_make(last, far, st_reach(e), near);
+        }
+        const bool enq = pass && Ph > int(st_reach(e));
+        const unsigned bal = __ballot_sync(kFull, enq);
+        if (bal) {
+          const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
+          if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = make_int2(Ph | (q << 16), slot);
+          st.qcount += __popc(bal);
+          __syncwarp();
+          if (st.qcount >= 32) flush_queue<kTrace>(a, w, st, 32, qc, b62, lane);
+        }
+        __syncwarp();
       }
-      // carry the last sentinel before the next iteration's first lane
-      const unsigned sl = sm & lastmask;
-      if (sl) lastsent = vp0 + (31 - __clz(sl));
-      base_slot += step;
+      // ---- advance the window ---------------------------------------------
+      const unsigned sl = sm & ((npos == 32) ? kFull : ((1u << npos) - 1u));
+      if (sl) lastsent = win + 31 - __clz(sl);
+      win += npos;
+      base_slot += npos;
       if (base_slot >= M) base_slot -= M;
     }
-    while (st.qcount > 0) flush_queue(a, w, st, min(st.qcount, 32), qc, b62, lane);
-    vbase += int(ch.end - ch.start) + M + A + 128;
+    while (st.qcount > 0) flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane);
+    // the next chunk continues the frame after a gap (stale state ages out)
+    frame = win + 64;
+    base_slot = (base_slot + 64) % M;
   }
+  cp_async_wait_all();
+}
+
+template <bool kTrace, bool kEither, typename OffT>
+cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_sms,
+                           cudaStream_t s) {
+  auto k = search_kernel<kTrace, kEither, OffT>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, warps * 32, smem);
+  if (e != cudaSuccess) return e;
+  if (per_sm < 1) return cudaErrorInvalidConfiguration;
+  int64_t grid = int64_t(num_sms) * per_sm;
+  const int64_t need = (int64_t(a.nchunks) + warps - 1) / warps;
+  if (grid > need) grid = need < 1 ? 1 : need;
+  k<<<unsigned(grid), warps * 32, smem, s>>>(a);
+  return cudaGetLastError();
 }
 
 }  // namespace
@@ -436,10 +543,12 @@ int search_ring_slots(int lq, int window) {
   return ((lq + window + 64) + 31) & ~31;
 }
 
-int search_hitbuf(int lq) { return lq <= 1100 ? 256 : 512; }
-
-size_t search_smem_bytes(int lq, int ring, int hitbuf, int warps) {
-  return 1024 + align16(size_t(lq)) + size_t(warps) * warp_smem_bytes(ring, hitbuf);
+size_t search_smem_bytes(int lq, int ring, int64_t table_entries, int warps) {
+  const size_t fixed = 1024 + align16(size_t(lq) + 2 * kQPad + 8);
+  const size_t table = table_entries < 0 ? 0
+                                         : align16(size_t((kWords + 1 + 7) & ~7) * 2 +
+                                                   size_t(table_entries) * 2);
+  return fixed + table + size_t(warps) * warp_smem_bytes(ring);
 }
 
 cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s) {
@@ -459,22 +568,34 @@ cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s) {
   int optin = 0;
   cudaError_t e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
-  // as many independent warps per CTA as the per-warp diagonal rings allow
-  int warps = kWarps;
-  while (warps > 1 && search_smem_bytes(a.qv.lq, a.ring, a.hitbuf, warps) > size_t(optin)) warps >>= 1;
-  const size_t smem = search_smem_bytes(a.qv.lq, a.ring, a.hitbuf, warps);
-  if (smem > size_t(optin)) return cudaErrorInvalidConfiguration;
-  e = cudaFuncSetAttribute(search_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-  if (e != cudaSuccess) return e;
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, search_kernel, warps * 32, smem);
-  if (e != cudaSuccess) return e;
-  if (per_sm < 1) return cudaErrorInvalidConfiguration;
-  int64_t grid = int64_t(num_sms) * per_sm;
-  const int64_t need = (int64_t(a.nchunks) + warps - 1) / warps;
-  if (grid > need) grid = need < 1 ? 1 : need;
-  search_kernel<<<unsigned(grid), warps * 32, smem, s>>>(a);
-  return cudaGetLastError();
+  const bool trace = a.trace[0] != nullptr;
+  const bool either = a.filter_mode == BLASTP_FILTER_EITHER;
+  // Table in shared memory when its offsets fit 16 bits and it leaves room
+  // for enough warps; otherwise the table stays in global memory (L1/L2).
+  int warps_s = 0;
+  if (a.table_entries < 65536) {
+    warps_s = kMaxWarps;
+    while (warps_s > 0 &&
+           search_smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s) > size_t(optin))
+      --warps_s;
+  }
+  int warps_g = kMaxWarps;
+  while (warps_g > 0 && search_smem_bytes(a.qv.lq, a.ring, -1, warps_g) > size_t(optin)) --warps_g;
+  if (warps_s >= 4 || (warps_s > 0 && warps_s * 2 >= warps_g)) {
+    const size_t smem = search_smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s);
+    if (trace)
+      return either ? launch_variant<true, true, uint16_t>(a, warps_s, smem, num_sms, s)
+                    : launch_variant<true, false, uint16_t>(a, warps_s, smem, num_sms, s);
+    return either ? launch_variant<false, true, uint16_t>(a, warps_s, smem, num_sms, s)
+                  : launch_variant<false, false, uint16_t>(a, warps_s, smem, num_sms, s);
+  }
+  if (warps_g < 1) return cudaErrorInvalidConfiguration;
+  const size_t smem = search_smem_bytes(a.qv.lq, a.ring, -1, warps_g);
+  if (trace)
+    return either ? launch_variant<true, true, uint32_t>(a, warps_g, smem, num_sms, s)
+                  : launch_variant<true, false, uint32_t>(a, warps_g, smem, num_sms, s);
+  return either ? launch_variant<false, true, uint32_t>(a, warps_g, smem, num_sms, s)
+                : launch_variant<false, false, uint32_t>(a, warps_g, smem, num_sms, s);
 }
 
 }  // namespace blastp
