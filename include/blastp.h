@@ -175,6 +175,15 @@ int blastp_debug_passing(const blastp_query_table *q, const blastp_db *db,
                          const blastp_params *p, void *cuda_stream,
                          blastp_hit *passing, int64_t cap, int64_t *n);
 
+/* Event counters of a traced search (synchronous): stats[i] for i < nstats,
+ * in this order: 32-position windows, 32-hit rounds, rounds with two hits
+ * on one diagonal, hits, passing hits, enqueued hits, extension batches,
+ * extensions computed, extensions accepted (R10), HSPs emitted, X-drop
+ * residues scored, X-drop lane slots (32 x longest lane per batch). */
+int blastp_debug_stats(const blastp_query_table *q, const blastp_db *db,
+                       const blastp_params *p, void *cuda_stream, int64_t *stats,
+                       int32_t nstats);
+
 void blastp_hsp_free(blastp_hsp *h);
 void blastp_query_table_free(blastp_query_table *q);
 void blastp_db_free(blastp_db *db);

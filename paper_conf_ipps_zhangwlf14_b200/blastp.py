@@ -84,6 +84,7 @@ def _load():
                                      vp, i64, P(i64)]
     L.blastp_debug_hits.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
     L.blastp_debug_passing.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
+    L.blastp_debug_stats.argtypes = [vp, vp, P(_CParams), vp, vp, i32]
     for f in ("blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"):
         getattr(L, f).argtypes = [vp]
         getattr(L, f).restype = None
@@ -96,7 +97,7 @@ EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "bl
             "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
             "blastp_shard_range", "blastp_db_info", "blastp_query_table_info",
             "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_sort_hsps_device",
-            "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing",
+            "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
 
 
@@ -274,6 +275,21 @@ def search_ungapped_device(table: QueryTable, db: Database, out_ptr: int, capaci
 
 def sort_hsps_device(ptr: int, n: int, stream=None):
     _check(lib.blastp_sort_hsps_device(ptr, n, _stream_handle(stream)), "blastp_sort_hsps_device")
+
+
+STAT_NAMES = ["windows", "rounds", "conflict_rounds", "hits", "passing", "enqueued", "flushes",
+              "extended", "accepted", "emitted", "xdrop_residues", "xdrop_lane_slots"]
+
+
+def debug_stats(table: QueryTable, db: Database, params: Params | None = None,
+                stream=None) -> dict:
+    """Event counters of a traced search (see blastp_debug_stats)."""
+    c = (params or table.params).c()
+    buf = (ctypes.c_int64 * len(STAT_NAMES))()
+    _check(lib.blastp_debug_stats(table.handle, db.handle, ctypes.byref(c),
+                                  _stream_handle(stream), buf, len(STAT_NAMES)),
+           "blastp_debug_stats")
+    return dict(zip(STAT_NAMES, list(buf)))
 
 
 @dataclass

@@ -461,7 +461,8 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
                           unsigned long long *count, TraceRec *const trace[3],
                           const int64_t trace_cap[3], unsigned long long *trace_count) {
   CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
-  if (trace_count) CUDA_TRY(cudaMemsetAsync(trace_count, 0, 3 * sizeof(unsigned long long), s));
+  if (trace_count)  // [0..3): trace record counts, [3..3+kNumStats): event counters
+    CUDA_TRY(cudaMemsetAsync(trace_count, 0, (3 + kNumStats) * sizeof(unsigned long long), s));
   if (db->nchunks == 0) return BLASTP_OK;
   for (const QueryDev &qd : q->q) {
     SearchArgs a{};
@@ -493,6 +494,7 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
       a.trace_cap[k] = trace ? trace_cap[k] : 0;
     }
     a.trace_count = trace_count;
+    a.stats = trace_count ? trace_count + 3 : nullptr;
     CUDA_TRY(cudaMemsetAsync(db->counters + 1, 0, sizeof(unsigned long long), s));
     CUDA_TRY(launch_search(a, db->sms, s));
   }
@@ -564,10 +566,11 @@ int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
 
 // ------------------------------------------------------------------- debug
 
-int blastp_debug_trace(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,
-                       void *cuda_stream, blastp_hit *hits, int64_t hits_cap, int64_t *n_hits,
-                       blastp_hit *passing, int64_t passing_cap, int64_t *n_passing,
-                       blastp_hsp *exts, int64_t exts_cap, int64_t *n_exts) {
+static int debug_run(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,
+                     void *cuda_stream, blastp_hit *hits, int64_t hits_cap, int64_t *n_hits,
+                     blastp_hit *passing, int64_t passing_cap, int64_t *n_passing,
+                     blastp_hsp *exts, int64_t exts_cap, int64_t *n_exts, int64_t *stats_out,
+                     int32_t nstats) {
   int rc = check_pair(q, db, p);
   if (rc) return rc;
   if (hits_cap < 0 || passing_cap < 0 || exts_cap < 0 || (hits_cap && !hits) ||
@@ -589,16 +592,21 @@ int blastp_debug_trace(const blastp_query_table *q, const blastp_db *db, const b
   for (int k = 0; k < 3; ++k)
     if (cudaMalloc(&tr[k], sizeof(TraceRec) * static_cast<size_t>(std::max<int64_t>(caps[k], 1))) != cudaSuccess)
       return cleanup(fail(BLASTP_E_NOMEM, "trace buffers"));
-  if (cudaMalloc(&tcount, 3 * sizeof(unsigned long long)) != cudaSuccess ||
+  if (cudaMalloc(&tcount, (3 + kNumStats) * sizeof(unsigned long long)) != cudaSuccess ||
       cudaMalloc(&hcount, sizeof(unsigned long long)) != cudaSuccess ||
       cudaMalloc(&dout, sizeof(blastp_hsp)) != cudaSuccess)
     return cleanup(fail(BLASTP_E_NOMEM, "trace counters"));
   rc = enqueue_search(q, db, p, s, dout, 0, hcount, tr, caps, tcount);
   if (rc) return cleanup(rc);
-  unsigned long long cnt[3] = {0, 0, 0};
+  unsigned long long cnt[3 + kNumStats] = {};
   if (cudaMemcpyAsync(cnt, tcount, sizeof(cnt), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
       cudaStreamSynchronize(s) != cudaSuccess)
     return cleanup(fail(BLASTP_E_CUDA, "trace readback: %s", cudaGetErrorString(cudaGetLastError())));
+  if (stats_out) {
+    for (int i = 0; i < nstats; ++i)
+      stats_out[i] = i < kNumStats ? static_cast<int64_t>(cnt[3 + i]) : 0;
+    return cleanup(BLASTP_OK);
+  }
   int64_t *outs[3] = {n_hits, n_passing, n_exts};
   bool over = false;
   std::vector<TraceRec> buf;
@@ -634,6 +642,21 @@ int blastp_debug_trace(const blastp_query_table *q, const blastp_db *db, const b
     }
   }
   return cleanup(over ? fail(BLASTP_E_CAPACITY, "trace capacity exceeded") : BLASTP_OK);
+}
+
+int blastp_debug_trace(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,
+                       void *cuda_stream, blastp_hit *hits, int64_t hits_cap, int64_t *n_hits,
+                       blastp_hit *passing, int64_t passing_cap, int64_t *n_passing,
+                       blastp_hsp *exts, int64_t exts_cap, int64_t *n_exts) {
+  return debug_run(q, db, p, cuda_stream, hits, hits_cap, n_hits, passing, passing_cap, n_passing,
+                   exts, exts_cap, n_exts, nullptr, 0);
+}
+
+int blastp_debug_stats(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,
+                       void *cuda_stream, int64_t *stats, int32_t nstats) {
+  if (!stats || nstats < 1) return fail(BLASTP_E_INVALID_ARG, "stats buffer");
+  return debug_run(q, db, p, cuda_stream, nullptr, 0, nullptr, nullptr, 0, nullptr, nullptr, 0,
+                   nullptr, stats, nstats);
 }
 
 int blastp_debug_hits(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,

@@ -95,6 +95,24 @@ struct SearchArgs {
   TraceRec *trace[3];                // hits, passing, extensions (or null)
   int64_t trace_cap[3];
   unsigned long long *trace_count;   // [3]
+  unsigned long long *stats;         // [kNumStats] event counters (trace runs only)
+};
+
+// Event counters collected by the tracing kernel variant (blastp_debug_stats).
+enum StatIndex {
+  kStatIterations = 0,   // 32-position windows
+  kStatRounds,           // 32-hit rounds
+  kStatConflictRounds,   // rounds with >= 2 hits on one diagonal
+  kStatHits,             // hits (R4)
+  kStatPassing,          // hits passing the two-hit test (R6)
+  kStatEnqueued,         // passing hits not covered at enqueue time
+  kStatFlushes,          // extension batches
+  kStatExtended,         // extensions computed (speculative included)
+  kStatAccepted,         // extensions accepted by the ext_reach chain (R10)
+  kStatEmitted,          // HSPs with score >= cutoff
+  kStatXdropSteps,       // residues scored by X-drop (both sides, all lanes)
+  kStatXdropLaneSlots,   // lanes x steps of the X-drop loops (utilisation)
+  kNumStats = 16
 };
 
 // Launch helpers implemented in search.cu / pack.cu / sort.cu.

@@ -135,7 +135,7 @@ __device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_
 // position by position (predicated) so the result is exactly R8.
 __device__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int q,
                              const uint8_t *qc, const int8_t *b62, int X, int &total, int &llen,
-                             int &rlen) {
+                             int &rlen, int &scanned) {
   const uint8_t *qq = qc + kQPad;
   const int seed = score(b62, qq[q], __ldg(stream + sp)) +
                    score(b62, qq[q + 1], __ldg(stream + sp + 1)) +
@@ -149,7 +149,8 @@ __device__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int
     uint32_t lo = ldg32(base), hi = ldg32(base + 4);
     const uint8_t *qp = qq + q + 3;
     bool stop = false;
-    for (int t = 0; !stop; t += 4) {
+    int t = 0;
+    for (; !stop; t += 4) {
       const uint32_t w = __funnelshift_r(lo, hi, sh);
       lo = hi;
       hi = ldg32(base + t + 8);
@@ -163,6 +164,7 @@ __device__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int
         }
       }
     }
+    scanned = t;
   }
   const int best_r = best;
   rlen = bl;
@@ -175,7 +177,8 @@ __device__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int
     uint32_t lo = ldg32(base), hi = ldg32(base + 4);
     const uint8_t *qp = qq + q - 1;
     bool stop = false;
-    for (int t = 0; !stop; t += 4) {
+    int t = 0;
+    for (; !stop; t += 4) {
       const uint32_t w = __funnelshift_r(lo, hi, sh);
       hi = lo;
       lo = ldg32(base - t - 4);
@@ -189,6 +192,7 @@ __device__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int
         }
       }
     }
+    scanned += t;
   }
   llen = bl;
   total = seed + best_r + best;
@@ -229,7 +233,13 @@ struct WarpState {
   int64_t spbase;  // stream position of frame position 0
   int64_t first_subj, last_subj;
   int qhead, qcount;
+  unsigned long long stat[kNumStats];  // tracing variant only (lane 0 sums)
 };
+
+template <bool kStats>
+__device__ __forceinline__ void stat_add(WarpState &st, int i, unsigned long long v) {
+  if (kStats) st.stat[i] += v;
+}
 
 // Extend up to 32 queued passing hits lane-parallel, then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order.
@@ -243,8 +253,16 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   const int q = int(uint32_t(ent.x) >> 16);
   const int slot = ent.y;
   const int64_t sp = st.spbase + P;
-  int total = 0, llen = 0, rlen = 0;
-  if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen);
+  int total = 0, llen = 0, rlen = 0, scanned = 0;
+  if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen, scanned);
+  if (kTrace) {
+    // residues scored per lane (in groups of 4); lane slots = the longest lane x 32
+    const int lenl = act ? scanned : 0;
+    stat_add<kTrace>(st, kStatFlushes, 1);
+    stat_add<kTrace>(st, kStatExtended, n);
+    stat_add<kTrace>(st, kStatXdropSteps, __reduce_add_sync(kFull, unsigned(lenl)));
+    stat_add<kTrace>(st, kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(lenl)));
+  }
   const int endp = min(P + 2 + rlen, 0xffff);  // HSP subject end (inclusive), frame
   const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
   const bool uniq = (grp == (1u << lane));
@@ -278,6 +296,10 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
     }
     __syncwarp();
     if (act && !uniq) acc = w.fs_acc[lane] != 0;
+  }
+  if (kTrace) {
+    stat_add<kTrace>(st, kStatAccepted, __popc(__ballot_sync(kFull, acc)));
+    stat_add<kTrace>(st, kStatEmitted, __popc(__ballot_sync(kFull, acc && total >= a.cutoff)));
   }
   if (acc) {
     if (kTrace) trace_push(a, 2, sp, q, llen, rlen, total);
@@ -349,6 +371,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
   const uint32_t nearmask = (1u << W) - 2u;  // bits 1 .. W-1
 
   WarpState st;
+  if (kTrace)
+    for (int i = 0; i < kNumStats; ++i) st.stat[i] = 0;
   int frame = kFrameMin;  // frame position of the next chunk's first residue
   int base_slot = 0;      // ring slot of diagonal (win - q + const) at q = lane = 0
   for (;;) {
@@ -384,6 +408,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
         end -= kFrameSpan;
         st.spbase += kFrameSpan;
       }
+      stat_add<kTrace>(st, kStatIterations, 1);
       const int64_t wsp = st.spbase + win;  // stream position of lane 0
       // ---- residues: stream[wsp .. wsp+33] staged, one block prefetched ---
       const int64_t need_blk = (wsp + 33) >> kResShift;
@@ -483,6 +508,14 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
         const int64_t sph = st.spbase + Ph;
         if (kEither && act && !pass)
           pass = has_successor(stream, sph, q, qc, b62, lq, W, A, a.threshold);
+        if (kTrace) {
+          stat_add<kTrace>(st, kStatRounds, 1);
+          stat_add<kTrace>(st, kStatConflictRounds, nearly ? 1 : 0);
+          stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, act)));
+          stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
+          stat_add<kTrace>(st, kStatEnqueued,
+                           __popc(__ballot_sync(kFull, pass && Ph > int(st_reach(e)))));
+        }
         if (kTrace && act) {
           trace_push(a, 0, sph, q, 0, 0, 0);
           if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
@@ -516,6 +549,9 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
     base_slot = (base_slot + 64) % M;
   }
   cp_async_wait_all();
+  if (kTrace && a.stats && lane == 0)
+    for (int i = 0; i < kNumStats; ++i)
+      if (st.stat[i]) atomicAdd(a.stats + i, st.stat[i]);
 }
 
 template <bool kTrace, bool kEither, typename OffT>

@@ -239,3 +239,18 @@ def test_bad_residue_reported(bp):
     with pytest.raises(bp.BlastpError) as e:
         bp.build_query_table("MKV1", bp.Params())
     assert e.value.status == bp.E_BAD_RESIDUE
+
+
+def test_debug_stats_match_oracle_counts(bp, orc):
+    """Event counters of the kernel agree with the oracle's lists (config 1)."""
+    (q,), db = config_workload(1)
+    p = bp.Params()
+    t = bp.build_query_table(q, p)
+    d = bp.pack_db(db.ascii, db.offsets)
+    s = bp.debug_stats(t, d, p)
+    r = oracle_run(orc, q, db.ascii, db.offsets, p, want_hits=True)
+    assert s["hits"] == len(r.hits)
+    assert s["passing"] == len(r.passing)
+    assert s["accepted"] == len(r.extensions)
+    assert s["emitted"] == len(r.hsps)
+    assert s["extended"] >= s["accepted"] and s["enqueued"] >= s["extended"] - 0
