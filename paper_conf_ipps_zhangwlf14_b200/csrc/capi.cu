@@ -469,6 +469,8 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.stream = db->stream;
     a.sstart = db->sstart;
     a.subject_base = db->subject_base;
+    a.nseq = db->nseq;
+    a.stream_len = db->stream_len;
     a.chunks = db->chunks;
     a.nchunks = db->nchunks;
     a.qv.woff = qd.woff;

@@ -81,6 +81,8 @@ struct QueryView {
 struct SearchArgs {
   const uint8_t *stream;
   const int64_t *sstart;  // [nseq]: stream position of each subject's first residue
+  int64_t nseq;           // subjects of the shard
+  int64_t stream_len;     // bytes of the packed stream
   int64_t subject_base;
   const Chunk *chunks;
   int32_t nchunks;
@@ -116,9 +118,11 @@ enum StatIndex {
 };
 
 // Launch helpers implemented in search.cu / pack.cu / sort.cu.
-size_t search_smem_bytes(int lq, int ring, int64_t table_entries, int warps);
 int search_ring_slots(int lq, int window);
+// Picks the kernel variant (search_cta.cu, else search.cu); the environment
+// variable BLASTP_KERNEL=warp|cta forces one (tests cover both).
 cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s);
+cudaError_t launch_search_warp(const SearchArgs &a, int num_sms, cudaStream_t s);
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
                         const int64_t *sstart, uint8_t *stream, int *err,
                         cudaStream_t s);

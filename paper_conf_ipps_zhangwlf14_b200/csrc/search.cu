@@ -1,15 +1,16 @@
-// search.cu -- the fused BLASTP ungapped hot path for sm_100a (v2).
+// search.cu -- "warp" variant of the fused BLASTP ungapped hot path (sm_100a).
 //
-// One kernel does the whole path of PAPER.md Sec. 3.2-3.4.  Each warp owns a
-// chunk of whole subjects at a time (work-stealing over chunks) and walks it
-// in ascending subject position:
+// Used for long queries (the CTA variant in search_cta.cu needs a
+// per-CTA diagonal ring of ~Lq + window slots plus the hit buckets).  Each
+// warp owns a chunk of whole subjects at a time (work-stealing over chunks)
+// and walks it in ascending subject position:
 //
 //   hit detection     Alg. 2: a 32-lane window of consecutive
 //                     word positions, residues staged per warp in shared
 //                     memory by cp.async ("coalesced"), lookup
-//                     table (R3) in shared memory (P:L1702-1730 hierarchical
-//                     buffering).  The window advances by just enough
-//                     positions that all their hits fit one 32-lane round.
+//                     table (R3) in shared memory when it fits (P:L1702-1730
+//                     hierarchical buffering).  The window advances by just
+//                     enough positions that all their hits fit one round.
 //   binning/sorting   P:L967-1343: replaced by a per-warp diagonal ring in
 //                     shared memory indexed by (s - q) mod M.  Positions are
 //                     visited in ascending s, so each diagonal's hits arrive
@@ -17,22 +18,19 @@
 //                     Hits of one round on the same diagonal are grouped by
 //                     __match_any_sync and ordered by lane (= s).
 //   two-hit filter    P:L1344-1351 (R6): exists p on the same diagonal and
-//                     subject with W <= h - p < A; the ring keeps, per
-//                     diagonal, the last hit, the last hit <= last - W
-//                     ("far") and a bit mask of the hits in between ("near").
+//                     subject with W <= h - p < A (ring state: last, far, near).
 //   extension         Alg. 3/5 + Fig. 8 (R7-R10): passing hits
 //                     not covered by ext_reach are queued; 32 at a time are
-//                     X-dropped lane-parallel (4 residues per load) and the
-//                     ext_reach chain is resolved per diagonal in queue order.
+//                     X-dropped lane-parallel and the ext_reach chain is
+//                     resolved per diagonal in queue order.
 //   output            P:L1352-1353: one global atomic per emitted HSP.
-//
-// Positions inside a warp are 16-bit "frame" positions (rebased every 32K
-// positions), so a diagonal's state is one 8-byte word.
 #include <cuda_runtime.h>
 
-#include "common.cuh"
+#include "search_common.cuh"
 
 namespace blastp {
+
+using namespace dev;
 
 namespace {
 
@@ -41,20 +39,12 @@ constexpr int kQcap = 64;       // extension queue slots per warp
 constexpr int kResShift = 9;    // residue staging block = 512 B (16 B per lane)
 constexpr int kResBlock = 1 << kResShift;
 constexpr int kResBlocks = 4;   // staging ring depth (blocks)
-constexpr int kQPad = 4;        // sentinel codes before the query codes
 constexpr int kFrameMin = 1024;    // first frame position (> window + margin)
 constexpr int kFrameSpan = 32768;  // rebase step
-constexpr unsigned kFull = 0xffffffffu;
 
 __constant__ int8_t c_b62[32 * 32];
 
-__host__ __device__ constexpr size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
-
-// Diagonal state (one per ring slot), frame positions, 0 = none.
-//   bits  0..15 last   most recent hit
-//   bits 16..31 far    largest hit <= last - W
-//   bits 32..47 reach  end (inclusive) of the last extension (R10)
-//   bits 48..55 near   bit j set iff a hit at last - j (1 <= j < W)
+// Ring slot state: bits 0..15 last, 16..31 far, 32..47 reach, 48..55 near.
 __device__ __forceinline__ uint32_t st_last(uint64_t e) { return uint32_t(e) & 0xffffu; }
 __device__ __forceinline__ uint32_t st_far(uint64_t e) { return uint32_t(e) >> 16; }
 __device__ __forceinline__ uint32_t st_reach(uint64_t e) { return uint32_t(e >> 32) & 0xffffu; }
@@ -62,26 +52,6 @@ __device__ __forceinline__ uint32_t st_near(uint64_t e) { return uint32_t(e >> 4
 __device__ __forceinline__ uint64_t st_make(uint32_t last, uint32_t far, uint32_t reach,
                                             uint32_t near) {
   return uint64_t(last | (far << 16)) | (uint64_t(reach | (near << 16)) << 32);
-}
-
-// Append a hit at position p (> last) to (last, far, near); W = min_gap.
-__device__ __forceinline__ void st_append(uint32_t &last, uint32_t &far, uint32_t &near, int p,
-                                          int W, uint32_t nearmask) {
-  if (last != 0) {
-    const int d = p - int(last);
-    if (d >= W) {
-      far = last;
-      near = 0;
-    } else {
-      // near hits that fall out of (p-W, p): the largest becomes `far`
-      const uint32_t gone = (near << d) & ~((1u << W) - 1u);
-      if (gone) far = uint32_t(p - (__ffs(gone) - 1));
-      near = ((near << d) | (1u << d)) & nearmask;
-    }
-  } else {
-    near = 0;
-  }
-  last = uint32_t(p);
 }
 
 struct WarpSmem {
@@ -110,130 +80,11 @@ __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
   return w;
 }
 
-__device__ __forceinline__ unsigned lanemask_lt(int lane) { return (1u << lane) - 1u; }
-
-__device__ __forceinline__ int score(const int8_t *b62, uint32_t qcode, uint32_t scode) {
-  return b62[(qcode << 5) | scode];
-}
-
-__device__ __forceinline__ uint32_t ldg32(const uint8_t *p) {
-  return __ldg(reinterpret_cast<const uint32_t *>(p));
-}
-
-__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
-  const unsigned s = static_cast<unsigned>(__cvta_generic_to_shared(smem));
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n"); }
-__device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_group 1;\n"); }
-
-// R7/R8: X-drop extension from the seed word at (q, sp).  qc is the query
-// with kQPad sentinels before it and >= 4 after it; the stream has sentinels
-// between subjects.  Sentinels score -128, which stops the walk at either
-// sequence end.  Four residues per 32-bit load; the stop rule is applied
-// position by position (predicated) so the result is exactly R8.
-__device__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int q,
-                             const uint8_t *qc, const int8_t *b62, int X, int &total, int &llen,
-                             int &rlen, int &scanned) {
-  const uint8_t *qq = qc + kQPad;
-  const int seed = score(b62, qq[q], __ldg(stream + sp)) +
-                   score(b62, qq[q + 1], __ldg(stream + sp + 1)) +
-                   score(b62, qq[q + 2], __ldg(stream + sp + 2));
-  // ---- right, from (q+3, sp+3)
-  int run = 0, best = 0, bl = 0;
-  {
-    const int64_t a = sp + 3;
-    const uint8_t *base = stream + (a & ~int64_t(3));
-    const uint32_t sh = uint32_t(a & 3) * 8;
-    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
-    const uint8_t *qp = qq + q + 3;
-    bool stop = false;
-    int t = 0;
-    for (; !stop; t += 4) {
-      const uint32_t w = __funnelshift_r(lo, hi, sh);
-      lo = hi;
-      hi = ldg32(base + t + 8);
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int s = score(b62, qp[t + j], (w >> (8 * j)) & 0xffu);
-        if (!stop) {
-          run += s;
-          if (run > best) { best = run; bl = t + j + 1; }
-          stop = best - run >= X;
-        }
-      }
-    }
-    scanned = t;
-  }
-  const int best_r = best;
-  rlen = bl;
-  // ---- left, from (q-1, sp-1) downwards
-  run = 0; best = 0; bl = 0;
-  {
-    const int64_t a3 = sp - 4;  // bytes a3 .. a3+3 = positions sp-4 .. sp-1
-    const uint8_t *base = stream + (a3 & ~int64_t(3));
-    const uint32_t sh = uint32_t(a3 & 3) * 8;
-    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
-    const uint8_t *qp = qq + q - 1;
-    bool stop = false;
-    int t = 0;
-    for (; !stop; t += 4) {
-      const uint32_t w = __funnelshift_r(lo, hi, sh);
-      hi = lo;
-      lo = ldg32(base - t - 4);
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int s = score(b62, qp[-(t + j)], (w >> (8 * (3 - j))) & 0xffu);
-        if (!stop) {
-          run += s;
-          if (run > best) { best = run; bl = t + j + 1; }
-          stop = best - run >= X;
-        }
-      }
-    }
-    scanned += t;
-  }
-  llen = bl;
-  total = seed + best_r + best;
-}
-
-// EITHER mode (R6, Fig. 7 reading): a hit at (q+k, sp+k) for some k in
-// [W, A-1], scored directly along the diagonal (the definition of a hit).
-__device__ bool has_successor(const uint8_t *__restrict__ stream, int64_t sp, int q,
-                              const uint8_t *qc, const int8_t *b62, int lq, int W, int A, int T) {
-  const uint8_t *qq = qc + kQPad;
-  const int kmax = min(A - 1, lq - 3 - q);
-  if (kmax < W) return false;
-  int s1 = score(b62, qq[q + 1], __ldg(stream + sp + 1));
-  int s2 = score(b62, qq[q + 2], __ldg(stream + sp + 2));
-  for (int j = 3; j <= kmax + 2; ++j) {
-    const uint32_t c = __ldg(stream + sp + j);
-    if (c == uint32_t(kSentinel)) return false;  // the subject ends: no later word
-    const int s3 = score(b62, qq[q + j], c);
-    if (j - 2 >= W && s1 + s2 + s3 >= T) return true;
-    s1 = s2;
-    s2 = s3;
-  }
-  return false;
-}
-
-__device__ __forceinline__ void trace_push(const SearchArgs &a, int which, int64_t sp, int q,
-                                           int llen, int rlen, int sc) {
-  unsigned long long i = atomicAdd(a.trace_count + which, 1ull);
-  if ((long long)i < a.trace_cap[which]) {
-    TraceRec r;
-    r.sp = sp; r.q = q; r.llen = llen; r.rlen = rlen; r.score = sc;
-    r.query_id = a.qv.query_id; r.pad = 0;
-    a.trace[which][i] = r;
-  }
-}
-
 struct WarpState {
   int64_t spbase;  // stream position of frame position 0
   int64_t first_subj, last_subj;
   int qhead, qcount;
-  unsigned long long stat[kNumStats];  // tracing variant only (lane 0 sums)
+  unsigned long long stat[kNumStats];  // tracing variant only
 };
 
 template <bool kStats>
@@ -256,12 +107,10 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   int total = 0, llen = 0, rlen = 0, scanned = 0;
   if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen, scanned);
   if (kTrace) {
-    // residues scored per lane (in groups of 4); lane slots = the longest lane x 32
-    const int lenl = act ? scanned : 0;
     stat_add<kTrace>(st, kStatFlushes, 1);
     stat_add<kTrace>(st, kStatExtended, n);
-    stat_add<kTrace>(st, kStatXdropSteps, __reduce_add_sync(kFull, unsigned(lenl)));
-    stat_add<kTrace>(st, kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(lenl)));
+    stat_add<kTrace>(st, kStatXdropSteps, __reduce_add_sync(kFull, unsigned(scanned)));
+    stat_add<kTrace>(st, kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(scanned)));
   }
   const int endp = min(P + 2 + rlen, 0xffff);  // HSP subject end (inclusive), frame
   const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
@@ -303,25 +152,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   }
   if (acc) {
     if (kTrace) trace_push(a, 2, sp, q, llen, rlen, total);
-    if (total >= a.cutoff) {
-      // subject of the seed: largest i with sstart[i] <= sp
-      int64_t lo = st.first_subj, hi = st.last_subj - 1;
-      while (lo < hi) {
-        const int64_t mid = (lo + hi + 1) >> 1;
-        if (__ldg(a.sstart + mid) <= sp) lo = mid; else hi = mid - 1;
-      }
-      const int64_t s_local = sp - __ldg(a.sstart + lo);
-      blastp_hsp h;
-      h.query_id = a.qv.query_id;
-      h.subject_id = int32_t(a.subject_base + lo);
-      h.q_start = q - llen;
-      h.s_start = int32_t(s_local) - llen;
-      h.diagonal = h.s_start - h.q_start;
-      h.length = llen + 3 + rlen;
-      h.score = total;
-      const unsigned long long idx = atomicAdd(a.hsp_count, 1ull);
-      if ((long long)idx < a.out_cap) a.out[idx] = h;
-    }
+    emit_hsp(a, sp, q, llen, rlen, total, st.first_subj, st.last_subj);
   }
   __syncwarp();
   st.qhead = (st.qhead + n) & (kQcap - 1);
@@ -330,7 +161,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
 
 // OffT: uint16_t (table in shared memory) or uint32_t (table in global memory)
 template <bool kTrace, bool kEither, typename OffT>
-__global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs a) {
+__global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const SearchArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
   int8_t *b62 = reinterpret_cast<int8_t *>(smem);
@@ -386,9 +217,9 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
     st.qhead = 0;
     st.qcount = 0;
     st.spbase = ch.start - frame;
-    int win = frame;                        // frame position of lane 0 of the window
-    int lastsent = frame - 1;               // the sentinel before the chunk
-    int64_t end = ch.end - st.spbase;       // frame position of the chunk end (exclusive)
+    int win = frame;                           // frame position of lane 0 of the window
+    int lastsent = frame - 1;                  // the sentinel before the chunk
+    int64_t end = ch.end - st.spbase;          // frame position of the chunk end (exclusive)
     int64_t next_blk = ch.start >> kResShift;  // next staging block to request
     cp_async_wait_all();
     __syncwarp();
@@ -479,18 +310,9 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
         // R6 predecessor among stored hits: the largest one <= Ph - W
         const int hi_ok = Ph - W;
         const int lo_ok = max(Ph - A + 1, ls + 1);  // within A, same subject
-        int cand = 0;
-        if (last != 0) {
-          if (int(last) <= hi_ok) {
-            cand = int(last);
-          } else {
-            const int jmin = int(last) - hi_ok;  // 1 .. W-1
-            const uint32_t m = near >> jmin;
-            cand = m ? int(last) - (jmin + __ffs(m) - 1) : int(far);
-          }
-        }
-        // earlier hits of this round on the same diagonal (rare): candidates,
-        // and appended to the state the group's last member writes back
+        int cand = st_pred(last, far, near, hi_ok);
+        // earlier hits of this round on the same diagonal: candidates, and
+        // appended to the state the group's last member writes back
         const int nearly = __reduce_max_sync(kFull, __popc(earlier));
         if (nearly) {
           unsigned rem = earlier;
@@ -515,10 +337,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
           stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
           stat_add<kTrace>(st, kStatEnqueued,
                            __popc(__ballot_sync(kFull, pass && Ph > int(st_reach(e)))));
-        }
-        if (kTrace && act) {
-          trace_push(a, 0, sph, q, 0, 0, 0);
-          if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
+          if (act) {
+            trace_push(a, 0, sph, q, 0, 0, 0);
+            if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
+          }
         }
         // the group's last member writes the diagonal state with its own hit
         if (act && (grp >> lane) == 1u) {
@@ -554,10 +376,18 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_kernel(const SearchArgs
       if (st.stat[i]) atomicAdd(a.stats + i, st.stat[i]);
 }
 
+size_t smem_bytes(int lq, int ring, int64_t table_entries, int warps) {
+  const size_t fixed = 1024 + align16(size_t(lq) + 2 * kQPad + 8);
+  const size_t table = table_entries < 0 ? 0
+                                         : align16(size_t((kWords + 1 + 7) & ~7) * 2 +
+                                                   size_t(table_entries) * 2);
+  return fixed + table + size_t(warps) * warp_smem_bytes(ring);
+}
+
 template <bool kTrace, bool kEither, typename OffT>
 cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_sms,
                            cudaStream_t s) {
-  auto k = search_kernel<kTrace, kEither, OffT>;
+  auto k = search_warp_kernel<kTrace, kEither, OffT>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
   int per_sm = 0;
@@ -579,28 +409,19 @@ int search_ring_slots(int lq, int window) {
   return ((lq + window + 64) + 31) & ~31;
 }
 
-size_t search_smem_bytes(int lq, int ring, int64_t table_entries, int warps) {
-  const size_t fixed = 1024 + align16(size_t(lq) + 2 * kQPad + 8);
-  const size_t table = table_entries < 0 ? 0
-                                         : align16(size_t((kWords + 1 + 7) & ~7) * 2 +
-                                                   size_t(table_entries) * 2);
-  return fixed + table + size_t(warps) * warp_smem_bytes(ring);
-}
-
-cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s) {
+cudaError_t launch_search_warp(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
   static unsigned long long b62_ready = 0;  // one bit per device
   int dev = 0;
   cudaGetDevice(&dev);
   if (!(b62_ready >> dev & 1ull)) {
     int8_t h[32 * 32];
-    for (int i = 0; i < 32; ++i)
-      for (int j = 0; j < 32; ++j)
-        h[i * 32 + j] = (i < kNumLetters && j < kNumLetters) ? kBlosum62[i][j]
-                                                              : int8_t(kSentinelScore);
+    fill_b62(h);
     cudaError_t e = cudaMemcpyToSymbol(c_b62, h, sizeof(h));
     if (e != cudaSuccess) return e;
     b62_ready |= 1ull << dev;
   }
+  SearchArgs a = a_in;
+  a.ring = search_ring_slots(a.qv.lq, a.window);
   int optin = 0;
   cudaError_t e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
@@ -611,14 +432,13 @@ cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s) {
   int warps_s = 0;
   if (a.table_entries < 65536) {
     warps_s = kMaxWarps;
-    while (warps_s > 0 &&
-           search_smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s) > size_t(optin))
+    while (warps_s > 0 && smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s) > size_t(optin))
       --warps_s;
   }
   int warps_g = kMaxWarps;
-  while (warps_g > 0 && search_smem_bytes(a.qv.lq, a.ring, -1, warps_g) > size_t(optin)) --warps_g;
+  while (warps_g > 0 && smem_bytes(a.qv.lq, a.ring, -1, warps_g) > size_t(optin)) --warps_g;
   if (warps_s >= 4 || (warps_s > 0 && warps_s * 2 >= warps_g)) {
-    const size_t smem = search_smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s);
+    const size_t smem = smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s);
     if (trace)
       return either ? launch_variant<true, true, uint16_t>(a, warps_s, smem, num_sms, s)
                     : launch_variant<true, false, uint16_t>(a, warps_s, smem, num_sms, s);
@@ -626,7 +446,7 @@ cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s) {
                   : launch_variant<false, false, uint16_t>(a, warps_s, smem, num_sms, s);
   }
   if (warps_g < 1) return cudaErrorInvalidConfiguration;
-  const size_t smem = search_smem_bytes(a.qv.lq, a.ring, -1, warps_g);
+  const size_t smem = smem_bytes(a.qv.lq, a.ring, -1, warps_g);
   if (trace)
     return either ? launch_variant<true, true, uint32_t>(a, warps_g, smem, num_sms, s)
                   : launch_variant<true, false, uint32_t>(a, warps_g, smem, num_sms, s);

@@ -1,0 +1,212 @@
+// search_common.cuh -- device helpers shared by the two search kernels
+// (search.cu: warp-private diagonal rings; search_cta.cu: CTA windows with
+// per-diagonal buckets and warp-specialised extension).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+namespace blastp {
+namespace dev {
+
+constexpr unsigned kFull = 0xffffffffu;
+constexpr int kQPad = 4;  // sentinel codes before (and >= 4 after) the query codes
+
+__host__ __device__ constexpr size_t align16(size_t x) { return (x + 15) & ~size_t(15); }
+
+// BLOSUM62 extended to 32x32 codes, sentinel / unused codes score -128 (R2).
+inline void fill_b62(int8_t *h) {
+  for (int i = 0; i < 32; ++i)
+    for (int j = 0; j < 32; ++j)
+      h[i * 32 + j] = (i < kNumLetters && j < kNumLetters) ? kBlosum62[i][j]
+                                                            : int8_t(kSentinelScore);
+}
+
+__device__ __forceinline__ unsigned lanemask_lt(int lane) { return (1u << lane) - 1u; }
+
+__device__ __forceinline__ int score(const int8_t *b62, uint32_t qcode, uint32_t scode) {
+  return b62[(qcode << 5) | scode];
+}
+
+__device__ __forceinline__ uint32_t ldg32(const uint8_t *p) {
+  return __ldg(reinterpret_cast<const uint32_t *>(p));
+}
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
+  const unsigned s = static_cast<unsigned>(__cvta_generic_to_shared(smem));
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n"); }
+__device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_group 1;\n"); }
+
+// Diagonal two-hit state, 16-bit positions, 0 = none:
+//   last  most recent hit; far  largest hit <= last - W;
+//   near  bit j set iff a hit at last - j (1 <= j < W).
+// Append a hit at position p (> last).
+__device__ __forceinline__ void st_append(uint32_t &last, uint32_t &far, uint32_t &near, int p,
+                                          int W, uint32_t nearmask) {
+  if (last != 0) {
+    const int d = p - int(last);
+    if (d >= W) {
+      far = last;
+      near = 0;
+    } else {
+      // near hits that fall out of (p-W, p): the largest becomes `far`
+      const uint32_t gone = (near << d) & ~((1u << W) - 1u);
+      if (gone) far = uint32_t(p - (__ffs(gone) - 1));
+      near = ((near << d) | (1u << d)) & nearmask;
+    }
+  } else {
+    near = 0;
+  }
+  last = uint32_t(p);
+}
+
+// Largest stored hit <= hi (hi > 0 frame position), or 0.
+__device__ __forceinline__ int st_pred(uint32_t last, uint32_t far, uint32_t near, int hi) {
+  if (last == 0) return 0;
+  if (int(last) <= hi) return int(last);
+  const int jmin = int(last) - hi;  // 1 .. W-1 when last < hi + W
+  const uint32_t m = jmin < 32 ? near >> jmin : 0u;
+  return m ? int(last) - (jmin + __ffs(m) - 1) : int(far);
+}
+
+// R7/R8: X-drop extension from the seed word at (q, sp).  qc is the query
+// with kQPad sentinels before it and >= 4 after it; the stream has sentinels
+// between subjects.  Sentinels score -128, which stops the walk at either
+// sequence end.  Four residues per 32-bit load; the stop rule is applied
+// position by position (predicated) so the result is exactly R8.
+// `scanned` = residues examined (both sides, in groups of 4).
+__device__ __forceinline__ void xdrop_extend(const uint8_t *__restrict__ stream, int64_t sp, int q,
+                                             const uint8_t *qc, const int8_t *b62, int X,
+                                             int &total, int &llen, int &rlen, int &scanned) {
+  const uint8_t *qq = qc + kQPad;
+  const int seed = score(b62, qq[q], __ldg(stream + sp)) +
+                   score(b62, qq[q + 1], __ldg(stream + sp + 1)) +
+                   score(b62, qq[q + 2], __ldg(stream + sp + 2));
+  int run = 0, best = 0, bl = 0;
+  {  // right, from (q+3, sp+3)
+    const int64_t a = sp + 3;
+    const uint8_t *base = stream + (a & ~int64_t(3));
+    const uint32_t sh = uint32_t(a & 3) * 8;
+    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
+    const uint8_t *qp = qq + q + 3;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      lo = hi;
+      hi = ldg32(base + t + 8);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int s = score(b62, qp[t + j], (w >> (8 * j)) & 0xffu);
+        const int nr = run + s;
+        const bool nb = !stop && nr > best;
+        best = nb ? nr : best;
+        bl = nb ? t + j + 1 : bl;
+        run = stop ? run : nr;
+        stop = stop || (best - nr >= X);
+      }
+    }
+    scanned = t;
+  }
+  const int best_r = best;
+  rlen = bl;
+  run = 0;
+  best = 0;
+  bl = 0;
+  {  // left, from (q-1, sp-1) downwards
+    const int64_t a3 = sp - 4;  // bytes a3 .. a3+3 = positions sp-4 .. sp-1
+    const uint8_t *base = stream + (a3 & ~int64_t(3));
+    const uint32_t sh = uint32_t(a3 & 3) * 8;
+    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
+    const uint8_t *qp = qq + q - 1;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      hi = lo;
+      lo = ldg32(base - t - 4);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int s = score(b62, qp[-(t + j)], (w >> (8 * (3 - j))) & 0xffu);
+        const int nr = run + s;
+        const bool nb = !stop && nr > best;
+        best = nb ? nr : best;
+        bl = nb ? t + j + 1 : bl;
+        run = stop ? run : nr;
+        stop = stop || (best - nr >= X);
+      }
+    }
+    scanned += t;
+  }
+  llen = bl;
+  total = seed + best_r + best;
+}
+
+// EITHER mode (R6, Fig. 7 reading): a hit at (q+k, sp+k) for some k in
+// [W, A-1], scored directly along the diagonal (the definition of a hit).
+__device__ __forceinline__ bool has_successor(const uint8_t *__restrict__ stream, int64_t sp,
+                                              int q, const uint8_t *qc, const int8_t *b62, int lq,
+                                              int W, int A, int T) {
+  const uint8_t *qq = qc + kQPad;
+  const int kmax = min(A - 1, lq - 3 - q);
+  if (kmax < W) return false;
+  int s1 = score(b62, qq[q + 1], __ldg(stream + sp + 1));
+  int s2 = score(b62, qq[q + 2], __ldg(stream + sp + 2));
+  for (int j = 3; j <= kmax + 2; ++j) {
+    const uint32_t c = __ldg(stream + sp + j);
+    if (c == uint32_t(kSentinel)) return false;  // the subject ends: no later word
+    const int s3 = score(b62, qq[q + j], c);
+    if (j - 2 >= W && s1 + s2 + s3 >= T) return true;
+    s1 = s2;
+    s2 = s3;
+  }
+  return false;
+}
+
+__device__ __forceinline__ void trace_push(const SearchArgs &a, int which, int64_t sp, int q,
+                                           int llen, int rlen, int sc) {
+  unsigned long long i = atomicAdd(a.trace_count + which, 1ull);
+  if ((long long)i < a.trace_cap[which]) {
+    TraceRec r;
+    r.sp = sp;
+    r.q = q;
+    r.llen = llen;
+    r.rlen = rlen;
+    r.score = sc;
+    r.query_id = a.qv.query_id;
+    r.pad = 0;
+    a.trace[which][i] = r;
+  }
+}
+
+// HSP record for an accepted extension of the seed at stream position sp;
+// appended to the output if its score reaches the cutoff (R10).  The subject
+// is found by binary search over [lo, hi) of the shard's subject starts.
+__device__ __forceinline__ bool emit_hsp(const SearchArgs &a, int64_t sp, int q, int llen,
+                                         int rlen, int total, int64_t lo, int64_t hi) {
+  if (total < a.cutoff) return false;
+  hi -= 1;
+  while (lo < hi) {
+    const int64_t mid = (lo + hi + 1) >> 1;
+    if (__ldg(a.sstart + mid) <= sp) lo = mid; else hi = mid - 1;
+  }
+  const int64_t s_local = sp - __ldg(a.sstart + lo);
+  blastp_hsp h;
+  h.query_id = a.qv.query_id;
+  h.subject_id = int32_t(a.subject_base + lo);
+  h.q_start = q - llen;
+  h.s_start = int32_t(s_local) - llen;
+  h.diagonal = h.s_start - h.q_start;
+  h.length = llen + 3 + rlen;
+  h.score = total;
+  const unsigned long long idx = atomicAdd(a.hsp_count, 1ull);
+  if ((long long)idx < a.out_cap) a.out[idx] = h;
+  return true;
+}
+
+}  // namespace dev
+}  // namespace blastp

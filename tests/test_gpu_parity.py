@@ -23,6 +23,13 @@ def bp():
     return blastp
 
 
+@pytest.fixture(params=["cta", "warp"], autouse=True)
+def kernel_variant(request, monkeypatch):
+    """Every parity test runs on both kernel variants (BLASTP_KERNEL)."""
+    monkeypatch.setenv("BLASTP_KERNEL", request.param)
+    return request.param
+
+
 def tuples(a):
     return [tuple(int(v) for v in x) for x in a.tolist()]
 
