@@ -589,7 +589,7 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
     }
     pbar(NP);
   }
-  if (lane == 0) st.flush(a);
+  st.flush(a);  // producer counters are per thread
 }
 
 template <bool kTrace, bool kEither, typename OffT>
