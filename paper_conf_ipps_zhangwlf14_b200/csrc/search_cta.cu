@@ -89,6 +89,8 @@ struct Smem {
   int *gcarry;         // [32] last sentinel before group
   uint32_t *scan_tmp;  // [32] warp totals of the bin scan
   uint32_t *gO, *gC;   // [32] group-0 offsets / counts (slow path)
+  uint32_t *posI;      // [nmax] inclusive hit count within the group, per position
+  uint32_t *posO;      // [nmax] lookup-table offset, per position
   Ctrl *ctrl;
   uint4 *fifo;         // [nc * qcap]: vpos, sp, q | slot << 16, seq
   unsigned int *ftail; // [nc] reservation counters
@@ -117,6 +119,7 @@ __host__ __device__ size_t smem_layout(const CtaConfig &c, int lq, int64_t entri
   take(12, size_t(c.nc) * c.qcap * 16);                   // fifo
   take(13, size_t(c.nc) * 4 * 2);                         // ftail, fhead
   take(14, size_t(c.nc) * 96 * 4);                        // fs
+  take(15, size_t(c.nmax) * 8);                           // posI, posO
   return o;
 }
 
@@ -153,8 +156,20 @@ __device__ void consumer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
   unsigned int head = 0;
   const unsigned qmask = unsigned(c.qcap) - 1u;
   for (;;) {
-    // entries are ready when their sequence number matches the slot's index
+    // entries are ready when their sequence number matches the slot's index;
+    // idle consumers probe one slot and sleep (they must not steal issue
+    // slots from the producers)
     const bool done = S.ctrl->done != 0;
+    if (!done) {
+      unsigned probe = 0;
+      if (lane == 0)
+        probe = reinterpret_cast<volatile unsigned int *>(&fifo[(head + 31u) & qmask].w)[0];
+      probe = __shfl_sync(kFull, probe, 0);
+      if (probe != head + 32u) {
+        __nanosleep(1000);
+        continue;
+      }
+    }
     const volatile unsigned int *seqp =
         reinterpret_cast<volatile unsigned int *>(&fifo[(head + lane) & qmask].w);
     const bool ready = (*seqp == head + unsigned(lane) + 1u);
@@ -335,9 +350,10 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
       const uint32_t t = __shfl_up_sync(kFull, incl, d);
       if (lane >= d) incl += t;
     }
-    const uint32_t excl = incl - cnt;
     if (lane == 31) S.gtot[warp] = incl;
     if (lane == 0) S.gsent[warp] = sm;
+    S.posI[32 * warp + lane] = incl;
+    S.posO[32 * warp + lane] = o;
     if (warp == 0) {
       S.gO[lane] = o;
       S.gC[lane] = cnt;
@@ -354,7 +370,6 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
     const unsigned fit = __ballot_sync(kFull, lane < NP && gincl <= uint32_t(c.cap));
     const int ngroups = __popc(fit);  // groups are a prefix (gincl non-decreasing)
     const uint32_t H = ngroups ? __shfl_sync(kFull, gincl, ngroups - 1) : 0u;
-    const uint32_t goff_mine = __shfl_sync(kFull, gincl - gt, warp);
     if (warp == 0) {
       // last sentinel before each group
       const uint32_t gs = lane < NP ? S.gsent[lane] : 0u;
@@ -416,23 +431,34 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
       }
     } else {
       // ---- (E) generate + bin by diagonal --------------------------------------
-      if (warp < ngroups) {
-        const uint32_t Hg = __shfl_sync(kFull, incl, 31);
-        for (uint32_t k0 = 0; k0 < Hg; k0 += 32) {
-          const uint32_t k = k0 + uint32_t(lane);
+      // 32-hit rounds of all consumed groups, dealt round-robin to the warps
+      // (groups differ in hit count; this keeps the phase balanced).
+      {
+        const uint32_t rg = (lane < ngroups) ? (gt + 31u) >> 5 : 0u;
+        uint32_t rincl = rg;
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const uint32_t t = __shfl_up_sync(kFull, rincl, d);
+          if (lane >= d) rincl += t;
+        }
+        const uint32_t rounds = __shfl_sync(kFull, rincl, 31);
+        for (uint32_t rho = warp; rho < rounds; rho += NP) {
+          const int gg = __popc(__ballot_sync(kFull, rincl <= rho));  // group of the round
+          const uint32_t r0g = __shfl_sync(kFull, rincl - rg, gg);
+          const uint32_t gofs = __shfl_sync(kFull, gincl - gt, gg);
+          const uint32_t Hg = __shfl_sync(kFull, gt, gg);
+          const uint32_t k = (rho - r0g) * 32u + uint32_t(lane);
+          const uint32_t *pi = S.posI + 32 * gg;
           int own = 0;
 #pragma unroll
-          for (int b = 16; b >= 1; b >>= 1) {
-            const uint32_t v = __shfl_sync(kFull, incl, own + b - 1);
-            if (v <= k) own += b;
-          }
-          const uint32_t o_own = __shfl_sync(kFull, o, own);
-          const uint32_t e_own = __shfl_sync(kFull, excl, own);
+          for (int b = 16; b >= 1; b >>= 1)
+            if (pi[own + b - 1] <= k) own += b;
           if (k < Hg) {
-            const int q = qpos[o_own + (k - e_own)];
-            const int prel = 32 * warp + own;
+            const uint32_t e_own = own ? pi[own - 1] : 0u;
+            const int q = qpos[S.posO[32 * gg + own] + (k - e_own)];
+            const int prel = 32 * gg + own;
             const int bin = prel - q + lq - 1;
-            const uint32_t idx = goff_mine + k;
+            const uint32_t idx = gofs + k;
             S.rec[idx] = (uint32_t(bin) << 11) | uint32_t(prel);
             S.rank[idx] = uint16_t(atomicAdd(&S.cnt[bin], 1u));
           }
@@ -491,10 +517,12 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
         const uint32_t s = S.cnt[bin], e = S.cnt[bin + 1];
         bool pass = false;
         int maxp = prel;
-        for (uint32_t j = s; j < e; ++j) {
-          const int p = S.bucketed[j];
-          maxp = max(maxp, p);
-          pass |= (p >= lo_ok) && (p <= hi_ok);
+        if (e - s > 1) {  // most bins hold a single hit
+          for (uint32_t j = s; j < e; ++j) {
+            const int p = S.bucketed[j];
+            maxp = max(maxp, p);
+            pass |= (p >= lo_ok) && (p <= hi_ok);
+          }
         }
         int slot = base_slot + bin;
         slot -= (slot >= M) ? M : 0;
@@ -530,7 +558,20 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
         const uint64_t old = S.ring[slot];
         const uint32_t olast = uint32_t(old) & 0xffffu, ofar = (uint32_t(old) >> 16) & 0xffffu,
                        onear = uint32_t(old >> 32) & 0xffu;
+        const unsigned reach_now = S.reach[slot];
+        if (e - s == 1) {  // single-hit bin: append to the old state, hand off
+          uint32_t last = olast, far = ofar, near = onear;
+          st_append(last, far, near, P, W, nearmask);
+          S.ring[slot] = uint64_t(last | (far << 16)) | (uint64_t(near) << 32);
+          const unsigned vp = vbase + unsigned(P);
+          if (S.pflag[s] && vp > reach_now) {
+            if (kTrace) st.add(kStatEnqueued, 1);
+            fifo_push(c, S, slot, vp, unsigned(spbase + P), prel - bin + lq - 1);
+          }
+          continue;
+        }
         uint32_t nnear = 0, nfar = 0;
+        int npass = 0;
         auto add = [&](int x) {
           if (x <= 0) return;
           const int d = P - x;
@@ -542,12 +583,14 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
           for (uint32_t m = onear; m; m &= m - 1) add(int(olast) - (__ffs(m) - 1));
           add(int(ofar));
         }
-        for (uint32_t j = s; j < e; ++j) add(win + int(S.bucketed[j]));
+        for (uint32_t j = s; j < e; ++j) {
+          add(win + int(S.bucketed[j]));
+          npass += S.pflag[j];
+        }
         S.ring[slot] = uint64_t(uint32_t(P) | (nfar << 16)) | (uint64_t(nnear) << 32);
         // passing hits of the bin, ascending s, not covered by a resolved reach
-        const unsigned reach_now = S.reach[slot];
         int prev = -1;
-        for (;;) {
+        for (int it = 0; it < npass; ++it) {
           int best = 0x7fffffff;
           for (uint32_t j = s; j < e; ++j) {
             const int p = S.bucketed[j];
@@ -619,6 +662,8 @@ __global__ void __launch_bounds__(kThreads, 1) search_cta_kernel(const SearchArg
   S.scan_tmp = g + 96;
   S.gO = g + 128;
   S.gC = g + 160;
+  S.posI = reinterpret_cast<uint32_t *>(smem + off[15]);
+  S.posO = S.posI + c.nmax;
   S.ctrl = reinterpret_cast<Ctrl *>(smem + off[11]);
   S.fifo = reinterpret_cast<uint4 *>(smem + off[12]);
   S.ftail = reinterpret_cast<unsigned int *>(smem + off[13]);
