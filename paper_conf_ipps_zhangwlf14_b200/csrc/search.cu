@@ -26,6 +26,10 @@
 //   output            P:L1352-1353: one global atomic per emitted HSP.
 #include <cuda_runtime.h>
 
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+
 #include "search_common.cuh"
 
 namespace blastp {
@@ -273,10 +277,11 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         if (lane >= d) incl += t;
       }
       const uint32_t excl = incl - cnt;
-      // positions consumed this iteration: all lanes whose hits fit one round
-      int npos = __popc(__ballot_sync(kFull, incl <= 32u));
-      if (npos == 0) npos = 1;  // a single word with > 32 hits: several rounds
-      const uint32_t Hn = __shfl_sync(kFull, incl, npos - 1);
+      // all 32 positions are consumed; their hits are processed in 32-hit
+      // rounds in lane-major (= s) order.  Hits of one diagonal in different
+      // rounds see each other through the ring (rounds are sequential).
+      const int npos = 32;
+      const uint32_t Hn = __shfl_sync(kFull, incl, 31);
       // last sentinel at or before each lane (before `win`: lastsent)
       const unsigned prior = sm & ((lane == 31) ? kFull : ((2u << lane) - 1u));
       const int ls_lane = prior ? (win + 31 - __clz(prior)) : lastsent;
@@ -429,13 +434,18 @@ cudaError_t launch_search_warp(const SearchArgs &a_in, int num_sms, cudaStream_t
   const bool either = a.filter_mode == BLASTP_FILTER_EITHER;
   // Table in shared memory when its offsets fit 16 bits and it leaves room
   // for enough warps; otherwise the table stays in global memory (L1/L2).
+  // experiment knobs: BLASTP_TABLE=global, BLASTP_WARPS=<max warps per CTA>
+  const char *tab_env = std::getenv("BLASTP_TABLE");
+  const bool force_global = tab_env && !std::strcmp(tab_env, "global");
+  const char *warps_env = std::getenv("BLASTP_WARPS");
+  const int max_warps = warps_env ? std::max(1, std::min(kMaxWarps, std::atoi(warps_env))) : kMaxWarps;
   int warps_s = 0;
-  if (a.table_entries < 65536) {
-    warps_s = kMaxWarps;
+  if (a.table_entries < 65536 && !force_global) {
+    warps_s = max_warps;
     while (warps_s > 0 && smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s) > size_t(optin))
       --warps_s;
   }
-  int warps_g = kMaxWarps;
+  int warps_g = max_warps;
   while (warps_g > 0 && smem_bytes(a.qv.lq, a.ring, -1, warps_g) > size_t(optin)) --warps_g;
   if (warps_s >= 4 || (warps_s > 0 && warps_s * 2 >= warps_g)) {
     const size_t smem = smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s);
