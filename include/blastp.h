@@ -52,7 +52,7 @@ extern "C" {
 typedef struct {
   int32_t word_len;    /* word length W; only 3 is supported     */
   int32_t threshold;   /* T: word v neighbours query word iff score >= T (R3) */
-  int32_t window;      /* A: two-hit window (R6), 1..4096       */
+  int32_t window;      /* A: two-hit window (R6), 1..256        */
   int32_t min_gap;     /* non-overlap distance (R6), 1..8; default = word_len */
   int32_t xdrop;       /* X: stop when best - run >= X (Fig. 8, R8), 1..127   */
   int32_t cutoff;      /* emit an extension iff score >= cutoff (R10)         */

@@ -67,8 +67,8 @@ int validate_params(const blastp_params *p) {
   if (p->word_len != 3) return fail(BLASTP_E_INVALID_ARG, "word_len %d unsupported (3 only)", p->word_len);
   if (p->min_gap < 1 || p->min_gap > 8)
     return fail(BLASTP_E_INVALID_ARG, "min_gap %d outside [1, 8]", p->min_gap);
-  if (p->window < 1 || p->window > 1024)
-    return fail(BLASTP_E_INVALID_ARG, "window %d outside [1, 1024]", p->window);
+  if (p->window < 1 || p->window > 256)
+    return fail(BLASTP_E_INVALID_ARG, "window %d outside [1, 256]", p->window);
   if (p->xdrop < 1 || p->xdrop > 127)
     return fail(BLASTP_E_INVALID_ARG, "xdrop %d outside [1, 127]", p->xdrop);
   if (p->threshold < -100 || p->threshold > 100)

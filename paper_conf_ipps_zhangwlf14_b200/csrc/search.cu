@@ -38,9 +38,9 @@ using namespace dev;
 
 namespace {
 
-constexpr int kMaxWarps = 16;   // warps per CTA (each independent)
+constexpr int kMaxWarps = 32;   // warps per CTA (each independent)
 constexpr int kQcap = 64;       // extension queue slots per warp
-constexpr int kResShift = 9;    // residue staging block = 512 B (16 B per lane)
+constexpr int kResShift = 8;    // residue staging block = 256 B (8 B per lane)
 constexpr int kResBlock = 1 << kResShift;
 constexpr int kResBlocks = 4;   // staging ring depth (blocks)
 constexpr int kFrameMin = 1024;    // first frame position (> window + margin)
@@ -48,32 +48,40 @@ constexpr int kFrameSpan = 32768;  // rebase step
 
 __constant__ int8_t c_b62[32 * 32];
 
-// Ring slot state: bits 0..15 last, 16..31 far, 32..47 reach, 48..55 near.
-__device__ __forceinline__ uint32_t st_last(uint64_t e) { return uint32_t(e) & 0xffffu; }
-__device__ __forceinline__ uint32_t st_far(uint64_t e) { return uint32_t(e) >> 16; }
-__device__ __forceinline__ uint32_t st_reach(uint64_t e) { return uint32_t(e >> 32) & 0xffffu; }
-__device__ __forceinline__ uint32_t st_near(uint64_t e) { return uint32_t(e >> 48) & 0xffu; }
-__device__ __forceinline__ uint64_t st_make(uint32_t last, uint32_t far, uint32_t reach,
-                                            uint32_t near) {
-  return uint64_t(last | (far << 16)) | (uint64_t(reach | (near << 16)) << 32);
+// Ring slot two-hit state, 32 bits: bits 0..15 last hit, 16..23 last - far
+// (0: none; a far hit more than 255 positions before `last` can never be
+// within the window A <= 256 of a later hit), 24..31 near mask.  The
+// ext_reach of the slot is a separate 16-bit array.
+__device__ __forceinline__ uint32_t st_last(uint32_t e) { return e & 0xffffu; }
+__device__ __forceinline__ uint32_t st_far(uint32_t e) {
+  const uint32_t fd = (e >> 16) & 0xffu;
+  return fd ? (e & 0xffffu) - fd : 0u;
+}
+__device__ __forceinline__ uint32_t st_near(uint32_t e) { return e >> 24; }
+__device__ __forceinline__ uint32_t st_make(uint32_t last, uint32_t far, uint32_t near) {
+  const uint32_t fd = (far != 0 && last - far <= 255u) ? last - far : 0u;
+  return last | (fd << 16) | (near << 24);
 }
 
 struct WarpSmem {
-  uint64_t *ring;   // [M]
+  uint32_t *ring;   // [M] two-hit state
+  uint16_t *reach;  // [M] ext_reach (frame position, 0 = none)
   uint8_t *res;     // [kResBlocks * kResBlock] residue staging ring
   int2 *queue;      // [kQcap]: x = P | q << 16, y = slot
   int *fs_vp, *fs_end, *fs_acc;  // [32] flush scratch
 };
 
 __host__ __device__ size_t warp_smem_bytes(int ring) {
-  return align16(size_t(ring) * 8) + size_t(kResBlocks) * kResBlock + size_t(kQcap) * 8 +
-         3 * 32 * 4;
+  return align16(size_t(ring) * 4) + align16(size_t(ring) * 2) +
+         size_t(kResBlocks) * kResBlock + size_t(kQcap) * 8 + 3 * 32 * 4;
 }
 
 __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
   WarpSmem w;
-  w.ring = reinterpret_cast<uint64_t *>(base);
-  base += align16(size_t(ring) * 8);
+  w.ring = reinterpret_cast<uint32_t *>(base);
+  base += align16(size_t(ring) * 4);
+  w.reach = reinterpret_cast<uint16_t *>(base);
+  base += align16(size_t(ring) * 2);
   w.res = base;
   base += size_t(kResBlocks) * kResBlock;
   w.queue = reinterpret_cast<int2 *>(base);
@@ -120,7 +128,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
   const bool uniq = (grp == (1u << lane));
   bool acc = false;
-  uint16_t *reach16 = reinterpret_cast<uint16_t *>(w.ring) + 4 * slot + 2;
+  uint16_t *reach16 = w.reach + slot;
   if (__all_sync(kFull, uniq || !act)) {
     if (act) {
       acc = P > int(*reach16);
@@ -198,7 +206,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int M = a.ring;
   WarpSmem w = carve(after_qc + table_bytes + size_t(warp) * warp_smem_bytes(M), M);
-  for (int i = lane; i < M; i += 32) w.ring[i] = 0;
+  for (int i = lane; i < M; i += 32) {
+    w.ring[i] = 0;
+    w.reach[i] = 0;
+  }
   __syncthreads();
 
   const uint8_t *__restrict__ stream = a.stream;
@@ -233,9 +244,11 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       if (win >= kFrameMin + kFrameSpan) {
         while (st.qcount > 0) flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane);
         for (int i = lane; i < M; i += 32) {
-          const uint64_t e = w.ring[i];
+          const uint32_t e = w.ring[i];
           auto rb = [](uint32_t v) { return v > uint32_t(kFrameSpan) ? v - kFrameSpan : 0u; };
-          w.ring[i] = st_make(rb(st_last(e)), rb(st_far(e)), rb(st_reach(e)), st_near(e));
+          const uint32_t nl = rb(st_last(e));
+          w.ring[i] = nl ? st_make(nl, rb(st_far(e)), st_near(e)) : 0u;
+          w.reach[i] = uint16_t(rb(w.reach[i]));
         }
         __syncwarp();
         win -= kFrameSpan;
@@ -249,8 +262,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       const int64_t need_blk = (wsp + 33) >> kResShift;
       if (next_blk <= need_blk + 1) {
         while (next_blk <= need_blk + 1) {
-          cp_async16(w.res + (next_blk & (kResBlocks - 1)) * kResBlock + lane * 16,
-                     stream + (next_blk << kResShift) + lane * 16);
+          cp_async8(w.res + (next_blk & (kResBlocks - 1)) * kResBlock + lane * 8,
+                    stream + (next_blk << kResShift) + lane * 8);
           cp_async_commit();
           ++next_blk;
         }
@@ -309,8 +322,11 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         }
         const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
         const unsigned earlier = grp & lanemask_lt(lane);
-        uint64_t e = 0;
-        if (act) e = w.ring[slot];
+        uint32_t e = 0, rch = 0;
+        if (act) {
+          e = w.ring[slot];
+          rch = w.reach[slot];
+        }
         uint32_t last = st_last(e), far = st_far(e), near = st_near(e);
         // R6 predecessor among stored hits: the largest one <= Ph - W
         const int hi_ok = Ph - W;
@@ -341,7 +357,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, act)));
           stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
           stat_add<kTrace>(st, kStatEnqueued,
-                           __popc(__ballot_sync(kFull, pass && Ph > int(st_reach(e)))));
+                           __popc(__ballot_sync(kFull, pass && Ph > int(rch))));
           if (act) {
             trace_push(a, 0, sph, q, 0, 0, 0);
             if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
@@ -350,9 +366,9 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         // the group's last member writes the diagonal state with its own hit
         if (act && (grp >> lane) == 1u) {
           st_append(last, far, near, Ph, W, nearmask);
-          w.ring[slot] = st_make(last, far, st_reach(e), near);
+          w.ring[slot] = st_make(last, far, near);
         }
-        const bool enq = pass && Ph > int(st_reach(e));
+        const bool enq = pass && Ph > int(rch);
         const unsigned bal = __ballot_sync(kFull, enq);
         if (bal) {
           const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
@@ -447,7 +463,11 @@ cudaError_t launch_search_warp(const SearchArgs &a_in, int num_sms, cudaStream_t
   }
   int warps_g = max_warps;
   while (warps_g > 0 && smem_bytes(a.qv.lq, a.ring, -1, warps_g) > size_t(optin)) --warps_g;
-  if (warps_s >= 4 || (warps_s > 0 && warps_s * 2 >= warps_g)) {
+  // More resident warps beat a shared-memory table once the table would cost
+  // more than a few warps (profiles/r01: q1054, 16 warps + L1/L2 table is
+  // faster than 11 warps + shared-memory table).
+  const bool force_smem = tab_env && !std::strcmp(tab_env, "smem");
+  if (warps_s > 0 && (force_smem || warps_s >= std::min(warps_g, 24))) {
     const size_t smem = smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s);
     if (trace)
       return either ? launch_variant<true, true, uint16_t>(a, warps_s, smem, num_sms, s)
