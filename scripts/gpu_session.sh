@@ -17,7 +17,7 @@ if [[ $what == ncu || $what == all ]]; then
     --log-file gpurun_out/launches.csv python bench.py --steps 3 --warmup 3 --no-e2e \
     --no-cpu-baseline > gpurun_out/ncu_launch_bench.json 2>&1
   echo "ncu launches rc=$?"
-  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:search_kernel \
+  timeout 1200 ncu --set full --clock-control none --import-source on -k regex:search_ \
     -s 3 -c 1 -o gpurun_out/prof_search python bench.py --steps 2 --warmup 3 --no-e2e \
     --no-cpu-baseline > gpurun_out/ncu_full.log 2>&1
   echo "ncu full rc=$?"; tail -3 gpurun_out/ncu_full.log
