@@ -147,14 +147,13 @@ def peaks():
     return 6650.0, "fallback (B200_PROFILING.md)"
 
 
-def ncu_traffic():
-    """Per-launch DRAM bytes of the search kernel from the committed ncu capture."""
+def ncu_capture():
+    """The committed ncu --set full summary of the search kernel (config 3)."""
     p = os.path.join(ROOT, "profiles", "ncu_search_kernel.json")
     if not os.path.exists(p):
-        return None, None
+        return {}
     with open(p) as f:
-        d = json.load(f)
-    return d.get("dram_bytes_per_launch"), d.get("source")
+        return json.load(f)
 
 
 # --------------------------------------------------------------- reference arm
@@ -301,7 +300,20 @@ def main():
     # + the HSP records written
     alg_bytes = gdb.residues * nq + n_hsp * 28
     achieved = alg_bytes / (statistics.mean(kern_ms) / 1e3) / 1e9
-    traffic, traffic_src = ncu_traffic()
+    cap = ncu_capture() if (args.config == 3 and world == 1 and nq == 1) else {}
+    traffic, traffic_src = cap.get("dram_bytes_per_launch"), cap.get("source")
+    # issue-rate roofline: warp instructions of the captured launch / this
+    # run's kernel time vs 148 SMs x 4 issue slots x the sampled SM clock
+    issue = None
+    if cap.get("smsp__inst_executed.sum") and clk.get("sm_mhz"):
+        inst = float(cap["smsp__inst_executed.sum"])
+        props = torch.cuda.get_device_properties(dev)
+        peak_i = props.multi_processor_count * 4 * clk["sm_mhz"] * 1e6
+        ach_i = inst / (kern_avg_ms / 1e3)
+        issue = {"bound": "issue", "achieved": ach_i, "peak": peak_i, "unit": "warp-inst/s",
+                 "frac": ach_i / peak_i, "inst_per_launch": inst,
+                 "peak_source": f"{props.multi_processor_count} SMs x 4 schedulers x sampled "
+                                f"SM clock", "source": traffic_src}
 
     # ---- e2e through the C-ABI with host buffers ---------------------------
     e2e = None
@@ -359,6 +371,7 @@ def main():
                          "kernel": "search_kernel", "kernel_ms": kern_avg_ms,
                          "alg_bytes_per_launch": alg_bytes // nq,
                          "peak_source": peak_src, "traffic_source": traffic_src},
+            "issue_roofline": issue,
             "clocks": clk,
             "e2e": e2e,
             "gpu_launches": args.steps * nq,
