@@ -171,8 +171,9 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   st.qcount -= n;
 }
 
-// OffT: uint16_t (table in shared memory) or uint32_t (table in global memory)
-template <bool kTrace, bool kEither, typename OffT>
+// OffT: uint16_t (table in shared memory) or uint32_t (table in global memory);
+// kW: min_gap fixed at compile time (3, the default) or 0 (runtime value).
+template <bool kTrace, bool kEither, typename OffT, int kW>
 __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const SearchArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
@@ -213,7 +214,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
   __syncthreads();
 
   const uint8_t *__restrict__ stream = a.stream;
-  const int W = a.min_gap, A = a.window;
+  const int W = kW ? kW : a.min_gap, A = a.window;  // kW: compile-time min_gap
   const uint32_t nearmask = (1u << W) - 2u;  // bits 1 .. W-1
 
   WarpState st;
@@ -408,7 +409,8 @@ size_t smem_bytes(int lq, int ring, int64_t table_entries, int warps) {
 template <bool kTrace, bool kEither, typename OffT>
 cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_sms,
                            cudaStream_t s) {
-  auto k = search_warp_kernel<kTrace, kEither, OffT>;
+  auto k = a.min_gap == 3 ? search_warp_kernel<kTrace, kEither, OffT, 3>
+                          : search_warp_kernel<kTrace, kEither, OffT, 0>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
   int per_sm = 0;
