@@ -239,6 +239,41 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     int64_t next_blk = ch.start >> kResShift;  // next staging block to request
     cp_async_wait_all();
     __syncwarp();
+    auto res_at = [&](int64_t x) -> uint32_t {
+      return w.res[((x >> kResShift) & (kResBlocks - 1)) * kResBlock + (x & (kResBlock - 1))];
+    };
+    // stage residues up to stream position `upto` (+ one block of prefetch)
+    auto stage = [&](int64_t upto) {
+      const int64_t need_blk = upto >> kResShift;
+      if (next_blk <= need_blk + 1) {
+        while (next_blk <= need_blk + 1) {
+          cp_async8(w.res + (next_blk & (kResBlocks - 1)) * kResBlock + lane * 8,
+                    stream + (next_blk << kResShift) + lane * 8);
+          cp_async_commit();
+          ++next_blk;
+        }
+        cp_async_wait_1();  // all but the prefetched block have landed
+        __syncwarp();
+      }
+    };
+    // table lookup of the window starting at frame position `wn` (software-
+    // pipelined: issued one window ahead, consumed by the next iteration)
+    uint32_t nx_r0 = 0, nx_o = 0, nx_c = 0;
+    auto lookup = [&](int wn) {
+      const int64_t pp = st.spbase + wn + lane;
+      stage(st.spbase + wn + 33);
+      const uint32_t r0 = res_at(pp), r1 = res_at(pp + 1), r2 = res_at(pp + 2);
+      const bool ok = (wn + lane < end) && (max(r0, max(r1, r2)) < uint32_t(kNumLetters));
+      nx_r0 = (wn + lane < end) ? r0 : 0u;
+      nx_o = 0;
+      nx_c = 0;
+      if (ok) {
+        const uint32_t c = (r0 * kNumLetters + r1) * kNumLetters + r2;
+        nx_o = woff[c];
+        nx_c = woff[c + 1];
+      }
+    };
+    lookup(win);
 
     while (win < end) {
       // ---- rebase the frame before positions outgrow 16 bits --------------
@@ -258,32 +293,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         st.spbase += kFrameSpan;
       }
       stat_add<kTrace>(st, kStatIterations, 1);
-      const int64_t wsp = st.spbase + win;  // stream position of lane 0
-      // ---- residues: stream[wsp .. wsp+33] staged, one block prefetched ---
-      const int64_t need_blk = (wsp + 33) >> kResShift;
-      if (next_blk <= need_blk + 1) {
-        while (next_blk <= need_blk + 1) {
-          cp_async8(w.res + (next_blk & (kResBlocks - 1)) * kResBlock + lane * 8,
-                    stream + (next_blk << kResShift) + lane * 8);
-          cp_async_commit();
-          ++next_blk;
-        }
-        cp_async_wait_1();  // all but the prefetched block have landed
-        __syncwarp();
-      }
-      const int64_t p = wsp + lane;
-      auto res_at = [&](int64_t x) -> uint32_t {
-        return w.res[((x >> kResShift) & (kResBlocks - 1)) * kResBlock + (x & (kResBlock - 1))];
-      };
-      const uint32_t r0 = res_at(p), r1 = res_at(p + 1), r2 = res_at(p + 2);
-      const bool valid = (win + lane < end) && (max(r0, max(r1, r2)) < uint32_t(kNumLetters));
-      const unsigned sm = __ballot_sync(kFull, r0 == uint32_t(kSentinel));
-      uint32_t o = 0, cnt = 0;
-      if (valid) {
-        const uint32_t c = (r0 * kNumLetters + r1) * kNumLetters + r2;
-        o = woff[c];
-        cnt = uint32_t(woff[c + 1]) - o;
-      }
+      // ---- this window's lookup (issued last iteration); issue the next ---
+      const uint32_t o = nx_o, cnt = nx_c - nx_o;
+      const unsigned sm = __ballot_sync(kFull, nx_r0 == uint32_t(kSentinel));
+      lookup(win + 32);
       uint32_t incl = cnt;
 #pragma unroll
       for (int d = 1; d < 32; d <<= 1) {
@@ -300,23 +313,40 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       const unsigned prior = sm & ((lane == 31) ? kFull : ((2u << lane) - 1u));
       const int ls_lane = prior ? (win + 31 - __clz(prior)) : lastsent;
 
-      for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
-        const uint32_t k = k0 + uint32_t(lane);
-        const bool act = k < Hn;
-        // owner lane of hit k: number of lanes with incl <= k
+      // round r's owner lane and query position are computed (and the query
+      // position load issued) one round ahead of its processing
+      auto owner_of = [&](uint32_t k) {  // number of lanes with incl <= k
         int own = 0;
 #pragma unroll
         for (int b = 16; b >= 1; b >>= 1) {
           const uint32_t v = __shfl_sync(kFull, incl, own + b - 1);
           if (v <= k) own += b;
         }
+        return own;
+      };
+      auto load_q = [&](uint32_t k, int own) -> int {
         const uint32_t o_own = __shfl_sync(kFull, o, own);
         const uint32_t e_own = __shfl_sync(kFull, excl, own);
+        return k < Hn ? int(qpos[o_own + (k - e_own)]) : 0;
+      };
+      int nown = 0, nq = 0;
+      if (Hn) {
+        nown = owner_of(uint32_t(lane));
+        nq = load_q(uint32_t(lane), nown);
+      }
+      for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
+        const uint32_t k = k0 + uint32_t(lane);
+        const bool act = k < Hn;
+        const int own = nown;
+        int q = nq;
+        if (k0 + 32 < Hn) {
+          nown = owner_of(k + 32);
+          nq = load_q(k + 32, nown);
+        }
         const int ls = __shfl_sync(kFull, ls_lane, own);
-        int q = 0, slot = 0;
+        int slot = 0;
         const int Ph = win + own;
         if (act) {
-          q = qpos[o_own + (k - e_own)];
           slot = base_slot + own - q;
           slot += (slot < 0) ? M : 0;
           slot -= (slot >= M) ? M : 0;
