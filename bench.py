@@ -226,11 +226,28 @@ def main():
     from paper_conf_ipps_zhangwlf14_b200.dist import gather_hsps
 
     rank, local_rank, world = env_rank()
+    # one GPU per rank; BLASTP_DIST_BACKEND=gloo lets several ranks share a
+    # device (a functional check of the sharded path on a 1-GPU box)
+    backend = os.environ.get("BLASTP_DIST_BACKEND", "nccl")
+    local_rank = local_rank % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
     stream = torch.cuda.current_stream()
+
+    def all_reduce_max(t):
+        if world > 1:
+            if backend == "nccl":
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            else:
+                c = t.cpu()
+                dist.all_reduce(c, op=dist.ReduceOp.MAX)
+                t.copy_(c)
+        return t
 
     queries, db, full_off, (lo, hi), desc = workload(args, rank, world)
     params = bp.Params()
@@ -288,8 +305,7 @@ def main():
     elapsed_ms = t_start.elapsed_time(t_end)
     kern_ms = [a.elapsed_time(b) for a, b in ev]
     t = torch.tensor([elapsed_ms, statistics.mean(kern_ms)], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    all_reduce_max(t)
     elapsed_ms, kern_avg_ms = float(t[0]), float(t[1])
     total_residues = int(full_off[-1] - full_off[0])
     value = total_residues * nq * args.steps / (elapsed_ms / 1e3)
@@ -337,8 +353,7 @@ def main():
             dt = time.perf_counter() - t0
             d.free()
             tt = torch.tensor([dt], dtype=torch.float64, device=dev)
-            if world > 1:
-                dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            all_reduce_max(tt)
             if k > 0:  # first e2e step is a warm-up
                 times.append(float(tt[0]))
             h2d = db.residues + 8 * (hi - lo + 1)

@@ -49,6 +49,10 @@ def gather_hsps(local, group=None, dst: int = 0):
 
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
+    if local.is_cuda and dist.get_backend(group) != "nccl":
+        # gloo (functional multi-rank checks on one device): collectives on host
+        out = gather_hsps(local.cpu(), group, dst)
+        return None if out is None else out.to(local.device)
     dev = local.device
     n = torch.tensor([local.shape[0]], dtype=torch.int64, device=dev)
     counts = [torch.zeros_like(n) for _ in range(world)]
