@@ -316,13 +316,13 @@ def main():
     # + the HSP records written
     alg_bytes = gdb.residues * nq + n_hsp * 28
     achieved = alg_bytes / (statistics.mean(kern_ms) / 1e3) / 1e9
-    cap = ncu_capture() if (args.config == 3 and world == 1 and nq == 1) else {}
-    traffic, traffic_src = cap.get("dram_bytes_per_launch"), cap.get("source")
+    capt = ncu_capture() if (args.config == 3 and world == 1 and nq == 1) else {}
+    traffic, traffic_src = capt.get("dram_bytes_per_launch"), capt.get("source")
     # issue-rate roofline: warp instructions of the captured launch / this
     # run's kernel time vs 148 SMs x 4 issue slots x the sampled SM clock
     issue = None
-    if cap.get("smsp__inst_executed.sum") and clk.get("sm_mhz"):
-        inst = float(cap["smsp__inst_executed.sum"])
+    if capt.get("smsp__inst_executed.sum") and clk.get("sm_mhz"):
+        inst = float(capt["smsp__inst_executed.sum"])
         props = torch.cuda.get_device_properties(dev)
         peak_i = props.multi_processor_count * 4 * clk["sm_mhz"] * 1e6
         ach_i = inst / (kern_avg_ms / 1e3)
