@@ -40,9 +40,6 @@ namespace {
 
 constexpr int kMaxWarps = 32;   // warps per CTA (each independent)
 constexpr int kQcap = 64;       // extension queue slots per warp
-constexpr int kResShift = 8;    // residue staging block = 256 B (8 B per lane)
-constexpr int kResBlock = 1 << kResShift;
-constexpr int kResBlocks = 4;   // staging ring depth (blocks)
 constexpr int kFrameMin = 1024;    // first frame position (> window + margin)
 constexpr int kFrameSpan = 32768;  // rebase step
 
@@ -64,16 +61,17 @@ __device__ __forceinline__ uint32_t st_make(uint32_t last, uint32_t far, uint32_
 }
 
 struct WarpSmem {
-  uint32_t *ring;   // [M] two-hit state
-  uint16_t *reach;  // [M] ext_reach (frame position, 0 = none)
-  uint8_t *res;     // [kResBlocks * kResBlock] residue staging ring
-  int2 *queue;      // [kQcap]: x = P | q << 16, y = slot
-  int *fs_vp, *fs_end, *fs_acc;  // [32] flush scratch
+  uint32_t *ring;    // [M] two-hit state
+  uint16_t *reach;   // [M] ext_reach (frame position, 0 = none)
+  uint32_t *queue;   // [kQcap]: P | q << 16 (the slot is recomputed at flush)
+  uint16_t *fs_p, *fs_end, *fs_acc;  // [32] flush scratch
 };
 
+// Per-warp shared memory: 6 B per diagonal slot + 352 B; small enough for
+// 30+ resident warps per SM at Lq ~ 1000 (occupancy is what this latency-
+// bound kernel runs on, profiles/r01).
 __host__ __device__ size_t warp_smem_bytes(int ring) {
-  return align16(size_t(ring) * 4) + align16(size_t(ring) * 2) +
-         size_t(kResBlocks) * kResBlock + size_t(kQcap) * 8 + 3 * 32 * 4;
+  return align16(size_t(ring) * 4) + align16(size_t(ring) * 2) + size_t(kQcap) * 4 + 3 * 32 * 2;
 }
 
 __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
@@ -82,13 +80,11 @@ __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
   base += align16(size_t(ring) * 4);
   w.reach = reinterpret_cast<uint16_t *>(base);
   base += align16(size_t(ring) * 2);
-  w.res = base;
-  base += size_t(kResBlocks) * kResBlock;
-  w.queue = reinterpret_cast<int2 *>(base);
-  base += size_t(kQcap) * 8;
-  w.fs_vp = reinterpret_cast<int *>(base);
-  w.fs_end = w.fs_vp + 32;
-  w.fs_acc = w.fs_vp + 64;
+  w.queue = reinterpret_cast<uint32_t *>(base);
+  base += size_t(kQcap) * 4;
+  w.fs_p = reinterpret_cast<uint16_t *>(base);
+  w.fs_end = w.fs_p + 32;
+  w.fs_acc = w.fs_p + 64;
   return w;
 }
 
@@ -108,13 +104,15 @@ __device__ __forceinline__ void stat_add(WarpState &st, int i, unsigned long lon
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order.
 template <bool kTrace>
 __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &st, int n,
-                            const uint8_t *qc, const int8_t *b62, int lane) {
+                            const uint8_t *qc, const int8_t *b62, int lane, int slotc, int M) {
   const bool act = lane < n;
-  int2 ent = make_int2(0, 0);
+  uint32_t ent = 0;
   if (act) ent = w.queue[(st.qhead + lane) & (kQcap - 1)];
-  const int P = ent.x & 0xffff;
-  const int q = int(uint32_t(ent.x) >> 16);
-  const int slot = ent.y;
+  const int P = int(ent & 0xffffu);
+  const int q = int(ent >> 16);
+  // ring slot of the diagonal: (base_slot - win) + P - q (mod M), slotc given
+  int slot = (P - q + slotc) % M;
+  slot += slot < 0 ? M : 0;
   const int64_t sp = st.spbase + P;
   int total = 0, llen = 0, rlen = 0, scanned = 0;
   if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen, scanned);
@@ -135,8 +133,8 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
       if (acc) *reach16 = uint16_t(endp);
     }
   } else {
-    w.fs_vp[lane] = P;
-    w.fs_end[lane] = endp;
+    w.fs_p[lane] = uint16_t(P);
+    w.fs_end[lane] = uint16_t(endp);
     __syncwarp();
     if (act) {
       if (uniq) {
@@ -148,7 +146,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
         while (g) {
           const int j = __ffs(g) - 1;
           g &= g - 1;
-          const bool aj = w.fs_vp[j] > r;
+          const bool aj = int(w.fs_p[j]) > r;
           if (aj) r = w.fs_end[j];
           w.fs_acc[j] = aj;
         }
@@ -236,33 +234,23 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     int win = frame;                           // frame position of lane 0 of the window
     int lastsent = frame - 1;                  // the sentinel before the chunk
     int64_t end = ch.end - st.spbase;          // frame position of the chunk end (exclusive)
-    int64_t next_blk = ch.start >> kResShift;  // next staging block to request
-    cp_async_wait_all();
-    __syncwarp();
-    auto res_at = [&](int64_t x) -> uint32_t {
-      return w.res[((x >> kResShift) & (kResBlocks - 1)) * kResBlock + (x & (kResBlock - 1))];
+    // Software pipeline over windows: residues are loaded two windows ahead
+    // (one coalesced byte per lane + 2 bytes of overlap), the table lookup is
+    // issued one window ahead and consumed by the next iteration.
+    uint32_t pf_r = 0, pf_x = 0;  // residues of the window after the next
+    auto load_res = [&](int wn) {
+      const int64_t pp = st.spbase + wn;
+      pf_r = __ldg(stream + pp + lane);
+      pf_x = lane < 2 ? __ldg(stream + pp + 32 + lane) : 0u;
     };
-    // stage residues up to stream position `upto` (+ one block of prefetch)
-    auto stage = [&](int64_t upto) {
-      const int64_t need_blk = upto >> kResShift;
-      if (next_blk <= need_blk + 1) {
-        while (next_blk <= need_blk + 1) {
-          cp_async8(w.res + (next_blk & (kResBlocks - 1)) * kResBlock + lane * 8,
-                    stream + (next_blk << kResShift) + lane * 8);
-          cp_async_commit();
-          ++next_blk;
-        }
-        cp_async_wait_1();  // all but the prefetched block have landed
-        __syncwarp();
-      }
-    };
-    // table lookup of the window starting at frame position `wn` (software-
-    // pipelined: issued one window ahead, consumed by the next iteration)
     uint32_t nx_r0 = 0, nx_o = 0, nx_c = 0;
-    auto lookup = [&](int wn) {
-      const int64_t pp = st.spbase + wn + lane;
-      stage(st.spbase + wn + 33);
-      const uint32_t r0 = res_at(pp), r1 = res_at(pp + 1), r2 = res_at(pp + 2);
+    auto lookup = [&](int wn) {  // consumes pf_* (residues of window wn)
+      const uint32_t r0 = pf_r;
+      uint32_t r1 = __shfl_down_sync(kFull, pf_r, 1), r2 = __shfl_down_sync(kFull, pf_r, 2);
+      const uint32_t x0 = __shfl_sync(kFull, pf_x, 0), x1 = __shfl_sync(kFull, pf_x, 1);
+      if (lane == 31) { r1 = x0; r2 = x1; }
+      if (lane == 30) r2 = x0;
+      load_res(wn + 32);
       const bool ok = (wn + lane < end) && (max(r0, max(r1, r2)) < uint32_t(kNumLetters));
       nx_r0 = (wn + lane < end) ? r0 : 0u;
       nx_o = 0;
@@ -273,12 +261,18 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         nx_c = woff[c + 1];
       }
     };
+    load_res(win);
     lookup(win);
+    auto slotc = [&]() {  // (base_slot - win) mod M: ring slot of (P, q) = P - q + slotc
+      int c = (base_slot - win) % M;
+      return c < 0 ? c + M : c;
+    };
 
     while (win < end) {
       // ---- rebase the frame before positions outgrow 16 bits --------------
       if (win >= kFrameMin + kFrameSpan) {
-        while (st.qcount > 0) flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane);
+        while (st.qcount > 0)
+          flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc(), M);
         for (int i = lane; i < M; i += 32) {
           const uint32_t e = w.ring[i];
           auto rb = [](uint32_t v) { return v > uint32_t(kFrameSpan) ? v - kFrameSpan : 0u; };
@@ -403,10 +397,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         const unsigned bal = __ballot_sync(kFull, enq);
         if (bal) {
           const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
-          if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = make_int2(Ph | (q << 16), slot);
+          if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = uint32_t(Ph) | (uint32_t(q) << 16);
           st.qcount += __popc(bal);
           __syncwarp();
-          if (st.qcount >= 32) flush_queue<kTrace>(a, w, st, 32, qc, b62, lane);
+          if (st.qcount >= 32) flush_queue<kTrace>(a, w, st, 32, qc, b62, lane, slotc(), M);
         }
         __syncwarp();
       }
@@ -417,7 +411,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       base_slot += npos;
       if (base_slot >= M) base_slot -= M;
     }
-    while (st.qcount > 0) flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane);
+    while (st.qcount > 0)
+      flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc(), M);
     // the next chunk continues the frame after a gap (stale state ages out)
     frame = win + 64;
     base_slot = (base_slot + 64) % M;
