@@ -452,9 +452,12 @@ cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_
 }  // namespace
 
 int search_ring_slots(int lq, int window) {
-  // M > lq + window + 32 keeps aliased slots (diagonal d and d+M) from ever
-  // looking recent; multiple of 32.
-  return ((lq + window + 64) + 31) & ~31;
+  // Diagonal d and d - M share a slot.  A stored hit of d - M lies before
+  // d - M + lq, so it can never be within `window` of a hit of d when
+  // M >= lq + window; and two diagonals hit inside one 32-position window
+  // are distinct slots when M >= lq + 32.
+  const int need = lq + (window > 32 ? window : 32) + 8;
+  return (need + 7) & ~7;
 }
 
 cudaError_t launch_search_warp(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
