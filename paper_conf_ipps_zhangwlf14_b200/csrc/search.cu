@@ -352,13 +352,16 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           e = w.ring[slot];
           rch = w.reach[slot];
         }
-        uint32_t last = st_last(e), far = st_far(e), near = st_near(e);
+        const uint32_t last = st_last(e), near = st_near(e);
         // R6 predecessor among stored hits: the largest one <= Ph - W
         const int hi_ok = Ph - W;
         const int lo_ok = max(Ph - A + 1, ls + 1);  // within A, same subject
-        int cand = st_pred(last, far, near, hi_ok);
-        // earlier hits of this round on the same diagonal: candidates, and
-        // appended to the state the group's last member writes back
+        const int cand_s = st_pred(last, st_far(e), near, hi_ok);
+        // earlier hits of this round on the same diagonal (rare per lane, but
+        // some in almost every round): the best predecessor among them and
+        // the mask of those within W of this hit
+        int cand_e = 0;
+        uint32_t nb = 0;
         const int nearly = __reduce_max_sync(kFull, __popc(earlier));
         if (nearly) {
           unsigned rem = earlier;
@@ -367,11 +370,13 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
             rem &= rem - 1;
             const int Pj = __shfl_sync(kFull, Ph, src);
             if (act && src != lane) {
-              if (Pj <= hi_ok && Pj > cand) cand = Pj;
-              st_append(last, far, near, Pj, W, nearmask);
+              if (Pj <= hi_ok) cand_e = max(cand_e, Pj);
+              const int d = Ph - Pj;
+              if (d < W) nb |= 1u << d;
             }
           }
         }
+        const int cand = max(cand_s, cand_e);
         bool pass = act && cand >= lo_ok;
         const int64_t sph = st.spbase + Ph;
         if (kEither && act && !pass)
@@ -388,10 +393,15 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
             if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
           }
         }
-        // the group's last member writes the diagonal state with its own hit
+        // the group's last member writes the diagonal state with its own hit:
+        // last = Ph, far = largest hit <= Ph - W (= cand), near = every hit
+        // (stored or earlier in the round) within W of Ph
         if (act && (grp >> lane) == 1u) {
-          st_append(last, far, near, Ph, W, nearmask);
-          w.ring[slot] = st_make(last, far, near);
+          if (last != 0) {
+            const int d = Ph - int(last);
+            if (d < W) nb |= ((near << d) | (1u << d));
+          }
+          w.ring[slot] = st_make(uint32_t(Ph), uint32_t(cand), nb & nearmask);
         }
         const bool enq = pass && Ph > int(rch);
         const unsigned bal = __ballot_sync(kFull, enq);
