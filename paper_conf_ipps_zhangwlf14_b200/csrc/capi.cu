@@ -309,15 +309,9 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   int64_t lo = 0, hi = 0;
   int rc = blastp_shard_range(offsets, nseq, shard_index, num_shards, &lo, &hi);
   if (rc) return rc;
-  for (int64_t i = 0; i < nseq; ++i) {
-    const int64_t L = offsets[i + 1] - offsets[i];
-    if (L < 0) return fail(BLASTP_E_INVALID_ARG, "offsets decrease at subject %lld", static_cast<long long>(i));
-    if (i >= lo && i < hi && L > BLASTP_MAX_SUBJECT_LEN)
-      return fail(BLASTP_E_TOO_LONG, "subject %lld has %lld residues", static_cast<long long>(i),
-                  static_cast<long long>(L));
-  }
   const int64_t n = hi - lo;
   const int64_t nres = offsets[hi] - offsets[lo];
+  if (nres < 0) return fail(BLASTP_E_INVALID_ARG, "offsets decrease");
   if (nres > 0 && !residues_ascii) return fail(BLASTP_E_INVALID_ARG, "residues is NULL");
   DeviceGuard g(device);
   if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
@@ -332,71 +326,56 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   db->subject_base = lo;
   // Stream layout: kStreamPadFront sentinels, then subject i at
   // sstart[i] = pad + (offsets[lo+i] - offsets[lo]) + i, each followed by
-  // one sentinel; kStreamPadBack trailing sentinels; 16-byte multiple.
-  db->h_sstart.resize(static_cast<size_t>(n));
-  for (int64_t i = 0; i < n; ++i)
-    db->h_sstart[static_cast<size_t>(i)] = kStreamPadFront + (offsets[lo + i] - offsets[lo]) + i;
+  // one sentinel; kStreamPadBack trailing sentinels; 512-byte multiple.
+  // Subject starts, length checks and the chunk plan are computed on the GPU.
   db->stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 511) & ~int64_t(511);
-
-  // Chunks of whole subjects, ~C residues each (>= 4 chunks per warp at
-  // 16 warps/SM), the long ones first so they start early.
-  int64_t C = nres / (int64_t(db->sms) * 16 * 4);
+  // Chunks of ~C residues of whole subjects (>= 4 per warp at 32 warps/SM).
+  int64_t C = nres / (int64_t(db->sms) * 32 * 4);
   C = std::min<int64_t>(std::max<int64_t>(C, 1024), 16384);
-  std::vector<Chunk> chunks;
-  for (int64_t i = 0; i < n;) {
-    const int64_t first = i;
-    int64_t acc = 0;
-    while (i < n) {
-      const int64_t L = offsets[lo + i + 1] - offsets[lo + i];
-      if (i != first && acc + L > C) break;
-      acc += L;
-      ++i;
-    }
-    Chunk c;
-    c.start = db->h_sstart[static_cast<size_t>(first)];
-    c.end = db->h_sstart[static_cast<size_t>(i - 1)] + (offsets[lo + i] - offsets[lo + i - 1]);
-    c.first_subj = first;
-    c.last_subj = i;
-    chunks.push_back(c);
-  }
-  std::stable_partition(chunks.begin(), chunks.end(),
-                        [&](const Chunk &c) { return c.end - c.start > 2 * C; });
-  db->nchunks = static_cast<int32_t>(chunks.size());
+  const int64_t nchunks = n > 0 ? (nres + C - 1) / C + 1 : 0;
+  db->nchunks = static_cast<int32_t>(nchunks);
 
+  // stream-ordered allocations from a pool that keeps its memory (repeated
+  // pack calls, e.g. the e2e benchmark, do not pay cudaMalloc again)
+  {
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+      uint64_t thr = ~uint64_t(0);
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
   uint8_t *d_ascii = nullptr;
   int64_t *d_off = nullptr;
   int *d_err = nullptr;
   auto cleanup = [&](int code) {
-    cudaFree(d_ascii);
-    cudaFree(d_off);
-    cudaFree(d_err);
-    if (code != BLASTP_OK) blastp_db_free(db);
+    cudaFreeAsync(d_ascii, s);
+    cudaFreeAsync(d_off, s);
+    cudaFreeAsync(d_err, s);
+    if (code != BLASTP_OK) {
+      cudaStreamSynchronize(s);
+      blastp_db_free(db);
+    }
     return code;
   };
-  if (cudaMalloc(&db->stream, static_cast<size_t>(db->stream_len)) != cudaSuccess ||
-      cudaMalloc(&db->sstart, sizeof(int64_t) * static_cast<size_t>(std::max<int64_t>(n, 1))) != cudaSuccess ||
-      cudaMalloc(&db->chunks, sizeof(Chunk) * std::max<size_t>(chunks.size(), 1)) != cudaSuccess ||
-      cudaMalloc(&db->counters, sizeof(unsigned long long) * 8) != cudaSuccess ||
-      cudaMalloc(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1))) != cudaSuccess ||
-      cudaMalloc(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1)) != cudaSuccess ||
-      cudaMalloc(&d_err, sizeof(int)) != cudaSuccess) {
+  if (cudaMallocAsync(&db->stream, static_cast<size_t>(db->stream_len), s) != cudaSuccess ||
+      cudaMallocAsync(&db->sstart, sizeof(int64_t) * static_cast<size_t>(std::max<int64_t>(n, 1)), s) != cudaSuccess ||
+      cudaMallocAsync(&db->chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1)), s) != cudaSuccess ||
+      cudaMallocAsync(&db->counters, sizeof(unsigned long long) * 8, s) != cudaSuccess ||
+      cudaMallocAsync(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1)), s) != cudaSuccess ||
+      cudaMallocAsync(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1), s) != cudaSuccess ||
+      cudaMallocAsync(&d_err, sizeof(int), s) != cudaSuccess) {
     cudaGetLastError();
     return cleanup(fail(BLASTP_E_NOMEM, "device allocation for the database failed"));
   }
   upload_encode_table();
   cudaError_t e = cudaMemsetAsync(db->stream, kSentinel, static_cast<size_t>(db->stream_len), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(d_err, 0, sizeof(int), s);
-  if (e == cudaSuccess && nres > 0)
-    e = cudaMemcpyAsync(d_ascii, residues_ascii + offsets[lo], static_cast<size_t>(nres),
-                        cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(d_off, offsets + lo, sizeof(int64_t) * static_cast<size_t>(n + 1),
                         cudaMemcpyHostToDevice, s);
-  if (e == cudaSuccess && n > 0)
-    e = cudaMemcpyAsync(db->sstart, db->h_sstart.data(), sizeof(int64_t) * static_cast<size_t>(n),
-                        cudaMemcpyHostToDevice, s);
-  if (e == cudaSuccess && !chunks.empty())
-    e = cudaMemcpyAsync(db->chunks, chunks.data(), sizeof(Chunk) * chunks.size(),
+  if (e == cudaSuccess) e = launch_layout(d_off, n, C, nchunks, db->sstart, db->chunks, d_err, s);
+  if (e == cudaSuccess && nres > 0)
+    e = cudaMemcpyAsync(d_ascii, residues_ascii + offsets[lo], static_cast<size_t>(nres),
                         cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess) e = launch_pack(d_ascii, d_off, n, db->sstart, db->stream, d_err, s);
   int h_err = 0;
@@ -404,6 +383,9 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess)
     return cleanup(fail(BLASTP_E_CUDA, "packing the database failed: %s", cudaGetErrorString(e)));
+  if (h_err & 2) return cleanup(fail(BLASTP_E_INVALID_ARG, "offsets decrease inside the shard"));
+  if (h_err & 4) return cleanup(fail(BLASTP_E_TOO_LONG, "a subject is longer than %d residues",
+                                     BLASTP_MAX_SUBJECT_LEN));
   if (h_err) {
     // find the offending byte on the host for a precise message
     for (int64_t k = offsets[lo]; k < offsets[hi]; ++k)
@@ -414,6 +396,18 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   }
   *out = db;
   return cleanup(BLASTP_OK);
+}
+
+// Host copy of the subject starts (debug traces only; fetched lazily).
+static const std::vector<int64_t> &host_sstart(const blastp_db *db) {
+  auto *mdb = const_cast<blastp_db *>(db);
+  if (static_cast<int64_t>(mdb->h_sstart.size()) != db->nseq) {
+    mdb->h_sstart.resize(static_cast<size_t>(db->nseq));
+    if (db->nseq > 0)
+      cudaMemcpy(mdb->h_sstart.data(), db->sstart, sizeof(int64_t) * static_cast<size_t>(db->nseq),
+                 cudaMemcpyDeviceToHost);
+  }
+  return mdb->h_sstart;
 }
 
 int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues, int64_t *subject_base,
@@ -623,9 +617,10 @@ static int debug_run(const blastp_query_table *q, const blastp_db *db, const bla
       return cleanup(fail(BLASTP_E_CUDA, "trace copy"));
     for (int64_t i = 0; i < m; ++i) {
       const TraceRec &r = buf[static_cast<size_t>(i)];
-      const auto it = std::upper_bound(db->h_sstart.begin(), db->h_sstart.end(), r.sp);
-      const int64_t subj = (it - db->h_sstart.begin()) - 1;
-      const int32_t sl = static_cast<int32_t>(r.sp - db->h_sstart[static_cast<size_t>(subj)]);
+      const std::vector<int64_t> &hs = host_sstart(db);
+      const auto it = std::upper_bound(hs.begin(), hs.end(), r.sp);
+      const int64_t subj = (it - hs.begin()) - 1;
+      const int32_t sl = static_cast<int32_t>(r.sp - hs[static_cast<size_t>(subj)]);
       const int32_t sid = static_cast<int32_t>(db->subject_base + subj);
       if (k < 2) {
         blastp_hit h{r.query_id, sid, r.q, sl};

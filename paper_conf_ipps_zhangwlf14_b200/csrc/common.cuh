@@ -126,6 +126,8 @@ cudaError_t launch_search_warp(const SearchArgs &a, int num_sms, cudaStream_t s)
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
                         const int64_t *sstart, uint8_t *stream, int *err,
                         cudaStream_t s);
+cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
+                          int64_t *sstart, Chunk *chunks, int *err, cudaStream_t s);
 cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
 void upload_encode_table();
 

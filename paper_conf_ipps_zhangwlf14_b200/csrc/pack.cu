@@ -32,7 +32,68 @@ __global__ void pack_kernel(const uint8_t *__restrict__ ascii, const int64_t *__
   }
 }
 
+// Stream layout: subject i starts at pad + (off[i] - off[0]) + i (one sentinel
+// after each subject).  Also validates the lengths (err bit 2: negative,
+// bit 4: longer than BLASTP_MAX_SUBJECT_LEN).
+__global__ void layout_kernel(const int64_t *__restrict__ off, int64_t n, int64_t *sstart,
+                              int *err) {
+  const int64_t base = off[0];
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n;
+       i += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t o = off[i], L = off[i + 1] - o;
+    sstart[i] = kStreamPadFront + (o - base) + i;
+    if (L < 0) atomicOr(err, 2);
+    if (L > BLASTP_MAX_SUBJECT_LEN) atomicOr(err, 4);
+  }
+}
+
+// Chunk k = the subjects whose first residue lies in [k*C, (k+1)*C) of the
+// shard's residues (binary search over the offsets); empty chunks have
+// start == end and are skipped by the search kernels.
+__global__ void chunk_kernel(const int64_t *__restrict__ off, int64_t n,
+                             const int64_t *__restrict__ sstart, int64_t C, int64_t nchunks,
+                             Chunk *chunks) {
+  const int64_t base = off[0];
+  auto first_at = [&](int64_t k) -> int64_t {
+    if (k >= nchunks) return n;
+    const int64_t target = k * C;
+    int64_t lo = 0, hi = n;
+    while (lo < hi) {
+      const int64_t m = (lo + hi) >> 1;
+      if (off[m] - base >= target) hi = m; else lo = m + 1;
+    }
+    return lo;
+  };
+  for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k < nchunks;
+       k += int64_t(gridDim.x) * blockDim.x) {
+    const int64_t f = first_at(k), l = first_at(k + 1);
+    Chunk c;
+    c.first_subj = f;
+    c.last_subj = l > f ? l : f;
+    if (l > f) {
+      c.start = sstart[f];
+      c.end = sstart[l - 1] + (off[l] - off[l - 1]);
+    } else {
+      c.start = c.end = 0;
+    }
+    chunks[k] = c;
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
+                          int64_t *sstart, Chunk *chunks, int *err, cudaStream_t s) {
+  if (n > 0) {
+    const int64_t blocks = (n + 255) / 256 > 4096 ? 4096 : (n + 255) / 256;
+    layout_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, err);
+  }
+  if (nchunks > 0) {
+    const int64_t blocks = (nchunks + 255) / 256 > 4096 ? 4096 : (nchunks + 255) / 256;
+    chunk_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, C, nchunks, chunks);
+  }
+  return cudaGetLastError();
+}
 
 void upload_encode_table() {
   uint8_t lut[256];
