@@ -261,3 +261,15 @@ def test_debug_stats_match_oracle_counts(bp, orc):
     assert s["accepted"] == len(r.extensions)
     assert s["emitted"] == len(r.hsps)
     assert s["extended"] >= s["accepted"] and s["enqueued"] >= s["extended"] - 0
+
+
+def test_pack_rejects_bad_offsets(bp):
+    ascii = np.frombuffer(b"MKVLAGGAAA", dtype=np.uint8).copy()
+    with pytest.raises(bp.BlastpError) as e:
+        bp.pack_db(ascii, np.array([0, 6, 4, 10], dtype=np.int64))
+    assert e.value.status == bp.E_INVALID_ARG
+
+
+def test_graft_smoke_entry(bp):
+    import __graft_entry__ as g
+    g.smoke()
