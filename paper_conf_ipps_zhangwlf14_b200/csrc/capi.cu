@@ -332,6 +332,7 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   // Chunks of ~C residues of whole subjects (>= 4 per warp at 32 warps/SM).
   int64_t C = nres / (int64_t(db->sms) * 32 * 4);
   C = std::min<int64_t>(std::max<int64_t>(C, 1024), 16384);
+  if (const char *ce = std::getenv("BLASTP_CHUNK")) C = std::max<int64_t>(64, std::atoll(ce));
   const int64_t nchunks = n > 0 ? (nres + C - 1) / C + 1 : 0;
   db->nchunks = static_cast<int32_t>(nchunks);
 
