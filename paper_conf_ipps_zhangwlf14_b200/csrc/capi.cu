@@ -112,9 +112,10 @@ struct blastp_db {
   uint8_t *stream = nullptr;
   int64_t *sstart = nullptr;
   Chunk *chunks = nullptr;
+  Chunk *long_chunks = nullptr;  // chunks > 2C residues, scheduled first (count at counters[6])
   int32_t nchunks = 0;
   std::vector<int64_t> h_sstart;
-  unsigned long long *counters = nullptr;  // [0] hsp count, [1] chunk cursor, [2..4] trace
+  unsigned long long *counters = nullptr;  // [0] hsp count, [1] chunk cursor, [6] long chunks
   blastp_hsp *out = nullptr;               // scratch for the host-array search
   int64_t out_cap = 0;
 };
@@ -361,6 +362,7 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   if (cudaMallocAsync(&db->stream, static_cast<size_t>(db->stream_len), s) != cudaSuccess ||
       cudaMallocAsync(&db->sstart, sizeof(int64_t) * static_cast<size_t>(std::max<int64_t>(n, 1)), s) != cudaSuccess ||
       cudaMallocAsync(&db->chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1)), s) != cudaSuccess ||
+      cudaMallocAsync(&db->long_chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1)), s) != cudaSuccess ||
       cudaMallocAsync(&db->counters, sizeof(unsigned long long) * 8, s) != cudaSuccess ||
       cudaMallocAsync(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1)), s) != cudaSuccess ||
       cudaMallocAsync(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1), s) != cudaSuccess ||
@@ -371,10 +373,13 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   upload_encode_table();
   cudaError_t e = cudaMemsetAsync(db->stream, kSentinel, static_cast<size_t>(db->stream_len), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(d_err, 0, sizeof(int), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(db->counters, 0, sizeof(unsigned long long) * 8, s);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(d_off, offsets + lo, sizeof(int64_t) * static_cast<size_t>(n + 1),
                         cudaMemcpyHostToDevice, s);
-  if (e == cudaSuccess) e = launch_layout(d_off, n, C, nchunks, db->sstart, db->chunks, d_err, s);
+  if (e == cudaSuccess)
+    e = launch_layout(d_off, n, C, nchunks, db->sstart, db->chunks, db->long_chunks,
+                      reinterpret_cast<int *>(db->counters + 6), d_err, s);
   if (e == cudaSuccess && nres > 0)
     e = cudaMemcpyAsync(d_ascii, residues_ascii + offsets[lo], static_cast<size_t>(nres),
                         cudaMemcpyHostToDevice, s);
@@ -428,6 +433,7 @@ void blastp_db_free(blastp_db *db) {
   cudaFree(db->stream);
   cudaFree(db->sstart);
   cudaFree(db->chunks);
+  cudaFree(db->long_chunks);
   cudaFree(db->counters);
   cudaFree(db->out);
   delete db;
@@ -468,6 +474,8 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.stream_len = db->stream_len;
     a.chunks = db->chunks;
     a.nchunks = db->nchunks;
+    a.long_chunks = db->long_chunks;
+    a.nlong = reinterpret_cast<const int *>(db->counters + 6);
     a.qv.woff = qd.woff;
     a.qv.qpos = qd.qpos;
     a.qv.qcodes = qd.qcodes;

@@ -86,6 +86,8 @@ struct SearchArgs {
   int64_t subject_base;
   const Chunk *chunks;
   int32_t nchunks;
+  const Chunk *long_chunks;  // scheduled before `chunks`
+  const int *nlong;          // device: number of long chunks
   QueryView qv;
   int32_t word_len, threshold, window, min_gap, xdrop, cutoff, filter_mode;
   int32_t ring;      // M: per-warp diagonal ring slots
@@ -127,7 +129,8 @@ cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
                         const int64_t *sstart, uint8_t *stream, int *err,
                         cudaStream_t s);
 cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
-                          int64_t *sstart, Chunk *chunks, int *err, cudaStream_t s);
+                          int64_t *sstart, Chunk *chunks, Chunk *long_chunks, int *nlong,
+                          int *err, cudaStream_t s);
 cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
 void upload_encode_table();
 

@@ -52,7 +52,7 @@ __global__ void layout_kernel(const int64_t *__restrict__ off, int64_t n, int64_
 // start == end and are skipped by the search kernels.
 __global__ void chunk_kernel(const int64_t *__restrict__ off, int64_t n,
                              const int64_t *__restrict__ sstart, int64_t C, int64_t nchunks,
-                             Chunk *chunks) {
+                             Chunk *chunks, Chunk *long_chunks, int *nlong) {
   const int64_t base = off[0];
   auto first_at = [&](int64_t k) -> int64_t {
     if (k >= nchunks) return n;
@@ -76,6 +76,12 @@ __global__ void chunk_kernel(const int64_t *__restrict__ off, int64_t n,
     } else {
       c.start = c.end = 0;
     }
+    // chunks much longer than C (long subjects) are scheduled first, so the
+    // single warp walking one never becomes the tail of the launch
+    if (c.end - c.start > 2 * C) {
+      long_chunks[atomicAdd(nlong, 1)] = c;
+      c.start = c.end = 0;
+    }
     chunks[k] = c;
   }
 }
@@ -83,14 +89,16 @@ __global__ void chunk_kernel(const int64_t *__restrict__ off, int64_t n,
 }  // namespace
 
 cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
-                          int64_t *sstart, Chunk *chunks, int *err, cudaStream_t s) {
+                          int64_t *sstart, Chunk *chunks, Chunk *long_chunks, int *nlong,
+                          int *err, cudaStream_t s) {
   if (n > 0) {
     const int64_t blocks = (n + 255) / 256 > 4096 ? 4096 : (n + 255) / 256;
     layout_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, err);
   }
   if (nchunks > 0) {
     const int64_t blocks = (nchunks + 255) / 256 > 4096 ? 4096 : (nchunks + 255) / 256;
-    chunk_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, C, nchunks, chunks);
+    chunk_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, C, nchunks, chunks, long_chunks,
+                                                  nlong);
   }
   return cudaGetLastError();
 }

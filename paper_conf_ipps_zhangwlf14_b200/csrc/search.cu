@@ -224,8 +224,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     unsigned long long ci = 0;
     if (lane == 0) ci = atomicAdd(a.chunk_cursor, 1ull);
     ci = __shfl_sync(kFull, ci, 0);
-    if (ci >= (unsigned long long)a.nchunks) break;
-    const Chunk ch = a.chunks[ci];
+    Chunk ch;
+    if (!fetch_chunk(a, ci, ch)) break;
     st.first_subj = ch.first_subj;
     st.last_subj = ch.last_subj;
     st.qhead = 0;

@@ -45,6 +45,20 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n"); }
 __device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_group 1;\n"); }
 
+// Work item ci of the chunk cursor: the long chunks first (their single warp
+// must not start last), then the regular plan.  False once all are taken.
+__device__ __forceinline__ bool fetch_chunk(const SearchArgs &a, unsigned long long ci, Chunk &ch) {
+  const unsigned long long nl = (unsigned long long)__ldg(a.nlong);
+  if (ci < nl) {
+    ch = a.long_chunks[ci];
+    return true;
+  }
+  ci -= nl;
+  if (ci >= (unsigned long long)a.nchunks) return false;
+  ch = a.chunks[ci];
+  return true;
+}
+
 // Diagonal two-hit state, 16-bit positions, 0 = none:
 //   last  most recent hit; far  largest hit <= last - W;
 //   near  bit j set iff a hit at last - j (1 <= j < W).

@@ -278,10 +278,10 @@ __device__ void producer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
     // ---- chunk management ---------------------------------------------------
     if (ptid == 0 && !C.have_chunk) {
       const unsigned long long ci = atomicAdd(a.chunk_cursor, 1ull);
-      if (ci >= (unsigned long long)a.nchunks) {
+      Chunk ch;
+      if (!fetch_chunk(a, ci, ch)) {
         C.have_chunk = -1;
       } else {
-        const Chunk ch = a.chunks[ci];
         const int frame = C.win;  // continue the frame (stale state ages out)
         C.spbase = ch.start - frame;
         C.end = ch.end - C.spbase;
