@@ -126,6 +126,14 @@ int blastp_shard_range(const int64_t *offsets, int64_t nseq,
 int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues,
                    int64_t *subject_base, int64_t *stream_bytes,
                    int64_t *num_chunks);
+/* Long-subject plan of the shard (implementation detail, exposed for tests
+ * and tuning): chunks longer than 2C residues that are scheduled first
+ * (*long_items), the segments they are split into for parallel two-hit
+ * filtering (*segments; 0 = every long chunk is walked whole) and the
+ * segment length in positions.  Results never depend on the plan.  Any
+ * pointer may be NULL.  Errors: INVALID_ARG (db NULL). */
+int blastp_db_long_info(const blastp_db *db, int64_t *long_items,
+                        int64_t *segments, int64_t *segment_len);
 int blastp_query_table_info(const blastp_query_table *q, int32_t *num_queries,
                             int64_t *table_entries);
 

@@ -76,6 +76,7 @@ def _load():
     L.blastp_pack_db.argtypes = [vp, vp, i64, i32, i32, ctypes.c_int, vp, P(vp)]
     L.blastp_shard_range.argtypes = [vp, i64, i32, i32, P(i64), P(i64)]
     L.blastp_db_info.argtypes = [vp, P(i64), P(i64), P(i64), P(i64), P(i64)]
+    L.blastp_db_long_info.argtypes = [vp, P(i64), P(i64), P(i64)]
     L.blastp_query_table_info.argtypes = [vp, P(i32), P(i64)]
     L.blastp_search_ungapped.argtypes = [vp, vp, P(_CParams), vp, P(vp), P(i64)]
     L.blastp_search_ungapped_device.argtypes = [vp, vp, P(_CParams), vp, vp, i64, vp]
@@ -95,7 +96,7 @@ lib = _load()
 
 EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "blastp_version",
             "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
-            "blastp_shard_range", "blastp_db_info", "blastp_query_table_info",
+            "blastp_shard_range", "blastp_db_info", "blastp_db_long_info", "blastp_query_table_info",
             "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_sort_hsps_device",
             "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
@@ -210,10 +211,7 @@ class Database:
                "blastp_pack_db")
         self.handle = h
         self.device = device
-        vals = [ctypes.c_int64() for _ in range(5)]
-        _check(lib.blastp_db_info(h, *[ctypes.byref(v) for v in vals]), "blastp_db_info")
-        self.nseq, self.residues, self.subject_base, self.stream_bytes, self.num_chunks = \
-            (v.value for v in vals)
+        self._info()
 
     @classmethod
     def from_pinned(cls, residues_ptr: int, offsets: np.ndarray, shard_index=0, num_shards=1,
@@ -227,11 +225,18 @@ class Database:
                "blastp_pack_db")
         self.handle = h
         self.device = device
+        self._info()
+        return self
+
+    def _info(self):
         vals = [ctypes.c_int64() for _ in range(5)]
-        _check(lib.blastp_db_info(h, *[ctypes.byref(v) for v in vals]), "blastp_db_info")
+        _check(lib.blastp_db_info(self.handle, *[ctypes.byref(v) for v in vals]), "blastp_db_info")
         self.nseq, self.residues, self.subject_base, self.stream_bytes, self.num_chunks = \
             (v.value for v in vals)
-        return self
+        vals = [ctypes.c_int64() for _ in range(3)]
+        _check(lib.blastp_db_long_info(self.handle, *[ctypes.byref(v) for v in vals]),
+               "blastp_db_long_info")
+        self.long_items, self.segments, self.segment_len = (v.value for v in vals)
 
     def free(self):
         if getattr(self, "handle", None):

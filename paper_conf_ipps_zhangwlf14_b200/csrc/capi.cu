@@ -112,13 +112,74 @@ struct blastp_db {
   uint8_t *stream = nullptr;
   int64_t *sstart = nullptr;
   Chunk *chunks = nullptr;
-  Chunk *long_chunks = nullptr;  // chunks > 2C residues, scheduled first (count at counters[6])
+  Chunk *long_chunks = nullptr;  // chunks > 2C residues (count at counters[6]), pack only
   int32_t nchunks = 0;
+  // long items, longest first, and their segments
+  LongItem *items = nullptr;
+  int32_t nlong = 0, nsegs = 0, seg_len = kSegLen, seg_cap = kSegCap;
+  int32_t *seg_item = nullptr, *seg_count = nullptr;
+  uint32_t *seg_list = nullptr;
+  unsigned *seg_done = nullptr;
+  unsigned seq = 0;  // search launches on this db (segment publication epoch)
   std::vector<int64_t> h_sstart;
   unsigned long long *counters = nullptr;  // [0] hsp count, [1] chunk cursor, [6] long chunks
   blastp_hsp *out = nullptr;               // scratch for the host-array search
   int64_t out_cap = 0;
 };
+
+// Long items (chunks > 2C, i.e. ending in a long subject), longest first;
+// those longer than 2 segments are split into segments (DESIGN.md "Long
+// subjects") while the segment budget lasts.  Knobs for tests/experiments:
+// BLASTP_SEGMENTS=0 (off), BLASTP_SEGLEN (256..16384; >= the largest window A
+// so a segment's warm-up stays inside its chunk), BLASTP_SEGCAP.
+static cudaError_t plan_long_items(blastp_db *db, int nlong, cudaStream_t s) {
+  std::vector<Chunk> lc(static_cast<size_t>(nlong));
+  cudaError_t e = cudaMemcpyAsync(lc.data(), db->long_chunks, sizeof(Chunk) * lc.size(),
+                                  cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) return e;
+  std::sort(lc.begin(), lc.end(), [](const Chunk &x, const Chunk &y) {
+    const int64_t lx = x.end - x.start, ly = y.end - y.start;
+    return lx != ly ? lx > ly : x.start < y.start;
+  });
+  const char *on = std::getenv("BLASTP_SEGMENTS");
+  const bool enabled = !(on && std::atoi(on) == 0);
+  if (const char *v = std::getenv("BLASTP_SEGLEN")) db->seg_len = std::max(256, std::min(16384, std::atoi(v)));
+  if (const char *v = std::getenv("BLASTP_SEGCAP")) db->seg_cap = std::max(1, std::atoi(v));
+  std::vector<LongItem> items(lc.size());
+  std::vector<int32_t> seg_item;
+  for (size_t i = 0; i < lc.size(); ++i) {
+    LongItem &it = items[i];
+    it = LongItem{};
+    it.c = lc[i];
+    const int64_t len = lc[i].end - lc[i].start;
+    const int64_t nseg = (len + db->seg_len - 1) / db->seg_len;
+    if (enabled && len > 2 * int64_t(db->seg_len) &&
+        int64_t(seg_item.size()) + nseg <= kMaxSegments) {
+      it.seg0 = static_cast<int32_t>(seg_item.size());
+      it.nseg = static_cast<int32_t>(nseg);
+      seg_item.insert(seg_item.end(), static_cast<size_t>(nseg), static_cast<int32_t>(i));
+    }
+  }
+  db->nlong = nlong;
+  db->nsegs = static_cast<int32_t>(seg_item.size());
+  const size_t ns = std::max<size_t>(seg_item.size(), 1);
+  if ((e = cudaMallocAsync(&db->items, sizeof(LongItem) * items.size(), s)) != cudaSuccess) return e;
+  if ((e = cudaMallocAsync(&db->seg_item, sizeof(int32_t) * ns, s)) != cudaSuccess) return e;
+  if ((e = cudaMallocAsync(&db->seg_count, sizeof(int32_t) * ns, s)) != cudaSuccess) return e;
+  if ((e = cudaMallocAsync(&db->seg_done, sizeof(unsigned) * ns, s)) != cudaSuccess) return e;
+  if ((e = cudaMallocAsync(&db->seg_list, sizeof(uint32_t) * ns * size_t(db->seg_cap), s)) != cudaSuccess)
+    return e;
+  if ((e = cudaMemcpyAsync(db->items, items.data(), sizeof(LongItem) * items.size(),
+                           cudaMemcpyHostToDevice, s)) != cudaSuccess)
+    return e;
+  if (!seg_item.empty() &&
+      (e = cudaMemcpyAsync(db->seg_item, seg_item.data(), sizeof(int32_t) * seg_item.size(),
+                           cudaMemcpyHostToDevice, s)) != cudaSuccess)
+    return e;
+  if ((e = cudaMemsetAsync(db->seg_done, 0, sizeof(unsigned) * ns, s)) != cudaSuccess) return e;
+  return cudaStreamSynchronize(s);  // the host vectors die here
+}
 
 static void free_query_dev(QueryDev &d) {
   cudaFree(d.woff);
@@ -384,8 +445,10 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
     e = cudaMemcpyAsync(d_ascii, residues_ascii + offsets[lo], static_cast<size_t>(nres),
                         cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess) e = launch_pack(d_ascii, d_off, n, db->sstart, db->stream, d_err, s);
-  int h_err = 0;
+  int h_err = 0, h_nlong = 0;
   if (e == cudaSuccess) e = cudaMemcpyAsync(&h_err, d_err, sizeof(int), cudaMemcpyDeviceToHost, s);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(&h_nlong, db->counters + 6, sizeof(int), cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess) e = cudaStreamSynchronize(s);
   if (e != cudaSuccess)
     return cleanup(fail(BLASTP_E_CUDA, "packing the database failed: %s", cudaGetErrorString(e)));
@@ -399,6 +462,10 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
         return cleanup(fail(BLASTP_E_BAD_RESIDUE, "database byte %lld (0x%02x) is not a residue",
                             static_cast<long long>(k), static_cast<unsigned char>(residues_ascii[k])));
     return cleanup(fail(BLASTP_E_BAD_RESIDUE, "database holds an invalid residue"));
+  }
+  if (h_nlong > 0 && plan_long_items(db, h_nlong, s) != cudaSuccess) {
+    cudaGetLastError();
+    return cleanup(fail(BLASTP_E_NOMEM, "device allocation for the long-subject plan failed"));
   }
   *out = db;
   return cleanup(BLASTP_OK);
@@ -414,6 +481,15 @@ static const std::vector<int64_t> &host_sstart(const blastp_db *db) {
                  cudaMemcpyDeviceToHost);
   }
   return mdb->h_sstart;
+}
+
+int blastp_db_long_info(const blastp_db *db, int64_t *long_items, int64_t *segments,
+                        int64_t *segment_len) {
+  if (!db) return fail(BLASTP_E_INVALID_ARG, "db is NULL");
+  if (long_items) *long_items = db->nlong;
+  if (segments) *segments = db->nsegs;
+  if (segment_len) *segment_len = db->seg_len;
+  return BLASTP_OK;
 }
 
 int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues, int64_t *subject_base,
@@ -434,6 +510,11 @@ void blastp_db_free(blastp_db *db) {
   cudaFree(db->sstart);
   cudaFree(db->chunks);
   cudaFree(db->long_chunks);
+  cudaFree(db->items);
+  cudaFree(db->seg_item);
+  cudaFree(db->seg_count);
+  cudaFree(db->seg_done);
+  cudaFree(db->seg_list);
   cudaFree(db->counters);
   cudaFree(db->out);
   delete db;
@@ -474,8 +555,16 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.stream_len = db->stream_len;
     a.chunks = db->chunks;
     a.nchunks = db->nchunks;
-    a.long_chunks = db->long_chunks;
-    a.nlong = reinterpret_cast<const int *>(db->counters + 6);
+    a.long_items = db->items;
+    a.nlong = db->nlong;
+    a.nsegs = db->nsegs;
+    a.seg_item = db->seg_item;
+    a.seg_list = db->seg_list;
+    a.seg_count = db->seg_count;
+    a.seg_done = db->seg_done;
+    a.seg_len = db->seg_len;
+    a.seg_cap = db->seg_cap;
+    a.seq = ++const_cast<blastp_db *>(db)->seq;
     a.qv.woff = qd.woff;
     a.qv.qpos = qd.qpos;
     a.qv.qcodes = qd.qcodes;

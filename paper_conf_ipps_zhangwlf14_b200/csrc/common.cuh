@@ -63,6 +63,19 @@ struct Chunk {
   int64_t first_subj, last_subj;
 };
 
+// A chunk longer than 2C (it ends in a long subject), scheduled before the
+// regular chunks.  With nseg > 0 the warp variant splits it (DESIGN.md "Long
+// subjects"): segment k covers emit positions [start + k*seg_len, +seg_len)
+// and is two-hit filtered by its own warp after a `window`-position warm-up,
+// writing its passing hits to a list; one walker warp then feeds the lists,
+// in s order, through extension and the ext_reach chain.  nseg == 0: the
+// chunk is walked whole by one warp.
+struct LongItem {
+  Chunk c;
+  int32_t seg0, nseg;  // segments [seg0, seg0 + nseg) of the segment arrays
+  int64_t pad;
+};
+
 // Trace record (debug entry points only): stream position of the hit /
 // seed, query position, and for extensions llen/rlen/score.
 struct TraceRec {
@@ -86,8 +99,17 @@ struct SearchArgs {
   int64_t subject_base;
   const Chunk *chunks;
   int32_t nchunks;
-  const Chunk *long_chunks;  // scheduled before `chunks`
-  const int *nlong;          // device: number of long chunks
+  // Work items of the chunk cursor, in order: segments [0, nsegs) (warp
+  // variant only), long items [0, nlong), regular chunks [0, nchunks).
+  const LongItem *long_items;
+  int32_t nlong;
+  int32_t nsegs;               // 0: no segment pipeline
+  const int32_t *seg_item;     // [nsegs] long item of each segment
+  uint32_t *seg_list;          // [nsegs * seg_cap] passing hits: (s - emit) | q << 16
+  int32_t *seg_count;          // [nsegs] list length, -1 = overflow
+  unsigned *seg_done;          // [nsegs] == seq once the segment's list is published
+  int32_t seg_len, seg_cap;
+  unsigned seq;                // launch sequence number of this search
   QueryView qv;
   int32_t word_len, threshold, window, min_gap, xdrop, cutoff, filter_mode;
   int32_t ring;      // M: per-warp diagonal ring slots
@@ -131,6 +153,10 @@ cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
 cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
                           int64_t *sstart, Chunk *chunks, Chunk *long_chunks, int *nlong,
                           int *err, cudaStream_t s);
+// Segment length / list capacity of the long-item pipeline.
+constexpr int kSegLen = 2048;
+constexpr int kSegCap = 2048;
+constexpr int kMaxSegments = 32768;  // 256 MB of lists at most
 cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
 void upload_encode_table();
 

@@ -27,6 +27,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <climits>
 #include <cstdlib>
 #include <cstring>
 
@@ -65,13 +66,16 @@ struct WarpSmem {
   uint16_t *reach;   // [M] ext_reach (frame position, 0 = none)
   uint32_t *queue;   // [kQcap]: P | q << 16 (the slot is recomputed at flush)
   uint16_t *fs_p, *fs_end, *fs_acc;  // [32] flush scratch
+  int *wk;           // [8] walker state: item, segment, entry, slot offset;
+                     // [4] segment being filtered (-1: none), [5] its list length
 };
 
 // Per-warp shared memory: 6 B per diagonal slot + 352 B; small enough for
 // 30+ resident warps per SM at Lq ~ 1000 (occupancy is what this latency-
 // bound kernel runs on, profiles/r01).
 __host__ __device__ size_t warp_smem_bytes(int ring) {
-  return align16(size_t(ring) * 4) + align16(size_t(ring) * 2) + size_t(kQcap) * 4 + 3 * 32 * 2;
+  return align16(size_t(ring) * 4) + align16(size_t(ring) * 2) + size_t(kQcap) * 4 + 3 * 32 * 2 +
+         32;
 }
 
 __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
@@ -85,6 +89,7 @@ __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
   w.fs_p = reinterpret_cast<uint16_t *>(base);
   w.fs_end = w.fs_p + 32;
   w.fs_acc = w.fs_p + 64;
+  w.wk = reinterpret_cast<int *>(w.fs_p + 96);
   return w;
 }
 
@@ -214,26 +219,204 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
   const uint8_t *__restrict__ stream = a.stream;
   const int W = kW ? kW : a.min_gap, A = a.window;  // kW: compile-time min_gap
   const uint32_t nearmask = (1u << W) - 2u;  // bits 1 .. W-1
+  const int warm = (A + 31) & ~31;           // segment warm-up, whole windows
 
   WarpState st;
   if (kTrace)
     for (int i = 0; i < kNumStats; ++i) st.stat[i] = 0;
+  st.qhead = 0;
+  st.qcount = 0;
   int frame = kFrameMin;  // frame position of the next chunk's first residue
   int base_slot = 0;      // ring slot of diagonal (win - q + const) at q = lane = 0
+  // subtract kFrameSpan from every stored frame position (0 = none stays 0)
+  auto rebase_ring = [&]() {
+    for (int i = lane; i < M; i += 32) {
+      const uint32_t e = w.ring[i];
+      auto rb = [](uint32_t v) { return v > uint32_t(kFrameSpan) ? v - kFrameSpan : 0u; };
+      const uint32_t nl = rb(st_last(e));
+      w.ring[i] = nl ? st_make(nl, rb(st_far(e)), st_near(e)) : 0u;
+      w.reach[i] = uint16_t(rb(w.reach[i]));
+    }
+    __syncwarp();
+    st.spbase += kFrameSpan;
+  };
+  const unsigned long long nsegs = (unsigned long long)a.nsegs;
+  const unsigned long long nitems = nsegs + (unsigned long long)a.nlong;
+  // Work items: segments (walk, queue spilled to a list), long items (walker, or a plain
+  // walk), regular chunks (walk).  Every queue drain outside the hot round
+  // loop happens at the single site at the bottom of this loop, so the
+  // X-drop code exists in three copies only (instruction-cache footprint);
+  // the walker therefore runs in steps that end whenever the queue must be
+  // drained, its state parked in shared memory (w.wk), not in registers.
+  int mode = 0;  // 0: take the next work item; 1: a walker is active
   for (;;) {
-    unsigned long long ci = 0;
-    if (lane == 0) ci = atomicAdd(a.chunk_cursor, 1ull);
-    ci = __shfl_sync(kFull, ci, 0);
-    Chunk ch;
-    if (!fetch_chunk(a, ci, ch)) break;
-    st.first_subj = ch.first_subj;
-    st.last_subj = ch.last_subj;
-    st.qhead = 0;
-    st.qcount = 0;
-    st.spbase = ch.start - frame;
+    int64_t wstart = 0, wend = 0, wemit = 0;
+    bool walk = false;
+    bool retrace = false;  // fallback walk: its hits were traced by the segments
+    int sg = -1;
+    int sc = 0;  // slot offset of the queued entries, for the drain below
+    if (mode == 0) {
+      unsigned long long ci = 0;
+      if (lane == 0) ci = atomicAdd(a.chunk_cursor, 1ull);
+      ci = __shfl_sync(kFull, ci, 0);
+      // a walk covers stream positions [wstart, wend); hits before wemit
+      // only warm the two-hit state (segments); a segment's queue is
+      // spilled to its list instead of being extended
+      if (ci < nsegs) {
+        sg = int(ci);
+        const LongItem &it = a.long_items[a.seg_item[sg]];
+        wemit = it.c.start + int64_t(sg - it.seg0) * a.seg_len;
+        wend = min(it.c.end, wemit + a.seg_len);
+        // R6 looks back < A positions: a warm-up of A rounded up to whole
+        // windows (seg_len >= 256 >= A keeps it inside the chunk)
+        wstart = sg == it.seg0 ? it.c.start : wemit - warm;
+        st.first_subj = it.c.first_subj;
+        st.last_subj = it.c.last_subj;
+        walk = true;
+      } else if (ci < nitems) {
+        const LongItem it = a.long_items[ci - nsegs];
+        st.first_subj = it.c.first_subj;
+        st.last_subj = it.c.last_subj;
+        if (it.nseg > 0) {
+          st.spbase = it.c.start - frame;
+          if (lane == 0) {
+            w.wk[0] = int(ci - nsegs);
+            w.wk[1] = 0;
+            w.wk[2] = 0;
+            w.wk[3] = ((base_slot - frame) % M + M) % M;  // slot = P - q + offset
+          }
+          __syncwarp();
+          mode = 1;
+        } else {
+          wstart = wemit = it.c.start;
+          wend = it.c.end;
+          walk = true;
+        }
+      } else {
+        const unsigned long long cj = ci - nitems;
+        if (cj >= (unsigned long long)a.nchunks) break;
+        const Chunk ch = a.chunks[cj];
+        st.first_subj = ch.first_subj;
+        st.last_subj = ch.last_subj;
+        wstart = wemit = ch.start;
+        wend = ch.end;
+        walk = true;
+      }
+    }
+    if (mode == 1) {
+      // ---- walker step: the segments' passing hits, in s order, into the
+      // extension queue (the ext_reach chain resolves at the drain, exactly
+      // as in a walk); returns whenever the queue must be drained first
+      const LongItem it = a.long_items[__shfl_sync(kFull, w.wk[0], 0)];
+      int k = __shfl_sync(kFull, w.wk[1], 0), i0 = __shfl_sync(kFull, w.wk[2], 0),
+          slotw = __shfl_sync(kFull, w.wk[3], 0);
+      // a rebase lowers every frame position by kFrameSpan: the slot offset
+      // rises by as much, so each diagonal keeps its slot
+      auto rebase_w = [&]() {
+        rebase_ring();
+        slotw = (slotw + kFrameSpan) % M;
+      };
+      for (;;) {
+        if (k == it.nseg) {
+          if (st.qcount > 0) break;
+          while (it.c.end - st.spbase >= kFrameMin + kFrameSpan) rebase_w();
+          frame = int(it.c.end - st.spbase) + 64;
+          base_slot = (frame + slotw) % M;
+          mode = 0;
+          break;
+        }
+        const int sgk = it.seg0 + k;
+        const int64_t emit = it.c.start + int64_t(k) * a.seg_len;
+        // wait (warp-uniformly) for the segment's list to be published
+        while (__shfl_sync(kFull, ld_acquire(a.seg_done + sgk), 0) != a.seq) __nanosleep(256);
+        // values that steer control flow are broadcast from lane 0: the
+        // compiler then knows they are warp-uniform (volatile loads are not)
+        const int n = __shfl_sync(kFull, *(volatile const int32_t *)(a.seg_count + sgk), 0);
+        if (n < 0) {
+          // the list overflowed: walk the rest of the chunk directly,
+          // continuing this frame and ext_reach state
+          if (st.qcount > 0) break;
+          wstart = k == 0 ? it.c.start : emit - warm;
+          wemit = emit;
+          wend = it.c.end;
+          while (wstart - st.spbase >= kFrameMin + kFrameSpan) rebase_w();
+          frame = int(wstart - st.spbase);
+          base_slot = (frame + slotw) % M;
+          walk = true;
+          retrace = true;
+          mode = 0;
+          break;
+        }
+        if (i0 >= n) {
+          ++k;
+          i0 = 0;
+          continue;
+        }
+        const volatile uint32_t *L = a.seg_list + int64_t(sgk) * a.seg_cap;
+        const uint32_t e0 = __shfl_sync(kFull, lane == 0 ? L[i0] : 0u, 0);
+        if (emit + int64_t(e0 & 0xffffu) - st.spbase >= kFrameMin + kFrameSpan) {
+          if (st.qcount > 0) break;
+          rebase_w();
+          continue;
+        }
+        const int i = i0 + lane;
+        const uint32_t e = i < n ? L[i] : 0u;
+        const int64_t P64 = emit + int64_t(e & 0xffffu) - st.spbase;
+        const bool act = i < n && P64 < kFrameMin + kFrameSpan + 32;  // a prefix
+        const int P = int(P64), q = int(e >> 16);
+        uint32_t rch = 0;
+        if (act) {
+          int slot = (P - q + slotw) % M;
+          slot += slot < 0 ? M : 0;
+          rch = w.reach[slot];
+        }
+        const bool enq = act && P > int(rch);
+        const unsigned bal = __ballot_sync(kFull, enq);
+        stat_add<kTrace>(st, kStatEnqueued, __popc(bal));
+        const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
+        if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = uint32_t(P) | (uint32_t(q) << 16);
+        st.qcount += __popc(bal);
+        i0 += __popc(__ballot_sync(kFull, act));
+        if (st.qcount >= 32) break;
+      }
+      __syncwarp();
+      if (lane == 0) {
+        w.wk[1] = k;
+        w.wk[2] = i0;
+        w.wk[3] = slotw;
+      }
+      __syncwarp();
+      sc = slotw;
+    }
+    if (walk) {
+    __syncwarp();
+    if (lane == 0) {
+      w.wk[4] = sg;
+      w.wk[5] = 0;
+    }
+    __syncwarp();
+    st.spbase = wstart - frame;
     int win = frame;                           // frame position of lane 0 of the window
     int lastsent = frame - 1;                  // the sentinel before the chunk
-    int64_t end = ch.end - st.spbase;          // frame position of the chunk end (exclusive)
+    int64_t end = wend - st.spbase;            // frame position of the chunk end (exclusive)
+    int emit_f = int(wemit - st.spbase);       // first frame position whose hits count
+    // Segment: move n queued entries to the segment's list as (s - emit) |
+    // q << 16 (passing hits in s order; ext_reach holds only stale values
+    // older than the frame there, so every passing hit was queued)
+    auto spill = [&](int n) {
+      const int sgw = __shfl_sync(kFull, w.wk[4], 0);
+      const int nl = __shfl_sync(kFull, w.wk[5], 0);
+      if (lane < n && nl + lane < a.seg_cap) {
+        const uint32_t ent = w.queue[(st.qhead + lane) & (kQcap - 1)];
+        a.seg_list[int64_t(sgw) * a.seg_cap + nl + lane] =
+            ((ent & 0xffffu) - uint32_t(emit_f)) | (ent & 0xffff0000u);
+      }
+      __syncwarp();
+      if (lane == 0) w.wk[5] = nl + n;
+      __syncwarp();
+      st.qhead = (st.qhead + n) & (kQcap - 1);
+      st.qcount -= n;
+    };
     // Software pipeline over windows: residues are loaded two windows ahead
     // (one coalesced byte per lane + 2 bytes of overlap), the table lookup is
     // issued one window ahead and consumed by the next iteration.
@@ -271,20 +454,18 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     while (win < end) {
       // ---- rebase the frame before positions outgrow 16 bits --------------
       if (win >= kFrameMin + kFrameSpan) {
-        while (st.qcount > 0)
-          flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc(), M);
-        for (int i = lane; i < M; i += 32) {
-          const uint32_t e = w.ring[i];
-          auto rb = [](uint32_t v) { return v > uint32_t(kFrameSpan) ? v - kFrameSpan : 0u; };
-          const uint32_t nl = rb(st_last(e));
-          w.ring[i] = nl ? st_make(nl, rb(st_far(e)), st_near(e)) : 0u;
-          w.reach[i] = uint16_t(rb(w.reach[i]));
+        if (__shfl_sync(kFull, w.wk[4], 0) >= 0) {
+          while (st.qcount > 0) spill(min(st.qcount, 32));
+        } else {
+          const int sc = slotc();
+          while (st.qcount > 0)
+            flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
         }
-        __syncwarp();
+        rebase_ring();
         win -= kFrameSpan;
         lastsent -= kFrameSpan;
         end -= kFrameSpan;
-        st.spbase += kFrameSpan;
+        emit_f -= kFrameSpan;
       }
       stat_add<kTrace>(st, kStatIterations, 1);
       // ---- this window's lookup (issued last iteration); issue the next ---
@@ -305,7 +486,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       const uint32_t Hn = __shfl_sync(kFull, incl, 31);
       // last sentinel at or before each lane (before `win`: lastsent)
       const unsigned prior = sm & ((lane == 31) ? kFull : ((2u << lane) - 1u));
-      const int ls_lane = prior ? (win + 31 - __clz(prior)) : lastsent;
+      int ls_lane = prior ? (win + 31 - __clz(prior)) : lastsent;
+      // a segment's warm-up windows (emit_f is window-aligned): a sentinel
+      // "after" every hit makes R6's lower bound unreachable, so no hit passes
+      if (win < emit_f) ls_lane = INT_MAX - 1;
 
       // round r's owner lane and query position are computed (and the query
       // position load issued) one round ahead of its processing
@@ -377,18 +561,23 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           }
         }
         const int cand = max(cand_s, cand_e);
-        bool pass = act && cand >= lo_ok;
+        // not a segment's warm-up (the LEFT test fails there by ls above)
+        const bool counts = act && (kTrace || kEither ? Ph >= emit_f : true);
+        bool pass = counts && cand >= lo_ok;
         const int64_t sph = st.spbase + Ph;
-        if (kEither && act && !pass)
+        if (kEither && counts && !pass)
           pass = has_successor(stream, sph, q, qc, b62, lq, W, A, a.threshold);
         if (kTrace) {
           stat_add<kTrace>(st, kStatRounds, 1);
           stat_add<kTrace>(st, kStatConflictRounds, nearly ? 1 : 0);
-          stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, act)));
-          stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
-          stat_add<kTrace>(st, kStatEnqueued,
-                           __popc(__ballot_sync(kFull, pass && Ph > int(rch))));
-          if (act) {
+          if (!retrace) {
+            stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, counts)));
+            stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
+          }
+          if (w.wk[4] < 0)
+            stat_add<kTrace>(st, kStatEnqueued,
+                             __popc(__ballot_sync(kFull, pass && Ph > int(rch))));
+          if (counts && !retrace) {
             trace_push(a, 0, sph, q, 0, 0, 0);
             if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
           }
@@ -410,7 +599,12 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = uint32_t(Ph) | (uint32_t(q) << 16);
           st.qcount += __popc(bal);
           __syncwarp();
-          if (st.qcount >= 32) flush_queue<kTrace>(a, w, st, 32, qc, b62, lane, slotc(), M);
+          if (st.qcount >= 32) {
+            if (__shfl_sync(kFull, w.wk[4], 0) >= 0)
+              spill(32);  // segment: to its list
+            else
+              flush_queue<kTrace>(a, w, st, 32, qc, b62, lane, slotc(), M);
+          }
         }
         __syncwarp();
       }
@@ -421,11 +615,23 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       base_slot += npos;
       if (base_slot >= M) base_slot -= M;
     }
-    while (st.qcount > 0)
-      flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc(), M);
+    if (const int sgw = __shfl_sync(kFull, w.wk[4], 0); sgw >= 0) {
+      while (st.qcount > 0) spill(min(st.qcount, 32));
+      const int nl = __shfl_sync(kFull, w.wk[5], 0);
+      __threadfence();
+      __syncwarp();
+      if (lane == 0) {
+        a.seg_count[sgw] = nl > a.seg_cap ? -1 : nl;
+        st_release(a.seg_done + sgw, a.seq);
+      }
+    }
+    sc = slotc();
     // the next chunk continues the frame after a gap (stale state ages out)
     frame = win + 64;
     base_slot = (base_slot + 64) % M;
+    }  // walk
+    // ---- the single drain site (chunk end, walker steps) -------------------
+    while (st.qcount > 0) flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
   }
   cp_async_wait_all();
   if (kTrace && a.stats && lane == 0)
@@ -453,7 +659,7 @@ cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_
   if (e != cudaSuccess) return e;
   if (per_sm < 1) return cudaErrorInvalidConfiguration;
   int64_t grid = int64_t(num_sms) * per_sm;
-  const int64_t need = (int64_t(a.nchunks) + warps - 1) / warps;
+  const int64_t need = (int64_t(a.nchunks) + a.nlong + a.nsegs + warps - 1) / warps;
   if (grid > need) grid = need < 1 ? 1 : need;
   k<<<unsigned(grid), warps * 32, smem, s>>>(a);
   return cudaGetLastError();

@@ -45,18 +45,28 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n"); }
 __device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_group 1;\n"); }
 
-// Work item ci of the chunk cursor: the long chunks first (their single warp
-// must not start last), then the regular plan.  False once all are taken.
+// Work item ci of the chunk cursor without the segment pipeline: the long
+// items whole (their single warp must not start last), then the regular
+// plan.  False once all are taken.
 __device__ __forceinline__ bool fetch_chunk(const SearchArgs &a, unsigned long long ci, Chunk &ch) {
-  const unsigned long long nl = (unsigned long long)__ldg(a.nlong);
+  const unsigned long long nl = (unsigned long long)a.nlong;
   if (ci < nl) {
-    ch = a.long_chunks[ci];
+    ch = a.long_items[ci].c;
     return true;
   }
   ci -= nl;
   if (ci >= (unsigned long long)a.nchunks) return false;
   ch = a.chunks[ci];
   return true;
+}
+
+__device__ __forceinline__ unsigned ld_acquire(const unsigned *p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(unsigned *p, unsigned v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
 }
 
 // Diagonal two-hit state, 16-bit positions, 0 = none:

@@ -735,7 +735,8 @@ cudaError_t launch_variant(const SearchArgs &a, const CtaConfig &c, size_t smem,
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
   int grid = num_sms;
-  if (grid > a.nchunks) grid = a.nchunks < 1 ? 1 : a.nchunks;
+  const int items = a.nchunks + a.nlong;
+  if (grid > items) grid = items < 1 ? 1 : items;
   k<<<unsigned(grid), kThreads, smem, s>>>(a, c);
   return cudaGetLastError();
 }
@@ -763,6 +764,7 @@ cudaError_t launch_search(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
   cudaError_t e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
   SearchArgs a = a_in;
+  a.nsegs = 0;  // no segment pipeline: long items are walked whole
   CtaConfig c{};
   c.np = 24;
   c.nc = 8;

@@ -184,6 +184,65 @@ def test_edge_cases(bp, orc):
     assert len(g) == 0
 
 
+def _long_subject_db(q):
+    """Long subjects (> 2C residues: split into segments) with copies of the
+    query planted across segment boundaries (exact ones, so an extension and
+    its ext_reach run from one segment into the next), one subject longer
+    than the 16-bit frame (65536), and short subjects around them."""
+    rng = np.random.default_rng(5)
+    L = len(q)
+
+    def subject(n, plants):
+        s = list(gen_query(int(rng.integers(1, 1 << 30)), n).decode())
+        for pos, exact in plants:
+            seg = list(q)
+            if not exact:
+                for i in np.nonzero(rng.random(L) < 0.3)[0]:
+                    seg[i] = ALPHA[int(rng.integers(0, 20))]
+            s[pos:pos + L] = seg
+        return "".join(s[:n])
+
+    subs = [gen_query(11, 120).decode(), "",
+            subject(40000, [(2048 - 100, True), (4096 - 7, False), (9000, True),
+                            (20480 - L // 2, True), (39000, False)]),
+            gen_query(12, 300).decode(),
+            subject(9000, [(100, True), (4000, True), (4100 + L, False)]),
+            subject(5000, [(2000, True)]),
+            subject(70000, [(1000, True), (32768 - 50, True), (65536 - 80, True), (69000, False)]),
+            q, gen_query(13, 700).decode(), "MK"]
+    ascii = np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy()
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    return ascii, off
+
+
+@pytest.mark.parametrize("knobs", [{}, {"BLASTP_SEGLEN": "256"}, {"BLASTP_SEGCAP": "4"},
+                                   {"BLASTP_SEGCAP": "150"}, {"BLASTP_SEGMENTS": "0"}],
+                         ids=["default", "seglen256", "overflow_all", "overflow_some", "off"])
+def test_long_subjects_segmented(bp, orc, monkeypatch, kernel_variant, knobs):
+    """The long-subject plan (segments filtered in parallel, one walker per
+    long chunk, list-overflow fallback) gives the oracle's results exactly:
+    hits, passing hits, extensions and HSPs, both filter readings."""
+    q = gen_query(21, 300).decode()
+    ascii, off = _long_subject_db(q)
+    for k, v in knobs.items():
+        monkeypatch.setenv(k, v)
+    d = bp.pack_db(ascii, off)
+    assert d.long_items >= 4
+    if knobs.get("BLASTP_SEGMENTS") == "0":
+        assert d.segments == 0
+    else:
+        assert d.segments >= (40000 + 9000 + 5000 + 70000) // d.segment_len
+    for mode, window in ((0, 40), (1, 40), (0, 80), (0, 256)):
+        p = bp.Params(filter_mode=mode, window=window)
+        g, r = assert_same(bp, orc, q, ascii, off, p, trace=True)
+        assert len(g) > 10
+    # repeated searches on one db (segment publication epochs)
+    t = bp.build_query_table(q, bp.Params())
+    first = tuples(bp.search_ungapped(t, d, bp.Params()))
+    for _ in range(3):
+        assert tuples(bp.search_ungapped(t, d, bp.Params())) == first
+
+
 def test_long_query_2000(bp, orc):
     q = gen_query(2000, 2000)
     db = gen_db(7, 8, n_subjects=400, mean_len=375.0, queries=[q], plant_frac=0.2)
