@@ -17,7 +17,9 @@ from dataclasses import dataclass
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libblastp.so")
+# BLASTP_LIB: load another build of the same library (A/B timing of kernel
+# revisions); it is still this package's C-ABI, never a fallback.
+LIB_PATH = os.environ.get("BLASTP_LIB") or os.path.join(_PKG, "libblastp.so")
 
 OK, E_INVALID_ARG, E_BAD_RESIDUE, E_TOO_LONG, E_NOMEM, E_CUDA, E_CAPACITY = 0, -1, -2, -3, -4, -5, -6
 FILTER_LEFT, FILTER_EITHER = 0, 1
@@ -76,7 +78,8 @@ def _load():
     L.blastp_pack_db.argtypes = [vp, vp, i64, i32, i32, ctypes.c_int, vp, P(vp)]
     L.blastp_shard_range.argtypes = [vp, i64, i32, i32, P(i64), P(i64)]
     L.blastp_db_info.argtypes = [vp, P(i64), P(i64), P(i64), P(i64), P(i64)]
-    L.blastp_db_long_info.argtypes = [vp, P(i64), P(i64), P(i64)]
+    if hasattr(L, "blastp_db_long_info"):  # absent in builds older than the long-item plan
+        L.blastp_db_long_info.argtypes = [vp, P(i64), P(i64), P(i64)]
     L.blastp_query_table_info.argtypes = [vp, P(i32), P(i64)]
     L.blastp_search_ungapped.argtypes = [vp, vp, P(_CParams), vp, P(vp), P(i64)]
     L.blastp_search_ungapped_device.argtypes = [vp, vp, P(_CParams), vp, vp, i64, vp]
@@ -233,10 +236,12 @@ class Database:
         _check(lib.blastp_db_info(self.handle, *[ctypes.byref(v) for v in vals]), "blastp_db_info")
         self.nseq, self.residues, self.subject_base, self.stream_bytes, self.num_chunks = \
             (v.value for v in vals)
-        vals = [ctypes.c_int64() for _ in range(3)]
-        _check(lib.blastp_db_long_info(self.handle, *[ctypes.byref(v) for v in vals]),
-               "blastp_db_long_info")
-        self.long_items, self.segments, self.segment_len = (v.value for v in vals)
+        self.long_items = self.segments = self.segment_len = None
+        if hasattr(lib, "blastp_db_long_info"):
+            vals = [ctypes.c_int64() for _ in range(3)]
+            _check(lib.blastp_db_long_info(self.handle, *[ctypes.byref(v) for v in vals]),
+                   "blastp_db_long_info")
+            self.long_items, self.segments, self.segment_len = (v.value for v in vals)
 
     def free(self):
         if getattr(self, "handle", None):
