@@ -126,6 +126,26 @@ int blastp_shard_range(const int64_t *offsets, int64_t nseq,
 int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues,
                    int64_t *subject_base, int64_t *stream_bytes,
                    int64_t *num_chunks);
+/* End-to-end search of a HOST-resident database shard (no blastp_db kept):
+ * the shard's subjects (blastp_shard_range) are cut into parts of whole
+ * subjects (num_parts > 0: that many residue-balanced parts; 0: automatic,
+ * growing 1.5x from ~1/64 of the shard) and each part is packed (H2D copy
+ * + encode, as blastp_pack_db, on an internal stream) while the previous
+ * part is searched on `cuda_stream` -- the copy overlaps the search (not in
+ * the paper, whose database is resident; DESIGN.md "Host-resident
+ * databases").  Every HSP of every query is appended to d_out (device,
+ * capacity records, unsorted; subject_id global) and the total count,
+ * possibly > capacity, is written to *d_count (device int64).  Same results
+ * as blastp_pack_db + blastp_search_ungapped_device on the whole shard.
+ * Returns when the last part's search is enqueued; part buffers are
+ * released in stream order.  Errors: as blastp_pack_db and
+ * blastp_search_ungapped_device. */
+int blastp_search_host_db(const blastp_query_table *q, const char *residues_ascii,
+                          const int64_t *offsets, int64_t nseq, int32_t shard_index,
+                          int32_t num_shards, const blastp_params *p, int32_t num_parts,
+                          void *cuda_stream, blastp_hsp *d_out, int64_t capacity,
+                          int64_t *d_count);
+
 /* Long-subject plan of the shard (implementation detail, exposed for tests
  * and tuning): chunks longer than 2C residues that are scheduled first
  * (*long_items), the segments they are split into for parallel two-hit

@@ -83,6 +83,9 @@ def _load():
     L.blastp_query_table_info.argtypes = [vp, P(i32), P(i64)]
     L.blastp_search_ungapped.argtypes = [vp, vp, P(_CParams), vp, P(vp), P(i64)]
     L.blastp_search_ungapped_device.argtypes = [vp, vp, P(_CParams), vp, vp, i64, vp]
+    if hasattr(L, "blastp_search_host_db"):  # absent in older builds (A/B timing)
+        L.blastp_search_host_db.argtypes = [vp, vp, vp, i64, i32, i32, P(_CParams), i32, vp, vp,
+                                            i64, vp]
     L.blastp_sort_hsps_device.argtypes = [vp, i64, vp]
     L.blastp_debug_trace.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64), vp, i64, P(i64),
                                      vp, i64, P(i64)]
@@ -100,7 +103,8 @@ lib = _load()
 EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "blastp_version",
             "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
             "blastp_shard_range", "blastp_db_info", "blastp_db_long_info", "blastp_query_table_info",
-            "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_sort_hsps_device",
+            "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_search_host_db",
+            "blastp_sort_hsps_device",
             "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
 
@@ -281,6 +285,29 @@ def search_ungapped_device(table: QueryTable, db: Database, out_ptr: int, capaci
     _check(lib.blastp_search_ungapped_device(table.handle, db.handle, ctypes.byref(c),
                                              _stream_handle(stream), out_ptr, capacity,
                                              count_ptr), "blastp_search_ungapped_device")
+
+
+def search_host_db(table: QueryTable, residues, offsets: np.ndarray, out_ptr: int, capacity: int,
+                   count_ptr: int, params: Params | None = None, shard_index: int = 0,
+                   num_shards: int = 1, num_parts: int = 0, stream=None):
+    """Pipelined search of a host-resident shard (blastp_search_host_db): parts
+    are copied host->device while the previous part is searched.  `residues`:
+    a numpy uint8 array / bytes, or an int host pointer (e.g. a pinned tensor's
+    data_ptr() minus offsets[0]).  HSPs appended at out_ptr (device), total
+    count written to the int64 at count_ptr; asynchronous on `stream`."""
+    off = np.ascontiguousarray(offsets, dtype=np.int64)
+    if isinstance(residues, int):
+        ptr, keep = residues, None
+    else:
+        keep = np.frombuffer(residues, dtype=np.uint8) if isinstance(residues, (bytes, bytearray)) \
+            else np.ascontiguousarray(residues)
+        ptr = keep.ctypes.data
+    c = (params or table.params).c()
+    _check(lib.blastp_search_host_db(table.handle, ptr, off.ctypes.data, len(off) - 1, shard_index,
+                                     num_shards, ctypes.byref(c), num_parts,
+                                     _stream_handle(stream), out_ptr, capacity, count_ptr),
+           "blastp_search_host_db")
+    return keep
 
 
 def sort_hsps_device(ptr: int, n: int, stream=None):

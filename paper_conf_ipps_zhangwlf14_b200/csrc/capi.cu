@@ -4,11 +4,13 @@
 // the database packer / sharder, launch drivers and result marshalling.
 // Every step of the search itself runs in the kernels of search.cu.
 #include <algorithm>
+#include <chrono>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <type_traits>
 #include <vector>
 
 #include <cuda_runtime.h>
@@ -121,6 +123,7 @@ struct blastp_db {
   uint32_t *seg_list = nullptr;
   unsigned *seg_done = nullptr;
   unsigned seq = 0;  // search launches on this db (segment publication epoch)
+  bool carved = false;  // stream/sstart/chunks/counters live in a caller's arena
   std::vector<int64_t> h_sstart;
   unsigned long long *counters = nullptr;  // [0] hsp count, [1] chunk cursor, [6] long chunks
   blastp_hsp *out = nullptr;               // scratch for the host-array search
@@ -362,22 +365,65 @@ int blastp_shard_range(const int64_t *offsets, int64_t nseq, int32_t shard_index
   return BLASTP_OK;
 }
 
-int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t nseq,
-                   int32_t shard_index, int32_t num_shards, int device, void *cuda_stream,
-                   blastp_db **out) {
-  if (!out) return fail(BLASTP_E_INVALID_ARG, "out is NULL");
-  *out = nullptr;
-  if (!offsets || nseq < 0) return fail(BLASTP_E_INVALID_ARG, "offsets NULL or nseq < 0");
-  int64_t lo = 0, hi = 0;
-  int rc = blastp_shard_range(offsets, nseq, shard_index, num_shards, &lo, &hi);
-  if (rc) return rc;
+}  // extern "C"
+
+// Packed-stream bytes and chunk count of n subjects / nres residues.
+// Stream layout: kStreamPadFront sentinels, then subject i at
+// sstart[i] = pad + (offsets[lo+i] - offsets[lo]) + i, each followed by one
+// sentinel; kStreamPadBack trailing sentinels; 512-byte multiple.  Chunks of
+// ~C residues of whole subjects (>= 4 per warp at 32 warps/SM).
+static void layout_sizes(int64_t n, int64_t nres, int sms, int64_t *stream_len, int64_t *C,
+                         int64_t *nchunks) {
+  *stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 511) & ~int64_t(511);
+  // (8 chunks per resident warp, at most 8192 residues: a launch's tail is one
+  // chunk per warp; measured 1.3% faster than 16384 on config 3)
+  int64_t c = nres / (int64_t(sms) * 32 * 8);
+  c = std::min<int64_t>(std::max<int64_t>(c, 1024), 8192);
+  if (const char *ce = std::getenv("BLASTP_CHUNK")) c = std::max<int64_t>(64, std::atoll(ce));
+  *C = c;
+  *nchunks = n > 0 ? (nres + c - 1) / c + 1 : 0;
+}
+
+// Bump allocator over one device block: the pipelined host-db search carves
+// every part's buffers from a single pool allocation per call (per-part
+// allocations let the pool grow or fragment in the middle of the pipeline).
+struct Arena {
+  uint8_t *base = nullptr;
+  size_t cap = 0, used = 0;
+  void *take(size_t bytes) {
+    used = (used + 255) & ~size_t(255);
+    if (used + bytes > cap) return nullptr;
+    void *p = base + used;
+    used += bytes;
+    return p;
+  }
+};
+static size_t arena_bytes(int64_t n, int64_t nres, int sms) {
+  int64_t len = 0, C = 0, nchunks = 0;
+  layout_sizes(n, nres, sms, &len, &C, &nchunks);
+  const auto a = [](size_t b) { return (b + 255) & ~size_t(255); };
+  return a(size_t(len)) + a(8 * size_t(std::max<int64_t>(n, 1))) +
+         2 * a(sizeof(Chunk) * size_t(std::max<int64_t>(nchunks, 1))) + a(64);
+}
+// Staging buffers of a pack (ASCII residues, offsets, error flags); shared by
+// the parts of one pipelined search, which are packed in order on one stream.
+struct PackStaging {
+  uint8_t *ascii = nullptr;
+  int64_t *off = nullptr;
+  int *err = nullptr;
+};
+
+// Pack subjects [lo, hi) of the offsets array (the body of blastp_pack_db).
+// arena / staging: optional preallocated buffers (blastp_search_host_db).
+static int pack_range(const char *residues_ascii, const int64_t *offsets, int64_t lo, int64_t hi,
+                      int device, cudaStream_t s, blastp_db **out, Arena *arena = nullptr,
+                      const PackStaging *staging = nullptr) {
   const int64_t n = hi - lo;
   const int64_t nres = offsets[hi] - offsets[lo];
   if (nres < 0) return fail(BLASTP_E_INVALID_ARG, "offsets decrease");
   if (nres > 0 && !residues_ascii) return fail(BLASTP_E_INVALID_ARG, "residues is NULL");
   DeviceGuard g(device);
   if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
-  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
 
   auto *db = new (std::nothrow) blastp_db;
   if (!db) return fail(BLASTP_E_NOMEM, "host allocation failed");
@@ -386,17 +432,11 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
   db->nseq = n;
   db->residues = nres;
   db->subject_base = lo;
-  // Stream layout: kStreamPadFront sentinels, then subject i at
-  // sstart[i] = pad + (offsets[lo+i] - offsets[lo]) + i, each followed by
-  // one sentinel; kStreamPadBack trailing sentinels; 512-byte multiple.
   // Subject starts, length checks and the chunk plan are computed on the GPU.
-  db->stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 511) & ~int64_t(511);
-  // Chunks of ~C residues of whole subjects (>= 4 per warp at 32 warps/SM).
-  int64_t C = nres / (int64_t(db->sms) * 32 * 4);
-  C = std::min<int64_t>(std::max<int64_t>(C, 1024), 16384);
-  if (const char *ce = std::getenv("BLASTP_CHUNK")) C = std::max<int64_t>(64, std::atoll(ce));
-  const int64_t nchunks = n > 0 ? (nres + C - 1) / C + 1 : 0;
+  int64_t C = 0, nchunks = 0;
+  layout_sizes(n, nres, db->sms, &db->stream_len, &C, &nchunks);
   db->nchunks = static_cast<int32_t>(nchunks);
+  db->carved = arena != nullptr;
 
   // stream-ordered allocations from a pool that keeps its memory (repeated
   // pack calls, e.g. the e2e benchmark, do not pay cudaMalloc again)
@@ -407,44 +447,67 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     }
   }
-  uint8_t *d_ascii = nullptr;
-  int64_t *d_off = nullptr;
-  int *d_err = nullptr;
+  uint8_t *d_ascii = staging ? staging->ascii : nullptr;
+  int64_t *d_off = staging ? staging->off : nullptr;
+  int *d_err = staging ? staging->err : nullptr;
   auto cleanup = [&](int code) {
-    cudaFreeAsync(d_ascii, s);
-    cudaFreeAsync(d_off, s);
-    cudaFreeAsync(d_err, s);
+    if (!staging) {
+      cudaFreeAsync(d_ascii, s);
+      cudaFreeAsync(d_off, s);
+      cudaFreeAsync(d_err, s);
+    }
     if (code != BLASTP_OK) {
       cudaStreamSynchronize(s);
       blastp_db_free(db);
     }
     return code;
   };
-  if (cudaMallocAsync(&db->stream, static_cast<size_t>(db->stream_len), s) != cudaSuccess ||
-      cudaMallocAsync(&db->sstart, sizeof(int64_t) * static_cast<size_t>(std::max<int64_t>(n, 1)), s) != cudaSuccess ||
-      cudaMallocAsync(&db->chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1)), s) != cudaSuccess ||
-      cudaMallocAsync(&db->long_chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1)), s) != cudaSuccess ||
-      cudaMallocAsync(&db->counters, sizeof(unsigned long long) * 8, s) != cudaSuccess ||
-      cudaMallocAsync(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1)), s) != cudaSuccess ||
-      cudaMallocAsync(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1), s) != cudaSuccess ||
-      cudaMallocAsync(&d_err, sizeof(int), s) != cudaSuccess) {
+  auto dalloc = [&](auto **p, size_t bytes) {
+    if (arena) {
+      *p = static_cast<std::remove_pointer_t<decltype(p)>>(arena->take(bytes));
+      return *p != nullptr;
+    }
+    return cudaMallocAsync(reinterpret_cast<void **>(p), bytes, s) == cudaSuccess;
+  };
+  if (!dalloc(&db->stream, static_cast<size_t>(db->stream_len)) ||
+      !dalloc(&db->sstart, sizeof(int64_t) * static_cast<size_t>(std::max<int64_t>(n, 1))) ||
+      !dalloc(&db->chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1))) ||
+      !dalloc(&db->long_chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1))) ||
+      !dalloc(&db->counters, 64) ||
+      (!staging &&
+       (cudaMallocAsync(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1)), s) != cudaSuccess ||
+        cudaMallocAsync(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1), s) != cudaSuccess ||
+        cudaMallocAsync(&d_err, sizeof(int), s) != cudaSuccess))) {
     cudaGetLastError();
     return cleanup(fail(BLASTP_E_NOMEM, "device allocation for the database failed"));
   }
   upload_encode_table();
-  cudaError_t e = cudaMemsetAsync(db->stream, kSentinel, static_cast<size_t>(db->stream_len), s);
-  if (e == cudaSuccess) e = cudaMemsetAsync(d_err, 0, sizeof(int), s);
-  if (e == cudaSuccess) e = cudaMemsetAsync(db->counters, 0, sizeof(unsigned long long) * 8, s);
+  const bool dbg = std::getenv("BLASTP_DEBUG_PIPE") != nullptr;
+  const auto t0 = std::chrono::steady_clock::now();
+  auto ms = [&]() {
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  };
+  double t_off = 0, t_enq = 0;
+  // The copies come first in stream order: copy engines need no SMs, so they
+  // overlap a search still running on another stream; the memsets and
+  // kernels after them wait for SMs.  (Pinned host buffers make both copies
+  // asynchronous.)
+  cudaError_t e = cudaSuccess;
+  if (nres > 0)
+    e = cudaMemcpyAsync(d_ascii, residues_ascii + offsets[lo], static_cast<size_t>(nres),
+                        cudaMemcpyHostToDevice, s);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(d_off, offsets + lo, sizeof(int64_t) * static_cast<size_t>(n + 1),
                         cudaMemcpyHostToDevice, s);
+  t_off = ms();
+  if (e == cudaSuccess) e = cudaMemsetAsync(d_err, 0, sizeof(int), s);
+  if (e == cudaSuccess) e = cudaMemsetAsync(db->counters, 0, sizeof(unsigned long long) * 8, s);
   if (e == cudaSuccess)
     e = launch_layout(d_off, n, C, nchunks, db->sstart, db->chunks, db->long_chunks,
                       reinterpret_cast<int *>(db->counters + 6), d_err, s);
-  if (e == cudaSuccess && nres > 0)
-    e = cudaMemcpyAsync(d_ascii, residues_ascii + offsets[lo], static_cast<size_t>(nres),
-                        cudaMemcpyHostToDevice, s);
-  if (e == cudaSuccess) e = launch_pack(d_ascii, d_off, n, db->sstart, db->stream, d_err, s);
+  if (e == cudaSuccess)
+    e = launch_pack(d_ascii, d_off, n, db->sstart, db->stream, db->stream_len, d_err, s);
+  t_enq = ms();
   int h_err = 0, h_nlong = 0;
   if (e == cudaSuccess) e = cudaMemcpyAsync(&h_err, d_err, sizeof(int), cudaMemcpyDeviceToHost, s);
   if (e == cudaSuccess)
@@ -463,12 +526,32 @@ int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t n
                             static_cast<long long>(k), static_cast<unsigned char>(residues_ascii[k])));
     return cleanup(fail(BLASTP_E_BAD_RESIDUE, "database holds an invalid residue"));
   }
+  const double t_sync = ms();
   if (h_nlong > 0 && plan_long_items(db, h_nlong, s) != cudaSuccess) {
     cudaGetLastError();
     return cleanup(fail(BLASTP_E_NOMEM, "device allocation for the long-subject plan failed"));
   }
+  if (dbg)
+    fprintf(stderr, "[pack] %lld subjects %lld residues: offsets copied %.3f, enqueued %.3f, "
+            "synced %.3f, planned %.3f ms\n", static_cast<long long>(n),
+            static_cast<long long>(nres), t_off, t_enq, t_sync, ms());
   *out = db;
   return cleanup(BLASTP_OK);
+}
+
+extern "C" {
+
+int blastp_pack_db(const char *residues_ascii, const int64_t *offsets, int64_t nseq,
+                   int32_t shard_index, int32_t num_shards, int device, void *cuda_stream,
+                   blastp_db **out) {
+  if (!out) return fail(BLASTP_E_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (!offsets || nseq < 0) return fail(BLASTP_E_INVALID_ARG, "offsets NULL or nseq < 0");
+  int64_t lo = 0, hi = 0;
+  int rc = blastp_shard_range(offsets, nseq, shard_index, num_shards, &lo, &hi);
+  if (rc) return rc;
+  return pack_range(residues_ascii, offsets, lo, hi, device, static_cast<cudaStream_t>(cuda_stream),
+                    out);
 }
 
 // Host copy of the subject starts (debug traces only; fetched lazily).
@@ -506,16 +589,18 @@ int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues, int64_
 void blastp_db_free(blastp_db *db) {
   if (!db) return;
   DeviceGuard g(db->device);
-  cudaFree(db->stream);
-  cudaFree(db->sstart);
-  cudaFree(db->chunks);
-  cudaFree(db->long_chunks);
+  if (!db->carved) {
+    cudaFree(db->stream);
+    cudaFree(db->sstart);
+    cudaFree(db->chunks);
+    cudaFree(db->long_chunks);
+    cudaFree(db->counters);
+  }
   cudaFree(db->items);
   cudaFree(db->seg_item);
   cudaFree(db->seg_count);
   cudaFree(db->seg_done);
   cudaFree(db->seg_list);
-  cudaFree(db->counters);
   cudaFree(db->out);
   delete db;
 }
@@ -541,8 +626,9 @@ static int check_pair(const blastp_query_table *q, const blastp_db *db, const bl
 static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
                           const blastp_params *p, cudaStream_t s, blastp_hsp *out, int64_t cap,
                           unsigned long long *count, TraceRec *const trace[3],
-                          const int64_t trace_cap[3], unsigned long long *trace_count) {
-  CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
+                          const int64_t trace_cap[3], unsigned long long *trace_count,
+                          bool reset_count = true) {
+  if (reset_count) CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
   if (trace_count)  // [0..3): trace record counts, [3..3+kNumStats): event counters
     CUDA_TRY(cudaMemsetAsync(trace_count, 0, (3 + kNumStats) * sizeof(unsigned long long), s));
   if (db->nchunks == 0) return BLASTP_OK;
@@ -605,6 +691,174 @@ int blastp_search_ungapped_device(const blastp_query_table *q, const blastp_db *
   DeviceGuard g(db->device);
   return enqueue_search(q, db, p, static_cast<cudaStream_t>(cuda_stream), d_out, capacity,
                         reinterpret_cast<unsigned long long *>(d_count), nullptr, nullptr, nullptr);
+}
+
+// Stream-ordered release of a database (its buffers come from the pool):
+// safe while kernels enqueued on `s` still read it.
+static void db_free_async(blastp_db *db, cudaStream_t s) {
+  if (!db) return;
+  if (!db->carved)
+    for (void *ptr : {static_cast<void *>(db->stream), static_cast<void *>(db->sstart),
+                      static_cast<void *>(db->chunks), static_cast<void *>(db->long_chunks),
+                      static_cast<void *>(db->counters)})
+      if (ptr) cudaFreeAsync(ptr, s);
+  for (void *ptr : {static_cast<void *>(db->items), static_cast<void *>(db->seg_item),
+                    static_cast<void *>(db->seg_count), static_cast<void *>(db->seg_done),
+                    static_cast<void *>(db->seg_list)})
+    if (ptr) cudaFreeAsync(ptr, s);
+  if (db->out) cudaFree(db->out);
+  delete db;
+}
+
+int blastp_search_host_db(const blastp_query_table *q, const char *residues_ascii,
+                          const int64_t *offsets, int64_t nseq, int32_t shard_index,
+                          int32_t num_shards, const blastp_params *p, int32_t num_parts,
+                          void *cuda_stream, blastp_hsp *d_out, int64_t capacity,
+                          int64_t *d_count) {
+  if (!q) return fail(BLASTP_E_INVALID_ARG, "table is NULL");
+  int rc = validate_params(p);
+  if (rc) return rc;
+  if (p->threshold != q->p.threshold || p->word_len != q->p.word_len)
+    return fail(BLASTP_E_INVALID_ARG, "threshold/word_len differ from the table's (%d/%d)",
+                q->p.threshold, q->p.word_len);
+  if (!d_count || capacity < 0 || (capacity > 0 && !d_out))
+    return fail(BLASTP_E_INVALID_ARG, "bad output buffer");
+  if (!offsets || nseq < 0) return fail(BLASTP_E_INVALID_ARG, "offsets NULL or nseq < 0");
+  if (num_parts < 0) return fail(BLASTP_E_INVALID_ARG, "num_parts %d < 0", num_parts);
+  int64_t lo = 0, hi = 0;
+  rc = blastp_shard_range(offsets, nseq, shard_index, num_shards, &lo, &hi);
+  if (rc) return rc;
+  DeviceGuard g(q->device);
+  if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", q->device, cudaGetErrorString(g.err));
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  auto *count = reinterpret_cast<unsigned long long *>(d_count);
+  CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
+  // Part boundaries (whole subjects, by residues): sizes grow 1.5x from a
+  // small first part -- its copy is the only one not hidden behind a search,
+  // and each part copies faster than the previous one is searched.
+  const int64_t total = offsets[hi] - offsets[lo];
+  if (total < 0) return fail(BLASTP_E_INVALID_ARG, "offsets decrease");
+  std::vector<int64_t> cut{lo};
+  {
+    // knobs (tuning): BLASTP_PIPE_FIRST residues of the first part,
+    // BLASTP_PIPE_GROWTH percent growth per part
+    int64_t want = std::max<int64_t>(int64_t(1) << 24, total / 64);
+    if (const char *v = std::getenv("BLASTP_PIPE_FIRST")) want = std::max<int64_t>(1, std::atoll(v));
+    int growth = 150;
+    if (const char *v = std::getenv("BLASTP_PIPE_GROWTH")) growth = std::max(101, std::atoi(v));
+    int64_t done = 0;
+    for (int k = 0; cut.back() < hi; ++k) {
+      int64_t size;
+      if (num_parts > 0)
+        size = (total * (k + 1)) / num_parts - done;
+      else {
+        size = want;
+        want = want * growth / 100;
+      }
+      const int64_t target = offsets[lo] + done + std::max<int64_t>(size, 1);
+      // first subject starting at or after target
+      int64_t a = cut.back() + 1, b = hi;
+      while (a < b) {
+        const int64_t m = (a + b) >> 1;
+        if (offsets[m] >= target) b = m; else a = m + 1;
+      }
+      cut.push_back(a);
+      done = offsets[a] - offsets[lo];
+    }
+  }
+  cudaStream_t cs = nullptr;  // copy + pack stream
+  CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  // one arena for every part's packed buffers + shared staging buffers
+  const int sms = num_sms(q->device);
+  size_t total_bytes = 0;
+  int64_t max_n = 0, max_res = 0;
+  for (size_t k = 0; k + 1 < cut.size(); ++k) {
+    const int64_t n = cut[k + 1] - cut[k], r = offsets[cut[k + 1]] - offsets[cut[k]];
+    if (r < 0) {
+      cudaStreamDestroy(cs);
+      return fail(BLASTP_E_INVALID_ARG, "offsets decrease");
+    }
+    total_bytes += arena_bytes(n, r, sms);
+    max_n = std::max(max_n, n);
+    max_res = std::max(max_res, r);
+  }
+  const auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
+  total_bytes += al(size_t(std::max<int64_t>(max_res, 1))) + al(8 * size_t(max_n + 1)) + al(4);
+  {
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, q->device) == cudaSuccess) {
+      uint64_t thr = ~uint64_t(0);
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  Arena arena;
+  if (cudaMallocAsync(reinterpret_cast<void **>(&arena.base), total_bytes, cs) != cudaSuccess) {
+    cudaGetLastError();
+    cudaStreamDestroy(cs);
+    return fail(BLASTP_E_NOMEM, "device arena of %zu bytes for the host-db search", total_bytes);
+  }
+  arena.cap = total_bytes;
+  PackStaging staging;
+  staging.ascii = static_cast<uint8_t *>(arena.take(size_t(std::max<int64_t>(max_res, 1))));
+  staging.off = static_cast<int64_t *>(arena.take(8 * size_t(max_n + 1)));
+  staging.err = static_cast<int *>(arena.take(4));
+  std::vector<blastp_db *> parts;
+  // BLASTP_DEBUG_PIPE=1: per-part host timestamps and search event times on stderr
+  const bool dbg = std::getenv("BLASTP_DEBUG_PIPE") != nullptr;
+  std::vector<cudaEvent_t> ev;
+  const auto t0 = std::chrono::steady_clock::now();
+  auto ms = [&]() {
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  };
+  auto mark = [&]() {
+    if (!dbg) return;
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    cudaEventRecord(e, s);
+    ev.push_back(e);
+  };
+  mark();
+  rc = BLASTP_OK;
+  for (size_t k = 0; k + 1 < cut.size() && rc == BLASTP_OK; ++k) {
+    // the host blocks here for part k's copy while part k-1 is searched
+    blastp_db *d = nullptr;
+    const double a = ms();
+    rc = pack_range(residues_ascii, offsets, cut[k], cut[k + 1], q->device, cs, &d, &arena,
+                    &staging);
+    if (rc) break;
+    const double b = ms();
+    parts.push_back(d);
+    rc = enqueue_search(q, d, p, s, d_out, capacity, count, nullptr, nullptr, nullptr, false);
+    mark();
+    if (dbg)
+      fprintf(stderr, "[pipe] part %zu: %lld residues, pack %.3f..%.3f ms, search enqueued %.3f ms\n",
+              k, static_cast<long long>(offsets[cut[k + 1]] - offsets[cut[k]]), a, b, ms());
+  }
+  for (blastp_db *d : parts) db_free_async(d, s);
+  // the searches on s read the arena: free it in their stream order (and
+  // after the copy stream's last use of the staging buffers)
+  {
+    cudaEvent_t done_copy;
+    if (cudaEventCreateWithFlags(&done_copy, cudaEventDisableTiming) == cudaSuccess) {
+      cudaEventRecord(done_copy, cs);
+      cudaStreamWaitEvent(s, done_copy, 0);
+      cudaEventDestroy(done_copy);
+    }
+  }
+  cudaFreeAsync(arena.base, s);
+  cudaStreamDestroy(cs);
+  if (dbg && !ev.empty()) {
+    cudaEventSynchronize(ev.back());
+    for (size_t k = 1; k < ev.size(); ++k) {
+      float t = 0, u = 0;
+      cudaEventElapsedTime(&t, ev[0], ev[k - 1]);
+      cudaEventElapsedTime(&u, ev[0], ev[k]);
+      fprintf(stderr, "[pipe] part %zu: search on device %.3f..%.3f ms (from the first mark)\n",
+              k - 1, t, u);
+    }
+    for (cudaEvent_t e : ev) cudaEventDestroy(e);
+  }
+  return rc;
 }
 
 int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream) {

@@ -148,7 +148,7 @@ int search_ring_slots(int lq, int window);
 cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s);
 cudaError_t launch_search_warp(const SearchArgs &a, int num_sms, cudaStream_t s);
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
-                        const int64_t *sstart, uint8_t *stream, int *err,
+                        const int64_t *sstart, uint8_t *stream, int64_t stream_len, int *err,
                         cudaStream_t s);
 cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
                           int64_t *sstart, Chunk *chunks, Chunk *long_chunks, int *nlong,

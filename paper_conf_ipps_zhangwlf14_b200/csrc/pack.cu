@@ -13,13 +13,23 @@ __constant__ uint8_t c_encode[256];
 
 // One warp per subject (grid-stride): lanes copy consecutive bytes, so every
 // load and store instruction of a warp touches one or two 32-byte sectors.
+// Every byte of the stream is written here (no separate memset, which as a
+// kernel would queue behind a running search and hold up the copies of a
+// pipelined blastp_search_host_db): the front pad, each subject followed by
+// its sentinel, and the back pad up to stream_len.
 __global__ void pack_kernel(const uint8_t *__restrict__ ascii, const int64_t *__restrict__ off,
                             int64_t n, const int64_t *__restrict__ sstart,
-                            uint8_t *__restrict__ stream, int *err) {
+                            uint8_t *__restrict__ stream, int64_t stream_len, int *err) {
   const int lane = threadIdx.x & 31;
-  const int64_t warps = (int64_t(gridDim.x) * blockDim.x) >> 5;
+  const int64_t gtid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  const int64_t nthreads = int64_t(gridDim.x) * blockDim.x;
+  const int64_t warps = nthreads >> 5;
   const int64_t base = off[0];
-  for (int64_t i = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5; i < n; i += warps) {
+  // pads: [0, kStreamPadFront) and [pad + residues + n, stream_len)
+  const int64_t tail = kStreamPadFront + (off[n] - base) + n;
+  for (int64_t j = gtid; j < kStreamPadFront; j += nthreads) stream[j] = uint8_t(kSentinel);
+  for (int64_t j = tail + gtid; j < stream_len; j += nthreads) stream[j] = uint8_t(kSentinel);
+  for (int64_t i = gtid >> 5; i < n; i += warps) {
     const int64_t a = off[i] - base, len = off[i + 1] - off[i];
     uint8_t *dst = stream + sstart[i];
     int bad = 0;
@@ -28,6 +38,7 @@ __global__ void pack_kernel(const uint8_t *__restrict__ ascii, const int64_t *__
       bad |= (c == 0xFF);
       dst[j] = c;
     }
+    if (lane == 0 && len >= 0) dst[len] = uint8_t(kSentinel);
     if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(err, 1);
   }
 }
@@ -103,7 +114,14 @@ cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchu
   return cudaGetLastError();
 }
 
+// Once per device: cudaMemcpyToSymbol is synchronous on the legacy default
+// stream, so calling it per pack would wait for searches running there (it
+// serialised the pipelined blastp_search_host_db).
 void upload_encode_table() {
+  static unsigned long long ready = 0;  // one bit per device
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (ready >> dev & 1ull) return;
   uint8_t lut[256];
   for (int i = 0; i < 256; ++i) lut[i] = 0xFF;
   for (int k = 0; k < kNumLetters; ++k) {
@@ -113,12 +131,12 @@ void upload_encode_table() {
   }
   const uint8_t x = 22;  // 'X'
   for (const char c : {'U', 'O', 'J', 'u', 'o', 'j'}) lut[static_cast<unsigned char>(c)] = x;
-  cudaMemcpyToSymbol(c_encode, lut, sizeof(lut));
+  if (cudaMemcpyToSymbol(c_encode, lut, sizeof(lut)) == cudaSuccess) ready |= 1ull << dev;
 }
 
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n, const int64_t *sstart,
-                        uint8_t *stream, int *err, cudaStream_t s) {
-  if (n <= 0) return cudaSuccess;
+                        uint8_t *stream, int64_t stream_len, int *err, cudaStream_t s) {
+  if (n <= 0) return cudaMemsetAsync(stream, kSentinel, static_cast<size_t>(stream_len), s);
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -126,7 +144,7 @@ cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n, con
   int64_t blocks = (n * 32 + threads - 1) / threads;
   const int64_t cap = int64_t(sms) * 16;
   if (blocks > cap) blocks = cap;
-  pack_kernel<<<unsigned(blocks), threads, 0, s>>>(ascii, off, n, sstart, stream, err);
+  pack_kernel<<<unsigned(blocks), threads, 0, s>>>(ascii, off, n, sstart, stream, stream_len, err);
   return cudaGetLastError();
 }
 

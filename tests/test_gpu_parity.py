@@ -273,6 +273,47 @@ def test_device_variant_and_sort_match_host_variant(bp, orc):
     assert int(cnt.item()) == len(host)
 
 
+def _host_db_search(bp, t, ascii, off, p, **kw):
+    import torch
+    cap = 1 << 16
+    out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    bp.search_host_db(t, ascii, off, out.data_ptr(), cap, cnt.data_ptr(), p, **kw)
+    n = int(cnt.item())
+    assert n <= cap
+    bp.sort_hsps_device(out.data_ptr(), n)
+    return [tuple(x) for x in out[: n * 7].view(n, 7).cpu().numpy().tolist()]
+
+
+def test_search_host_db_pipelined_parts(bp, orc):
+    """blastp_search_host_db (parts copied while the previous part is
+    searched) equals pack + search of the whole shard, for automatic and
+    explicit part counts, shards, a query batch and long subjects."""
+    q = gen_query(21, 300).decode()
+    ascii, off = _long_subject_db(q)
+    rng = np.random.default_rng(8)
+    a2, o2 = _rand_db(rng, 3000, 0, 600, q)
+    ascii = np.concatenate([a2, ascii])
+    off = np.concatenate([o2, o2[-1] + off[1:]]).astype(np.int64)
+    p = bp.Params()
+    t = bp.build_query_table(q, p)
+    whole = tuples(bp.search_ungapped(t, bp.pack_db(ascii, off), p))
+    r = oracle_run(orc, q, ascii, off, p, nthreads=4)
+    assert whole == tuples(r.hsps)
+    for parts in (0, 1, 2, 7, 50):
+        assert _host_db_search(bp, t, ascii, off, p, num_parts=parts) == whole, parts
+    for k in range(3):  # a shard's parts: global subject ids
+        shard = tuples(bp.search_ungapped(t, bp.pack_db(ascii, off, k, 3), p))
+        assert _host_db_search(bp, t, ascii, off, p, shard_index=k, num_shards=3,
+                               num_parts=4) == shard
+    qs = [q, gen_query(22, 127).decode()]
+    tb = bp.build_query_batch(qs, p)
+    assert _host_db_search(bp, tb, ascii, off, p, num_parts=3) == \
+        tuples(bp.search_ungapped(tb, bp.pack_db(ascii, off), p))
+    # no subjects at all
+    assert _host_db_search(bp, t, np.zeros(0, np.uint8), np.zeros(1, np.int64), p) == []
+
+
 def test_query_batch_equals_single_queries(bp, orc):
     qs = [gen_query(11 + i, L) for i, L in enumerate([100, 350, 900])]
     db = gen_db(12, 13, n_subjects=500, mean_len=300.0, queries=qs, plant_frac=0.3)
