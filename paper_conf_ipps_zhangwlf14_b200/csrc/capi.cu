@@ -367,21 +367,27 @@ int blastp_shard_range(const int64_t *offsets, int64_t nseq, int32_t shard_index
 
 }  // extern "C"
 
-// Packed-stream bytes and chunk count of n subjects / nres residues.
+// Packed-stream bytes and chunk plan of n subjects / nres residues.
 // Stream layout: kStreamPadFront sentinels, then subject i at
 // sstart[i] = pad + (offsets[lo+i] - offsets[lo]) + i, each followed by one
 // sentinel; kStreamPadBack trailing sentinels; 512-byte multiple.  Chunks of
-// ~C residues of whole subjects (>= 4 per warp at 32 warps/SM).
-static void layout_sizes(int64_t n, int64_t nres, int sms, int64_t *stream_len, int64_t *C,
-                         int64_t *nchunks) {
+// C residues of whole subjects (8 per resident warp, at most 8192: measured
+// 1.3% faster than 16384 on config 3), the last 2 C per resident warp in
+// chunks of C/4 (ChunkPlan).
+static void layout_sizes(int64_t n, int64_t nres, int sms, int64_t *stream_len, ChunkPlan *plan) {
   *stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 511) & ~int64_t(511);
-  // (8 chunks per resident warp, at most 8192 residues: a launch's tail is one
-  // chunk per warp; measured 1.3% faster than 16384 on config 3)
-  int64_t c = nres / (int64_t(sms) * 32 * 8);
+  const int64_t warps = int64_t(sms) * 32;
+  int64_t c = nres / (warps * 8);
   c = std::min<int64_t>(std::max<int64_t>(c, 1024), 8192);
   if (const char *ce = std::getenv("BLASTP_CHUNK")) c = std::max<int64_t>(64, std::atoll(ce));
-  *C = c;
-  *nchunks = n > 0 ? (nres + c - 1) / c + 1 : 0;
+  plan->C = c;
+  plan->Ct = std::min<int64_t>(c, std::max<int64_t>(1024, c / 4));
+  if (const char *v = std::getenv("BLASTP_TAIL_CHUNKS")) {  // knob: 0 = uniform chunks
+    if (std::atoi(v) == 0) plan->Ct = c;
+  }
+  plan->K1 = std::max<int64_t>(0, nres - 2 * warps * c) / c;
+  const int64_t rest = nres - plan->K1 * c;
+  plan->nchunks = n > 0 ? plan->K1 + (rest + plan->Ct - 1) / plan->Ct + 1 : 0;
 }
 
 // Bump allocator over one device block: the pipelined host-db search carves
@@ -399,8 +405,10 @@ struct Arena {
   }
 };
 static size_t arena_bytes(int64_t n, int64_t nres, int sms) {
-  int64_t len = 0, C = 0, nchunks = 0;
-  layout_sizes(n, nres, sms, &len, &C, &nchunks);
+  int64_t len = 0;
+  ChunkPlan plan{};
+  layout_sizes(n, nres, sms, &len, &plan);
+  const int64_t nchunks = plan.nchunks;
   const auto a = [](size_t b) { return (b + 255) & ~size_t(255); };
   return a(size_t(len)) + a(8 * size_t(std::max<int64_t>(n, 1))) +
          2 * a(sizeof(Chunk) * size_t(std::max<int64_t>(nchunks, 1))) + a(64);
@@ -433,8 +441,9 @@ static int pack_range(const char *residues_ascii, const int64_t *offsets, int64_
   db->residues = nres;
   db->subject_base = lo;
   // Subject starts, length checks and the chunk plan are computed on the GPU.
-  int64_t C = 0, nchunks = 0;
-  layout_sizes(n, nres, db->sms, &db->stream_len, &C, &nchunks);
+  ChunkPlan plan{};
+  layout_sizes(n, nres, db->sms, &db->stream_len, &plan);
+  const int64_t nchunks = plan.nchunks;
   db->nchunks = static_cast<int32_t>(nchunks);
   db->carved = arena != nullptr;
 
@@ -503,7 +512,7 @@ static int pack_range(const char *residues_ascii, const int64_t *offsets, int64_
   if (e == cudaSuccess) e = cudaMemsetAsync(d_err, 0, sizeof(int), s);
   if (e == cudaSuccess) e = cudaMemsetAsync(db->counters, 0, sizeof(unsigned long long) * 8, s);
   if (e == cudaSuccess)
-    e = launch_layout(d_off, n, C, nchunks, db->sstart, db->chunks, db->long_chunks,
+    e = launch_layout(d_off, n, plan, db->sstart, db->chunks, db->long_chunks,
                       reinterpret_cast<int *>(db->counters + 6), d_err, s);
   if (e == cudaSuccess)
     e = launch_pack(d_ascii, d_off, n, db->sstart, db->stream, db->stream_len, d_err, s);

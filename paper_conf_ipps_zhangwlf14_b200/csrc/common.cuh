@@ -150,9 +150,20 @@ cudaError_t launch_search_warp(const SearchArgs &a, int num_sms, cudaStream_t s)
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
                         const int64_t *sstart, uint8_t *stream, int64_t stream_len, int *err,
                         cudaStream_t s);
-cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
-                          int64_t *sstart, Chunk *chunks, Chunk *long_chunks, int *nlong,
-                          int *err, cudaStream_t s);
+// Chunk plan: chunk k covers the subjects whose first residue lies in
+// [target(k), target(k+1)) of the shard's residues; chunks [0, K1) are C
+// residues apart, the rest (the last ~2 chunks' worth per resident warp) Ct =
+// C/4 apart, so the tail of a launch -- warps finishing their last chunk --
+// is a fraction of a small chunk.
+struct ChunkPlan {
+  int64_t C, Ct, K1, nchunks;
+};
+__host__ __device__ inline int64_t chunk_target(const ChunkPlan &p, int64_t k) {
+  return k < p.K1 ? k * p.C : p.K1 * p.C + (k - p.K1) * p.Ct;
+}
+cudaError_t launch_layout(const int64_t *off, int64_t n, const ChunkPlan &plan, int64_t *sstart,
+                          Chunk *chunks, Chunk *long_chunks, int *nlong, int *err,
+                          cudaStream_t s);
 // Segment length / list capacity of the long-item pipeline.
 constexpr int kSegLen = 2048;
 constexpr int kSegCap = 2048;

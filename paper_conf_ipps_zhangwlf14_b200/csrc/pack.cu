@@ -58,16 +58,17 @@ __global__ void layout_kernel(const int64_t *__restrict__ off, int64_t n, int64_
   }
 }
 
-// Chunk k = the subjects whose first residue lies in [k*C, (k+1)*C) of the
-// shard's residues (binary search over the offsets); empty chunks have
-// start == end and are skipped by the search kernels.
+// Chunk k = the subjects whose first residue lies in [target(k),
+// target(k+1)) of the shard's residues (ChunkPlan; binary search over the
+// offsets); empty chunks have start == end and are skipped by the kernels.
 __global__ void chunk_kernel(const int64_t *__restrict__ off, int64_t n,
-                             const int64_t *__restrict__ sstart, int64_t C, int64_t nchunks,
+                             const int64_t *__restrict__ sstart, ChunkPlan plan,
                              Chunk *chunks, Chunk *long_chunks, int *nlong) {
   const int64_t base = off[0];
+  const int64_t nchunks = plan.nchunks;
   auto first_at = [&](int64_t k) -> int64_t {
     if (k >= nchunks) return n;
-    const int64_t target = k * C;
+    const int64_t target = chunk_target(plan, k);
     int64_t lo = 0, hi = n;
     while (lo < hi) {
       const int64_t m = (lo + hi) >> 1;
@@ -89,7 +90,7 @@ __global__ void chunk_kernel(const int64_t *__restrict__ off, int64_t n,
     }
     // chunks much longer than C (long subjects) are scheduled first, so the
     // single warp walking one never becomes the tail of the launch
-    if (c.end - c.start > 2 * C) {
+    if (c.end - c.start > 2 * (chunk_target(plan, k + 1) - chunk_target(plan, k))) {
       long_chunks[atomicAdd(nlong, 1)] = c;
       c.start = c.end = 0;
     }
@@ -99,16 +100,17 @@ __global__ void chunk_kernel(const int64_t *__restrict__ off, int64_t n,
 
 }  // namespace
 
-cudaError_t launch_layout(const int64_t *off, int64_t n, int64_t C, int64_t nchunks,
-                          int64_t *sstart, Chunk *chunks, Chunk *long_chunks, int *nlong,
-                          int *err, cudaStream_t s) {
+cudaError_t launch_layout(const int64_t *off, int64_t n, const ChunkPlan &plan, int64_t *sstart,
+                          Chunk *chunks, Chunk *long_chunks, int *nlong, int *err,
+                          cudaStream_t s) {
+  const int64_t nchunks = plan.nchunks;
   if (n > 0) {
     const int64_t blocks = (n + 255) / 256 > 4096 ? 4096 : (n + 255) / 256;
     layout_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, err);
   }
   if (nchunks > 0) {
     const int64_t blocks = (nchunks + 255) / 256 > 4096 ? 4096 : (nchunks + 255) / 256;
-    chunk_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, C, nchunks, chunks, long_chunks,
+    chunk_kernel<<<unsigned(blocks), 256, 0, s>>>(off, n, sstart, plan, chunks, long_chunks,
                                                   nlong);
   }
   return cudaGetLastError();
