@@ -11,6 +11,7 @@
  *   diagonal             d = s - q            (R5)
  *   two-hit filter       P:L1344-1351         (R6)
  *   coverage / ext_reach Alg. 3 L12-23        (R10)
+ *   hit-based extension  Alg. 4 L9-14          (ext_mode 1)
  *   X-drop extension     Fig. 8, P:L1579-1693 (R7-R9)
  *
  * Build: gcc -O2 -std=c99 -shared -fPIC -pthread oracle.c -o liboracle.so
@@ -285,7 +286,9 @@ static void search_range(range_job *J) {
         if (!pass[k]) continue;
         const int32_t h = H[k], q = h - d;
         hitlist_push(J->passing, subj, q, h);
-        if (h <= ext_reach) continue;
+        /* Alg. 3 L19: skip a hit covered by the previous extension of the
+         * diagonal (DIAGONAL); Alg. 4 L9-14 extends every hit (HIT). */
+        if (p->ext_mode == 0 && h <= ext_reach) continue;
         /* R7: seed word [q, q+w) x [h, h+w), then independent X-drop to the
          * right (from q+w, h+w) and to the left (from q-1, h-1). */
         int32_t s0 = 0;

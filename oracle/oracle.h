@@ -26,7 +26,9 @@
  *   oracle_two_hit           pinned: Fig. 7 example (both modes), O(n^2) brute force
  *   oracle_search            pinned: P5-P9 invariants, independent oracle-B
  *                                    (oracle/oracle_b.py) on random tiny cases,
- *                                    planted exact copies, E[hits] closed form.
+ *                                    planted exact copies, E[hits] closed form;
+ *                                    HIT mode: oracle-B, one extension per
+ *                                    passing hit, Alg. 3 chain of HIT = DIAGONAL.
  *   Whole HSP list vs FSA-BLAST: parity unpinned (FSA-BLAST's rules are not
  *   in the paper); see DESIGN.md.
  */
@@ -54,6 +56,9 @@ typedef struct {
   int32_t xdrop;       /* X: stop when best - run >= X (R8)                  */
   int32_t cutoff;      /* emit iff score >= cutoff (R10)                     */
   int32_t filter_mode; /* 0 = LEFT (R6 default), 1 = EITHER (Fig. 7 reading) */
+  int32_t ext_mode;    /* 0 = DIAGONAL: Alg. 3 coverage chain (R10, default);
+                          1 = HIT: Alg. 4, every
+                          passing hit extended independently, duplicates kept */
 } oracle_params;
 
 /* One ungapped extension (R10/R11).  diagonal = s_start - q_start. */

@@ -40,7 +40,7 @@ class _Params(ctypes.Structure):
     _fields_ = [("word_len", ctypes.c_int32), ("threshold", ctypes.c_int32),
                 ("window", ctypes.c_int32), ("min_gap", ctypes.c_int32),
                 ("xdrop", ctypes.c_int32), ("cutoff", ctypes.c_int32),
-                ("filter_mode", ctypes.c_int32)]
+                ("filter_mode", ctypes.c_int32), ("ext_mode", ctypes.c_int32)]
 
 
 class _HitList(ctypes.Structure):
@@ -58,10 +58,11 @@ class Params:
     xdrop: int = 16
     cutoff: int = 41
     filter_mode: int = 0  # 0 LEFT, 1 EITHER
+    ext_mode: int = 0  # 0 DIAGONAL (Alg. 3 coverage chain), 1 HIT (Alg. 4)
 
     def _c(self) -> _Params:
         return _Params(self.word_len, self.threshold, self.window, self.min_gap, self.xdrop,
-                       self.cutoff, self.filter_mode)
+                       self.cutoff, self.filter_mode, self.ext_mode)
 
 
 _lib = None

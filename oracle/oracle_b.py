@@ -9,7 +9,8 @@ with oracle.c except the definition of the method in PAPER.md:
   (P:L1344-1351, R6);
 * X-drop is a direct loop over the diagonal, written from the ChangeSinceBest
   / DropFlag description of Fig. 8 (P:L1579-1693, R8);
-* coverage follows Alg. 3 L19-23 (R10).
+* coverage follows Alg. 3 L19-23 (R10); ext_mode=1 is Alg. 4
+  (P:L1465-1486): every passing hit is extended, no coverage test.
 
 Results are returned as a sorted list of 7-tuples (R11).
 """
@@ -34,7 +35,7 @@ def _extend_one_side(Q, S, q0, s0, step, M, X):
 
 
 def search_b(Q, subjects, M, *, T=11, w=3, A=40, W=3, X=16, cutoff=41, mode=0,
-             query_id=0, subject_base=0):
+             query_id=0, subject_base=0, ext_mode=0):
     """Return (hsps, extensions) as sorted lists of 7-tuples
     (query_id, subject_id, diagonal, q_start, s_start, length, score)."""
     Q = [int(c) for c in Q]
@@ -61,7 +62,7 @@ def search_b(Q, subjects, M, *, T=11, w=3, A=40, W=3, X=16, cutoff=41, mode=0,
                     ok = any(W <= h - p < A for p in H)
                 else:
                     ok = any(W <= abs(h - p) < A for p in H)
-                if not ok or h <= reach:
+                if not ok or (ext_mode == 0 and h <= reach):
                     continue
                 q = h - d
                 seed = sum(M[Q[q + j]][S[h + j]] for j in range(w))

@@ -314,15 +314,16 @@ def test_oracle_b_agrees_on_random_tiny_cases(orc, B62):
     checked_ext = 0
     for i, (Q, subs) in enumerate(_oracle_b_cases(rng, al, n)):
         mode = i % 2
+        ext_mode = (i // 2) % 2  # DIAGONAL (Alg. 3) / HIT (Alg. 4)
         T = 11 if i % 5 else 9
         X = int(rng.choice([16, 16, 5, 30]))
         cutoff = int(rng.choice([41, 20]))
         offs = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
         db = np.concatenate(subs).astype(np.uint8) if offs[-1] else np.zeros(0, np.uint8)
-        p = orc.Params(threshold=T, xdrop=X, cutoff=cutoff, filter_mode=mode)
+        p = orc.Params(threshold=T, xdrop=X, cutoff=cutoff, filter_mode=mode, ext_mode=ext_mode)
         r = orc.search(Q, db, offs, p, query_id=3, subject_base=10)
         hb, eb = search_b(Q, subs, M, T=T, X=X, cutoff=cutoff, mode=mode, query_id=3,
-                          subject_base=10)
+                          subject_base=10, ext_mode=ext_mode)
         assert [tuple(x) for x in r.hsps.tolist()] == hb, i
         assert [tuple(x) for x in r.extensions.tolist()] == eb, i
         checked_ext += len(eb)
@@ -338,3 +339,28 @@ def test_multithreaded_equals_single(orc):
     r4 = orc.search(Q, codes, db.offsets, nthreads=4)
     assert (r1.hsps == r4.hsps).all() and (r1.extensions == r4.extensions).all()
     assert len(r1.hsps) > 50
+
+
+@pytest.mark.parametrize("mode", [0, 1])
+def test_hit_mode_extends_every_passing_hit(orc, mode):
+    """Alg. 4 (P:L1465-1486): one extension per passing hit, duplicates kept;
+    the diagonal-based (Alg. 3) extensions are a sub-multiset of them (a
+    covered hit is skipped, an uncovered one is extended identically)."""
+    from collections import Counter
+    q = gen_query(31, 400)
+    db = gen_db(32, 33, n_subjects=600, mean_len=250, queries=[q], plant_frac=0.3)
+    Q = orc.encode(q)
+    codes = orc.encode(db.ascii.tobytes())
+    hit = orc.search(Q, codes, db.offsets, orc.Params(filter_mode=mode, ext_mode=1),
+                     want_hits=True)
+    diag = orc.search(Q, codes, db.offsets, orc.Params(filter_mode=mode, ext_mode=0),
+                      want_hits=True)
+    assert len(hit.extensions) == len(hit.passing) == len(diag.passing)
+    ch = Counter(tuple(x) for x in hit.extensions.tolist())
+    cd = Counter(tuple(x) for x in diag.extensions.tolist())
+    assert not (cd - ch)
+    assert len(hit.extensions) > len(diag.extensions) > 50
+    # duplicates: several seeds inside one planted copy give the same HSP
+    assert any(v > 1 for v in ch.values())
+    assert sorted(tuple(x) for x in hit.hsps.tolist()) == \
+        sorted(x for x in (tuple(y) for y in hit.extensions.tolist()) if x[6] >= 41)
