@@ -52,7 +52,9 @@ def parse_args():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--config", type=int, default=3, choices=[1, 2, 3])
+    ap.add_argument("--config", type=int, default=3, choices=[1, 2, 3, 5],
+                    help="BASELINE config; 5 = 64 queries vs the nr-shaped DB cut into 8 "
+                         "shards, rank r searching shard r (weak scaling)")
     ap.add_argument("--query-lens", default="1054",
                     help="comma list of query lengths searched as one batch (config 4: 127,517,1054)")
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -69,14 +71,27 @@ def env_rank():
 
 # --------------------------------------------------------------- workload
 
+def shard_plan(args, world):
+    """(shard count, whole-job residues are those of shards [0, world)).
+    Configs 1-3: the DB is cut into `world` shards (strong scaling, config 4).
+    Config 5: the DB is cut into max(8, world) shards and rank r owns shard r
+    (weak scaling: per-GPU work is fixed; at N = 8 the job is all of config 5)."""
+    return max(8, world) if args.config == 5 else world
+
+
 def workload(args, rank, world):
     from paper_conf_ipps_zhangwlf14_b200.dist import shard_subjects
-    from synth import CONFIGS, config_offsets, gen_db, gen_query
+    from synth import CONFIGS, config_offsets, gen_db, gen_queries, gen_query
     c = CONFIGS[args.config]
-    lens = [int(x) for x in args.query_lens.split(",")] if args.config == 3 else [c["query_len"]]
-    queries = [gen_query(c["query_seed"] if L == c["query_len"] else L, L) for L in lens]
+    if args.config == 5:
+        queries = gen_queries(c["query_seed"], 64, 100, 2000)
+        lens = [len(q) for q in queries]
+    else:
+        lens = [int(x) for x in args.query_lens.split(",")] if args.config == 3 else [c["query_len"]]
+        queries = [gen_query(c["query_seed"] if L == c["query_len"] else L, L) for L in lens]
     full_off = config_offsets(args.config, args.scale)
-    lo, hi = shard_subjects(full_off, rank, world)
+    nshards = shard_plan(args, world)
+    lo, hi = shard_subjects(full_off, rank, nshards)
     ns, tr = c["n_subjects"], c["total_residues"]
     if args.scale != 1.0:
         ns = None if ns is None else max(1, int(ns * args.scale))
@@ -84,9 +99,17 @@ def workload(args, rank, world):
     db = gen_db(c["db_seed"], c["plant_seed"], n_subjects=ns, total_residues=tr,
                 mean_len=c["mean_len"], queries=queries, plant_frac=c["plant_frac"],
                 subject_range=(lo, hi))
-    desc = (f"config{args.config}{'/4' if world > 1 else ''}: q{'+'.join(map(str, lens))} vs "
-            f"{c['name'].split('_vs_')[-1]} synthetic DB ({len(full_off) - 1} subjects, "
-            f"{int(full_off[-1])} residues)" + (f", sharded over {world} GPUs" if world > 1 else ""))
+    if args.config == 5:
+        _, job_hi = shard_subjects(full_off, world - 1, nshards)
+        desc = (f"config5: 64 queries (len U[100,2000], {sum(lens)} residues) vs "
+                f"{c['name'].split('_vs_')[-1]} synthetic DB ({len(full_off) - 1} subjects, "
+                f"{int(full_off[-1])} residues) cut into {nshards} shards; shards 0..{world - 1} "
+                f"searched, one per GPU ({int(full_off[job_hi] - full_off[0])} residues)")
+    else:
+        desc = (f"config{args.config}{'/4' if world > 1 else ''}: q{'+'.join(map(str, lens))} vs "
+                f"{c['name'].split('_vs_')[-1]} synthetic DB ({len(full_off) - 1} subjects, "
+                f"{int(full_off[-1])} residues)" +
+                (f", sharded over {world} GPUs" if world > 1 else ""))
     return queries, db, full_off, (lo, hi), desc
 
 
@@ -166,7 +189,8 @@ def run_reference(args):
     queries, db, full_off, (lo, hi), desc = workload(args, 0, 1)
     Qs = [o.encode(q) for q in queries]
     tables = [o.neighbourhood(Q, o.blosum62(), 11) for Q in Qs]
-    nsub = int(np.searchsorted(db.offsets, CPU_SAMPLE_RESIDUES // max(1, args.steps + args.warmup)))
+    budget = CPU_SAMPLE_RESIDUES * 1054 // max(1, sum(len(q) for q in queries))
+    nsub = int(np.searchsorted(db.offsets, budget // max(1, args.steps + args.warmup)))
     nsub = max(1, min(nsub, db.nseq))
     sub_off = db.offsets[: nsub + 1]
     codes = o.encode(db.ascii[: sub_off[-1]].tobytes())
@@ -183,7 +207,7 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "scaling": "weak" if args.config == 5 else "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
             "config": {"workload": desc, "sample_subjects": nsub,
                        "sample_residues": int(sub_off[-1])},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
@@ -200,7 +224,8 @@ def cpu_baseline(queries, db):
     from oracle import oracle as o
     Qs = [o.encode(q) for q in queries]
     tables = [o.neighbourhood(Q, o.blosum62(), 11) for Q in Qs]
-    nsub = max(1, min(int(np.searchsorted(db.offsets, CPU_SAMPLE_RESIDUES)), db.nseq))
+    budget = CPU_SAMPLE_RESIDUES * 1054 // max(1, sum(len(q) for q in queries))
+    nsub = max(1, min(int(np.searchsorted(db.offsets, budget)), db.nseq))
     sub_off = db.offsets[: nsub + 1]
     codes = o.encode(db.ascii[: sub_off[-1]].tobytes())
     cores = os.cpu_count() or 1
@@ -260,7 +285,8 @@ def main():
     # the offsets are step input too: pinned, so their copy is asynchronous
     off_pinned = torch.from_numpy(np.ascontiguousarray(full_off, dtype=np.int64)).pin_memory()
     full_off = off_pinned.numpy()
-    gdb = bp.Database.from_pinned(base_ptr, full_off, rank, world, device=local_rank,
+    nshards = shard_plan(args, world)
+    gdb = bp.Database.from_pinned(base_ptr, full_off, rank, nshards, device=local_rank,
                                   stream=stream)
     assert gdb.subject_base == lo and gdb.residues == db.residues
     cap = max(1 << 20, gdb.residues // 500 * nq)
@@ -310,7 +336,9 @@ def main():
     t = torch.tensor([elapsed_ms, statistics.mean(kern_ms)], dtype=torch.float64, device=dev)
     all_reduce_max(t)
     elapsed_ms, kern_avg_ms = float(t[0]), float(t[1])
-    total_residues = int(full_off[-1] - full_off[0])
+    # whole-job residues: every shard a rank searched (configs 1-3: the DB)
+    from paper_conf_ipps_zhangwlf14_b200.dist import shard_subjects
+    total_residues = int(full_off[shard_subjects(full_off, world - 1, nshards)[1]] - full_off[0])
     value = total_residues * nq * args.steps / (elapsed_ms / 1e3)
 
     # ---- roofline of the dominant kernel (search_kernel) --------------------
@@ -346,7 +374,7 @@ def main():
             # the public end-to-end entry point for a host-resident shard:
             # parts are copied H2D while the previous part is searched
             bp.search_host_db(table, base_ptr, full_off, out.data_ptr(), cap, cnt.data_ptr(),
-                              params, shard_index=rank, num_shards=world, stream=stream)
+                              params, shard_index=rank, num_shards=nshards, stream=stream)
             n = int(cnt.item())
             res = out[: min(n, cap)]
             if world > 1:
@@ -376,14 +404,17 @@ def main():
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": max(args.warmup, 3),
             "ms_per_step": elapsed_ms / args.steps, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "scaling": "weak" if args.config == 5 else "strong", "vs_baseline": None,
+            "dtype": "int32", "data": "synthetic",
             "config": {"workload": desc, "query_lens": [len(q) for q in queries],
                        "db_subjects": int(len(full_off) - 1), "db_residues": total_residues,
                        "shard_residues_rank0": int(gdb.residues),
                        "params": {"word_len": 3, "T": 11, "A": 40, "X": 16, "cutoff": 41,
                                   "filter": "LEFT"},
                        "l2": "inputs larger than L2 (DB shard >> 126 MB), no flush",
-                       "hsps_per_step": n_hsp, "parallelism": f"db-shard{world}"},
+                       "hsps_per_step": n_hsp,
+                       "parallelism": f"db-shard{world}" + (f" (of {nshards})" if nshards != world
+                                                             else "")},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel": "search_kernel", "kernel_ms": kern_avg_ms,

@@ -46,6 +46,10 @@ extern "C" {
 #define BLASTP_MAX_SUBJECT_LEN (1 << 30)
 #define BLASTP_FILTER_LEFT 0   /* R6 default: W <= h - p < A              */
 #define BLASTP_FILTER_EITHER 1 /* Fig. 7 reading: W <= |h - p| < A        */
+#define BLASTP_EXT_DIAGONAL 0  /* Alg. 3: a passing hit covered by the
+                                  previous extension of its diagonal is skipped (R10) */
+#define BLASTP_EXT_HIT 1       /* Alg. 4: every passing
+                                  hit is extended independently; duplicates kept      */
 
 /* Search parameters.  Defaults (blastp_params_default) are the BASELINE.json
  * configuration: w = 3, T = 11, A = 40, X = 7 bits -> 16 raw, cutoff 41. */
@@ -57,6 +61,7 @@ typedef struct {
   int32_t xdrop;       /* X: stop when best - run >= X (Fig. 8, R8), 1..127   */
   int32_t cutoff;      /* emit an extension iff score >= cutoff (R10)         */
   int32_t filter_mode; /* BLASTP_FILTER_LEFT or BLASTP_FILTER_EITHER          */
+  int32_t ext_mode;    /* BLASTP_EXT_DIAGONAL (default) or BLASTP_EXT_HIT      */
 } blastp_params;
 
 /* One ungapped extension ("start and end position of this extension with
@@ -160,7 +165,9 @@ int blastp_query_table_info(const blastp_query_table *q, int32_t *num_queries,
 /* Ungapped search (Alg. 1-5; R4-R10): every hit of every query against
  * every subject of the shard, the two-hit filter per (subject, diagonal),
  * X-drop extension of passing hits not covered by a previous extension of
- * the same diagonal, and every extension with score >= cutoff returned.
+ * the same diagonal (ext_mode DIAGONAL; ext_mode HIT extends every passing
+ * hit, so one HSP may be returned once per seed inside it), and every
+ * extension with score >= cutoff returned.
  * HOST variant: *out_host (library-malloc'd, free with blastp_hsp_free) gets
  * *out_count HSPs in canonical order (R11: lexicographic on all 7 fields).
  * Synchronous on cuda_stream.  `p` must equal the params of the table for

@@ -23,6 +23,7 @@ LIB_PATH = os.environ.get("BLASTP_LIB") or os.path.join(_PKG, "libblastp.so")
 
 OK, E_INVALID_ARG, E_BAD_RESIDUE, E_TOO_LONG, E_NOMEM, E_CUDA, E_CAPACITY = 0, -1, -2, -3, -4, -5, -6
 FILTER_LEFT, FILTER_EITHER = 0, 1
+EXT_DIAGONAL, EXT_HIT = 0, 1
 
 HSP_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("diagonal", "<i4"),
                       ("q_start", "<i4"), ("s_start", "<i4"), ("length", "<i4"),
@@ -39,7 +40,8 @@ class BlastpError(RuntimeError):
 
 class _CParams(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int32) for n in
-                ("word_len", "threshold", "window", "min_gap", "xdrop", "cutoff", "filter_mode")]
+                ("word_len", "threshold", "window", "min_gap", "xdrop", "cutoff", "filter_mode",
+                 "ext_mode")]
 
 
 @dataclass
@@ -52,10 +54,11 @@ class Params:
     xdrop: int = 16
     cutoff: int = 41
     filter_mode: int = FILTER_LEFT
+    ext_mode: int = EXT_DIAGONAL  # Alg. 3 coverage chain; EXT_HIT = Alg. 4
 
     def c(self) -> _CParams:
         return _CParams(self.word_len, self.threshold, self.window, self.min_gap, self.xdrop,
-                        self.cutoff, self.filter_mode)
+                        self.cutoff, self.filter_mode, self.ext_mode)
 
 
 def _load():

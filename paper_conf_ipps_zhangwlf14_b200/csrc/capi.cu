@@ -77,6 +77,8 @@ int validate_params(const blastp_params *p) {
     return fail(BLASTP_E_INVALID_ARG, "threshold %d outside [-100, 100]", p->threshold);
   if (p->filter_mode != BLASTP_FILTER_LEFT && p->filter_mode != BLASTP_FILTER_EITHER)
     return fail(BLASTP_E_INVALID_ARG, "filter_mode %d unknown", p->filter_mode);
+  if (p->ext_mode != BLASTP_EXT_DIAGONAL && p->ext_mode != BLASTP_EXT_HIT)
+    return fail(BLASTP_E_INVALID_ARG, "ext_mode %d unknown", p->ext_mode);
   return BLASTP_OK;
 }
 
@@ -202,6 +204,7 @@ void blastp_params_default(blastp_params *p) {
   p->xdrop = 16;
   p->cutoff = 41;
   p->filter_mode = BLASTP_FILTER_LEFT;
+  p->ext_mode = BLASTP_EXT_DIAGONAL;
 }
 
 const char *blastp_strerror(int status) {
@@ -672,6 +675,7 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.xdrop = p->xdrop;
     a.cutoff = p->cutoff;
     a.filter_mode = p->filter_mode;
+    a.ext_mode = p->ext_mode;
     a.ring = search_ring_slots(qd.lq, p->window);
     a.table_entries = qd.entries;
     a.out = out;

@@ -112,6 +112,7 @@ struct SearchArgs {
   unsigned seq;                // launch sequence number of this search
   QueryView qv;
   int32_t word_len, threshold, window, min_gap, xdrop, cutoff, filter_mode;
+  int32_t ext_mode;  // BLASTP_EXT_DIAGONAL (Alg. 3 ext_reach chain) / BLASTP_EXT_HIT (Alg. 4)
   int32_t ring;      // M: per-warp diagonal ring slots
   int64_t table_entries;  // CSR entries of the query table (positions)
   blastp_hsp *out;

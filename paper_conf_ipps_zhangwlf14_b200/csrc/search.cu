@@ -128,11 +128,15 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
     stat_add<kTrace>(st, kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(scanned)));
   }
   const int endp = min(P + 2 + rlen, 0xffff);  // HSP subject end (inclusive), frame
-  const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
-  const bool uniq = (grp == (1u << lane));
   bool acc = false;
   uint16_t *reach16 = w.reach + slot;
-  if (__all_sync(kFull, uniq || !act)) {
+  if (a.ext_mode == BLASTP_EXT_HIT) {
+    // Alg. 4: every passing hit is extended and kept; ext_reach
+    // is never written, so every passing hit was also queued
+    acc = act;
+  } else if (const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane),
+             uniq = (grp == (1u << lane));
+             __all_sync(kFull, uniq || !act)) {
     if (act) {
       acc = P > int(*reach16);
       if (acc) *reach16 = uint16_t(endp);

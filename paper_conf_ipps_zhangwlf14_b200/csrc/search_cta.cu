@@ -188,7 +188,9 @@ __device__ void consumer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
     const int q = int(ent.z & 0xffffu);
     const int slot = int(ent.z >> 16);
     // skip hits already covered by an extension resolved in an earlier batch
-    const bool pre = act && vpos > S.reach[slot];
+    // (ext_mode HIT, Alg. 4: ext_reach stays 0, every passing hit is extended)
+    const bool hitm = a.ext_mode == BLASTP_EXT_HIT;
+    const bool pre = act && (hitm || vpos > S.reach[slot]);
     int total = 0, llen = 0, rlen = 0, scanned = 0;
     if (pre) xdrop_extend(a.stream, sp, q, S.qc, S.b62, a.xdrop, total, llen, rlen, scanned);
     if (kTrace) {
@@ -198,10 +200,12 @@ __device__ void consumer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
       st.add(kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(scanned)));
     }
     const unsigned endv = vpos + 2u + unsigned(rlen);  // subject end of the HSP (vpos)
-    const unsigned grp = __match_any_sync(kFull, pre ? slot : -1 - lane);
-    const bool uniq = grp == (1u << lane);
     bool acc = false;
-    if (__all_sync(kFull, uniq || !pre)) {
+    if (hitm) {
+      acc = pre;
+    } else if (const unsigned grp = __match_any_sync(kFull, pre ? slot : -1 - lane),
+               uniq = grp == (1u << lane);
+               __all_sync(kFull, uniq || !pre)) {
       if (pre) {
         acc = vpos > S.reach[slot];
         if (acc) S.reach[slot] = endv;

@@ -43,8 +43,8 @@ def test_built_for_sm100a(bp):
 
 def test_params_default_matches_baseline(bp):
     p = bp.params_default()
-    assert (p.word_len, p.threshold, p.window, p.min_gap, p.xdrop, p.cutoff, p.filter_mode) == \
-        (3, 11, 40, 3, 16, 41, 0)
+    assert (p.word_len, p.threshold, p.window, p.min_gap, p.xdrop, p.cutoff, p.filter_mode,
+            p.ext_mode) == (3, 11, 40, 3, 16, 41, 0, 0)
     assert bp.Params() == p
 
 
@@ -88,7 +88,7 @@ def test_shard_range_rejects_bad_arguments(bp):
 
 def test_invalid_params_rejected_before_any_gpu_work(bp):
     for bad in [dict(word_len=4), dict(min_gap=0), dict(window=0), dict(xdrop=0),
-                dict(xdrop=200), dict(filter_mode=7), dict(threshold=500)]:
+                dict(xdrop=200), dict(filter_mode=7), dict(ext_mode=2), dict(threshold=500)]:
         with pytest.raises(bp.BlastpError) as e:
             bp.build_query_table("MKVLAAGIVALLA", bp.Params(**bad))
         assert e.value.status == bp.E_INVALID_ARG, bad
