@@ -13,6 +13,9 @@ __constant__ uint8_t c_encode[256];
 
 // One warp per subject (grid-stride): lanes copy consecutive bytes, so every
 // load and store instruction of a warp touches one or two 32-byte sectors.
+// The encode table is staged in shared memory: lanes look up different
+// letters, which a __constant__ table would serialise (one address per
+// cycle); four bytes per lane are in flight per iteration.
 // Every byte of the stream is written here (no separate memset, which as a
 // kernel would queue behind a running search and hold up the copies of a
 // pipelined blastp_search_host_db): the front pad, each subject followed by
@@ -20,6 +23,9 @@ __constant__ uint8_t c_encode[256];
 __global__ void pack_kernel(const uint8_t *__restrict__ ascii, const int64_t *__restrict__ off,
                             int64_t n, const int64_t *__restrict__ sstart,
                             uint8_t *__restrict__ stream, int64_t stream_len, int *err) {
+  __shared__ uint8_t lut[256];
+  for (int i = threadIdx.x; i < 256; i += blockDim.x) lut[i] = c_encode[i];
+  __syncthreads();
   const int lane = threadIdx.x & 31;
   const int64_t gtid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   const int64_t nthreads = int64_t(gridDim.x) * blockDim.x;
@@ -32,9 +38,21 @@ __global__ void pack_kernel(const uint8_t *__restrict__ ascii, const int64_t *__
   for (int64_t i = gtid >> 5; i < n; i += warps) {
     const int64_t a = off[i] - base, len = off[i + 1] - off[i];
     uint8_t *dst = stream + sstart[i];
+    const uint8_t *src = ascii + a;
     int bad = 0;
-    for (int64_t j = lane; j < len; j += 32) {
-      const uint8_t c = c_encode[__ldg(ascii + a + j)];
+    int64_t j = lane;
+    for (; j + 96 < len; j += 128) {
+      const uint8_t c0 = __ldg(src + j), c1 = __ldg(src + j + 32), c2 = __ldg(src + j + 64),
+                    c3 = __ldg(src + j + 96);
+      const uint8_t e0 = lut[c0], e1 = lut[c1], e2 = lut[c2], e3 = lut[c3];
+      bad |= (e0 == 0xFF) | (e1 == 0xFF) | (e2 == 0xFF) | (e3 == 0xFF);
+      dst[j] = e0;
+      dst[j + 32] = e1;
+      dst[j + 64] = e2;
+      dst[j + 96] = e3;
+    }
+    for (; j < len; j += 32) {
+      const uint8_t c = lut[__ldg(src + j)];
       bad |= (c == 0xFF);
       dst[j] = c;
     }

@@ -101,6 +101,24 @@ __device__ __forceinline__ int st_pred(uint32_t last, uint32_t far, uint32_t nea
   return m ? int(last) - (jmin + __ffs(m) - 1) : int(far);
 }
 
+// Four consecutive steps of the R8 scan (Fig. 8) on scores s0..s3 at offsets
+// t..t+3, branch-free and exact: p_j = running sums, m_j = best after step j
+// (max of the old best and p_0..p_j); the scan stops at the first j with
+// m_j - p_j >= X, so the best is m_j* (= m_3 without a stop) and, if it rose,
+// its length is the first step reaching it (strict >: shortest argmax).
+// `run` is only meaningful while no stop has occurred.
+__device__ __forceinline__ void xdrop_group4(int s0, int s1, int s2, int s3, int X, int t,
+                                             int &run, int &best, int &bl, bool &stop) {
+  const int p0 = run + s0, p1 = p0 + s1, p2 = p1 + s2, p3 = p2 + s3;
+  const int m0 = max(best, p0), m1 = max(m0, p1), m2 = max(m1, p2), m3 = max(m2, p3);
+  const bool st0 = m0 - p0 >= X, st1 = m1 - p1 >= X, st2 = m2 - p2 >= X, st3 = m3 - p3 >= X;
+  const int mf = st0 ? m0 : st1 ? m1 : st2 ? m2 : m3;
+  if (mf > best) bl = t + (p0 == mf ? 1 : p1 == mf ? 2 : p2 == mf ? 3 : 4);
+  best = mf;
+  run = p3;
+  stop = st0 || st1 || st2 || st3;
+}
+
 // R7/R8: X-drop extension from the seed word at (q, sp).  qc is the query
 // with kQPad sentinels before it and >= 4 after it; the stream has sentinels
 // between subjects.  Sentinels score -128, which stops the walk at either
@@ -127,16 +145,9 @@ __device__ __forceinline__ void xdrop_extend(const uint8_t *__restrict__ stream,
       const uint32_t w = __funnelshift_r(lo, hi, sh);
       lo = hi;
       hi = ldg32(base + t + 8);
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int s = score(b62, qp[t + j], (w >> (8 * j)) & 0xffu);
-        const int nr = run + s;
-        const bool nb = !stop && nr > best;
-        best = nb ? nr : best;
-        bl = nb ? t + j + 1 : bl;
-        run = stop ? run : nr;
-        stop = stop || (best - nr >= X);
-      }
+      xdrop_group4(score(b62, qp[t], w & 0xffu), score(b62, qp[t + 1], (w >> 8) & 0xffu),
+                   score(b62, qp[t + 2], (w >> 16) & 0xffu), score(b62, qp[t + 3], w >> 24), X,
+                   t, run, best, bl, stop);
     }
     scanned = t;
   }
@@ -157,16 +168,9 @@ __device__ __forceinline__ void xdrop_extend(const uint8_t *__restrict__ stream,
       const uint32_t w = __funnelshift_r(lo, hi, sh);
       hi = lo;
       lo = ldg32(base - t - 4);
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const int s = score(b62, qp[-(t + j)], (w >> (8 * (3 - j))) & 0xffu);
-        const int nr = run + s;
-        const bool nb = !stop && nr > best;
-        best = nb ? nr : best;
-        bl = nb ? t + j + 1 : bl;
-        run = stop ? run : nr;
-        stop = stop || (best - nr >= X);
-      }
+      xdrop_group4(score(b62, qp[-t], w >> 24), score(b62, qp[-(t + 1)], (w >> 16) & 0xffu),
+                   score(b62, qp[-(t + 2)], (w >> 8) & 0xffu), score(b62, qp[-(t + 3)], w & 0xffu),
+                   X, t, run, best, bl, stop);
     }
     scanned += t;
   }
