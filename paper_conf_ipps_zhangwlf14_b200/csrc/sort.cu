@@ -1,8 +1,12 @@
 // sort.cu -- canonical order of HSP lists on the GPU (R11): lexicographic on
-// (query_id, subject_id, diagonal, q_start, ...).  HSPs are unique in their
-// first four fields (successive extensions of a diagonal start beyond the
-// previous reach), so four stable LSD passes on those fields give the full
-// 7-field order.  Output formatting only -- not part of the timed hot path.
+// (query_id, subject_id, diagonal, q_start, s_start, length, score).
+// s_start = q_start + diagonal and the score is a function of the segment,
+// so five stable LSD passes (length, q_start, diagonal, subject_id,
+// query_id) give the full 7-field order.  The first four fields alone are
+// not unique: a later seed of a diagonal lies beyond the previous HSP's end,
+// but its left extension may reach back to the same start (and ext_mode HIT
+// returns one extension per seed, R14).  Output formatting only -- not part
+// of the timed hot path.
 #include <cub/device/device_radix_sort.cuh>
 #include <cuda_runtime.h>
 
@@ -58,7 +62,7 @@ cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s) {
   if (e == cudaSuccess) {
     const int blocks = int((n + 255) / 256 > 4096 ? 4096 : (n + 255) / 256);
     iota_kernel<<<blocks, 256, 0, s>>>(idx, n);
-    const int fields[4] = {3, 2, 1, 0};  // q_start, diagonal, subject_id, query_id
+    const int fields[5] = {5, 3, 2, 1, 0};  // length, q_start, diagonal, subject_id, query_id
     for (int f : fields) {
       key_kernel<<<blocks, 256, 0, s>>>(d, idx, key, n, f);
       e = cub::DeviceRadixSort::SortPairs(temp, temp_bytes, key, key2, idx, idx2, ni, 0, 32, s);

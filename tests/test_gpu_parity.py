@@ -418,6 +418,41 @@ def test_search_host_db_pipelined_parts(bp, orc):
     assert _host_db_search(bp, t, np.zeros(0, np.uint8), np.zeros(1, np.int64), p) == []
 
 
+def _same_start_db(orc):
+    """A seeded DB whose oracle HSP list holds two HSPs of one diagonal with
+    the same start and different ends (a later seed beyond the first HSP's
+    end whose left extension reaches back to the same start): the canonical
+    order then depends on the length field (R11)."""
+    rng = np.random.default_rng(7)
+    q = gen_query(77, 300).decode()
+    for _ in range(40):
+        subs = []
+        for _ in range(50):
+            s = list(rng.choice(list(ALPHA[:20]), size=400))
+            a, b, n = int(rng.integers(0, 200)), int(rng.integers(0, 300)), int(rng.integers(30, 90))
+            seg = list(q[a:a + n])
+            for i in np.nonzero(rng.random(len(seg)) < 0.35)[0]:
+                seg[i] = ALPHA[int(rng.integers(0, 20))]
+            s[b:b + len(seg)] = seg
+            subs.append("".join(s[:400]))
+        ascii = np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy()
+        off = np.arange(0, 50 * 400 + 1, 400, dtype=np.int64)
+        h = tuples(orc.search(orc.encode(q), orc.encode(ascii.tobytes()), off).hsps)
+        if len({x[:4] for x in h}) < len(h):
+            return q, ascii, off
+    raise AssertionError("no same-start HSP pair generated")
+
+
+def test_same_start_hsps_canonical_order(bp, orc):
+    """HSPs equal in (query, subject, diagonal, q_start) are ordered by
+    length as R11 requires, on the host (GPU-sorted) and device variants."""
+    q, ascii, off = _same_start_db(orc)
+    for ext_mode in (0, 1):
+        p = bp.Params(ext_mode=ext_mode)
+        g, r = assert_same(bp, orc, q, ascii, off, p, trace=True)
+        assert len({x[:4] for x in tuples(g)}) < len(g)
+
+
 def test_query_batch_equals_single_queries(bp, orc):
     qs = [gen_query(11 + i, L) for i, L in enumerate([100, 350, 900])]
     db = gen_db(12, 13, n_subjects=500, mean_len=300.0, queries=qs, plant_frac=0.3)
