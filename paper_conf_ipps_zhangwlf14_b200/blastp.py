@@ -181,7 +181,8 @@ class QueryTable:
         return e.value
 
     def free(self):
-        if getattr(self, "handle", None):
+        # lib is None during interpreter shutdown (module globals cleared)
+        if getattr(self, "handle", None) and lib is not None:
             lib.blastp_query_table_free(self.handle)
             self.handle = None
 
@@ -251,7 +252,7 @@ class Database:
             self.long_items, self.segments, self.segment_len = (v.value for v in vals)
 
     def free(self):
-        if getattr(self, "handle", None):
+        if getattr(self, "handle", None) and lib is not None:
             lib.blastp_db_free(self.handle)
             self.handle = None
 

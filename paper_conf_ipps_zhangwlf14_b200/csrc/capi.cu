@@ -831,6 +831,28 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
     ev.push_back(e);
   };
   mark();
+  // Consecutive parts are searched on two alternating streams: part k+1's
+  // search kernel fills the SMs that part k's launch leaves idle in its
+  // tail (the CTAs of one search are resident one per SM and retire
+  // unevenly).  Parts have separate counters; they share only the HSP
+  // output counter, which is atomic.  BLASTP_PIPE_STREAMS=1: one stream.
+  int nstreams = 2;
+  if (const char *v = std::getenv("BLASTP_PIPE_STREAMS")) nstreams = std::atoi(v) == 1 ? 1 : 2;
+  cudaStream_t s2 = s;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  if (nstreams == 2) {
+    if (cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&ev_join, cudaEventDisableTiming) != cudaSuccess) {
+      cudaGetLastError();
+      if (s2 != s) cudaStreamDestroy(s2);
+      cudaFreeAsync(arena.base, cs);
+      cudaStreamDestroy(cs);
+      return fail(BLASTP_E_CUDA, "could not create the second search stream");
+    }
+    cudaEventRecord(ev_fork, s);  // after the count reset
+    cudaStreamWaitEvent(s2, ev_fork, 0);
+  }
   rc = BLASTP_OK;
   for (size_t k = 0; k + 1 < cut.size() && rc == BLASTP_OK; ++k) {
     // the host blocks here for part k's copy while part k-1 is searched
@@ -841,11 +863,19 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
     if (rc) break;
     const double b = ms();
     parts.push_back(d);
-    rc = enqueue_search(q, d, p, s, d_out, capacity, count, nullptr, nullptr, nullptr, false);
+    rc = enqueue_search(q, d, p, (k & 1) ? s2 : s, d_out, capacity, count, nullptr, nullptr,
+                        nullptr, false);
     mark();
     if (dbg)
       fprintf(stderr, "[pipe] part %zu: %lld residues, pack %.3f..%.3f ms, search enqueued %.3f ms\n",
               k, static_cast<long long>(offsets[cut[k + 1]] - offsets[cut[k]]), a, b, ms());
+  }
+  if (s2 != s) {  // join: s waits for the searches on s2
+    cudaEventRecord(ev_join, s2);
+    cudaStreamWaitEvent(s, ev_join, 0);
+    cudaEventDestroy(ev_fork);
+    cudaEventDestroy(ev_join);
+    cudaStreamDestroy(s2);
   }
   for (blastp_db *d : parts) db_free_async(d, s);
   // the searches on s read the arena: free it in their stream order (and

@@ -288,6 +288,40 @@ def test_edge_cases(bp, orc):
     assert len(g) == 0
 
 
+def test_pack_tiny_and_mixed_subjects(bp, orc):
+    """Runs of empty and 1-5 residue subjects (more than 32 subject starts in
+    one 512-byte pack tile: the pack kernel's general path), lowercase and
+    U/O/J residues, and ordinary subjects between them: every hit, passing
+    hit, extension and HSP identical to the oracle (a word spanning two
+    subjects, a wrong sentinel or a shifted residue would show up as a hit)."""
+    rng = np.random.default_rng(31)
+    q = gen_query(32, 400).decode()
+    subs = []
+    for blk in range(60):
+        if blk % 3 == 0:
+            subs += ["".join(rng.choice(list(ALPHA[:20]), size=int(L)))
+                     for L in rng.integers(0, 6, size=int(rng.integers(40, 300)))]
+        else:
+            L = int(rng.integers(50, 900))
+            s = list(rng.choice(list(ALPHA[:20] + "uojbzx"), size=L))
+            a, n = int(rng.integers(0, 300)), int(rng.integers(20, 100))
+            b = int(rng.integers(0, max(1, L - n)))
+            s[b:b + n] = list(q[a:a + n])[:max(0, L - b)]
+            subs.append("".join(s[:L]))
+    ascii = np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy()
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    g, r = assert_same(bp, orc, q, ascii, off, bp.Params(), trace=True)
+    assert len(g) > 20
+    for k in range(3):  # shards start at arbitrary subjects
+        shard = tuples(bp.search_ungapped(bp.build_query_table(q), bp.pack_db(ascii, off, k, 3)))
+        assert shard == [h for h in tuples(g) if h[1] in range(*_shard_ids(bp, off, k, 3))]
+
+
+def _shard_ids(bp, off, k, n):
+    d = bp.pack_db(np.zeros(int(off[-1]), np.uint8) + ord("A"), off, k, n)
+    return d.subject_base, d.subject_base + d.nseq
+
+
 def _long_subject_db(q):
     """Long subjects (> 2C residues: split into segments) with copies of the
     query planted across segment boundaries (exact ones, so an extension and
@@ -351,6 +385,20 @@ def test_long_query_2000(bp, orc):
     q = gen_query(2000, 2000)
     db = gen_db(7, 8, n_subjects=400, mean_len=375.0, queries=[q], plant_frac=0.2)
     assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(), trace=True)
+
+
+def test_longest_query(bp, orc):
+    """BLASTP_MAX_QUERY_LEN (16,000): the diagonal ring is ~96 KB per warp,
+    so a CTA holds two warps and the lookup table stays in global memory;
+    results identical to the oracle.  One residue more is rejected."""
+    q = gen_query(16000, 16000)
+    db = gen_db(9, 10, n_subjects=150, mean_len=375.0, queries=[q], plant_frac=0.3)
+    g, _ = assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(), trace=False,
+                       nthreads=os.cpu_count() or 8)
+    assert len(g) > 20
+    with pytest.raises(bp.BlastpError) as e:
+        bp.build_query_table(gen_query(16001, 16001))
+    assert e.value.status == -3  # BLASTP_E_TOO_LONG
 
 
 # ------------------------------------------------------------------ API
