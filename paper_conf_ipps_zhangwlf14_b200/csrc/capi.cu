@@ -239,6 +239,30 @@ static int build_one_query(const char *ascii, int32_t len, const blastp_params *
                            static_cast<unsigned char>(ascii[i]));
     Q[static_cast<size_t>(i)] = static_cast<uint8_t>(c);
   }
+  out.lq = len;
+  const char *how = std::getenv("BLASTP_TABLE_BUILD");  // "host": the host enumeration below
+  if (!(how && !std::strcmp(how, "host"))) {
+    // GPU build (table.cu): one thread per word counts, scans, fills
+    if (cudaMallocAsync(&out.woff, sizeof(uint32_t) * (kWords + 1), s) != cudaSuccess ||
+        cudaMallocAsync(&out.qcodes, static_cast<size_t>(len) + 16, s) != cudaSuccess) {
+      cudaGetLastError();
+      free_query_dev(out);
+      return fail(BLASTP_E_NOMEM, "device allocation for the query table failed");
+    }
+    CUDA_TRY(cudaMemcpyAsync(out.qcodes, Q.data(), Q.size(), cudaMemcpyHostToDevice, s));
+    int64_t total = 0;
+    CUDA_TRY(launch_table_count(out.qcodes, len, p->threshold, out.woff, &total, s));
+    out.entries = total;
+    if (cudaMallocAsync(&out.qpos, sizeof(uint16_t) * size_t(std::max<int64_t>(total, 1)), s) !=
+        cudaSuccess) {
+      cudaGetLastError();
+      free_query_dev(out);
+      return fail(BLASTP_E_NOMEM, "device allocation for the query table failed");
+    }
+    CUDA_TRY(launch_table_fill(out.qcodes, len, p->threshold, out.woff, out.qpos, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+    return BLASTP_OK;
+  }
   // Neighbourhood words by pruned enumeration: for each query word, walk the
   // 24^3 words letter by letter and cut a branch as soon as even the best
   // remaining letters cannot reach T.  Same set as the brute-force

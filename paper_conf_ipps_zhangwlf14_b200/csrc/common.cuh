@@ -148,6 +148,12 @@ int search_ring_slots(int lq, int window);
 // variable BLASTP_KERNEL=warp|cta forces one (tests cover both).
 cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s);
 cudaError_t launch_search_warp(const SearchArgs &a, int num_sms, cudaStream_t s);
+// Query lookup table on the GPU (table.cu): woff (kWords + 1) from the query
+// codes, the entry count returned on the host (synchronises s), then qpos.
+cudaError_t launch_table_count(const uint8_t *qcodes, int lq, int T, uint32_t *woff,
+                               int64_t *total, cudaStream_t s);
+cudaError_t launch_table_fill(const uint8_t *qcodes, int lq, int T, const uint32_t *woff,
+                              uint16_t *qpos, cudaStream_t s);
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,
                         const int64_t *sstart, uint8_t *stream, int64_t stream_len, int *err,
                         cudaStream_t s);

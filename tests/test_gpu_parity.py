@@ -223,6 +223,23 @@ def test_config5_shard_sampled(bp, orc, kernel_variant):
         assert_sampled_parity(bp, orc, queries, db.ascii, off, g, p, blocks, subject_base=lo)
 
 
+@pytest.mark.parametrize("T", [8, 11, 13])
+def test_query_table_builders_agree(bp, orc, monkeypatch, T):
+    """The GPU table builder (default) and the host enumeration
+    (BLASTP_TABLE_BUILD=host) give the same table: same entry count and the
+    same hit trace as the oracle's brute-force neighbourhood (R3)."""
+    q = gen_query(41, 600).decode() + "WWWCCCBZX*"
+    db = gen_db(42, 43, n_subjects=120, mean_len=300.0, queries=[q.encode()], plant_frac=0.3)
+    p = bp.Params(threshold=T)
+    entries = []
+    for how in ("gpu", "host"):
+        monkeypatch.setenv("BLASTP_TABLE_BUILD", how)
+        entries.append(bp.build_query_table(q, p).entries)
+        assert_same(bp, orc, q, db.ascii, db.offsets, p, trace=True)
+    off, pos = orc.neighbourhood(orc.encode(q), orc.blosum62(), T)
+    assert entries[0] == entries[1] == len(pos)
+
+
 # ------------------------------------------------------------------ fuzz
 
 def _rand_db(rng, n, lo, hi, q=None, plant=0.3):
@@ -387,12 +404,18 @@ def test_long_query_2000(bp, orc):
     assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(), trace=True)
 
 
-def test_longest_query(bp, orc):
+def test_longest_query(bp, orc, kernel_variant):
     """BLASTP_MAX_QUERY_LEN (16,000): the diagonal ring is ~96 KB per warp,
     so a CTA holds two warps and the lookup table stays in global memory;
-    results identical to the oracle.  One residue more is rejected."""
+    results identical to the oracle.  One residue more is rejected.  The
+    CTA variant's per-CTA diagonal state does not fit shared memory at this
+    length: forcing it (BLASTP_KERNEL=cta) fails loudly."""
     q = gen_query(16000, 16000)
     db = gen_db(9, 10, n_subjects=150, mean_len=375.0, queries=[q], plant_frac=0.3)
+    if kernel_variant == "cta":
+        with pytest.raises(bp.BlastpError, match="invalid configuration"):
+            gpu_run(bp, q, db.ascii, db.offsets, bp.Params())
+        return
     g, _ = assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(), trace=False,
                        nthreads=os.cpu_count() or 8)
     assert len(g) > 20
