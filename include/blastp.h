@@ -50,6 +50,10 @@ extern "C" {
                                   previous extension of its diagonal is skipped (R10) */
 #define BLASTP_EXT_HIT 1       /* Alg. 4: every passing
                                   hit is extended independently; duplicates kept      */
+#define BLASTP_EXT_WINDOW 2    /* Alg. 5 + Fig. 8: Alg. 3's coverage rule,
+                                  each extension a warp-wide window scan (prefix sum,
+                                  running max, drop flag over 32 positions at a time);
+                                  results identical to DIAGONAL                       */
 
 /* Search parameters.  Defaults (blastp_params_default) are the BASELINE.json
  * configuration: w = 3, T = 11, A = 40, X = 7 bits -> 16 raw, cutoff 41. */
@@ -61,7 +65,7 @@ typedef struct {
   int32_t xdrop;       /* X: stop when best - run >= X (Fig. 8, R8), 1..127   */
   int32_t cutoff;      /* emit an extension iff score >= cutoff (R10)         */
   int32_t filter_mode; /* BLASTP_FILTER_LEFT or BLASTP_FILTER_EITHER          */
-  int32_t ext_mode;    /* BLASTP_EXT_DIAGONAL (default) or BLASTP_EXT_HIT      */
+  int32_t ext_mode;    /* BLASTP_EXT_DIAGONAL (default), _HIT or _WINDOW       */
 } blastp_params;
 
 /* One ungapped extension ("start and end position of this extension with
@@ -188,6 +192,15 @@ int blastp_search_ungapped_device(const blastp_query_table *q,
 
 /* Canonical order (R11) of n device HSPs, in place, on the GPU. */
 int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream);
+
+/* De-duplication of a canonically ordered (blastp_sort_hsps_device) device
+ * HSP list, in place: runs of identical records collapse to one.  This is the
+ * step Alg. 4 (ext_mode HIT) leaves before gapped extension ("requires a
+ * de-duplication step"); a DIAGONAL-mode list has no
+ * duplicates.  *d_n_out (device int64) receives the new count; asynchronous
+ * on cuda_stream.  Errors: INVALID_ARG (n < 0, NULL buffers), NOMEM, CUDA. */
+int blastp_unique_hsps_device(blastp_hsp *d_hsps, int64_t n, int64_t *d_n_out,
+                              void *cuda_stream);
 
 /* Debug / parity entry points (synchronous, host buffers).  They run the
  * same kernel as the search with tracing enabled and return:

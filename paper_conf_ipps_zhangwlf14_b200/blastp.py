@@ -23,7 +23,7 @@ LIB_PATH = os.environ.get("BLASTP_LIB") or os.path.join(_PKG, "libblastp.so")
 
 OK, E_INVALID_ARG, E_BAD_RESIDUE, E_TOO_LONG, E_NOMEM, E_CUDA, E_CAPACITY = 0, -1, -2, -3, -4, -5, -6
 FILTER_LEFT, FILTER_EITHER = 0, 1
-EXT_DIAGONAL, EXT_HIT = 0, 1
+EXT_DIAGONAL, EXT_HIT, EXT_WINDOW = 0, 1, 2
 
 HSP_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("diagonal", "<i4"),
                       ("q_start", "<i4"), ("s_start", "<i4"), ("length", "<i4"),
@@ -90,6 +90,7 @@ def _load():
         L.blastp_search_host_db.argtypes = [vp, vp, vp, i64, i32, i32, P(_CParams), i32, vp, vp,
                                             i64, vp]
     L.blastp_sort_hsps_device.argtypes = [vp, i64, vp]
+    L.blastp_unique_hsps_device.argtypes = [vp, i64, vp, vp]
     L.blastp_debug_trace.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64), vp, i64, P(i64),
                                      vp, i64, P(i64)]
     L.blastp_debug_hits.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
@@ -107,7 +108,7 @@ EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "bl
             "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
             "blastp_shard_range", "blastp_db_info", "blastp_db_long_info", "blastp_query_table_info",
             "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_search_host_db",
-            "blastp_sort_hsps_device",
+            "blastp_sort_hsps_device", "blastp_unique_hsps_device",
             "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
 
@@ -316,6 +317,13 @@ def search_host_db(table: QueryTable, residues, offsets: np.ndarray, out_ptr: in
 
 def sort_hsps_device(ptr: int, n: int, stream=None):
     _check(lib.blastp_sort_hsps_device(ptr, n, _stream_handle(stream)), "blastp_sort_hsps_device")
+
+
+def unique_hsps_device(ptr: int, n: int, count_ptr: int, stream=None):
+    """Collapse duplicates of a canonically sorted device HSP list in place;
+    the new count is written to the device int64 at count_ptr."""
+    _check(lib.blastp_unique_hsps_device(ptr, n, count_ptr, _stream_handle(stream)),
+           "blastp_unique_hsps_device")
 
 
 STAT_NAMES = ["windows", "rounds", "conflict_rounds", "hits", "passing", "enqueued", "flushes",

@@ -77,7 +77,8 @@ int validate_params(const blastp_params *p) {
     return fail(BLASTP_E_INVALID_ARG, "threshold %d outside [-100, 100]", p->threshold);
   if (p->filter_mode != BLASTP_FILTER_LEFT && p->filter_mode != BLASTP_FILTER_EITHER)
     return fail(BLASTP_E_INVALID_ARG, "filter_mode %d unknown", p->filter_mode);
-  if (p->ext_mode != BLASTP_EXT_DIAGONAL && p->ext_mode != BLASTP_EXT_HIT)
+  if (p->ext_mode != BLASTP_EXT_DIAGONAL && p->ext_mode != BLASTP_EXT_HIT &&
+      p->ext_mode != BLASTP_EXT_WINDOW)
     return fail(BLASTP_E_INVALID_ARG, "ext_mode %d unknown", p->ext_mode);
   return BLASTP_OK;
 }
@@ -931,6 +932,14 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
 int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream) {
   if (n < 0 || (n > 0 && !d_hsps)) return fail(BLASTP_E_INVALID_ARG, "bad HSP buffer");
   CUDA_TRY(sort_hsps(d_hsps, n, static_cast<cudaStream_t>(cuda_stream)));
+  return BLASTP_OK;
+}
+
+int blastp_unique_hsps_device(blastp_hsp *d_hsps, int64_t n, int64_t *d_n_out,
+                              void *cuda_stream) {
+  if (n < 0 || (n > 0 && !d_hsps) || !d_n_out)
+    return fail(BLASTP_E_INVALID_ARG, "bad HSP buffer");
+  CUDA_TRY(unique_hsps(d_hsps, n, d_n_out, static_cast<cudaStream_t>(cuda_stream)));
   return BLASTP_OK;
 }
 

@@ -176,6 +176,7 @@ constexpr int kSegLen = 2048;
 constexpr int kSegCap = 2048;
 constexpr int kMaxSegments = 32768;  // 256 MB of lists at most
 cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
+cudaError_t unique_hsps(blastp_hsp *d, int64_t n, int64_t *d_n_out, cudaStream_t s);
 void upload_encode_table();
 
 }  // namespace blastp

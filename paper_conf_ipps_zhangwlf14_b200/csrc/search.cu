@@ -105,11 +105,107 @@ __device__ __forceinline__ void stat_add(WarpState &st, int i, unsigned long lon
   if (kStats) st.stat[i] += v;
 }
 
+// One direction of the window-based X-drop (Alg. 5 / Fig. 8):
+// the warp scores 32 consecutive positions of the diagonal at a time, lane i
+// the position t0 + i (step +1 right from (q0, s0), -1 left), then forms the
+// PrefixSum (inclusive scan seeded with the running sum), the running best
+// (inclusive max scan seeded with the best so far) and the DropFlag
+// (best - prefix >= X); the first flagged lane stops the scan.  The best is
+// the largest prefix at or before the stop, its length the first lane that
+// reaches it (strict >, R8).  Returns (best, length); warp-uniform.
+__device__ __forceinline__ void window_xdrop(const uint8_t *__restrict__ stream, int64_t s0,
+                                             const uint8_t *qq, int q0, int step,
+                                             const int8_t *b62, int X, int lane, int &best_out,
+                                             int &len_out) {
+  int run = 0, best = 0, blen = 0;
+  for (int t0 = 0;; t0 += 32) {
+    const int t = t0 + lane;
+    const int64_t sp = s0 + int64_t(step) * t;
+    const int qi = q0 + step * t;
+    // lanes past a sentinel (sequence end) read clamped addresses: the scan
+    // stops at the sentinel, so their values are never used
+    const uint32_t sc = __ldg(stream + (sp < 0 ? 0 : sp));
+    const uint32_t qcv = qq[qi < -kQPad ? -kQPad : qi];
+    int P = score(b62, qcv, sc);
+    if (lane == 0) P += run;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int v = __shfl_up_sync(kFull, P, d);
+      if (lane >= d) P += v;
+    }
+    int Mx = max(P, best);
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const int v = __shfl_up_sync(kFull, Mx, d);
+      if (lane >= d) Mx = max(Mx, v);
+    }
+    const unsigned drop = __ballot_sync(kFull, Mx - P >= X);
+    const int stop = drop ? __ffs(drop) - 1 : 31;  // last lane that counts
+    const int mx = __shfl_sync(kFull, Mx, stop);
+    if (mx > best) {
+      const unsigned at = __ballot_sync(kFull, lane <= stop && P == mx);
+      blen = t0 + __ffs(at);
+      best = mx;
+    }
+    if (drop) break;
+    run = __shfl_sync(kFull, P, 31);
+  }
+  best_out = best;
+  len_out = blen;
+}
+
+// Alg. 5 (ext_mode WINDOW): the queued passing hits in queue (= s) order, one
+// at a time; a hit covered by its diagonal's ext_reach is skipped before any
+// work (Alg. 3 L19), otherwise the warp extends it with window_xdrop in both
+// directions and sets ext_reach = the HSP's subject end (R10).
+template <bool kTrace>
+__device__ void flush_queue_window(const SearchArgs &a, const WarpSmem &w, WarpState &st, int n,
+                                   const uint8_t *qc, const int8_t *b62, int lane, int slotc,
+                                   int M) {
+  const uint8_t *qq = qc + kQPad;
+  for (int j = 0; j < n; ++j) {
+    const uint32_t ent = w.queue[(st.qhead + j) & (kQcap - 1)];
+    const int P = int(ent & 0xffffu), q = int(ent >> 16);
+    int slot = (P - q + slotc) % M;
+    slot += slot < 0 ? M : 0;
+    if (P <= int(w.reach[slot])) continue;  // covered (warp-uniform)
+    const int64_t sp = st.spbase + P;
+    const int seed = score(b62, qq[q], __ldg(a.stream + sp)) +
+                     score(b62, qq[q + 1], __ldg(a.stream + sp + 1)) +
+                     score(b62, qq[q + 2], __ldg(a.stream + sp + 2));
+    int br, rlen, bl, llen;
+    window_xdrop(a.stream, sp + 3, qq, q + 3, 1, b62, a.xdrop, lane, br, rlen);
+    window_xdrop(a.stream, sp - 1, qq, q - 1, -1, b62, a.xdrop, lane, bl, llen);
+    const int total = seed + br + bl;
+    __syncwarp();
+    if (lane == 0) w.reach[slot] = uint16_t(min(P + 2 + rlen, 0xffff));
+    __syncwarp();
+    if (kTrace) {
+      stat_add<kTrace>(st, kStatExtended, 1);
+      stat_add<kTrace>(st, kStatAccepted, 1);
+      stat_add<kTrace>(st, kStatEmitted, total >= a.cutoff ? 1 : 0);
+    }
+    if (lane == 0) {
+      if (kTrace) trace_push(a, 2, sp, q, llen, rlen, total);
+      emit_hsp(a, sp, q, llen, rlen, total, st.first_subj, st.last_subj);
+    }
+  }
+  __syncwarp();
+  st.qhead = (st.qhead + n) & (kQcap - 1);
+  st.qcount -= n;
+}
+
 // Extend up to 32 queued passing hits lane-parallel, then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order.
-template <bool kTrace>
+// kWin: ext_mode WINDOW, a kernel instantiation of its own (the window scan
+// inlined into the default kernel cost it 15% through register allocation).
+template <bool kTrace, bool kWin>
 __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &st, int n,
                             const uint8_t *qc, const int8_t *b62, int lane, int slotc, int M) {
+  if constexpr (kWin) {
+    flush_queue_window<kTrace>(a, w, st, n, qc, b62, lane, slotc, M);
+    return;
+  }
   const bool act = lane < n;
   uint32_t ent = 0;
   if (act) ent = w.queue[(st.qhead + lane) & (kQcap - 1)];
@@ -180,7 +276,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
 
 // OffT: uint16_t (table in shared memory) or uint32_t (table in global memory);
 // kW: min_gap fixed at compile time (3, the default) or 0 (runtime value).
-template <bool kTrace, bool kEither, typename OffT, int kW>
+template <bool kTrace, bool kEither, typename OffT, int kW, bool kWin>
 __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const SearchArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
@@ -463,7 +559,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         } else {
           const int sc = slotc();
           while (st.qcount > 0)
-            flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
+            flush_queue<kTrace, kWin>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
         }
         rebase_ring();
         win -= kFrameSpan;
@@ -607,7 +703,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
             if (__shfl_sync(kFull, w.wk[4], 0) >= 0)
               spill(32);  // segment: to its list
             else
-              flush_queue<kTrace>(a, w, st, 32, qc, b62, lane, slotc(), M);
+              flush_queue<kTrace, kWin>(a, w, st, 32, qc, b62, lane, slotc(), M);
           }
         }
         __syncwarp();
@@ -635,7 +731,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     base_slot = (base_slot + 64) % M;
     }  // walk
     // ---- the single drain site (chunk end, walker steps) -------------------
-    while (st.qcount > 0) flush_queue<kTrace>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
+    while (st.qcount > 0) flush_queue<kTrace, kWin>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
   }
   cp_async_wait_all();
   if (kTrace && a.stats && lane == 0)
@@ -654,8 +750,9 @@ size_t smem_bytes(int lq, int ring, int64_t table_entries, int warps) {
 template <bool kTrace, bool kEither, typename OffT>
 cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_sms,
                            cudaStream_t s) {
-  auto k = a.min_gap == 3 ? search_warp_kernel<kTrace, kEither, OffT, 3>
-                          : search_warp_kernel<kTrace, kEither, OffT, 0>;
+  auto k = a.ext_mode == BLASTP_EXT_WINDOW ? search_warp_kernel<kTrace, kEither, OffT, 0, true>
+           : a.min_gap == 3                ? search_warp_kernel<kTrace, kEither, OffT, 3, false>
+                                           : search_warp_kernel<kTrace, kEither, OffT, 0, false>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
   int per_sm = 0;

@@ -8,9 +8,17 @@
 // returns one extension per seed, R14).  Output formatting only -- not part
 // of the timed hot path.
 #include <cub/device/device_radix_sort.cuh>
+#include <cub/device/device_select.cuh>
 #include <cuda_runtime.h>
 
 #include "common.cuh"
+
+// record equality (all 7 fields) for cub::DeviceSelect::Unique
+__host__ __device__ inline bool operator==(const blastp_hsp &a, const blastp_hsp &b) {
+  return a.query_id == b.query_id && a.subject_id == b.subject_id && a.diagonal == b.diagonal &&
+         a.q_start == b.q_start && a.s_start == b.s_start && a.length == b.length &&
+         a.score == b.score;
+}
 
 namespace blastp {
 
@@ -78,6 +86,28 @@ cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s) {
   cudaFreeAsync(idx2, s);
   cudaFreeAsync(key, s);
   cudaFreeAsync(key2, s);
+  cudaFreeAsync(tmp, s);
+  cudaFreeAsync(temp, s);
+  if (e != cudaSuccess) return e;
+  return cudaGetLastError();
+}
+
+// Adjacent duplicates of a sorted list collapse to one (cub::DeviceSelect::Unique
+// into a temporary, then copied back); the count lands in *d_n_out (device).
+cudaError_t unique_hsps(blastp_hsp *d, int64_t n, int64_t *d_n_out, cudaStream_t s) {
+  if (n <= 0) return cudaMemsetAsync(d_n_out, 0, sizeof(int64_t), s);
+  if (n > int64_t(0x7fffffff)) return cudaErrorInvalidValue;
+  blastp_hsp *tmp = nullptr;
+  void *temp = nullptr;
+  size_t temp_bytes = 0;
+  cudaError_t e = cub::DeviceSelect::Unique(nullptr, temp_bytes, d, tmp, d_n_out, n, s);
+  if (e != cudaSuccess) return e;
+  if ((e = cudaMallocAsync(&tmp, size_t(n) * sizeof(blastp_hsp), s)) != cudaSuccess) return e;
+  if ((e = cudaMallocAsync(&temp, temp_bytes, s)) == cudaSuccess) {
+    e = cub::DeviceSelect::Unique(temp, temp_bytes, d, tmp, d_n_out, n, s);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(d, tmp, size_t(n) * sizeof(blastp_hsp), cudaMemcpyDeviceToDevice, s);
+  }
   cudaFreeAsync(tmp, s);
   cudaFreeAsync(temp, s);
   if (e != cudaSuccess) return e;

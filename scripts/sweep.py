@@ -1,6 +1,7 @@
 """Strategy sweep on B200 (the paper's E1-E3 comparisons, re-run
 on this implementation): kernel variant (warp rings / CTA bins, BLASTP_KERNEL)
-x extension strategy (diagonal-based Alg. 3 / hit-based Alg. 4) x two-hit
+x extension strategy (diagonal-based Alg. 3 / hit-based Alg. 4 / window-based
+Alg. 5, warp variant; the CTA variant runs Alg. 3 for WINDOW) x two-hit
 reading (LEFT / EITHER) on configs 1-3.  Device time per search (CUDA events
 on the launch stream, median of `reps` after 2 warm-ups), residues/s and the
 HSP/extension counts of each cell.
@@ -31,7 +32,7 @@ for cfg in (1, 2, 3):
     cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
     for kernel in ("warp", "cta"):
         os.environ["BLASTP_KERNEL"] = kernel
-        for ext_mode in (0, 1):
+        for ext_mode in (0, 1, 2):
             for filt in (0, 1):
                 p = bp.Params(filter_mode=filt, ext_mode=ext_mode)
                 t = bp.build_query_table(q, p, stream=stream)
@@ -48,7 +49,7 @@ for cfg in (1, 2, 3):
                 n = int(cnt.item())
                 med = statistics.median(ms)
                 row = {"config": cfg, "query_len": len(q), "residues": db.residues,
-                       "kernel": kernel, "ext_mode": ["DIAGONAL", "HIT"][ext_mode],
+                       "kernel": kernel, "ext_mode": ["DIAGONAL", "HIT", "WINDOW"][ext_mode],
                        "filter": ["LEFT", "EITHER"][filt], "ms": med,
                        "residues_per_s": db.residues / (med / 1e3), "hsps": n}
                 rows.append(row)

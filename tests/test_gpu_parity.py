@@ -39,9 +39,10 @@ def hit_set(a):
 
 
 def oracle_run(orc, q_ascii, ascii, offsets, p, want_hits=False, nthreads=1, query_id=0):
+    # ext_mode WINDOW (Alg. 5) computes Alg. 3's extensions: the oracle's DIAGONAL mode
     P = orc.Params(word_len=p.word_len, threshold=p.threshold, window=p.window,
                    min_gap=p.min_gap, xdrop=p.xdrop, cutoff=p.cutoff, filter_mode=p.filter_mode,
-                   ext_mode=p.ext_mode)
+                   ext_mode=1 if p.ext_mode == 1 else 0)
     codes = orc.encode(ascii.tobytes() if hasattr(ascii, "tobytes") else ascii)
     return orc.search(orc.encode(q_ascii), codes, np.asarray(offsets, dtype=np.int64), P,
                       want_hits=want_hits, nthreads=nthreads, query_id=query_id)
@@ -72,11 +73,12 @@ def assert_same(bp, orc, q, ascii, offsets, p, trace=True, nthreads=1):
 # ------------------------------------------------------------------ configs
 
 @pytest.mark.parametrize("mode", [0, 1])
-@pytest.mark.parametrize("ext_mode", [0, 1])
+@pytest.mark.parametrize("ext_mode", [0, 1, 2])
 def test_config1_full_trace(bp, orc, mode, ext_mode):
     """Config 1 (q127 vs 1,000 subjects): hits, passing hits, every extension
-    and the HSP list identical to the oracle, both filter readings, both
-    extension strategies (Alg. 3 diagonal-based, Alg. 4 hit-based)."""
+    and the HSP list identical to the oracle, both filter readings, all three
+    extension strategies (Alg. 3 diagonal-based, Alg. 4 hit-based, Alg. 5
+    window-based = Alg. 3's results)."""
     (q,), db = config_workload(1)
     p = bp.Params(filter_mode=mode, ext_mode=ext_mode)
     g, r = assert_same(bp, orc, q, db.ascii, db.offsets, p)
@@ -119,7 +121,7 @@ def assert_sampled_parity(bp, orc, queries, ascii, offsets, g, p, blocks, subjec
         assert B[Q[h["q_start"]:h["q_start"] + h["length"]], S].sum() == h["score"]
     P = orc.Params(word_len=p.word_len, threshold=p.threshold, window=p.window,
                    min_gap=p.min_gap, xdrop=p.xdrop, cutoff=p.cutoff, filter_mode=p.filter_mode,
-                   ext_mode=p.ext_mode)
+                   ext_mode=1 if p.ext_mode == 1 else 0)
     tables = [orc.neighbourhood(Q, B, p.threshold) for Q in Qs]
     for lo, hi in blocks:
         sub_off = offsets[lo:hi + 1]
@@ -271,7 +273,7 @@ def test_fuzz_small_random(bp, orc):
                       min_gap=int(rng.choice([3, 3, 1, 2, 5])),
                       xdrop=int(rng.choice([16, 16, 5, 30])),
                       cutoff=int(rng.choice([41, 20, 0])),
-                      filter_mode=int(case % 2), ext_mode=int((case // 2) % 2))
+                      filter_mode=int(case % 2), ext_mode=int((case // 2) % 3))
         assert_same(bp, orc, q, ascii, off, p, trace=True)
 
 
@@ -285,6 +287,7 @@ def test_adversarial_low_complexity(bp, orc):
     for mode in (0, 1):
         assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=mode), trace=True)
     assert_same(bp, orc, q, ascii, off, bp.Params(ext_mode=1), trace=True)
+    assert_same(bp, orc, q, ascii, off, bp.Params(ext_mode=2), trace=True)
 
 
 def test_edge_cases(bp, orc):
@@ -387,7 +390,8 @@ def test_long_subjects_segmented(bp, orc, monkeypatch, kernel_variant, knobs):
         assert d.segments == 0
     else:
         assert d.segments >= (40000 + 9000 + 5000 + 70000) // d.segment_len
-    for mode, window, ext in ((0, 40, 0), (1, 40, 0), (0, 80, 0), (0, 256, 0), (0, 40, 1)):
+    for mode, window, ext in ((0, 40, 0), (1, 40, 0), (0, 80, 0), (0, 256, 0), (0, 40, 1),
+                              (0, 40, 2)):
         p = bp.Params(filter_mode=mode, window=window, ext_mode=ext)
         g, r = assert_same(bp, orc, q, ascii, off, p, trace=True)
         assert len(g) > 10
@@ -446,6 +450,34 @@ def test_device_variant_and_sort_match_host_variant(bp, orc):
     small = torch.zeros(7 * 3, dtype=torch.int32, device="cuda")
     bp.search_ungapped_device(t, d, small.data_ptr(), 3, cnt.data_ptr(), p)
     assert int(cnt.item()) == len(host)
+
+
+def test_hit_mode_dedup_device(bp, orc):
+    """Alg. 4 (ext_mode HIT) returns one extension per passing hit; the
+    de-duplication step the paper leaves before gapped extension
+    (blastp_unique_hsps_device after the canonical sort) gives exactly the
+    distinct HSPs of the oracle's HIT list; on a DIAGONAL list it is a no-op."""
+    import torch
+    (q,), db = config_workload(1)
+    d = bp.pack_db(db.ascii, db.offsets)
+    for ext_mode in (1, 0):
+        p = bp.Params(ext_mode=ext_mode)
+        t = bp.build_query_table(q, p)
+        cap = 1 << 16
+        out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+        cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+        bp.search_ungapped_device(t, d, out.data_ptr(), cap, cnt.data_ptr(), p)
+        n = int(cnt.item())
+        bp.sort_hsps_device(out.data_ptr(), n)
+        bp.unique_hsps_device(out.data_ptr(), n, cnt.data_ptr())
+        m = int(cnt.item())
+        got = [tuple(x) for x in out[: m * 7].view(m, 7).cpu().numpy().tolist()]
+        ref = tuples(oracle_run(orc, q, db.ascii, db.offsets, p).hsps)
+        assert got == sorted(set(ref))
+        if ext_mode == 1:
+            assert m < n  # there were duplicates
+        else:
+            assert m == n
 
 
 def _host_db_search(bp, t, ascii, off, p, **kw):
@@ -518,7 +550,7 @@ def test_same_start_hsps_canonical_order(bp, orc):
     """HSPs equal in (query, subject, diagonal, q_start) are ordered by
     length as R11 requires, on the host (GPU-sorted) and device variants."""
     q, ascii, off = _same_start_db(orc)
-    for ext_mode in (0, 1):
+    for ext_mode in (0, 1, 2):
         p = bp.Params(ext_mode=ext_mode)
         g, r = assert_same(bp, orc, q, ascii, off, p, trace=True)
         assert len({x[:4] for x in tuples(g)}) < len(g)
