@@ -155,6 +155,45 @@ void oracle_two_hit(const int32_t *s, int32_t n, int32_t min_gap,
   }
 }
 
+/* Alg. 1 L8-19, filter_mode 2 (STATEFUL; reading R15): walk
+ * the hits of one diagonal in ascending s with one `lasthit`.  distance =
+ * h - lasthit; no lasthit (first hit of the diagonal in this subject) or
+ * distance >= window: lasthit <- h (L17-19); min_gap <= distance < window:
+ * extend from h (L12-14) and lasthit <- the end of the extension, ext.sub_pos
+ * (L15-16; R10 reads it as the HSP's subject end, inclusive); distance <
+ * min_gap (an overlapping word, or a hit inside the last extension): no
+ * change (FSA-BLAST's rule, R15).  end_of(ctx, k) returns the subject end of
+ * the extension from hit k, which does not depend on the walk (R7). */
+typedef int32_t (*ext_end_fn)(void *ctx, int32_t k);
+
+static void stateful_walk(const int32_t *s, int32_t n, int32_t min_gap,
+                          int32_t window, ext_end_fn end_of, void *ctx,
+                          uint8_t *trigger) {
+  int32_t have = 0, lasthit = 0;
+  for (int32_t k = 0; k < n; ++k) {
+    trigger[k] = 0;
+    const int32_t h = s[k];
+    if (!have || h - lasthit >= window) { /* L17-19 */
+      lasthit = h;
+      have = 1;
+      continue;
+    }
+    if (h - lasthit < min_gap) continue; /* R15 */
+    trigger[k] = 1;                      /* L11-14 */
+    lasthit = end_of(ctx, k);            /* L15-16 */
+  }
+}
+
+static int32_t end_from_array(void *ctx, int32_t k) {
+  return ((const int32_t *)ctx)[k];
+}
+
+void oracle_two_hit_stateful(const int32_t *s, int32_t n,
+                             const int32_t *ext_end, int32_t min_gap,
+                             int32_t window, uint8_t *trigger) {
+  stateful_walk(s, n, min_gap, window, end_from_array, (void *)ext_end, trigger);
+}
+
 /* ---------------------------------------------------------- search, R4-R11 */
 
 typedef struct {
@@ -209,10 +248,65 @@ typedef struct {
   const int32_t *pos;
   oracle_hitlist *hits, *passing;
   int collect_ext; /* keep every extension (else only count them) */
+  int64_t cur_subject; /* subject being searched (index in offsets) */
   /* outputs */
   hsp_vec out, ext;
   int err;
 } range_job;
+
+/* R7-R9: the extension from the hit at subject position h of diagonal d:
+ * seed word [q, q+w) x [h, h+w), then independent X-drop to the right (from
+ * q+w, h+w) and to the left (from q-1, h-1).  Returns the HSP's subject end
+ * (inclusive), the ext_reach / lasthit value of R10 / R15. */
+static int32_t extend_hit(const range_job *J, const uint8_t *S, int32_t ls,
+                          int32_t d, int32_t h, oracle_hsp *e) {
+  const oracle_params *p = J->p;
+  const int32_t w = p->word_len, lq = J->lq, na = J->na, q = h - d;
+  int32_t s0 = 0;
+  for (int32_t k2 = 0; k2 < w; ++k2)
+    s0 += J->matrix[J->query[q + k2] * na + S[h + k2]];
+  int32_t nr = lq - (q + w), nl = q;
+  if (ls - (h + w) < nr) nr = ls - (h + w);
+  if (h < nl) nl = h;
+  int32_t bestR, rlen, stepsR, bestL, llen, stepsL;
+  oracle_xdrop_pairs(J->query + q + w, S + h + w, nr, +1, J->matrix, na,
+                     p->xdrop, &bestR, &rlen, &stepsR);
+  oracle_xdrop_pairs(J->query + q - 1, S + h - 1, nl, -1, J->matrix, na,
+                     p->xdrop, &bestL, &llen, &stepsL);
+  e->query_id = J->query_id;
+  e->subject_id = (int32_t)(J->subject_base + J->cur_subject);
+  e->diagonal = d;
+  e->q_start = q - llen;
+  e->s_start = h - llen;
+  e->length = llen + w + rlen;
+  e->score = s0 + bestL + bestR;
+  return h + w - 1 + rlen; /* HSP subject end, inclusive */
+}
+
+/* Keep an extension (every one, emitted or not) and emit it iff its score
+ * reaches the cutoff (R10).  Nonzero on allocation failure. */
+static int record_ext(range_job *J, const oracle_hsp *e) {
+  if (J->collect_ext) {
+    if (hsp_push(&J->ext, e)) return 1;
+  } else {
+    J->ext.n++;
+  }
+  if (e->score >= J->p->cutoff && hsp_push(&J->out, e)) return 1;
+  return 0;
+}
+
+typedef struct {
+  range_job *J;
+  const uint8_t *S;
+  int32_t ls, d;
+  const int32_t *H;
+  oracle_hsp scratch;
+} ext_ctx;
+
+static int32_t ext_end_of(void *ctx, int32_t k) {
+  ext_ctx *X = (ext_ctx *)ctx;
+  return extend_hit(X->J, X->S, X->ls, X->d, X->H[k], &X->scratch);
+}
 
 static void search_range(range_job *J) {
   const oracle_params *p = J->p;
@@ -225,6 +319,7 @@ static void search_range(range_job *J) {
     const uint8_t *S = J->db + J->offsets[i];
     const int32_t ls = (int32_t)(J->offsets[i + 1] - J->offsets[i]);
     const int32_t subj = (int32_t)(J->subject_base + i);
+    J->cur_subject = i;
     if (ls < w || lq < w) continue;
 
     /* Hit detection (Alg. 1 L1-4; R4): scan the subject left to
@@ -276,6 +371,24 @@ static void search_range(range_job *J) {
       if (n == 0) continue;
       const int32_t d = di - (lq - w);
       const int32_t *H = hs + dstart[di];
+      if (p->filter_mode == 2) {
+        /* Alg. 1 L8-19 (STATEFUL, R15): the walk decides which hits are
+         * extended; each extension is the same R7-R9 extension as below. */
+        ext_ctx X = {J, S, ls, d, H, {0, 0, 0, 0, 0, 0, 0}};
+        stateful_walk(H, n, p->min_gap, p->window, ext_end_of, &X, pass);
+        for (int32_t k = 0; k < n; ++k) {
+          if (!pass[k]) continue;
+          hitlist_push(J->passing, subj, H[k] - d, H[k]);
+        }
+        /* record the extensions (recomputed: the walk only kept the ends) */
+        for (int32_t k = 0; k < n && !J->err; ++k) {
+          if (!pass[k]) continue;
+          oracle_hsp e;
+          extend_hit(J, S, ls, d, H[k], &e);
+          if (record_ext(J, &e)) J->err = 1;
+        }
+        continue;
+      }
       /* Two-hit filter (R6). */
       oracle_two_hit(H, n, p->min_gap, p->window, p->filter_mode, pass);
       /* Diagonal-based ungapped extension (Alg. 3): walk the
@@ -284,39 +397,14 @@ static void search_range(range_job *J) {
       int32_t ext_reach = -1;
       for (int32_t k = 0; k < n; ++k) {
         if (!pass[k]) continue;
-        const int32_t h = H[k], q = h - d;
-        hitlist_push(J->passing, subj, q, h);
+        const int32_t h = H[k];
+        hitlist_push(J->passing, subj, h - d, h);
         /* Alg. 3 L19: skip a hit covered by the previous extension of the
          * diagonal (DIAGONAL); Alg. 4 L9-14 extends every hit (HIT). */
         if (p->ext_mode == 0 && h <= ext_reach) continue;
-        /* R7: seed word [q, q+w) x [h, h+w), then independent X-drop to the
-         * right (from q+w, h+w) and to the left (from q-1, h-1). */
-        int32_t s0 = 0;
-        for (int32_t k2 = 0; k2 < w; ++k2)
-          s0 += J->matrix[J->query[q + k2] * na + S[h + k2]];
-        int32_t nr = lq - (q + w), nl = q;
-        if (ls - (h + w) < nr) nr = ls - (h + w);
-        if (h < nl) nl = h;
-        int32_t bestR, rlen, stepsR, bestL, llen, stepsL;
-        oracle_xdrop_pairs(J->query + q + w, S + h + w, nr, +1, J->matrix, na,
-                           p->xdrop, &bestR, &rlen, &stepsR);
-        oracle_xdrop_pairs(J->query + q - 1, S + h - 1, nl, -1, J->matrix, na,
-                           p->xdrop, &bestL, &llen, &stepsL);
         oracle_hsp e;
-        e.query_id = J->query_id;
-        e.subject_id = subj;
-        e.diagonal = d;
-        e.q_start = q - llen;
-        e.s_start = h - llen;
-        e.length = llen + w + rlen;
-        e.score = s0 + bestL + bestR;
-        ext_reach = h + w - 1 + rlen; /* HSP subject end, inclusive */
-        if (J->collect_ext) {
-          if (hsp_push(&J->ext, &e)) { J->err = 1; break; }
-        } else {
-          J->ext.n++;
-        }
-        if (e.score >= p->cutoff && hsp_push(&J->out, &e)) { J->err = 1; break; }
+        ext_reach = extend_hit(J, S, ls, d, h, &e);
+        if (record_ext(J, &e)) { J->err = 1; break; }
       }
     }
   }

@@ -24,6 +24,10 @@
  *                                    neighbourhood-size statistics
  *   oracle_xdrop_pairs       pinned: Fig. 8 worked example, X=inf closed form
  *   oracle_two_hit           pinned: Fig. 7 example (both modes), O(n^2) brute force
+ *   oracle_two_hit_stateful  pinned: hand-walked Alg. 1 examples (tests/golden/
+ *                                    alg1_stateful.json), = LEFT on diagonals of
+ *                                    <= 2 hits, covering-extension special case,
+ *                                    trigger spacing invariant
  *   oracle_search            pinned: P5-P9 invariants, independent oracle-B
  *                                    (oracle/oracle_b.py) on random tiny cases,
  *                                    planted exact copies, E[hits] closed form;
@@ -55,7 +59,9 @@ typedef struct {
   int32_t min_gap;     /* non-overlap distance, = word_len (R6)              */
   int32_t xdrop;       /* X: stop when best - run >= X (R8)                  */
   int32_t cutoff;      /* emit iff score >= cutoff (R10)                     */
-  int32_t filter_mode; /* 0 = LEFT (R6 default), 1 = EITHER (Fig. 7 reading) */
+  int32_t filter_mode; /* 0 = LEFT (R6 default), 1 = EITHER (Fig. 7 reading),
+                          2 = STATEFUL: Alg. 1 L8-19's lasthit walk (R15),
+                          which also decides coverage (ext_mode ignored) */
   int32_t ext_mode;    /* 0 = DIAGONAL: Alg. 3 coverage chain (R10, default);
                           1 = HIT: Alg. 4, every
                           passing hit extended independently, duplicates kept */
@@ -104,6 +110,17 @@ void oracle_xdrop_pairs(const uint8_t *a, const uint8_t *b, int32_t n,
  * range for some m. */
 void oracle_two_hit(const int32_t *s, int32_t n, int32_t min_gap,
                     int32_t window, int32_t mode, uint8_t *pass);
+
+/* Alg. 1 L8-19 (R15): the STATEFUL walk over the ascending
+ * subject positions s[0..n) of the hits of ONE diagonal of ONE subject.
+ * ext_end[k] = subject end (inclusive) of the extension from hit k (R7-R10;
+ * it does not depend on the walk).  trigger[k] = 1 iff hit k is extended:
+ * lasthit <- h when there is none or h - lasthit >= window; extend when
+ * min_gap <= h - lasthit < window, then lasthit <- ext_end[k]; otherwise
+ * (h - lasthit < min_gap) nothing changes. */
+void oracle_two_hit_stateful(const int32_t *s, int32_t n,
+                             const int32_t *ext_end, int32_t min_gap,
+                             int32_t window, uint8_t *trigger);
 
 /* Full search of one query against the subjects of `db` (codes,
  * concatenated; subject i is db[offsets[i] .. offsets[i+1]) ).

@@ -57,7 +57,7 @@ class Params:
     min_gap: int = 3
     xdrop: int = 16
     cutoff: int = 41
-    filter_mode: int = 0  # 0 LEFT, 1 EITHER
+    filter_mode: int = 0  # 0 LEFT, 1 EITHER, 2 STATEFUL (Alg. 1 lasthit walk, R15)
     ext_mode: int = 0  # 0 DIAGONAL (Alg. 3 coverage chain), 1 HIT (Alg. 4)
 
     def _c(self) -> _Params:
@@ -88,6 +88,9 @@ def lib():
         L.oracle_two_hit.restype = None
         L.oracle_two_hit.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
                                      ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]
+        L.oracle_two_hit_stateful.restype = None
+        L.oracle_two_hit_stateful.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p,
+                                              ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]
         L.oracle_search.restype = ctypes.c_int64
         L.oracle_search.argtypes = [
             ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,  # query, lq, qid
@@ -157,6 +160,17 @@ def two_hit(s, min_gap: int = 3, window: int = 40, mode: int = 0) -> np.ndarray:
     s = np.ascontiguousarray(s, dtype=np.int32)
     out = np.zeros(len(s), dtype=np.uint8)
     lib().oracle_two_hit(_ptr(s), len(s), min_gap, window, mode, _ptr(out))
+    return out.astype(bool)
+
+
+def two_hit_stateful(s, ext_end, min_gap: int = 3, window: int = 40) -> np.ndarray:
+    """Alg. 1 L8-19 walk (R15): which hits of one diagonal are extended, given the
+    subject end of the extension from each hit."""
+    s = np.ascontiguousarray(s, dtype=np.int32)
+    e = np.ascontiguousarray(ext_end, dtype=np.int32)
+    assert len(e) == len(s)
+    out = np.zeros(len(s), dtype=np.uint8)
+    lib().oracle_two_hit_stateful(_ptr(s), len(s), _ptr(e), min_gap, window, _ptr(out))
     return out.astype(bool)
 
 

@@ -10,7 +10,9 @@ with oracle.c except the definition of the method in PAPER.md:
 * X-drop is a direct loop over the diagonal, written from the ChangeSinceBest
   / DropFlag description of Fig. 8 (P:L1579-1693, R8);
 * coverage follows Alg. 3 L19-23 (R10); ext_mode=1 is Alg. 4
-  (P:L1465-1486): every passing hit is extended, no coverage test.
+  (P:L1465-1486): every passing hit is extended, no coverage test;
+* mode=2 (STATEFUL, R15) is Alg. 1 L8-19 written as a scan of
+  the diagonal position by position with the lasthit register.
 
 Results are returned as a sorted list of 7-tuples (R11).
 """
@@ -55,6 +57,24 @@ def search_b(Q, subjects, M, *, T=11, w=3, A=40, W=3, X=16, cutoff=41, mode=0,
                 if sum(M[Q[q + j]][S[s + j]] for j in range(w)) >= T:
                     H.append(s)
             if not H:
+                continue
+            if mode == 2:
+                # Alg. 1: one register per diagonal, updated at every hit
+                lasthit = None
+                for h in H:
+                    dist = None if lasthit is None else h - lasthit
+                    if dist is None or dist >= A:
+                        lasthit = h          # L17-19
+                    elif dist >= W:          # L11-16
+                        q = h - d
+                        seed = sum(M[Q[q + j]][S[h + j]] for j in range(w))
+                        gr, rl = _extend_one_side(Q, S, q + w, h + w, +1, M, X)
+                        gl, ll = _extend_one_side(Q, S, q - 1, h - 1, -1, M, X)
+                        rec = (query_id, sid, d, q - ll, h - ll, ll + w + rl, seed + gl + gr)
+                        exts.append(rec)
+                        if rec[6] >= cutoff:
+                            hsps.append(rec)
+                        lasthit = h + w - 1 + rl
                 continue
             reach = -1
             for h in H:
