@@ -46,6 +46,12 @@ extern "C" {
 #define BLASTP_MAX_SUBJECT_LEN (1 << 30)
 #define BLASTP_FILTER_LEFT 0   /* R6 default: W <= h - p < A              */
 #define BLASTP_FILTER_EITHER 1 /* Fig. 7 reading: W <= |h - p| < A        */
+#define BLASTP_FILTER_STATEFUL 2 /* Alg. 1 L8-19, reading R15: one lasthit per
+                                    diagonal; h - lasthit >= A (or none): lasthit <- h;
+                                    W <= h - lasthit < A: extend, lasthit <- HSP subject
+                                    end; else no change.  Decides coverage itself, so it
+                                    requires ext_mode BLASTP_EXT_DIAGONAL.  Warp kernel
+                                    only; long subjects are walked whole (no segments). */
 #define BLASTP_EXT_DIAGONAL 0  /* Alg. 3: a passing hit covered by the
                                   previous extension of its diagonal is skipped (R10) */
 #define BLASTP_EXT_HIT 1       /* Alg. 4: every passing
@@ -64,7 +70,7 @@ typedef struct {
   int32_t min_gap;     /* non-overlap distance (R6), 1..8; default = word_len */
   int32_t xdrop;       /* X: stop when best - run >= X (Fig. 8, R8), 1..127   */
   int32_t cutoff;      /* emit an extension iff score >= cutoff (R10)         */
-  int32_t filter_mode; /* BLASTP_FILTER_LEFT or BLASTP_FILTER_EITHER          */
+  int32_t filter_mode; /* BLASTP_FILTER_LEFT, _EITHER or _STATEFUL            */
   int32_t ext_mode;    /* BLASTP_EXT_DIAGONAL (default), _HIT or _WINDOW       */
 } blastp_params;
 

@@ -75,8 +75,12 @@ int validate_params(const blastp_params *p) {
     return fail(BLASTP_E_INVALID_ARG, "xdrop %d outside [1, 127]", p->xdrop);
   if (p->threshold < -100 || p->threshold > 100)
     return fail(BLASTP_E_INVALID_ARG, "threshold %d outside [-100, 100]", p->threshold);
-  if (p->filter_mode != BLASTP_FILTER_LEFT && p->filter_mode != BLASTP_FILTER_EITHER)
+  if (p->filter_mode != BLASTP_FILTER_LEFT && p->filter_mode != BLASTP_FILTER_EITHER &&
+      p->filter_mode != BLASTP_FILTER_STATEFUL)
     return fail(BLASTP_E_INVALID_ARG, "filter_mode %d unknown", p->filter_mode);
+  if (p->filter_mode == BLASTP_FILTER_STATEFUL && p->ext_mode != BLASTP_EXT_DIAGONAL)
+    return fail(BLASTP_E_INVALID_ARG, "filter_mode STATEFUL decides coverage itself: ext_mode "
+                "must be DIAGONAL (got %d)", p->ext_mode);
   if (p->ext_mode != BLASTP_EXT_DIAGONAL && p->ext_mode != BLASTP_EXT_HIT &&
       p->ext_mode != BLASTP_EXT_WINDOW)
     return fail(BLASTP_E_INVALID_ARG, "ext_mode %d unknown", p->ext_mode);
@@ -680,7 +684,9 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.nchunks = db->nchunks;
     a.long_items = db->items;
     a.nlong = db->nlong;
-    a.nsegs = db->nsegs;
+    // STATEFUL's walk state at a segment start depends on the whole subject
+    // before it (extension ends), so long subjects are walked whole
+    a.nsegs = p->filter_mode == BLASTP_FILTER_STATEFUL ? 0 : db->nsegs;
     a.seg_item = db->seg_item;
     a.seg_list = db->seg_list;
     a.seg_count = db->seg_count;

@@ -195,22 +195,78 @@ __device__ void flush_queue_window(const SearchArgs &a, const WarpSmem &w, WarpS
   st.qcount -= n;
 }
 
+// ext_mode DIAGONAL without speculation: of the n flushed entries, those
+// covered by their diagonal's ext_reach are dropped; of the rest, the first
+// of each diagonal (queue = s order) is extended (and always accepted: it is
+// beyond ext_reach, Alg. 3 L19), its ext_reach set to the HSP end (R10); the
+// later entries of that diagonal stay at the head of the queue for the next
+// flush, where ext_reach has moved past the extension just made.  No
+// extension is computed and then thrown away.
+template <bool kTrace>
+__device__ void flush_queue_defer(const SearchArgs &a, const WarpSmem &w, WarpState &st, int n,
+                                  const uint8_t *qc, const int8_t *b62, int lane, int slotc,
+                                  int M) {
+  const bool act = lane < n;
+  const uint32_t ent = act ? w.queue[(st.qhead + lane) & (kQcap - 1)] : 0u;
+  const int P = int(ent & 0xffffu);
+  const int q = int(ent >> 16);
+  int slot = (P - q + slotc) % M;
+  slot += slot < 0 ? M : 0;
+  const bool unc = act && P > int(w.reach[slot]);
+  const unsigned grp = __match_any_sync(kFull, unc ? slot : -1 - lane);
+  const bool ext = unc && (grp & lanemask_lt(lane)) == 0u;
+  const bool keep = unc && !ext;
+  const int64_t sp = st.spbase + P;
+  int total = 0, llen = 0, rlen = 0, scanned = 0;
+  if (ext) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen, scanned);
+  if (kTrace) {
+    stat_add<kTrace>(st, kStatFlushes, 1);
+    stat_add<kTrace>(st, kStatExtended, __popc(__ballot_sync(kFull, ext)));
+    stat_add<kTrace>(st, kStatXdropSteps, __reduce_add_sync(kFull, unsigned(scanned)));
+    stat_add<kTrace>(st, kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(scanned)));
+    stat_add<kTrace>(st, kStatAccepted, __popc(__ballot_sync(kFull, ext)));
+    stat_add<kTrace>(st, kStatEmitted, __popc(__ballot_sync(kFull, ext && total >= a.cutoff)));
+  }
+  if (ext) {
+    w.reach[slot] = uint16_t(min(P + 2 + rlen, 0xffff));  // one extending lane per slot
+    if (kTrace) trace_push(a, 2, sp, q, llen, rlen, total);
+    emit_hsp(a, sp, q, llen, rlen, total, st.first_subj, st.last_subj);
+  }
+  const unsigned kb = __ballot_sync(kFull, keep);
+  const int nk = __popc(kb);
+  __syncwarp();
+  if (keep) w.queue[(st.qhead + n - nk + __popc(kb & lanemask_lt(lane))) & (kQcap - 1)] = ent;
+  __syncwarp();
+  st.qhead = (st.qhead + n - nk) & (kQcap - 1);
+  st.qcount -= n - nk;
+}
+
 // Extend up to 32 queued passing hits lane-parallel, then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order.
 // kWin: ext_mode WINDOW, a kernel instantiation of its own (the window scan
 // inlined into the default kernel cost it 15% through register allocation).
-template <bool kTrace, bool kWin>
+// kSt: filter mode STATEFUL (Alg. 1 L8-19, R15): the queued entries' walk
+// is finished here (see the round code in search_warp_kernel).
+template <bool kTrace, bool kWin, int kSt>
 __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &st, int n,
                             const uint8_t *qc, const int8_t *b62, int lane, int slotc, int M) {
   if constexpr (kWin) {
     flush_queue_window<kTrace>(a, w, st, n, qc, b62, lane, slotc, M);
     return;
   }
+#ifdef BLASTP_FLUSH_DEFER
+  if constexpr (!kSt) {
+    if (a.ext_mode == BLASTP_EXT_DIAGONAL) {
+      flush_queue_defer<kTrace>(a, w, st, n, qc, b62, lane, slotc, M);
+      return;
+    }
+  }
+#endif
   const bool act = lane < n;
   uint32_t ent = 0;
   if (act) ent = w.queue[(st.qhead + lane) & (kQcap - 1)];
   const int P = int(ent & 0xffffu);
-  const int q = int(ent >> 16);
+  const int q = kSt ? int((ent >> 16) & 0x3fffu) : int(ent >> 16);
   // ring slot of the diagonal: (base_slot - win) + P - q (mod M), slotc given
   int slot = (P - q + slotc) % M;
   slot += slot < 0 ? M : 0;
@@ -226,7 +282,48 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   const int endp = min(P + 2 + rlen, 0xffff);  // HSP subject end (inclusive), frame
   bool acc = false;
   uint16_t *reach16 = w.reach + slot;
-  if (a.ext_mode == BLASTP_EXT_HIT) {
+  if constexpr (kSt) {
+    // Finish Alg. 1's walk over the flushed entries of each diagonal, in
+    // queue (= s) order, from the slot's lasthit: a trigger (bit 31) was
+    // decided at enqueue; a fresh entry (bit 30) starts a new subject (no
+    // lasthit); any other entry applies L11-19 to the lasthit the walk has
+    // reached.  An accepted extension sets lasthit = its subject end.
+    const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
+    const uint32_t e = act ? w.ring[slot] : 0u;
+    uint32_t cur = e & 0xffffu;
+    const int gmax = __reduce_max_sync(kFull, act ? __popc(grp) : 0);
+    const uint32_t fl = ent >> 30;
+    unsigned rem = act ? grp : 0u;
+    for (int it = 0; it < gmax; ++it) {
+      const int src = rem ? __ffs(rem) - 1 : lane;
+      const bool valid = rem != 0;
+      rem &= rem - 1;
+      const int Pj = __shfl_sync(kFull, P, src);
+      const int Ej = __shfl_sync(kFull, endp, src);
+      const uint32_t fj = __shfl_sync(kFull, fl, src);
+      if (valid) {
+        bool aj;
+        if (fj & 2u) {
+          aj = true;
+        } else {
+          if (fj & 1u) cur = 0;
+          const int d = Pj - int(cur);
+          aj = false;
+          if (cur == 0 || d >= a.window) cur = uint32_t(Pj);
+          else if (d >= a.min_gap) aj = true;
+        }
+        if (aj) cur = uint32_t(Ej);
+        if (src == lane) acc = aj;
+      }
+    }
+    __syncwarp();
+    if (act && (grp >> lane) == 1u) w.ring[slot] = cur | (((e >> 16) - __popc(grp)) << 16);
+    __syncwarp();
+    if (kTrace) {
+      stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, acc)));
+      if (acc) trace_push(a, 1, sp, q, 0, 0, 0);
+    }
+  } else if (a.ext_mode == BLASTP_EXT_HIT) {
     // Alg. 4: every passing hit is extended and kept; ext_reach
     // is never written, so every passing hit was also queued
     acc = act;
@@ -274,10 +371,13 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   st.qcount -= n;
 }
 
+// kF: filter mode, BLASTP_FILTER_LEFT / _EITHER / _STATEFUL;
 // OffT: uint16_t (table in shared memory) or uint32_t (table in global memory);
 // kW: min_gap fixed at compile time (3, the default) or 0 (runtime value).
-template <bool kTrace, bool kEither, typename OffT, int kW, bool kWin>
+template <bool kTrace, int kF, typename OffT, int kW, bool kWin>
 __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const SearchArgs a) {
+  constexpr bool kEither = kF == BLASTP_FILTER_EITHER;
+  constexpr int kSt = kF == BLASTP_FILTER_STATEFUL;
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
   int8_t *b62 = reinterpret_cast<int8_t *>(smem);
@@ -377,7 +477,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         const LongItem it = a.long_items[ci - nsegs];
         st.first_subj = it.c.first_subj;
         st.last_subj = it.c.last_subj;
-        if (it.nseg > 0) {
+        if (it.nseg > 0 && !kSt) {
           st.spbase = it.c.start - frame;
           if (lane == 0) {
             w.wk[0] = int(ci - nsegs);
@@ -403,7 +503,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         walk = true;
       }
     }
-    if (mode == 1) {
+    if (!kSt && mode == 1) {
       // ---- walker step: the segments' passing hits, in s order, into the
       // extension queue (the ext_reach chain resolves at the drain, exactly
       // as in a walk); returns whenever the queue must be drained first
@@ -559,7 +659,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         } else {
           const int sc = slotc();
           while (st.qcount > 0)
-            flush_queue<kTrace, kWin>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
+            flush_queue<kTrace, kWin, kSt>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
         }
         rebase_ring();
         win -= kFrameSpan;
@@ -593,34 +693,35 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
 
       // round r's owner lane and query position are computed (and the query
       // position load issued) one round ahead of its processing
-      auto owner_of = [&](uint32_t k) {  // number of lanes with incl <= k
-        int own = 0;
-#pragma unroll
-        for (int b = 16; b >= 1; b >>= 1) {
-          const uint32_t v = __shfl_sync(kFull, incl, own + b - 1);
-          if (v <= k) own += b;
-        }
-        return own;
-      };
-      auto load_q = [&](uint32_t k, int own) -> int {
-        const uint32_t o_own = __shfl_sync(kFull, o, own);
-        const uint32_t e_own = __shfl_sync(kFull, excl, own);
-        return k < Hn ? int(qpos[o_own + (k - e_own)]) : 0;
+      // Owner lane and query position of hit kb + lane, through a 32-entry
+      // per-warp scratch (the flush scratch; free here): each lane whose run
+      // of hits intersects [kb, kb + 32) stores (lane, table offset - excl)
+      // at the slot of its run's first hit in the round; a hit's owner is the
+      // last run start at or before it, from the OR-reduced start mask
+      // (measured: 1.1% faster than a 5-step shuffle binary search over the
+      // inclusive counts, profiles/r01/ab_locate.txt)
+      uint32_t *scr = reinterpret_cast<uint32_t *>(w.fs_p);
+      auto locate = [&](uint32_t kb, int &own_out, int &q_out) {
+        const bool wr = cnt != 0u && excl < kb + 32u && incl > kb;
+        const int p0 = wr ? max(int(excl) - int(kb), 0) : 0;
+        if (wr) scr[p0] = uint32_t(lane) | ((o - excl) << 5);
+        const unsigned S = __reduce_or_sync(kFull, wr ? (1u << p0) : 0u);
+        __syncwarp();
+        const int src = 31 - __clz(S & (kFull >> (31 - lane)));
+        const uint32_t v = scr[src];
+        own_out = int(v & 31u);
+        const uint32_t k = kb + uint32_t(lane);
+        q_out = k < Hn ? int(qpos[((v >> 5) + k) & 0x7ffffffu]) : 0;
+        __syncwarp();
       };
       int nown = 0, nq = 0;
-      if (Hn) {
-        nown = owner_of(uint32_t(lane));
-        nq = load_q(uint32_t(lane), nown);
-      }
+      if (Hn) locate(0u, nown, nq);
       for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
         const uint32_t k = k0 + uint32_t(lane);
         const bool act = k < Hn;
         const int own = nown;
         int q = nq;
-        if (k0 + 32 < Hn) {
-          nown = owner_of(k + 32);
-          nq = load_q(k + 32, nown);
-        }
+        if (k0 + 32 < Hn) locate(k0 + 32u, nown, nq);
         const int ls = __shfl_sync(kFull, ls_lane, own);
         int slot = 0;
         const int Ph = win + own;
@@ -636,74 +737,131 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           e = w.ring[slot];
           rch = w.reach[slot];
         }
-        const uint32_t last = st_last(e), near = st_near(e);
-        // R6 predecessor among stored hits: the largest one <= Ph - W
-        const int hi_ok = Ph - W;
-        const int lo_ok = max(Ph - A + 1, ls + 1);  // within A, same subject
-        const int cand_s = st_pred(last, st_far(e), near, hi_ok);
-        // earlier hits of this round on the same diagonal (rare per lane, but
-        // some in almost every round): the best predecessor among them and
-        // the mask of those within W of this hit
-        int cand_e = 0;
-        uint32_t nb = 0;
-        const int nearly = __reduce_max_sync(kFull, __popc(earlier));
-        if (nearly) {
-          unsigned rem = earlier;
-          for (int it = 0; it < nearly; ++it) {
+        bool enq = false;
+        uint32_t eflags = 0;  // STATEFUL queue-entry flags (bit 31 trigger, bit 30 fresh)
+        if constexpr (kSt) {
+          // Alg. 1 L8-19 (R15) at enqueue time.  Slot state: lasthit L (0:
+          // none) | count of queued, unresolved entries << 16; reach[] = the
+          // position of the last queued entry.  While entries are queued the
+          // lasthit depends on their extensions: later hits are queued too
+          // (conditional) and the walk finishes at the flush, in queue order.
+          // Members of a round group replay the group's walk in lane (= s)
+          // order; each keeps its own decision.
+          uint32_t L = e & 0xffffu, cnt = e >> 16, rq = rch;
+          const int gmax = __reduce_max_sync(kFull, act ? __popc(grp) : 0);
+          unsigned rem = act ? grp : 0u;
+          for (int it = 0; it < gmax; ++it) {
             const int src = rem ? __ffs(rem) - 1 : lane;
+            const bool valid = rem != 0;
             rem &= rem - 1;
             const int Pj = __shfl_sync(kFull, Ph, src);
-            if (act && src != lane) {
-              if (Pj <= hi_ok) cand_e = max(cand_e, Pj);
-              const int d = Ph - Pj;
-              if (d < W) nb |= 1u << d;
+            const int lsj = __shfl_sync(kFull, ls, src);
+            if (valid) {
+              bool ej = false;
+              uint32_t fj = 0;
+              if (cnt > 0) {
+                ej = true;
+                fj = int(rq) <= lsj ? (1u << 30) : 0u;  // pending entries of an earlier subject
+                ++cnt;
+                rq = uint32_t(Pj);
+              } else {
+                const int d = Pj - int(L);
+                if (L == 0 || int(L) <= lsj || d >= A) {
+                  L = uint32_t(Pj);  // L17-19
+                } else if (d >= W) {  // L11-14: extend (lasthit from the flush)
+                  ej = true;
+                  fj = 1u << 31;
+                  cnt = 1;
+                  rq = uint32_t(Pj);
+                }
+              }
+              if (src == lane) {
+                enq = ej;
+                eflags = fj;
+              }
             }
           }
-        }
-        const int cand = max(cand_s, cand_e);
-        // not a segment's warm-up (the LEFT test fails there by ls above)
-        const bool counts = act && (kTrace || kEither ? Ph >= emit_f : true);
-        bool pass = counts && cand >= lo_ok;
-        const int64_t sph = st.spbase + Ph;
-        if (kEither && counts && !pass)
-          pass = has_successor(stream, sph, q, qc, b62, lq, W, A, a.threshold);
-        if (kTrace) {
-          stat_add<kTrace>(st, kStatRounds, 1);
-          stat_add<kTrace>(st, kStatConflictRounds, nearly ? 1 : 0);
-          if (!retrace) {
-            stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, counts)));
-            stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
+          if (kTrace) {
+            stat_add<kTrace>(st, kStatRounds, 1);
+            stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, act)));
+            stat_add<kTrace>(st, kStatEnqueued, __popc(__ballot_sync(kFull, enq)));
+            if (act) trace_push(a, 0, st.spbase + Ph, q, 0, 0, 0);
           }
-          if (w.wk[4] < 0)
-            stat_add<kTrace>(st, kStatEnqueued,
-                             __popc(__ballot_sync(kFull, pass && Ph > int(rch))));
-          if (counts && !retrace) {
-            trace_push(a, 0, sph, q, 0, 0, 0);
-            if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
+          __syncwarp();
+          if (act && (grp >> lane) == 1u) {
+            w.ring[slot] = L | (cnt << 16);
+            w.reach[slot] = uint16_t(rq);
           }
-        }
-        // the group's last member writes the diagonal state with its own hit:
-        // last = Ph, far = largest hit <= Ph - W (= cand), near = every hit
-        // (stored or earlier in the round) within W of Ph
-        if (act && (grp >> lane) == 1u) {
-          if (last != 0) {
-            const int d = Ph - int(last);
-            if (d < W) nb |= ((near << d) | (1u << d));
+        } else {
+          const uint32_t last = st_last(e), near = st_near(e);
+          // R6 predecessor among stored hits: the largest one <= Ph - W
+          const int hi_ok = Ph - W;
+          const int lo_ok = max(Ph - A + 1, ls + 1);  // within A, same subject
+          const int cand_s = st_pred(last, st_far(e), near, hi_ok);
+          // earlier hits of this round on the same diagonal (rare per lane, but
+          // some in almost every round): the best predecessor among them and
+          // the mask of those within W of this hit
+          int cand_e = 0;
+          uint32_t nb = 0;
+          if (const int nearly = __reduce_max_sync(kFull, __popc(earlier)); nearly) {
+            unsigned rem = earlier;
+            for (int it = 0; it < nearly; ++it) {
+              const int src = rem ? __ffs(rem) - 1 : lane;
+              rem &= rem - 1;
+              const int Pj = __shfl_sync(kFull, Ph, src);
+              if (act && src != lane) {
+                if (Pj <= hi_ok) cand_e = max(cand_e, Pj);
+                const int d = Ph - Pj;
+                if (d < W) nb |= 1u << d;
+              }
+            }
           }
-          w.ring[slot] = st_make(uint32_t(Ph), uint32_t(cand), nb & nearmask);
+          const int cand = max(cand_s, cand_e);
+          // not a segment's warm-up (the LEFT test fails there by ls above)
+          const bool counts = act && (kTrace || kEither ? Ph >= emit_f : true);
+          bool pass = counts && cand >= lo_ok;
+          const int64_t sph = st.spbase + Ph;
+          if (kEither && counts && !pass)
+            pass = has_successor(stream, sph, q, qc, b62, lq, W, A, a.threshold);
+          if (kTrace) {
+            stat_add<kTrace>(st, kStatRounds, 1);
+            stat_add<kTrace>(st, kStatConflictRounds, __any_sync(kFull, earlier != 0) ? 1 : 0);
+            if (!retrace) {
+              stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, counts)));
+              stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
+            }
+            if (w.wk[4] < 0)
+              stat_add<kTrace>(st, kStatEnqueued,
+                               __popc(__ballot_sync(kFull, pass && Ph > int(rch))));
+            if (counts && !retrace) {
+              trace_push(a, 0, sph, q, 0, 0, 0);
+              if (pass) trace_push(a, 1, sph, q, 0, 0, 0);
+            }
+          }
+          // the group's last member writes the diagonal state with its own hit:
+          // last = Ph, far = largest hit <= Ph - W (= cand), near = every hit
+          // (stored or earlier in the round) within W of Ph
+          if (act && (grp >> lane) == 1u) {
+            if (last != 0) {
+              const int d = Ph - int(last);
+              if (d < W) nb |= ((near << d) | (1u << d));
+            }
+            w.ring[slot] = st_make(uint32_t(Ph), uint32_t(cand), nb & nearmask);
+          }
+          enq = pass && Ph > int(rch);
         }
-        const bool enq = pass && Ph > int(rch);
         const unsigned bal = __ballot_sync(kFull, enq);
         if (bal) {
           const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
-          if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = uint32_t(Ph) | (uint32_t(q) << 16);
+          if (enq)
+            w.queue[(st.qhead + pos) & (kQcap - 1)] = uint32_t(Ph) | (uint32_t(q) << 16) | eflags;
           st.qcount += __popc(bal);
           __syncwarp();
-          if (st.qcount >= 32) {
+          while (st.qcount >= 32) {  // a flush may keep entries queued
             if (__shfl_sync(kFull, w.wk[4], 0) >= 0)
               spill(32);  // segment: to its list
             else
-              flush_queue<kTrace, kWin>(a, w, st, 32, qc, b62, lane, slotc(), M);
+              flush_queue<kTrace, kWin, kSt>(a, w, st, 32, qc, b62, lane, slotc(), M);
           }
         }
         __syncwarp();
@@ -731,7 +889,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     base_slot = (base_slot + 64) % M;
     }  // walk
     // ---- the single drain site (chunk end, walker steps) -------------------
-    while (st.qcount > 0) flush_queue<kTrace, kWin>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
+    while (st.qcount > 0)
+      flush_queue<kTrace, kWin, kSt>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
   }
   cp_async_wait_all();
   if (kTrace && a.stats && lane == 0)
@@ -747,12 +906,14 @@ size_t smem_bytes(int lq, int ring, int64_t table_entries, int warps) {
   return fixed + table + size_t(warps) * warp_smem_bytes(ring);
 }
 
-template <bool kTrace, bool kEither, typename OffT>
+template <bool kTrace, int kF, typename OffT>
 cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_sms,
                            cudaStream_t s) {
-  auto k = a.ext_mode == BLASTP_EXT_WINDOW ? search_warp_kernel<kTrace, kEither, OffT, 0, true>
-           : a.min_gap == 3                ? search_warp_kernel<kTrace, kEither, OffT, 3, false>
-                                           : search_warp_kernel<kTrace, kEither, OffT, 0, false>;
+  void (*k)(const SearchArgs) = search_warp_kernel<kTrace, kF, OffT, 0, false>;
+  if constexpr (kF != BLASTP_FILTER_STATEFUL) {
+    if (a.ext_mode == BLASTP_EXT_WINDOW) k = search_warp_kernel<kTrace, kF, OffT, 0, true>;
+    else if (a.min_gap == 3) k = search_warp_kernel<kTrace, kF, OffT, 3, false>;
+  }
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
   int per_sm = 0;
@@ -794,10 +955,7 @@ cudaError_t launch_search_warp(const SearchArgs &a_in, int num_sms, cudaStream_t
   cudaError_t e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
   const bool trace = a.trace[0] != nullptr;
-  const bool either = a.filter_mode == BLASTP_FILTER_EITHER;
-  // Table in shared memory when its offsets fit 16 bits and it leaves room
-  // for enough warps; otherwise the table stays in global memory (L1/L2).
-  // experiment knobs: BLASTP_TABLE=global, BLASTP_WARPS=<max warps per CTA>
+  const int fm = a.filter_mode;
   const char *tab_env = std::getenv("BLASTP_TABLE");
   const bool force_global = tab_env && !std::strcmp(tab_env, "global");
   const char *warps_env = std::getenv("BLASTP_WARPS");
@@ -814,21 +972,22 @@ cudaError_t launch_search_warp(const SearchArgs &a_in, int num_sms, cudaStream_t
   // more than a few warps (profiles/r01: q1054, 16 warps + L1/L2 table is
   // faster than 11 warps + shared-memory table).
   const bool force_smem = tab_env && !std::strcmp(tab_env, "smem");
-  if (warps_s > 0 && (force_smem || warps_s >= std::min(warps_g, 24))) {
-    const size_t smem = smem_bytes(a.qv.lq, a.ring, a.table_entries, warps_s);
-    if (trace)
-      return either ? launch_variant<true, true, uint16_t>(a, warps_s, smem, num_sms, s)
-                    : launch_variant<true, false, uint16_t>(a, warps_s, smem, num_sms, s);
-    return either ? launch_variant<false, true, uint16_t>(a, warps_s, smem, num_sms, s)
-                  : launch_variant<false, false, uint16_t>(a, warps_s, smem, num_sms, s);
-  }
-  if (warps_g < 1) return cudaErrorInvalidConfiguration;
-  const size_t smem = smem_bytes(a.qv.lq, a.ring, -1, warps_g);
-  if (trace)
-    return either ? launch_variant<true, true, uint32_t>(a, warps_g, smem, num_sms, s)
-                  : launch_variant<true, false, uint32_t>(a, warps_g, smem, num_sms, s);
-  return either ? launch_variant<false, true, uint32_t>(a, warps_g, smem, num_sms, s)
-                : launch_variant<false, false, uint32_t>(a, warps_g, smem, num_sms, s);
+  const bool use_s = warps_s > 0 && (force_smem || warps_s >= std::min(warps_g, 24));
+  if (!use_s && warps_g < 1) return cudaErrorInvalidConfiguration;
+  const int warps = use_s ? warps_s : warps_g;
+  const size_t smem = smem_bytes(a.qv.lq, a.ring, use_s ? a.table_entries : -1, warps);
+  auto pick = [&](auto off_tag) -> cudaError_t {
+    using OffT = decltype(off_tag);
+    if (trace) {
+      if (fm == BLASTP_FILTER_EITHER) return launch_variant<true, 1, OffT>(a, warps, smem, num_sms, s);
+      if (fm == BLASTP_FILTER_STATEFUL) return launch_variant<true, 2, OffT>(a, warps, smem, num_sms, s);
+      return launch_variant<true, 0, OffT>(a, warps, smem, num_sms, s);
+    }
+    if (fm == BLASTP_FILTER_EITHER) return launch_variant<false, 1, OffT>(a, warps, smem, num_sms, s);
+    if (fm == BLASTP_FILTER_STATEFUL) return launch_variant<false, 2, OffT>(a, warps, smem, num_sms, s);
+    return launch_variant<false, 0, OffT>(a, warps, smem, num_sms, s);
+  };
+  return use_s ? pick(uint16_t{}) : pick(uint32_t{});
 }
 
 }  // namespace blastp

@@ -760,7 +760,8 @@ cudaError_t launch_search(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
   // The warp variant is the default (faster on B200, profiles/r01); the CTA
   // variant runs when BLASTP_KERNEL=cta.
   const int choice = kernel_choice();
-  if (choice != 2) return launch_search_warp(a_in, num_sms, s);
+  if (choice != 2 || a_in.filter_mode == BLASTP_FILTER_STATEFUL)
+    return launch_search_warp(a_in, num_sms, s);  // STATEFUL: warp variant only
   static unsigned long long b62_ready = 0;  // one bit per device
   int dev = 0;
   cudaGetDevice(&dev);

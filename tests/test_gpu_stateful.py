@@ -1,0 +1,123 @@
+"""GPU parity of filter_mode STATEFUL (Alg. 1 L8-19; reading R15):
+the warp kernel's lasthit walk (decided at enqueue, finished at the flush in
+queue order) vs the CPU oracle, element by element -- every hit, every
+extended hit, every extension and the HSP list.  Run with -m gpu on a B200."""
+import os
+
+import numpy as np
+import pytest
+
+from synth import config_workload, gen_db, gen_query
+from test_gpu_parity import (_config3, _long_subject_db, _rand_db, assert_same,
+                             assert_sampled_parity, tuples, ALPHA)
+
+pytestmark = pytest.mark.gpu
+ST = 2  # BLASTP_FILTER_STATEFUL
+
+
+@pytest.fixture(scope="module")
+def bp():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_ipps_zhangwlf14_b200 import build
+    build.build()
+    from paper_conf_ipps_zhangwlf14_b200 import blastp
+    assert blastp.FILTER_STATEFUL == ST
+    return blastp
+
+
+@pytest.fixture(params=["warp", "cta"], autouse=True)
+def kernel_variant(request, monkeypatch):
+    """BLASTP_KERNEL=cta must route STATEFUL to the warp kernel, same results."""
+    monkeypatch.setenv("BLASTP_KERNEL", request.param)
+    return request.param
+
+
+def test_config1_full_trace(bp, orc):
+    (q,), db = config_workload(1)
+    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=ST))
+    assert len(g) > 10 and len(r.passing) > 100
+
+
+def test_config2_full(bp, orc):
+    (q,), db = config_workload(2)
+    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=ST), trace=False,
+                       nthreads=os.cpu_count() or 8)
+    assert len(g) > 1000
+
+
+def test_fuzz_small_random(bp, orc):
+    rng = np.random.default_rng(1515)
+    for case in range(80):
+        lq = int(rng.choice([3, 5, 17, 64, 127, 300, 517]))
+        q = "".join(rng.choice(list(ALPHA[:20] if case % 4 else ALPHA), size=lq))
+        ascii, off = _rand_db(rng, int(rng.integers(1, 60)), 0, 400, q)
+        p = bp.Params(threshold=int(rng.choice([11, 11, 9, 13])),
+                      window=int(rng.choice([40, 40, 10, 80, 3])),
+                      min_gap=int(rng.choice([3, 3, 1, 2, 5])),
+                      xdrop=int(rng.choice([16, 16, 5, 30])),
+                      cutoff=int(rng.choice([41, 20, 0])), filter_mode=ST)
+        assert_same(bp, orc, q, ascii, off, p, trace=True)
+
+
+def test_adversarial_low_complexity(bp, orc):
+    """Every (q, s) a hit: long runs of hits per diagonal inside one round and
+    across flushes (many conditional entries per diagonal, chains split over
+    two flushes), fresh-subject entries on a still-pending diagonal."""
+    q = "W" * 300 + "AAAAQQQQ" * 10 + "W" * 50
+    subs = ["W" * 1000, "A" * 200 + "W" * 40, "WA" * 300, "Q" * 500, "W" * 3, "W" * 45,
+            "W" * 44, "CW" * 30]
+    ascii = np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy()
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    for window, W in ((40, 3), (10, 3), (80, 1), (3, 2)):
+        assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=ST, window=window, min_gap=W),
+                    trace=True)
+
+
+def test_long_subjects_walked_whole(bp, orc):
+    """Long subjects (> 2C residues, segmented in LEFT mode) are walked whole
+    by one warp in STATEFUL mode; one subject is longer than the 16-bit frame
+    (rebases with pending entries flushed first)."""
+    q = gen_query(21, 300).decode()
+    ascii, off = _long_subject_db(q)
+    d = bp.pack_db(ascii, off)
+    assert d.segments > 0
+    for window in (40, 256):
+        g, _ = assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=ST, window=window),
+                           trace=True)
+        assert len(g) > 10
+
+
+def test_long_query_2000(bp, orc):
+    q = gen_query(2000, 2000)
+    db = gen_db(7, 8, n_subjects=400, mean_len=375.0, queries=[q], plant_frac=0.2)
+    assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=ST), trace=True)
+
+
+def test_config3_full_size_sampled(bp, orc, kernel_variant):
+    """Config 3 at full size in STATEFUL mode: sampled subject blocks re-searched
+    by the oracle, every sampled GPU HSP re-scored from the sequences."""
+    if kernel_variant == "cta":
+        pytest.skip("same kernel as the warp run")
+    (q,), db = _config3()
+    p = bp.Params(filter_mode=ST)
+    t = bp.build_query_table(q, p)
+    d = bp.pack_db(db.ascii, db.offsets)
+    g = bp.search_ungapped(t, d, p)
+    left = bp.search_ungapped(t, d, bp.Params())
+    assert len(g) > 10000 and len(g) != len(left)
+    n = db.nseq
+    blocks = [(k, min(k + 2000, n)) for k in range(0, n, n // 8)][:8]
+    blocks.append((n // 2 - 5, n // 2 + 5))  # the 36,805-residue subject
+    assert_sampled_parity(bp, orc, [q], db.ascii, db.offsets, g, p, blocks)
+
+
+def test_stateful_requires_diagonal_ext_mode(bp):
+    q = gen_query(3, 100).decode()
+    for ext in (1, 2):
+        with pytest.raises(bp.BlastpError) as e:
+            t = bp.build_query_table(q, bp.Params())
+            d = bp.pack_db(np.frombuffer(q.encode(), np.uint8).copy(), np.array([0, len(q)]))
+            bp.search_ungapped(t, d, bp.Params(filter_mode=ST, ext_mode=ext))
+        assert e.value.status == -1  # BLASTP_E_INVALID_ARG
