@@ -195,54 +195,12 @@ __device__ void flush_queue_window(const SearchArgs &a, const WarpSmem &w, WarpS
   st.qcount -= n;
 }
 
-// ext_mode DIAGONAL without speculation: of the n flushed entries, those
-// covered by their diagonal's ext_reach are dropped; of the rest, the first
-// of each diagonal (queue = s order) is extended (and always accepted: it is
-// beyond ext_reach, Alg. 3 L19), its ext_reach set to the HSP end (R10); the
-// later entries of that diagonal stay at the head of the queue for the next
-// flush, where ext_reach has moved past the extension just made.  No
-// extension is computed and then thrown away.
-template <bool kTrace>
-__device__ void flush_queue_defer(const SearchArgs &a, const WarpSmem &w, WarpState &st, int n,
-                                  const uint8_t *qc, const int8_t *b62, int lane, int slotc,
-                                  int M) {
-  const bool act = lane < n;
-  const uint32_t ent = act ? w.queue[(st.qhead + lane) & (kQcap - 1)] : 0u;
-  const int P = int(ent & 0xffffu);
-  const int q = int(ent >> 16);
-  int slot = (P - q + slotc) % M;
-  slot += slot < 0 ? M : 0;
-  const bool unc = act && P > int(w.reach[slot]);
-  const unsigned grp = __match_any_sync(kFull, unc ? slot : -1 - lane);
-  const bool ext = unc && (grp & lanemask_lt(lane)) == 0u;
-  const bool keep = unc && !ext;
-  const int64_t sp = st.spbase + P;
-  int total = 0, llen = 0, rlen = 0, scanned = 0;
-  if (ext) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen, scanned);
-  if (kTrace) {
-    stat_add<kTrace>(st, kStatFlushes, 1);
-    stat_add<kTrace>(st, kStatExtended, __popc(__ballot_sync(kFull, ext)));
-    stat_add<kTrace>(st, kStatXdropSteps, __reduce_add_sync(kFull, unsigned(scanned)));
-    stat_add<kTrace>(st, kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(scanned)));
-    stat_add<kTrace>(st, kStatAccepted, __popc(__ballot_sync(kFull, ext)));
-    stat_add<kTrace>(st, kStatEmitted, __popc(__ballot_sync(kFull, ext && total >= a.cutoff)));
-  }
-  if (ext) {
-    w.reach[slot] = uint16_t(min(P + 2 + rlen, 0xffff));  // one extending lane per slot
-    if (kTrace) trace_push(a, 2, sp, q, llen, rlen, total);
-    emit_hsp(a, sp, q, llen, rlen, total, st.first_subj, st.last_subj);
-  }
-  const unsigned kb = __ballot_sync(kFull, keep);
-  const int nk = __popc(kb);
-  __syncwarp();
-  if (keep) w.queue[(st.qhead + n - nk + __popc(kb & lanemask_lt(lane))) & (kQcap - 1)] = ent;
-  __syncwarp();
-  st.qhead = (st.qhead + n - nk) & (kQcap - 1);
-  st.qcount -= n - nk;
-}
-
 // Extend up to 32 queued passing hits lane-parallel, then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order.
+// Speculation (extending entries the chain may then reject, 22% of them on
+// config 3) is cheaper than extending only each diagonal's first uncovered
+// entry and keeping the rest queued: +8.7% per config-3 step measured
+// (profiles/r01/ab_flush_defer_rejected.txt).
 // kWin: ext_mode WINDOW, a kernel instantiation of its own (the window scan
 // inlined into the default kernel cost it 15% through register allocation).
 // kSt: filter mode STATEFUL (Alg. 1 L8-19, R15): the queued entries' walk
@@ -254,14 +212,6 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
     flush_queue_window<kTrace>(a, w, st, n, qc, b62, lane, slotc, M);
     return;
   }
-#ifdef BLASTP_FLUSH_DEFER
-  if constexpr (!kSt) {
-    if (a.ext_mode == BLASTP_EXT_DIAGONAL) {
-      flush_queue_defer<kTrace>(a, w, st, n, qc, b62, lane, slotc, M);
-      return;
-    }
-  }
-#endif
   const bool act = lane < n;
   uint32_t ent = 0;
   if (act) ent = w.queue[(st.qhead + lane) & (kQcap - 1)];

@@ -45,8 +45,9 @@ def test_gpu_arm_json_line():
     d = run_bench("--config", "1", "--steps", "3", "--warmup", "3", "--e2e-steps", "1")
     for k in REQUIRED + ["roofline", "clocks", "e2e", "gpu_launches", "cpu_baseline"]:
         assert k in d, k
-    r = d["roofline"]
+    r = d["hbm_roofline"]
     assert r["bound"] == "hbm" and 0 < r["frac"] < 1 and r["peak"] > 1000
+    assert d["roofline"]["bound"] in ("hbm", "alu") and 0 < d["roofline"]["frac"] < 1
     assert d["gpu_launches"] == 3
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle"
