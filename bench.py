@@ -415,6 +415,47 @@ def main():
                        "of part k) + "
                        + ("NCCL gather + " if world > 1 else "") + "D2H of the HSP list"}
 
+    # ---- e2e from a formatted host database (the makeblastdb layout: the
+    # shard packed once into pinned host memory, outside the timed region):
+    # every step copies each part H2D on a copy stream and searches it as soon
+    # as it lands (no per-part kernel or host synchronisation) + D2H of the HSPs
+    e2e_fmt = None
+    if not args.no_e2e and args.e2e_steps > 0 and hasattr(bp.lib, "blastp_format_host_db"):
+        t0 = time.perf_counter()
+        hdb = bp.format_host_db(base_ptr, full_off, shard_index=rank, num_shards=nshards,
+                                stream=stream)
+        fmt_ms = 1e3 * (time.perf_counter() - t0)
+        times = []
+        for k in range(args.e2e_steps + 1):
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            bp.search_formatted_db(table, hdb, out.data_ptr(), cap, cnt.data_ptr(), params,
+                                   stream=stream)
+            n = int(cnt.item())
+            res = out[: min(n, cap)]
+            if world > 1:
+                res = gather_hsps(res)
+            host = res.cpu() if res is not None else None
+            torch.cuda.synchronize()
+            dt = time.perf_counter() - t0
+            tt = torch.tensor([dt], dtype=torch.float64, device=dev)
+            all_reduce_max(tt)
+            if k > 0:
+                times.append(float(tt[0]))
+        h2d = hdb.host_bytes
+        d2h = 8 + (host.numel() * 4 if host is not None else 0)
+        e2e_fmt = {"value": total_residues * nq / statistics.mean(times), "unit": UNIT,
+                   "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+                   "ms_per_step": 1e3 * statistics.mean(times),
+                   "format_ms": fmt_ms, "parts": hdb.num_parts,
+                   "path": "blastp_format_host_db once (pinned host image of the packed parts, "
+                           "outside the timed region), then per step blastp_search_formatted_db "
+                           "(H2D of part k+1 on a copy stream while part k is searched) + "
+                           + ("NCCL gather + " if world > 1 else "") + "D2H of the HSP list"}
+        hdb.free()
+
     # ---- e2e with the shard resident in HBM (a search service: the database
     # is loaded once; each step's inputs are the query strings, its result the
     # HSP list): query table build from host strings (H2D + GPU build) +
@@ -481,7 +522,11 @@ def main():
                               "queries; blastp_pack_db of the rank's shard from pinned host "
                               "memory (H2D + encode kernels)"},
             "clocks": clk,
-            "e2e": e2e,
+            # e2e: the formatted host database streamed every step (the
+            # production layout); the ASCII-streaming and HBM-resident paths
+            # beside it
+            "e2e": e2e_fmt or e2e,
+            "e2e_ascii_db": e2e if e2e_fmt else None,
             "e2e_resident_db": e2e_res,
             "gpu_launches": args.steps * nq,
             "cpu_baseline": cpu,

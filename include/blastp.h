@@ -161,6 +161,32 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
                           void *cuda_stream, blastp_hsp *d_out, int64_t capacity,
                           int64_t *d_count);
 
+/* Formatted host database (the makeblastdb step): the shard `shard_index`
+ * of `num_shards` (as blastp_pack_db) is packed on `device` in parts
+ * (num_parts > 0: that many residue-balanced parts; 0: parts growing 1.5x
+ * from a small first one, as blastp_search_host_db) and each part's device
+ * image -- code stream, subject starts, chunk plan, long-item plan -- is
+ * copied back into one pinned host buffer owned by the handle.  Synchronous.
+ * blastp_search_formatted_db then streams the parts: one host->device copy
+ * per part on a copy stream (no kernel, no host synchronisation between
+ * parts) and the part's search on one of two alternating search streams
+ * once its copy has landed; HSPs are appended to d_out / *d_count exactly as
+ * blastp_search_ungapped_device does for the whole shard (same results as
+ * blastp_pack_db + blastp_search_ungapped_device).  Asynchronous on
+ * cuda_stream; the device image is released in stream order.  Errors: as
+ * blastp_pack_db (format) and blastp_search_ungapped_device (search),
+ * E_NOMEM if the pinned image or the device image cannot be allocated. */
+typedef struct blastp_host_db blastp_host_db;
+int blastp_format_host_db(const char *residues_ascii, const int64_t *offsets, int64_t nseq,
+                          int32_t shard_index, int32_t num_shards, int32_t num_parts,
+                          int device, void *cuda_stream, blastp_host_db **out);
+int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db *h,
+                               const blastp_params *p, void *cuda_stream, blastp_hsp *d_out,
+                               int64_t capacity, int64_t *d_count);
+int blastp_host_db_info(const blastp_host_db *h, int64_t *nseq, int64_t *residues,
+                        int64_t *subject_base, int32_t *num_parts, int64_t *host_bytes);
+void blastp_host_db_free(blastp_host_db *h);
+
 /* Long-subject plan of the shard (implementation detail, exposed for tests
  * and tuning): chunks longer than 2C residues that are scheduled first
  * (*long_items), the segments they are split into for parallel two-hit

@@ -89,6 +89,12 @@ def _load():
     if hasattr(L, "blastp_search_host_db"):  # absent in older builds (A/B timing)
         L.blastp_search_host_db.argtypes = [vp, vp, vp, i64, i32, i32, P(_CParams), i32, vp, vp,
                                             i64, vp]
+    if hasattr(L, "blastp_format_host_db"):  # absent in older builds (A/B timing)
+        L.blastp_format_host_db.argtypes = [vp, vp, i64, i32, i32, i32, ctypes.c_int, vp, P(vp)]
+        L.blastp_search_formatted_db.argtypes = [vp, vp, P(_CParams), vp, vp, i64, vp]
+        L.blastp_host_db_info.argtypes = [vp, P(i64), P(i64), P(i64), P(i32), P(i64)]
+        L.blastp_host_db_free.argtypes = [vp]
+        L.blastp_host_db_free.restype = None
     L.blastp_sort_hsps_device.argtypes = [vp, i64, vp]
     L.blastp_unique_hsps_device.argtypes = [vp, i64, vp, vp]
     L.blastp_debug_trace.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64), vp, i64, P(i64),
@@ -108,6 +114,8 @@ EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "bl
             "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
             "blastp_shard_range", "blastp_db_info", "blastp_db_long_info", "blastp_query_table_info",
             "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_search_host_db",
+            "blastp_format_host_db", "blastp_search_formatted_db", "blastp_host_db_info",
+            "blastp_host_db_free",
             "blastp_sort_hsps_device", "blastp_unique_hsps_device",
             "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
@@ -313,6 +321,57 @@ def search_host_db(table: QueryTable, residues, offsets: np.ndarray, out_ptr: in
                                      _stream_handle(stream), out_ptr, capacity, count_ptr),
            "blastp_search_host_db")
     return keep
+
+
+class HostDb:
+    """A shard formatted into pinned host memory (blastp_format_host_db)."""
+
+    def __init__(self, handle):
+        self.handle = handle
+        vals = [ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int32(),
+                ctypes.c_int64()]
+        _check(lib.blastp_host_db_info(handle, *[ctypes.byref(v) for v in vals]),
+               "blastp_host_db_info")
+        self.nseq, self.residues, self.subject_base, self.num_parts, self.host_bytes = \
+            (v.value for v in vals)
+
+    def free(self):
+        if self.handle:
+            lib.blastp_host_db_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def format_host_db(residues, offsets: np.ndarray, shard_index: int = 0, num_shards: int = 1,
+                   num_parts: int = 0, device: int = 0, stream=None) -> HostDb:
+    """Pack a shard once into ready-to-stream parts in pinned host memory."""
+    off = np.ascontiguousarray(offsets, dtype=np.int64)
+    if isinstance(residues, int):
+        ptr = residues
+    else:
+        keep = np.frombuffer(residues, dtype=np.uint8) if isinstance(residues, (bytes, bytearray)) \
+            else np.ascontiguousarray(residues)
+        ptr = keep.ctypes.data
+    h = ctypes.c_void_p()
+    _check(lib.blastp_format_host_db(ptr, off.ctypes.data, len(off) - 1, shard_index, num_shards,
+                                     num_parts, device, _stream_handle(stream), ctypes.byref(h)),
+           "blastp_format_host_db")
+    return HostDb(h.value)
+
+
+def search_formatted_db(table: QueryTable, hdb: HostDb, out_ptr: int, capacity: int,
+                        count_ptr: int, params: Params | None = None, stream=None):
+    """Stream a formatted host shard through the search (blastp_search_formatted_db):
+    HSPs appended at out_ptr (device), count at count_ptr; asynchronous."""
+    c = (params or table.params).c()
+    _check(lib.blastp_search_formatted_db(table.handle, hdb.handle, ctypes.byref(c),
+                                          _stream_handle(stream), out_ptr, capacity, count_ptr),
+           "blastp_search_formatted_db")
 
 
 def sort_hsps_device(ptr: int, n: int, stream=None):

@@ -754,6 +754,42 @@ static void db_free_async(blastp_db *db, cudaStream_t s) {
   delete db;
 }
 
+// Part boundaries of a streamed shard [lo, hi) (whole subjects, by
+// residues): num_parts equal parts, or (num_parts = 0) sizes growing 1.5x
+// from a small first part -- its copy is the only one not hidden behind a
+// search, and each part copies faster than the previous one is searched.
+static std::vector<int64_t> part_cuts(const int64_t *offsets, int64_t lo, int64_t hi,
+                                      int32_t num_parts) {
+  const int64_t total = offsets[hi] - offsets[lo];
+  std::vector<int64_t> cut{lo};
+  // knobs (tuning): BLASTP_PIPE_FIRST residues of the first part,
+  // BLASTP_PIPE_GROWTH percent growth per part
+  int64_t want = std::max<int64_t>(int64_t(1) << 24, total / 64);
+  if (const char *v = std::getenv("BLASTP_PIPE_FIRST")) want = std::max<int64_t>(1, std::atoll(v));
+  int growth = 150;
+  if (const char *v = std::getenv("BLASTP_PIPE_GROWTH")) growth = std::max(101, std::atoi(v));
+  int64_t done = 0;
+  for (int k = 0; cut.back() < hi; ++k) {
+    int64_t size;
+    if (num_parts > 0)
+      size = (total * (k + 1)) / num_parts - done;
+    else {
+      size = want;
+      want = want * growth / 100;
+    }
+    const int64_t target = offsets[lo] + done + std::max<int64_t>(size, 1);
+    // first subject starting at or after target
+    int64_t a = cut.back() + 1, b = hi;
+    while (a < b) {
+      const int64_t m = (a + b) >> 1;
+      if (offsets[m] >= target) b = m; else a = m + 1;
+    }
+    cut.push_back(a);
+    done = offsets[a] - offsets[lo];
+  }
+  return cut;
+}
+
 int blastp_search_host_db(const blastp_query_table *q, const char *residues_ascii,
                           const int64_t *offsets, int64_t nseq, int32_t shard_index,
                           int32_t num_shards, const blastp_params *p, int32_t num_parts,
@@ -777,39 +813,9 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
   cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
   auto *count = reinterpret_cast<unsigned long long *>(d_count);
   CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
-  // Part boundaries (whole subjects, by residues): sizes grow 1.5x from a
-  // small first part -- its copy is the only one not hidden behind a search,
-  // and each part copies faster than the previous one is searched.
   const int64_t total = offsets[hi] - offsets[lo];
   if (total < 0) return fail(BLASTP_E_INVALID_ARG, "offsets decrease");
-  std::vector<int64_t> cut{lo};
-  {
-    // knobs (tuning): BLASTP_PIPE_FIRST residues of the first part,
-    // BLASTP_PIPE_GROWTH percent growth per part
-    int64_t want = std::max<int64_t>(int64_t(1) << 24, total / 64);
-    if (const char *v = std::getenv("BLASTP_PIPE_FIRST")) want = std::max<int64_t>(1, std::atoll(v));
-    int growth = 150;
-    if (const char *v = std::getenv("BLASTP_PIPE_GROWTH")) growth = std::max(101, std::atoi(v));
-    int64_t done = 0;
-    for (int k = 0; cut.back() < hi; ++k) {
-      int64_t size;
-      if (num_parts > 0)
-        size = (total * (k + 1)) / num_parts - done;
-      else {
-        size = want;
-        want = want * growth / 100;
-      }
-      const int64_t target = offsets[lo] + done + std::max<int64_t>(size, 1);
-      // first subject starting at or after target
-      int64_t a = cut.back() + 1, b = hi;
-      while (a < b) {
-        const int64_t m = (a + b) >> 1;
-        if (offsets[m] >= target) b = m; else a = m + 1;
-      }
-      cut.push_back(a);
-      done = offsets[a] - offsets[lo];
-    }
-  }
+  const std::vector<int64_t> cut = part_cuts(offsets, lo, hi, num_parts);
   cudaStream_t cs = nullptr;  // copy + pack stream
   CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
   // one arena for every part's packed buffers + shared staging buffers
@@ -932,6 +938,258 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
     }
     for (cudaEvent_t e : ev) cudaEventDestroy(e);
   }
+  return rc;
+}
+
+// ------------------------------------------------- formatted host database
+// A shard packed once (the makeblastdb step of a BLAST installation) and kept
+// in pinned host memory as ready-to-copy parts: each part's code stream,
+// subject starts, chunk plan and long-item plan are the device buffers of a
+// blastp_pack_db of that part, copied back.  A search then only copies them
+// (copy engine, no kernel and no host synchronisation per part) and searches.
+struct HostPart {
+  int64_t nseq = 0, residues = 0, subject_base = 0, stream_len = 0;
+  int32_t nchunks = 0, nlong = 0, nsegs = 0, seg_len = kSegLen, seg_cap = kSegCap;
+  size_t off_stream = 0, off_sstart = 0, off_chunks = 0, off_items = 0, off_seg_item = 0;
+};
+struct blastp_host_db {
+  int device = 0;
+  int64_t nseq = 0, residues = 0, subject_base = 0;
+  std::vector<HostPart> parts;
+  uint8_t *buf = nullptr;  // pinned
+  size_t bytes = 0;
+};
+
+static size_t al256(size_t b) { return (b + 255) & ~size_t(255); }
+
+int blastp_format_host_db(const char *residues_ascii, const int64_t *offsets, int64_t nseq,
+                          int32_t shard_index, int32_t num_shards, int32_t num_parts,
+                          int device, void *cuda_stream, blastp_host_db **out) {
+  if (!out) return fail(BLASTP_E_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (!offsets || nseq < 0) return fail(BLASTP_E_INVALID_ARG, "offsets NULL or nseq < 0");
+  if (num_parts < 0) return fail(BLASTP_E_INVALID_ARG, "num_parts %d < 0", num_parts);
+  int64_t lo = 0, hi = 0;
+  int rc = blastp_shard_range(offsets, nseq, shard_index, num_shards, &lo, &hi);
+  if (rc) return rc;
+  if (offsets[hi] - offsets[lo] < 0) return fail(BLASTP_E_INVALID_ARG, "offsets decrease");
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  const std::vector<int64_t> cut = part_cuts(offsets, lo, hi, num_parts);
+  auto *h = new (std::nothrow) blastp_host_db;
+  if (!h) return fail(BLASTP_E_NOMEM, "host allocation failed");
+  h->device = device;
+  h->nseq = hi - lo;
+  h->residues = offsets[hi] - offsets[lo];
+  h->subject_base = lo;
+  std::vector<blastp_db *> dbs;
+  auto cleanup = [&](int code) {
+    for (blastp_db *d : dbs) blastp_db_free(d);
+    if (code != BLASTP_OK) blastp_host_db_free(h);
+    return code;
+  };
+  // pack every part on the device and lay out the host image; then copy
+  // each part back
+  size_t bytes = 0;
+  for (size_t k = 0; k + 1 < cut.size(); ++k) {
+    blastp_db *d = nullptr;
+    rc = pack_range(residues_ascii, offsets, cut[k], cut[k + 1], device, s, &d);
+    if (rc) return cleanup(rc);
+    HostPart hp;
+    hp.nseq = d->nseq;
+    hp.residues = d->residues;
+    hp.subject_base = d->subject_base;
+    hp.stream_len = d->stream_len;
+    hp.nchunks = d->nchunks;
+    hp.nlong = d->nlong;
+    hp.nsegs = d->nsegs;
+    hp.seg_len = d->seg_len;
+    hp.seg_cap = d->seg_cap;
+    hp.off_stream = bytes;
+    bytes += al256(size_t(hp.stream_len));
+    hp.off_sstart = bytes;
+    bytes += al256(sizeof(int64_t) * size_t(std::max<int64_t>(hp.nseq, 1)));
+    hp.off_chunks = bytes;
+    bytes += al256(sizeof(Chunk) * size_t(std::max(hp.nchunks, 1)));
+    hp.off_items = bytes;
+    bytes += al256(sizeof(LongItem) * size_t(std::max(hp.nlong, 1)));
+    hp.off_seg_item = bytes;
+    bytes += al256(sizeof(int32_t) * size_t(std::max(hp.nsegs, 1)));
+    h->parts.push_back(hp);
+    dbs.push_back(d);  // kept until the host image (sized by all parts) exists
+  }
+  if (cudaMallocHost(reinterpret_cast<void **>(&h->buf), std::max<size_t>(bytes, 1)) != cudaSuccess) {
+    cudaGetLastError();
+    return cleanup(fail(BLASTP_E_NOMEM, "pinned host image of %zu bytes", bytes));
+  }
+  h->bytes = bytes;
+  cudaError_t e = cudaSuccess;
+  for (size_t k = 0; k < dbs.size() && e == cudaSuccess; ++k) {
+    const blastp_db *d = dbs[k];
+    const HostPart &hp = h->parts[k];
+    e = cudaMemcpyAsync(h->buf + hp.off_stream, d->stream, size_t(hp.stream_len),
+                        cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && hp.nseq > 0)
+      e = cudaMemcpyAsync(h->buf + hp.off_sstart, d->sstart, sizeof(int64_t) * size_t(hp.nseq),
+                          cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && hp.nchunks > 0)
+      e = cudaMemcpyAsync(h->buf + hp.off_chunks, d->chunks, sizeof(Chunk) * size_t(hp.nchunks),
+                          cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && hp.nlong > 0)
+      e = cudaMemcpyAsync(h->buf + hp.off_items, d->items, sizeof(LongItem) * size_t(hp.nlong),
+                          cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess && hp.nsegs > 0)
+      e = cudaMemcpyAsync(h->buf + hp.off_seg_item, d->seg_item,
+                          sizeof(int32_t) * size_t(hp.nsegs), cudaMemcpyDeviceToHost, s);
+  }
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess)
+    return cleanup(fail(BLASTP_E_CUDA, "copying the formatted parts back: %s", cudaGetErrorString(e)));
+  *out = h;
+  return cleanup(BLASTP_OK);
+}
+
+int blastp_host_db_info(const blastp_host_db *h, int64_t *nseq, int64_t *residues,
+                        int64_t *subject_base, int32_t *num_parts, int64_t *host_bytes) {
+  if (!h) return fail(BLASTP_E_INVALID_ARG, "host db is NULL");
+  if (nseq) *nseq = h->nseq;
+  if (residues) *residues = h->residues;
+  if (subject_base) *subject_base = h->subject_base;
+  if (num_parts) *num_parts = static_cast<int32_t>(h->parts.size());
+  if (host_bytes) *host_bytes = static_cast<int64_t>(h->bytes);
+  return BLASTP_OK;
+}
+
+void blastp_host_db_free(blastp_host_db *h) {
+  if (!h) return;
+  if (h->buf) cudaFreeHost(h->buf);
+  delete h;
+}
+
+int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db *h,
+                               const blastp_params *p, void *cuda_stream, blastp_hsp *d_out,
+                               int64_t capacity, int64_t *d_count) {
+  if (!q || !h) return fail(BLASTP_E_INVALID_ARG, "table or host db is NULL");
+  int rc = validate_params(p);
+  if (rc) return rc;
+  if (p->threshold != q->p.threshold || p->word_len != q->p.word_len)
+    return fail(BLASTP_E_INVALID_ARG, "threshold/word_len differ from the table's (%d/%d)",
+                q->p.threshold, q->p.word_len);
+  if (q->device != h->device)
+    return fail(BLASTP_E_INVALID_ARG, "table on device %d, host db formatted for device %d",
+                q->device, h->device);
+  if (!d_count || capacity < 0 || (capacity > 0 && !d_out))
+    return fail(BLASTP_E_INVALID_ARG, "bad output buffer");
+  DeviceGuard g(q->device);
+  if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", q->device, cudaGetErrorString(g.err));
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  auto *count = reinterpret_cast<unsigned long long *>(d_count);
+  CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
+  // device image: the host image's layout plus per-part scratch (counters,
+  // segment lists / counts / publication flags)
+  std::vector<size_t> scratch_off(h->parts.size());
+  size_t bytes = al256(h->bytes);
+  for (size_t k = 0; k < h->parts.size(); ++k) {
+    const HostPart &hp = h->parts[k];
+    const size_t ns = size_t(std::max(hp.nsegs, 1));
+    scratch_off[k] = bytes;
+    bytes += al256(64) + al256(4 * ns) + al256(4 * ns) + al256(4 * ns * size_t(hp.seg_cap));
+  }
+  {
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, q->device) == cudaSuccess) {
+      uint64_t thr = ~uint64_t(0);
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  cudaStream_t cs = nullptr, s2 = nullptr;
+  CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+  if (cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking) != cudaSuccess) {
+    cudaGetLastError();
+    cudaStreamDestroy(cs);
+    return fail(BLASTP_E_CUDA, "could not create the second search stream");
+  }
+  bytes = std::max<size_t>(bytes, 256);
+  uint8_t *dev = nullptr;
+  // the arena is allocated in s's order; the copies on cs wait for that
+  if (cudaMallocAsync(reinterpret_cast<void **>(&dev), bytes, s) != cudaSuccess) {
+    cudaGetLastError();
+    cudaStreamDestroy(cs);
+    cudaStreamDestroy(s2);
+    return fail(BLASTP_E_NOMEM, "device image of %zu bytes for the formatted search", bytes);
+  }
+  std::vector<cudaEvent_t> evs;
+  auto event = [&]() {
+    cudaEvent_t e = nullptr;
+    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) == cudaSuccess) evs.push_back(e);
+    return e;
+  };
+  cudaEvent_t ev_start = event();
+  cudaEventRecord(ev_start, s);  // arena allocated, count reset
+  cudaStreamWaitEvent(cs, ev_start, 0);
+  cudaStreamWaitEvent(s2, ev_start, 0);
+  std::vector<blastp_db> dbs(h->parts.size());
+  rc = BLASTP_OK;
+  for (size_t k = 0; k < h->parts.size() && rc == BLASTP_OK; ++k) {
+    const HostPart &hp = h->parts[k];
+    blastp_db &d = dbs[k];
+    d.device = h->device;
+    d.sms = num_sms(h->device);
+    d.nseq = hp.nseq;
+    d.residues = hp.residues;
+    d.subject_base = hp.subject_base;
+    d.stream_len = hp.stream_len;
+    d.nchunks = hp.nchunks;
+    d.nlong = hp.nlong;
+    d.nsegs = hp.nsegs;
+    d.seg_len = hp.seg_len;
+    d.seg_cap = hp.seg_cap;
+    d.carved = true;
+    d.stream = dev + hp.off_stream;
+    d.sstart = reinterpret_cast<int64_t *>(dev + hp.off_sstart);
+    d.chunks = reinterpret_cast<Chunk *>(dev + hp.off_chunks);
+    d.items = reinterpret_cast<LongItem *>(dev + hp.off_items);
+    d.seg_item = reinterpret_cast<int32_t *>(dev + hp.off_seg_item);
+    const size_t ns = size_t(std::max(hp.nsegs, 1));
+    uint8_t *sc = dev + scratch_off[k];
+    d.counters = reinterpret_cast<unsigned long long *>(sc);
+    sc += al256(64);
+    d.seg_count = reinterpret_cast<int32_t *>(sc);
+    sc += al256(4 * ns);
+    d.seg_done = reinterpret_cast<unsigned *>(sc);
+    sc += al256(4 * ns);
+    d.seg_list = reinterpret_cast<uint32_t *>(sc);
+    // copy engine only: the part's image in one copy (its buffers are
+    // contiguous in the image)
+    const size_t end = k + 1 < h->parts.size() ? h->parts[k + 1].off_stream : h->bytes;
+    cudaError_t e = cudaMemcpyAsync(dev + hp.off_stream, h->buf + hp.off_stream,
+                                    end - hp.off_stream, cudaMemcpyHostToDevice, cs);
+    cudaEvent_t ready = event();
+    if (e == cudaSuccess) e = cudaEventRecord(ready, cs);
+    cudaStream_t ss = (k & 1) ? s2 : s;
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(ss, ready, 0);
+    // per-part scratch reset (segment epochs start at 0; searches bump seq)
+    if (e == cudaSuccess) e = cudaMemsetAsync(d.seg_done, 0, 4 * ns, ss);
+    if (e == cudaSuccess) e = cudaMemsetAsync(d.counters, 0, 64, ss);
+    if (e != cudaSuccess) {
+      rc = fail(BLASTP_E_CUDA, "enqueueing part %zu: %s", k, cudaGetErrorString(e));
+      break;
+    }
+    rc = enqueue_search(q, &d, p, ss, d_out, capacity, count, nullptr, nullptr, nullptr, false);
+  }
+  // join s2 into s, then release the arena in s's order
+  cudaEvent_t ev_join = event();
+  cudaEventRecord(ev_join, s2);
+  cudaStreamWaitEvent(s, ev_join, 0);
+  cudaEvent_t ev_copy = event();
+  cudaEventRecord(ev_copy, cs);
+  cudaStreamWaitEvent(s, ev_copy, 0);
+  cudaFreeAsync(dev, s);
+  for (cudaEvent_t e : evs) cudaEventDestroy(e);
+  cudaStreamDestroy(cs);
+  cudaStreamDestroy(s2);
+  for (blastp_db &d : dbs) d.carved = true;  // nothing owned: the arena holds it all
   return rc;
 }
 

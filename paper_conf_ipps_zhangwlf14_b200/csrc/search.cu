@@ -61,35 +61,43 @@ __device__ __forceinline__ uint32_t st_make(uint32_t last, uint32_t far, uint32_
   return last | (fd << 16) | (near << 24);
 }
 
+// Per-warp shared-memory area: the fixed-size parts first, so that every
+// address is the warp's base plus a constant (reach: plus a launch-uniform
+// offset) -- one base register, no per-array pointers to keep or recompute.
+//   [0, 256)     queue[kQcap]: P | q << 16 (the slot is recomputed at flush)
+//   [256, 448)   flush scratch fs_p, fs_end, fs_acc [32] u16 (also the
+//                owner-lookup scratch, 32 u32 over fs_p/fs_end)
+//   [448, 480)   wk[8]: walker state: item, segment, entry, slot offset;
+//                [4] segment being filtered (-1: none), [5] its list length
+//   [480, ...)   ring[M] two-hit state, then reach[M] ext_reach (16-bit)
+constexpr int kRingOff = 480;
 struct WarpSmem {
-  uint32_t *ring;    // [M] two-hit state
-  uint16_t *reach;   // [M] ext_reach (frame position, 0 = none)
-  uint32_t *queue;   // [kQcap]: P | q << 16 (the slot is recomputed at flush)
-  uint16_t *fs_p, *fs_end, *fs_acc;  // [32] flush scratch
-  int *wk;           // [8] walker state: item, segment, entry, slot offset;
-                     // [4] segment being filtered (-1: none), [5] its list length
+  uint8_t *base;
+  int reach_off;  // kRingOff + align16(4 M)
+  __device__ __forceinline__ uint32_t *queue() const { return reinterpret_cast<uint32_t *>(base); }
+  __device__ __forceinline__ uint16_t *fs_p() const { return reinterpret_cast<uint16_t *>(base + 256); }
+  __device__ __forceinline__ uint16_t *fs_end() const { return fs_p() + 32; }
+  __device__ __forceinline__ uint16_t *fs_acc() const { return fs_p() + 64; }
+  __device__ __forceinline__ int *wk() const { return reinterpret_cast<int *>(base + 448); }
+  __device__ __forceinline__ uint32_t *ring() const {
+    return reinterpret_cast<uint32_t *>(base + kRingOff);
+  }
+  __device__ __forceinline__ uint16_t *reach() const {
+    return reinterpret_cast<uint16_t *>(base + reach_off);
+  }
 };
 
-// Per-warp shared memory: 6 B per diagonal slot + 352 B; small enough for
+// Per-warp shared memory: 6 B per diagonal slot + 480 B; small enough for
 // 30+ resident warps per SM at Lq ~ 1000 (occupancy is what this latency-
 // bound kernel runs on, profiles/r01).
 __host__ __device__ size_t warp_smem_bytes(int ring) {
-  return align16(size_t(ring) * 4) + align16(size_t(ring) * 2) + size_t(kQcap) * 4 + 3 * 32 * 2 +
-         32;
+  return kRingOff + align16(size_t(ring) * 4) + align16(size_t(ring) * 2);
 }
 
 __device__ __forceinline__ WarpSmem carve(uint8_t *base, int ring) {
   WarpSmem w;
-  w.ring = reinterpret_cast<uint32_t *>(base);
-  base += align16(size_t(ring) * 4);
-  w.reach = reinterpret_cast<uint16_t *>(base);
-  base += align16(size_t(ring) * 2);
-  w.queue = reinterpret_cast<uint32_t *>(base);
-  base += size_t(kQcap) * 4;
-  w.fs_p = reinterpret_cast<uint16_t *>(base);
-  w.fs_end = w.fs_p + 32;
-  w.fs_acc = w.fs_p + 64;
-  w.wk = reinterpret_cast<int *>(w.fs_p + 96);
+  w.base = base;
+  w.reach_off = kRingOff + int(align16(size_t(ring) * 4));
   return w;
 }
 
@@ -164,11 +172,11 @@ __device__ void flush_queue_window(const SearchArgs &a, const WarpSmem &w, WarpS
                                    int M) {
   const uint8_t *qq = qc + kQPad;
   for (int j = 0; j < n; ++j) {
-    const uint32_t ent = w.queue[(st.qhead + j) & (kQcap - 1)];
+    const uint32_t ent = w.queue()[(st.qhead + j) & (kQcap - 1)];
     const int P = int(ent & 0xffffu), q = int(ent >> 16);
     int slot = (P - q + slotc) % M;
     slot += slot < 0 ? M : 0;
-    if (P <= int(w.reach[slot])) continue;  // covered (warp-uniform)
+    if (P <= int(w.reach()[slot])) continue;  // covered (warp-uniform)
     const int64_t sp = st.spbase + P;
     const int seed = score(b62, qq[q], __ldg(a.stream + sp)) +
                      score(b62, qq[q + 1], __ldg(a.stream + sp + 1)) +
@@ -178,7 +186,7 @@ __device__ void flush_queue_window(const SearchArgs &a, const WarpSmem &w, WarpS
     window_xdrop(a.stream, sp - 1, qq, q - 1, -1, b62, a.xdrop, lane, bl, llen);
     const int total = seed + br + bl;
     __syncwarp();
-    if (lane == 0) w.reach[slot] = uint16_t(min(P + 2 + rlen, 0xffff));
+    if (lane == 0) w.reach()[slot] = uint16_t(min(P + 2 + rlen, 0xffff));
     __syncwarp();
     if (kTrace) {
       stat_add<kTrace>(st, kStatExtended, 1);
@@ -214,7 +222,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   }
   const bool act = lane < n;
   uint32_t ent = 0;
-  if (act) ent = w.queue[(st.qhead + lane) & (kQcap - 1)];
+  if (act) ent = w.queue()[(st.qhead + lane) & (kQcap - 1)];
   const int P = int(ent & 0xffffu);
   const int q = kSt ? int((ent >> 16) & 0x3fffu) : int(ent >> 16);
   // ring slot of the diagonal: (base_slot - win) + P - q (mod M), slotc given
@@ -231,7 +239,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
   }
   const int endp = min(P + 2 + rlen, 0xffff);  // HSP subject end (inclusive), frame
   bool acc = false;
-  uint16_t *reach16 = w.reach + slot;
+  uint16_t *reach16 = w.reach() + slot;
   if constexpr (kSt) {
     // Finish Alg. 1's walk over the flushed entries of each diagonal, in
     // queue (= s) order, from the slot's lasthit: a trigger (bit 31) was
@@ -239,7 +247,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
     // lasthit); any other entry applies L11-19 to the lasthit the walk has
     // reached.  An accepted extension sets lasthit = its subject end.
     const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
-    const uint32_t e = act ? w.ring[slot] : 0u;
+    const uint32_t e = act ? w.ring()[slot] : 0u;
     uint32_t cur = e & 0xffffu;
     const int gmax = __reduce_max_sync(kFull, act ? __popc(grp) : 0);
     const uint32_t fl = ent >> 30;
@@ -267,7 +275,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
       }
     }
     __syncwarp();
-    if (act && (grp >> lane) == 1u) w.ring[slot] = cur | (((e >> 16) - __popc(grp)) << 16);
+    if (act && (grp >> lane) == 1u) w.ring()[slot] = cur | (((e >> 16) - __popc(grp)) << 16);
     __syncwarp();
     if (kTrace) {
       stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, acc)));
@@ -285,8 +293,8 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
       if (acc) *reach16 = uint16_t(endp);
     }
   } else {
-    w.fs_p[lane] = uint16_t(P);
-    w.fs_end[lane] = uint16_t(endp);
+    w.fs_p()[lane] = uint16_t(P);
+    w.fs_end()[lane] = uint16_t(endp);
     __syncwarp();
     if (act) {
       if (uniq) {
@@ -298,15 +306,15 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
         while (g) {
           const int j = __ffs(g) - 1;
           g &= g - 1;
-          const bool aj = int(w.fs_p[j]) > r;
-          if (aj) r = w.fs_end[j];
-          w.fs_acc[j] = aj;
+          const bool aj = int(w.fs_p()[j]) > r;
+          if (aj) r = w.fs_end()[j];
+          w.fs_acc()[j] = aj;
         }
         *reach16 = uint16_t(r);
       }
     }
     __syncwarp();
-    if (act && !uniq) acc = w.fs_acc[lane] != 0;
+    if (act && !uniq) acc = w.fs_acc()[lane] != 0;
   }
   if (kTrace) {
     stat_add<kTrace>(st, kStatAccepted, __popc(__ballot_sync(kFull, acc)));
@@ -361,8 +369,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
   const int M = a.ring;
   WarpSmem w = carve(after_qc + table_bytes + size_t(warp) * warp_smem_bytes(M), M);
   for (int i = lane; i < M; i += 32) {
-    w.ring[i] = 0;
-    w.reach[i] = 0;
+    w.ring()[i] = 0;
+    w.reach()[i] = 0;
   }
   __syncthreads();
 
@@ -381,11 +389,11 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
   // subtract kFrameSpan from every stored frame position (0 = none stays 0)
   auto rebase_ring = [&]() {
     for (int i = lane; i < M; i += 32) {
-      const uint32_t e = w.ring[i];
+      const uint32_t e = w.ring()[i];
       auto rb = [](uint32_t v) { return v > uint32_t(kFrameSpan) ? v - kFrameSpan : 0u; };
       const uint32_t nl = rb(st_last(e));
-      w.ring[i] = nl ? st_make(nl, rb(st_far(e)), st_near(e)) : 0u;
-      w.reach[i] = uint16_t(rb(w.reach[i]));
+      w.ring()[i] = nl ? st_make(nl, rb(st_far(e)), st_near(e)) : 0u;
+      w.reach()[i] = uint16_t(rb(w.reach()[i]));
     }
     __syncwarp();
     st.spbase += kFrameSpan;
@@ -397,7 +405,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
   // loop happens at the single site at the bottom of this loop, so the
   // X-drop code exists in three copies only (instruction-cache footprint);
   // the walker therefore runs in steps that end whenever the queue must be
-  // drained, its state parked in shared memory (w.wk), not in registers.
+  // drained, its state parked in shared memory (w.wk()), not in registers.
   int mode = 0;  // 0: take the next work item; 1: a walker is active
   for (;;) {
     int64_t wstart = 0, wend = 0, wemit = 0;
@@ -430,10 +438,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         if (it.nseg > 0 && !kSt) {
           st.spbase = it.c.start - frame;
           if (lane == 0) {
-            w.wk[0] = int(ci - nsegs);
-            w.wk[1] = 0;
-            w.wk[2] = 0;
-            w.wk[3] = ((base_slot - frame) % M + M) % M;  // slot = P - q + offset
+            w.wk()[0] = int(ci - nsegs);
+            w.wk()[1] = 0;
+            w.wk()[2] = 0;
+            w.wk()[3] = ((base_slot - frame) % M + M) % M;  // slot = P - q + offset
           }
           __syncwarp();
           mode = 1;
@@ -457,9 +465,9 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       // ---- walker step: the segments' passing hits, in s order, into the
       // extension queue (the ext_reach chain resolves at the drain, exactly
       // as in a walk); returns whenever the queue must be drained first
-      const LongItem it = a.long_items[__shfl_sync(kFull, w.wk[0], 0)];
-      int k = __shfl_sync(kFull, w.wk[1], 0), i0 = __shfl_sync(kFull, w.wk[2], 0),
-          slotw = __shfl_sync(kFull, w.wk[3], 0);
+      const LongItem it = a.long_items[__shfl_sync(kFull, w.wk()[0], 0)];
+      int k = __shfl_sync(kFull, w.wk()[1], 0), i0 = __shfl_sync(kFull, w.wk()[2], 0),
+          slotw = __shfl_sync(kFull, w.wk()[3], 0);
       // a rebase lowers every frame position by kFrameSpan: the slot offset
       // rises by as much, so each diagonal keeps its slot
       auto rebase_w = [&]() {
@@ -518,22 +526,22 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         if (act) {
           int slot = (P - q + slotw) % M;
           slot += slot < 0 ? M : 0;
-          rch = w.reach[slot];
+          rch = w.reach()[slot];
         }
         const bool enq = act && P > int(rch);
         const unsigned bal = __ballot_sync(kFull, enq);
         stat_add<kTrace>(st, kStatEnqueued, __popc(bal));
         const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
-        if (enq) w.queue[(st.qhead + pos) & (kQcap - 1)] = uint32_t(P) | (uint32_t(q) << 16);
+        if (enq) w.queue()[(st.qhead + pos) & (kQcap - 1)] = uint32_t(P) | (uint32_t(q) << 16);
         st.qcount += __popc(bal);
         i0 += __popc(__ballot_sync(kFull, act));
         if (st.qcount >= 32) break;
       }
       __syncwarp();
       if (lane == 0) {
-        w.wk[1] = k;
-        w.wk[2] = i0;
-        w.wk[3] = slotw;
+        w.wk()[1] = k;
+        w.wk()[2] = i0;
+        w.wk()[3] = slotw;
       }
       __syncwarp();
       sc = slotw;
@@ -541,8 +549,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     if (walk) {
     __syncwarp();
     if (lane == 0) {
-      w.wk[4] = sg;
-      w.wk[5] = 0;
+      w.wk()[4] = sg;
+      w.wk()[5] = 0;
     }
     __syncwarp();
     st.spbase = wstart - frame;
@@ -554,15 +562,15 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     // q << 16 (passing hits in s order; ext_reach holds only stale values
     // older than the frame there, so every passing hit was queued)
     auto spill = [&](int n) {
-      const int sgw = __shfl_sync(kFull, w.wk[4], 0);
-      const int nl = __shfl_sync(kFull, w.wk[5], 0);
+      const int sgw = __shfl_sync(kFull, w.wk()[4], 0);
+      const int nl = __shfl_sync(kFull, w.wk()[5], 0);
       if (lane < n && nl + lane < a.seg_cap) {
-        const uint32_t ent = w.queue[(st.qhead + lane) & (kQcap - 1)];
+        const uint32_t ent = w.queue()[(st.qhead + lane) & (kQcap - 1)];
         a.seg_list[int64_t(sgw) * a.seg_cap + nl + lane] =
             ((ent & 0xffffu) - uint32_t(emit_f)) | (ent & 0xffff0000u);
       }
       __syncwarp();
-      if (lane == 0) w.wk[5] = nl + n;
+      if (lane == 0) w.wk()[5] = nl + n;
       __syncwarp();
       st.qhead = (st.qhead + n) & (kQcap - 1);
       st.qcount -= n;
@@ -604,7 +612,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     while (win < end) {
       // ---- rebase the frame before positions outgrow 16 bits --------------
       if (win >= kFrameMin + kFrameSpan) {
-        if (__shfl_sync(kFull, w.wk[4], 0) >= 0) {
+        if (__shfl_sync(kFull, w.wk()[4], 0) >= 0) {
           while (st.qcount > 0) spill(min(st.qcount, 32));
         } else {
           const int sc = slotc();
@@ -650,7 +658,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       // last run start at or before it, from the OR-reduced start mask
       // (measured: 1.1% faster than a 5-step shuffle binary search over the
       // inclusive counts, profiles/r01/ab_locate.txt)
-      uint32_t *scr = reinterpret_cast<uint32_t *>(w.fs_p);
+      uint32_t *scr = reinterpret_cast<uint32_t *>(w.fs_p());
       auto locate = [&](uint32_t kb, int &own_out, int &q_out) {
         const bool wr = cnt != 0u && excl < kb + 32u && incl > kb;
         const int p0 = wr ? max(int(excl) - int(kb), 0) : 0;
@@ -684,8 +692,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         const unsigned earlier = grp & lanemask_lt(lane);
         uint32_t e = 0, rch = 0;
         if (act) {
-          e = w.ring[slot];
-          rch = w.reach[slot];
+          e = w.ring()[slot];
+          rch = w.reach()[slot];
         }
         bool enq = false;
         uint32_t eflags = 0;  // STATEFUL queue-entry flags (bit 31 trigger, bit 30 fresh)
@@ -739,8 +747,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           }
           __syncwarp();
           if (act && (grp >> lane) == 1u) {
-            w.ring[slot] = L | (cnt << 16);
-            w.reach[slot] = uint16_t(rq);
+            w.ring()[slot] = L | (cnt << 16);
+            w.reach()[slot] = uint16_t(rq);
           }
         } else {
           const uint32_t last = st_last(e), near = st_near(e);
@@ -780,7 +788,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
               stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, counts)));
               stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
             }
-            if (w.wk[4] < 0)
+            if (w.wk()[4] < 0)
               stat_add<kTrace>(st, kStatEnqueued,
                                __popc(__ballot_sync(kFull, pass && Ph > int(rch))));
             if (counts && !retrace) {
@@ -796,7 +804,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
               const int d = Ph - int(last);
               if (d < W) nb |= ((near << d) | (1u << d));
             }
-            w.ring[slot] = st_make(uint32_t(Ph), uint32_t(cand), nb & nearmask);
+            w.ring()[slot] = st_make(uint32_t(Ph), uint32_t(cand), nb & nearmask);
           }
           enq = pass && Ph > int(rch);
         }
@@ -804,11 +812,11 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         if (bal) {
           const int pos = st.qcount + __popc(bal & lanemask_lt(lane));
           if (enq)
-            w.queue[(st.qhead + pos) & (kQcap - 1)] = uint32_t(Ph) | (uint32_t(q) << 16) | eflags;
+            w.queue()[(st.qhead + pos) & (kQcap - 1)] = uint32_t(Ph) | (uint32_t(q) << 16) | eflags;
           st.qcount += __popc(bal);
           __syncwarp();
           while (st.qcount >= 32) {  // a flush may keep entries queued
-            if (__shfl_sync(kFull, w.wk[4], 0) >= 0)
+            if (__shfl_sync(kFull, w.wk()[4], 0) >= 0)
               spill(32);  // segment: to its list
             else
               flush_queue<kTrace, kWin, kSt>(a, w, st, 32, qc, b62, lane, slotc(), M);
@@ -823,9 +831,9 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       base_slot += npos;
       if (base_slot >= M) base_slot -= M;
     }
-    if (const int sgw = __shfl_sync(kFull, w.wk[4], 0); sgw >= 0) {
+    if (const int sgw = __shfl_sync(kFull, w.wk()[4], 0); sgw >= 0) {
       while (st.qcount > 0) spill(min(st.qcount, 32));
-      const int nl = __shfl_sync(kFull, w.wk[5], 0);
+      const int nl = __shfl_sync(kFull, w.wk()[5], 0);
       __threadfence();
       __syncwarp();
       if (lane == 0) {

@@ -521,6 +521,57 @@ def test_search_host_db_pipelined_parts(bp, orc):
     assert _host_db_search(bp, t, np.zeros(0, np.uint8), np.zeros(1, np.int64), p) == []
 
 
+def _formatted_search(bp, t, hdb, p):
+    import torch
+    cap = 1 << 16
+    out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    bp.search_formatted_db(t, hdb, out.data_ptr(), cap, cnt.data_ptr(), p)
+    n = int(cnt.item())
+    assert n <= cap
+    bp.sort_hsps_device(out.data_ptr(), n)
+    return [tuple(x) for x in out[: n * 7].view(n, 7).cpu().numpy().tolist()]
+
+
+def test_formatted_host_db(bp, orc):
+    """blastp_format_host_db + blastp_search_formatted_db (parts packed once
+    into pinned host memory, streamed by copies only) equals pack + search of
+    the whole shard: automatic and explicit part counts, shards, repeated
+    searches of one image, a query batch, every filter mode and long subjects
+    (segment plans travel with the image)."""
+    q = gen_query(21, 300).decode()
+    ascii, off = _long_subject_db(q)
+    rng = np.random.default_rng(9)
+    a2, o2 = _rand_db(rng, 3000, 0, 600, q)
+    ascii = np.concatenate([a2, ascii])
+    off = np.concatenate([o2, o2[-1] + off[1:]]).astype(np.int64)
+    t = bp.build_query_table(q, bp.Params())
+    d = bp.pack_db(ascii, off)
+    for p in (bp.Params(), bp.Params(filter_mode=1), bp.Params(filter_mode=2),
+              bp.Params(ext_mode=1)):
+        whole = tuples(bp.search_ungapped(t, d, p))
+        for parts in (0, 1, 3, 7):
+            hdb = bp.format_host_db(ascii, off, num_parts=parts)
+            assert hdb.nseq == len(off) - 1 and hdb.residues == int(off[-1])
+            assert parts == 0 or hdb.num_parts == parts
+            assert _formatted_search(bp, t, hdb, p) == whole, (p, parts)
+            assert _formatted_search(bp, t, hdb, p) == whole  # the image is reusable
+            hdb.free()
+    p = bp.Params()
+    assert tuples(bp.search_ungapped(t, d, p)) == tuples(oracle_run(orc, q, ascii, off, p,
+                                                                    nthreads=4).hsps)
+    for k in range(3):
+        shard = tuples(bp.search_ungapped(t, bp.pack_db(ascii, off, k, 3), p))
+        hdb = bp.format_host_db(ascii, off, shard_index=k, num_shards=3, num_parts=2)
+        assert _formatted_search(bp, t, hdb, p) == shard
+    qs = [q, gen_query(22, 127).decode()]
+    tb = bp.build_query_batch(qs, p)
+    hdb = bp.format_host_db(ascii, off, num_parts=4)
+    assert _formatted_search(bp, tb, hdb, p) == tuples(bp.search_ungapped(tb, d, p))
+    empty = bp.format_host_db(np.zeros(0, np.uint8), np.zeros(1, np.int64))
+    assert _formatted_search(bp, t, empty, p) == []
+
+
 def _same_start_db(orc):
     """A seeded DB whose oracle HSP list holds two HSPs of one diagonal with
     the same start and different ends (a later seed beyond the first HSP's
