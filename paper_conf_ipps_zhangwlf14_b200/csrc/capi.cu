@@ -759,14 +759,13 @@ static void db_free_async(blastp_db *db, cudaStream_t s) {
 // from a small first part -- its copy is the only one not hidden behind a
 // search, and each part copies faster than the previous one is searched.
 static std::vector<int64_t> part_cuts(const int64_t *offsets, int64_t lo, int64_t hi,
-                                      int32_t num_parts) {
+                                      int32_t num_parts, int growth = 150) {
   const int64_t total = offsets[hi] - offsets[lo];
   std::vector<int64_t> cut{lo};
   // knobs (tuning): BLASTP_PIPE_FIRST residues of the first part,
   // BLASTP_PIPE_GROWTH percent growth per part
   int64_t want = std::max<int64_t>(int64_t(1) << 24, total / 64);
   if (const char *v = std::getenv("BLASTP_PIPE_FIRST")) want = std::max<int64_t>(1, std::atoll(v));
-  int growth = 150;
   if (const char *v = std::getenv("BLASTP_PIPE_GROWTH")) growth = std::max(101, std::atoi(v));
   int64_t done = 0;
   for (int k = 0; cut.back() < hi; ++k) {
@@ -976,7 +975,11 @@ int blastp_format_host_db(const char *residues_ascii, const int64_t *offsets, in
   DeviceGuard g(device);
   if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
   cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
-  const std::vector<int64_t> cut = part_cuts(offsets, lo, hi, num_parts);
+  // growth 1.4x: a part's copy (~55 GB/s from pinned memory) must not take
+  // longer than the previous part's search (~38 G residues/s at q1054):
+  // measured 33.1 ms vs 33.7 (1.5x), 38.5 (2x) on config 3
+  // (profiles/r01/fmt_sweep_v2.txt)
+  const std::vector<int64_t> cut = part_cuts(offsets, lo, hi, num_parts, 140);
   auto *h = new (std::nothrow) blastp_host_db;
   if (!h) return fail(BLASTP_E_NOMEM, "host allocation failed");
   h->device = device;

@@ -16,7 +16,7 @@ import torch  # noqa: E402
 from paper_conf_ipps_zhangwlf14_b200 import blastp as bp  # noqa: E402
 from synth import config_workload  # noqa: E402
 
-scale = float(sys.argv[1]) if len(sys.argv) > 1 else 1.0
+scale = float(sys.argv[1]) if len(sys.argv) > 1 and sys.argv[1][0].isdigit() else 1.0
 (q,), db = config_workload(3, scale=scale)
 pinned = torch.empty(db.residues, dtype=torch.uint8, pin_memory=True)
 pinned.copy_(torch.from_numpy(db.ascii))
@@ -25,7 +25,7 @@ t = bp.build_query_table(q)
 cap = 1 << 22
 out = torch.empty(cap * 7, dtype=torch.int32, device="cuda")
 cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
-d = bp.pack_db(pinned.data_ptr(), off)
+d = bp.Database.from_pinned(pinned.data_ptr(), off, 0, 1)
 for _ in range(3):
     bp.search_ungapped_device(t, d, out.data_ptr(), cap, cnt.data_ptr())
 torch.cuda.synchronize()
@@ -35,8 +35,11 @@ for _ in range(5):
 torch.cuda.synchronize()
 print(f"resident search: {1e3 * (time.perf_counter() - t0) / 5:.2f} ms", flush=True)
 d.free()
-for first, growth, parts in [(1 << 24, 150, 0), (1 << 24, 200, 0), (1 << 24, 300, 0),
-                             (1 << 23, 200, 0), (1 << 25, 200, 0), (0, 0, 4), (0, 0, 16)]:
+grid = [(1 << 24, 150, 0), (1 << 24, 140, 0), (1 << 24, 130, 0), (1 << 24, 120, 0),
+        (1 << 23, 130, 0), (1 << 25, 130, 0), (1 << 23, 140, 0), (0, 0, 32), (0, 0, 48)]
+if "--wide" in sys.argv:
+    grid += [(1 << 24, 200, 0), (1 << 24, 300, 0), (0, 0, 4), (0, 0, 16)]
+for first, growth, parts in grid:
     if parts == 0:
         os.environ["BLASTP_PIPE_FIRST"] = str(first)
         os.environ["BLASTP_PIPE_GROWTH"] = str(growth)
