@@ -360,13 +360,21 @@ def main():
     # + the HSP records written
     alg_bytes = gdb.residues * nq + n_hsp * 28
     achieved = alg_bytes / (statistics.mean(kern_ms) / 1e3) / 1e9
-    capt = ncu_capture() if (args.config == 3 and world == 1 and nq == 1) else {}
-    traffic, traffic_src = capt.get("dram_bytes_per_launch"), capt.get("source")
+    # the committed capture is one config-3 launch over the whole DB; a rank's
+    # shard of it (N > 1) is credited its residue fraction of the counts
+    capt = ncu_capture() if (args.config == 3 and nq == 1) else {}
+    frac_shard = gdb.residues / max(1, total_residues)
+    traffic = capt.get("dram_bytes_per_launch")
+    traffic = traffic * frac_shard if traffic is not None else None
+    traffic_src = capt.get("source")
+    if capt and world > 1:
+        traffic_src = f"{traffic_src}, x {frac_shard:.4f} (this rank's residue share)"
+
     # issue-rate roofline: warp instructions of the captured launch / this
     # run's kernel time vs 148 SMs x 4 issue slots x the sampled SM clock
     issue = None
     if capt.get("smsp__inst_executed.sum") and clk.get("sm_mhz"):
-        inst = float(capt["smsp__inst_executed.sum"])
+        inst = float(capt["smsp__inst_executed.sum"]) * frac_shard
         props = torch.cuda.get_device_properties(dev)
         peak_i = props.multi_processor_count * 4 * clk["sm_mhz"] * 1e6
         ach_i = inst / (kern_avg_ms / 1e3)
