@@ -403,14 +403,17 @@ int blastp_shard_range(const int64_t *offsets, int64_t nseq, int32_t shard_index
 // Stream layout: kStreamPadFront sentinels, then subject i at
 // sstart[i] = pad + (offsets[lo+i] - offsets[lo]) + i, each followed by one
 // sentinel; kStreamPadBack trailing sentinels; 512-byte multiple.  Chunks of
-// C residues of whole subjects (8 per resident warp, at most 8192: measured
+// C residues of whole subjects (8 per resident warp, 128 <= C <= 8192: measured
 // 1.3% faster than 16384 on config 3), the last 2 C per resident warp in
 // chunks of C/4 (ChunkPlan).
 static void layout_sizes(int64_t n, int64_t nres, int sms, int64_t *stream_len, ChunkPlan *plan) {
   *stream_len = (kStreamPadFront + nres + n + kStreamPadBack + 511) & ~int64_t(511);
   const int64_t warps = int64_t(sms) * 32;
   int64_t c = nres / (warps * 8);
-  c = std::min<int64_t>(std::max<int64_t>(c, 1024), 8192);
+  // at least 128: a small shard still spreads over many warps (config 1,
+  // 250k residues: 0.066 ms vs 0.095 ms with a 1024 minimum; config 2
+  // unchanged; profiles/r01/chunk_sweep.txt)
+  c = std::min<int64_t>(std::max<int64_t>(c, 128), 8192);
   if (const char *ce = std::getenv("BLASTP_CHUNK")) c = std::max<int64_t>(64, std::atoll(ce));
   plan->C = c;
   plan->Ct = std::min<int64_t>(c, std::max<int64_t>(1024, c / 4));

@@ -572,6 +572,37 @@ def test_formatted_host_db(bp, orc):
     assert _formatted_search(bp, t, empty, p) == []
 
 
+def test_formatted_host_db_config3_full_size(bp):
+    """Config 3 at full size (the bench's e2e path): the formatted image
+    streamed in parts gives exactly the resident shard's HSP list (the
+    resident list is itself pinned to the oracle by
+    test_config3_full_size_sampled)."""
+    import torch
+    (q,), db = _config3()
+    p = bp.Params()
+    t = bp.build_query_table(q, p)
+    cap = 1 << 20
+    outs = []
+    for mode in ("resident", "formatted"):
+        out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+        cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+        if mode == "resident":
+            d = bp.pack_db(db.ascii, db.offsets)
+            bp.search_ungapped_device(t, d, out.data_ptr(), cap, cnt.data_ptr(), p)
+            n = int(cnt.item())
+            d.free()
+        else:
+            h = bp.format_host_db(db.ascii, db.offsets)
+            assert h.num_parts > 4
+            bp.search_formatted_db(t, h, out.data_ptr(), cap, cnt.data_ptr(), p)
+            n = int(cnt.item())
+            h.free()
+        assert 10000 < n <= cap
+        bp.sort_hsps_device(out.data_ptr(), n)
+        outs.append(out[: n * 7].cpu())
+    assert torch.equal(outs[0], outs[1])
+
+
 def _same_start_db(orc):
     """A seeded DB whose oracle HSP list holds two HSPs of one diagonal with
     the same start and different ends (a later seed beyond the first HSP's
