@@ -548,7 +548,8 @@ def main():
             "e2e": e2e_fmt or e2e,
             "e2e_ascii_db": e2e if e2e_fmt else None,
             "e2e_resident_db": e2e_res,
-            "gpu_launches": args.steps * nq,
+            "gpu_launches": args.steps * (table.launches(params)
+                                          if hasattr(table, "launches") else nq),
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)

@@ -110,7 +110,13 @@ int blastp_build_query_table(const char *query_ascii, int32_t len,
                              const blastp_params *p, int device,
                              void *cuda_stream, blastp_query_table **out);
 
-/* Same for `nq` queries; query_id of results = index in `queries`. */
+/* Same for `nq` queries; query_id of results = index in `queries`.
+ * Queries of a batch are also packed into query groups (SURVEY 8(f) rank 1:
+ * one database scan for several queries): first-fit decreasing into groups
+ * of combined length <= 1024 with p->window + 8 sentinel codes between
+ * members (BLASTP_GROUP=0 disables).  A search uses the groups when its
+ * window A satisfies A + 8 <= that gap (else, and for the debug entry
+ * points, it searches query by query); results are identical either way. */
 int blastp_build_query_batch(const char *const *queries, const int32_t *lens,
                              int32_t nq, const blastp_params *p, int device,
                              void *cuda_stream, blastp_query_table **out);
@@ -197,6 +203,12 @@ int blastp_db_long_info(const blastp_db *db, int64_t *long_items,
                         int64_t *segments, int64_t *segment_len);
 int blastp_query_table_info(const blastp_query_table *q, int32_t *num_queries,
                             int64_t *table_entries);
+/* Query groups of a batch table: *groups (searched as one scan each),
+ * *alone (queries searched by themselves) and the sentinel *gap between
+ * members; a search with window A launches groups + alone kernels per
+ * shard when A + 8 <= gap, else num_queries.  Any pointer may be NULL. */
+int blastp_query_table_groups(const blastp_query_table *q, int32_t *groups, int32_t *alone,
+                              int32_t *gap);
 
 /* Ungapped search (Alg. 1-5; R4-R10): every hit of every query against
  * every subject of the shard, the two-hit filter per (subject, diagonal),

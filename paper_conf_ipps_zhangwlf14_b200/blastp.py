@@ -84,6 +84,8 @@ def _load():
     if hasattr(L, "blastp_db_long_info"):  # absent in builds older than the long-item plan
         L.blastp_db_long_info.argtypes = [vp, P(i64), P(i64), P(i64)]
     L.blastp_query_table_info.argtypes = [vp, P(i32), P(i64)]
+    if hasattr(L, "blastp_query_table_groups"):
+        L.blastp_query_table_groups.argtypes = [vp, P(i32), P(i32), P(i32)]
     L.blastp_search_ungapped.argtypes = [vp, vp, P(_CParams), vp, P(vp), P(i64)]
     L.blastp_search_ungapped_device.argtypes = [vp, vp, P(_CParams), vp, vp, i64, vp]
     if hasattr(L, "blastp_search_host_db"):  # absent in older builds (A/B timing)
@@ -113,6 +115,7 @@ lib = _load()
 EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "blastp_version",
             "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
             "blastp_shard_range", "blastp_db_info", "blastp_db_long_info", "blastp_query_table_info",
+            "blastp_query_table_groups",
             "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_search_host_db",
             "blastp_format_host_db", "blastp_search_formatted_db", "blastp_host_db_info",
             "blastp_host_db_free",
@@ -180,6 +183,20 @@ class QueryTable:
         _check(lib.blastp_query_table_info(self.handle, ctypes.byref(n), ctypes.byref(e)),
                "blastp_query_table_info")
         return n.value
+
+    @property
+    def groups(self) -> tuple[int, int, int]:
+        """(query groups, queries searched alone, sentinel gap) of a batch table."""
+        g, a, gap = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+        _check(lib.blastp_query_table_groups(self.handle, ctypes.byref(g), ctypes.byref(a),
+                                             ctypes.byref(gap)), "blastp_query_table_groups")
+        return g.value, a.value, gap.value
+
+    def launches(self, params: Params | None = None) -> int:
+        """Search kernels per shard for a search with `params` (groups when the window fits)."""
+        g, a, gap = self.groups
+        p = params or self.params
+        return g + a if g and p.window + 8 <= gap else self.num_queries
 
     @property
     def entries(self) -> int:

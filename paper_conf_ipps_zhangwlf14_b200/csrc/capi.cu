@@ -105,6 +105,11 @@ struct QueryDev {
   uint8_t *qcodes = nullptr;
   int32_t lq = 0;
   int64_t entries = 0;
+  // a group of queries searched as one: the member
+  // queries' codes concatenated with sentinel gaps; member k starts at
+  // combined position sub_off[k] and is query sub_id[k] of the batch
+  int32_t nsub = 0;
+  int32_t *sub = nullptr;  // device: sub_off[nsub], then sub_id[nsub]
 };
 
 struct blastp_query_table {
@@ -112,6 +117,10 @@ struct blastp_query_table {
   blastp_params p{};
   std::vector<QueryDev> q;
   int64_t entries = 0;
+  // query groups of a batch and the queries left alone (indices into q)
+  std::vector<QueryDev> groups;
+  std::vector<int32_t> alone;
+  int32_t group_gap = 0;  // sentinel positions between the members of a group
 };
 
 struct blastp_db {
@@ -195,6 +204,7 @@ static void free_query_dev(QueryDev &d) {
   cudaFree(d.woff);
   cudaFree(d.qpos);
   cudaFree(d.qcodes);
+  cudaFree(d.sub);
   d = QueryDev{};
 }
 
@@ -231,19 +241,27 @@ const char *blastp_version(void) { return "blastp-b200 0.1 (sm_100a)"; }
 
 // ------------------------------------------------------- query table (R3)
 
-static int build_one_query(const char *ascii, int32_t len, const blastp_params *p, QueryDev &out,
-                           cudaStream_t s) {
+static int encode_query(const char *ascii, int32_t len, std::vector<uint8_t> &Q) {
   if (!ascii) return fail(BLASTP_E_INVALID_ARG, "query is NULL");
   if (len < 3) return fail(BLASTP_E_INVALID_ARG, "query length %d < 3", len);
   if (len > BLASTP_MAX_QUERY_LEN)
     return fail(BLASTP_E_TOO_LONG, "query length %d > %d", len, BLASTP_MAX_QUERY_LEN);
-  std::vector<uint8_t> Q(static_cast<size_t>(len));
+  Q.resize(static_cast<size_t>(len));
   for (int32_t i = 0; i < len; ++i) {
     const int c = encode_char(static_cast<unsigned char>(ascii[i]));
     if (c < 0) return fail(BLASTP_E_BAD_RESIDUE, "query byte %d (0x%02x) is not a residue", i,
                            static_cast<unsigned char>(ascii[i]));
     Q[static_cast<size_t>(i)] = static_cast<uint8_t>(c);
   }
+  return BLASTP_OK;
+}
+
+// Lookup table (R3) of the query codes Q (a query, or a group's members
+// separated by sentinel codes: a word touching a sentinel scores -1000 per
+// sentinel letter and neighbours nothing).
+static int build_table(const std::vector<uint8_t> &Q, const blastp_params *p, QueryDev &out,
+                       cudaStream_t s) {
+  const int32_t len = static_cast<int32_t>(Q.size());
   out.lq = len;
   const char *how = std::getenv("BLASTP_TABLE_BUILD");  // "host": the host enumeration below
   if (!(how && !std::strcmp(how, "host"))) {
@@ -283,6 +301,7 @@ static int build_one_query(const char *ascii, int32_t len, const blastp_params *
   auto enumerate = [&](auto &&emit) {
     for (int32_t q = 0; q + 3 <= len; ++q) {
       const int a0 = Q[q], a1 = Q[q + 1], a2 = Q[q + 2];
+      if (a0 >= kNumLetters || a1 >= kNumLetters || a2 >= kNumLetters) continue;  // group gap
       for (int x = 0; x < kNumLetters; ++x) {
         const int s1 = kBlosum62[a0][x];
         if (s1 + rowmax[a1] + rowmax[a2] < T) continue;
@@ -319,6 +338,79 @@ static int build_one_query(const char *ascii, int32_t len, const blastp_params *
   return BLASTP_OK;
 }
 
+static int build_one_query(const char *ascii, int32_t len, const blastp_params *p, QueryDev &out,
+                           cudaStream_t s) {
+  std::vector<uint8_t> Q;
+  int rc = encode_query(ascii, len, Q);
+  return rc ? rc : build_table(Q, p, out, s);
+}
+
+// Query groups of a batch (one DB scan for several
+// queries).  Members are concatenated with `gap` sentinel codes between
+// them, gap >= A + 8: two members' hits that share a combined diagonal lie
+// >= A apart in the subject, so no two-hit pair, lasthit or ext_reach ever
+// links them, and every X-drop stops at the sentinels of its own member --
+// the group's search returns exactly the members' searches.
+// First-fit decreasing into groups of combined length <= kGroupLen (the
+// size that still keeps 32 warps per SM resident, like a q1054 search).
+constexpr int32_t kGroupLen = 1024;
+static int build_groups(blastp_query_table *t, const char *const *queries, const int32_t *lens,
+                        int32_t nq, cudaStream_t s) {
+  const char *env = std::getenv("BLASTP_GROUP");  // knob: BLASTP_GROUP=0 disables grouping
+  if ((env && std::atoi(env) == 0) || nq < 2) {
+    for (int32_t i = 0; i < nq; ++i) t->alone.push_back(i);
+    return BLASTP_OK;
+  }
+  const int32_t gap = t->p.window + 8;
+  t->group_gap = gap;
+  std::vector<int32_t> order(static_cast<size_t>(nq));
+  for (int32_t i = 0; i < nq; ++i) order[static_cast<size_t>(i)] = i;
+  std::stable_sort(order.begin(), order.end(),
+                   [&](int32_t a, int32_t b) { return lens[a] > lens[b]; });
+  std::vector<std::vector<int32_t>> bins;
+  std::vector<int32_t> used;
+  for (int32_t i : order) {
+    size_t b = 0;
+    for (; b < bins.size(); ++b)
+      if (used[b] + gap + lens[i] <= kGroupLen) break;
+    if (b == bins.size()) {
+      bins.push_back({});
+      used.push_back(-gap);
+    }
+    bins[b].push_back(i);
+    used[b] += gap + lens[i];
+  }
+  for (auto &members : bins) {
+    if (members.size() == 1) {
+      t->alone.push_back(members[0]);
+      continue;
+    }
+    std::sort(members.begin(), members.end());
+    std::vector<uint8_t> Q, M;
+    std::vector<int32_t> sub;
+    for (int32_t i : members) {
+      if (!Q.empty()) Q.insert(Q.end(), static_cast<size_t>(gap), uint8_t(kSentinel));
+      sub.push_back(static_cast<int32_t>(Q.size()));
+      int rc = encode_query(queries[i], lens[i], M);
+      if (rc) return rc;
+      Q.insert(Q.end(), M.begin(), M.end());
+    }
+    for (int32_t i : members) sub.push_back(i);
+    QueryDev g;
+    int rc = build_table(Q, &t->p, g, s);
+    if (rc) return rc;
+    g.nsub = static_cast<int32_t>(members.size());
+    if (cudaMalloc(&g.sub, sizeof(int32_t) * sub.size()) != cudaSuccess) {
+      cudaGetLastError();
+      free_query_dev(g);
+      return fail(BLASTP_E_NOMEM, "device allocation for a query group failed");
+    }
+    t->groups.push_back(g);
+    CUDA_TRY(cudaMemcpy(g.sub, sub.data(), sizeof(int32_t) * sub.size(), cudaMemcpyHostToDevice));
+  }
+  return BLASTP_OK;
+}
+
 int blastp_build_query_batch(const char *const *queries, const int32_t *lens, int32_t nq,
                              const blastp_params *p, int device, void *cuda_stream,
                              blastp_query_table **out) {
@@ -343,6 +435,11 @@ int blastp_build_query_batch(const char *const *queries, const int32_t *lens, in
     }
     t->entries += t->q[static_cast<size_t>(i)].entries;
   }
+  rc = build_groups(t, queries, lens, nq, static_cast<cudaStream_t>(cuda_stream));
+  if (rc) {
+    blastp_query_table_free(t);
+    return rc;
+  }
   *out = t;
   return BLASTP_OK;
 }
@@ -352,6 +449,15 @@ int blastp_build_query_table(const char *query_ascii, int32_t len, const blastp_
   const char *qs[1] = {query_ascii};
   int32_t ls[1] = {len};
   return blastp_build_query_batch(qs, ls, 1, p, device, cuda_stream, out);
+}
+
+int blastp_query_table_groups(const blastp_query_table *q, int32_t *groups, int32_t *alone,
+                              int32_t *gap) {
+  if (!q) return fail(BLASTP_E_INVALID_ARG, "table is NULL");
+  if (groups) *groups = static_cast<int32_t>(q->groups.size());
+  if (alone) *alone = static_cast<int32_t>(q->alone.size());
+  if (gap) *gap = q->group_gap;
+  return BLASTP_OK;
 }
 
 int blastp_query_table_info(const blastp_query_table *q, int32_t *num_queries,
@@ -366,6 +472,7 @@ void blastp_query_table_free(blastp_query_table *q) {
   if (!q) return;
   DeviceGuard g(q->device);
   for (auto &d : q->q) free_query_dev(d);
+  for (auto &d : q->groups) free_query_dev(d);
   delete q;
 }
 
@@ -676,7 +783,27 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
   if (trace_count)  // [0..3): trace record counts, [3..3+kNumStats): event counters
     CUDA_TRY(cudaMemsetAsync(trace_count, 0, (3 + kNumStats) * sizeof(unsigned long long), s));
   if (db->nchunks == 0) return BLASTP_OK;
-  for (const QueryDev &qd : q->q) {
+  // a batch's query groups (one scan per group) when the two-hit window fits
+  // the sentinel gap they were built with; traced runs search query by query
+  std::vector<const QueryDev *> list;
+  std::vector<int32_t> ids;
+  if (!q->groups.empty() && trace == nullptr && p->window + 8 <= q->group_gap) {
+    for (const QueryDev &g : q->groups) {
+      list.push_back(&g);
+      ids.push_back(-1);
+    }
+    for (int32_t i : q->alone) {
+      list.push_back(&q->q[static_cast<size_t>(i)]);
+      ids.push_back(i);
+    }
+  } else {
+    for (size_t i = 0; i < q->q.size(); ++i) {
+      list.push_back(&q->q[i]);
+      ids.push_back(static_cast<int32_t>(i));
+    }
+  }
+  for (size_t li = 0; li < list.size(); ++li) {
+    const QueryDev &qd = *list[li];
     SearchArgs a{};
     a.stream = db->stream;
     a.sstart = db->sstart;
@@ -701,7 +828,9 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.qv.qpos = qd.qpos;
     a.qv.qcodes = qd.qcodes;
     a.qv.lq = qd.lq;
-    a.qv.query_id = static_cast<int32_t>(&qd - q->q.data());
+    a.qv.query_id = ids[li];
+    a.qv.nsub = qd.nsub;
+    a.qv.sub = qd.sub;
     a.word_len = p->word_len;
     a.threshold = p->threshold;
     a.window = p->window;

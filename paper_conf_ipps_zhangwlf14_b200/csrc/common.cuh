@@ -89,6 +89,10 @@ struct QueryView {
   const uint16_t *qpos;   // [entries], ascending within a word
   const uint8_t *qcodes;  // [lq] query codes
   int32_t lq, query_id;
+  // a query group (nsub >= 2): member k starts at combined position sub[k]
+  // and is batch query sub[nsub + k]; 0 for a single query
+  int32_t nsub;
+  const int32_t *sub;
 };
 
 struct SearchArgs {

@@ -229,6 +229,17 @@ __device__ __forceinline__ bool emit_hsp(const SearchArgs &a, int64_t sp, int q,
   const int64_t s_local = sp - __ldg(a.sstart + lo);
   blastp_hsp h;
   h.query_id = a.qv.query_id;
+  if (a.qv.nsub > 1) {
+    // a query group: the member whose codes hold the seed (every extension
+    // stops at the sentinels between members)
+    int k = 0, hi_k = a.qv.nsub - 1;
+    while (k < hi_k) {
+      const int mid = (k + hi_k + 1) >> 1;
+      if (__ldg(a.qv.sub + mid) <= q) k = mid; else hi_k = mid - 1;
+    }
+    q -= __ldg(a.qv.sub + k);
+    h.query_id = __ldg(a.qv.sub + a.qv.nsub + k);
+  }
   h.subject_id = int32_t(a.subject_base + lo);
   h.q_start = q - llen;
   h.s_start = int32_t(s_local) - llen;

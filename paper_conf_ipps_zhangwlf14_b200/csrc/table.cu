@@ -36,10 +36,12 @@ template <bool kFill>
 __global__ void __launch_bounds__(kTableThreads)
     table_kernel(const Matrix B, const uint8_t *__restrict__ qcodes, int lq, int T,
                  uint32_t *__restrict__ woff, uint16_t *__restrict__ qpos) {
-  __shared__ int bt[kNumLetters * 32];
-  for (int i = threadIdx.x; i < kNumLetters * 32; i += blockDim.x) {
+  // rows for every 5-bit query code: the sentinels between the members of a
+  // query group score -1000 against everything (no word touching one)
+  __shared__ int bt[32 * 32];
+  for (int i = threadIdx.x; i < 32 * 32; i += blockDim.x) {
     const int a = i >> 5, x = i & 31;
-    bt[i] = x < kNumLetters ? int(B.m[a * kNumLetters + x]) : -1000;
+    bt[i] = (a < kNumLetters && x < kNumLetters) ? int(B.m[a * kNumLetters + x]) : -1000;
   }
   __syncthreads();
   const int w = blockIdx.x * blockDim.x + threadIdx.x;

@@ -650,6 +650,59 @@ def test_query_batch_equals_single_queries(bp, orc):
     assert tuples(batch) == sorted(exp)
 
 
+def test_query_groups_equal_single_queries(bp, orc):
+    """A batch of short queries is searched as query groups (members
+    concatenated with sentinel gaps >= A + 8, one scan per group; SURVEY 8(f)
+    rank 1): HSPs identical to the oracle's per-query searches for every
+    filter and extension mode, for a window that fits the gap (groups) and one
+    that does not (query by query), with planted homologs of every member,
+    long subjects (segments) and the formatted host database path."""
+    import torch
+    rng = np.random.default_rng(77)
+    lens = [60, 90, 120, 150, 200, 240, 310, 400, 3, 17, 520, 700, 45]
+    qs = [gen_query(300 + i, L) for i, L in enumerate(lens)]
+    db = gen_db(301, 302, n_subjects=400, mean_len=300.0, queries=qs, plant_frac=0.5)
+    lq, lo = _long_subject_db(qs[7].decode())
+    ascii = np.concatenate([db.ascii, lq])
+    off = np.concatenate([db.offsets, db.offsets[-1] + lo[1:]]).astype(np.int64)
+    d = bp.pack_db(ascii, off)
+    for build_window in (40, 256):
+        tb = bp.build_query_batch(qs, bp.Params(window=build_window))
+        g, alone, gap = tb.groups
+        assert g >= 2 and gap == build_window + 8
+        for p in (bp.Params(), bp.Params(filter_mode=1), bp.Params(filter_mode=2),
+                  bp.Params(ext_mode=1), bp.Params(ext_mode=2), bp.Params(window=80),
+                  bp.Params(window=256)):
+            assert tb.launches(p) == (g + alone if p.window + 8 <= gap else len(qs))
+            got = tuples(bp.search_ungapped(tb, d, p))
+            exp = []
+            for i, q in enumerate(qs):
+                exp += tuples(oracle_run(orc, q, ascii, off, p, query_id=i, nthreads=4).hsps)
+            assert got == sorted(exp), (build_window, p)
+            assert len(got) > 100
+    # the formatted host database streams the groups too
+    tb = bp.build_query_batch(qs, bp.Params())
+    h = bp.format_host_db(ascii, off, num_parts=3)
+    cap = 1 << 18
+    out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    bp.search_formatted_db(tb, h, out.data_ptr(), cap, cnt.data_ptr())
+    n = int(cnt.item())
+    bp.sort_hsps_device(out.data_ptr(), n)
+    assert [tuple(x) for x in out[: n * 7].view(n, 7).cpu().numpy().tolist()] == \
+        tuples(bp.search_ungapped(tb, d, bp.Params()))
+    # grouping off: same results
+    import os as _os
+    _os.environ["BLASTP_GROUP"] = "0"
+    try:
+        t0 = bp.build_query_batch(qs, bp.Params())
+        assert t0.groups[0] == 0
+        assert tuples(bp.search_ungapped(t0, d, bp.Params())) == \
+            tuples(bp.search_ungapped(tb, d, bp.Params()))
+    finally:
+        del _os.environ["BLASTP_GROUP"]
+
+
 def test_sharded_union_equals_whole(bp, orc):
     (q,), db = config_workload(1)
     p = bp.Params()
