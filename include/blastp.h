@@ -113,7 +113,7 @@ int blastp_build_query_table(const char *query_ascii, int32_t len,
 /* Same for `nq` queries; query_id of results = index in `queries`.
  * Queries of a batch are also packed into query groups (SURVEY 8(f) rank 1:
  * one database scan for several queries): first-fit decreasing into groups
- * of combined length <= 1024 with p->window + 8 sentinel codes between
+ * of combined length <= 1280 with p->window + 8 sentinel codes between
  * members (BLASTP_GROUP=0 disables).  A search uses the groups when its
  * window A satisfies A + 8 <= that gap (else, and for the debug entry
  * points, it searches query by query); results are identical either way. */

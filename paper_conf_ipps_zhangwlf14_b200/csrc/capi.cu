@@ -351,9 +351,11 @@ static int build_one_query(const char *ascii, int32_t len, const blastp_params *
 // >= A apart in the subject, so no two-hit pair, lasthit or ext_reach ever
 // links them, and every X-drop stops at the sentinels of its own member --
 // the group's search returns exactly the members' searches.
-// First-fit decreasing into groups of combined length <= kGroupLen (the
-// size that still keeps 32 warps per SM resident, like a q1054 search).
-constexpr int32_t kGroupLen = 1024;
+// First-fit decreasing into groups of combined length <= kGroupLen
+// (config 5 sweep, profiles/r01/group_sweep.txt: 768 757 ms, 1024 742,
+// 1280 732, 1536 746, 2048 824 -- longer groups cost resident warps --
+// vs 786 ms query by query).
+constexpr int32_t kGroupLen = 1280;
 static int build_groups(blastp_query_table *t, const char *const *queries, const int32_t *lens,
                         int32_t nq, cudaStream_t s) {
   const char *env = std::getenv("BLASTP_GROUP");  // knob: BLASTP_GROUP=0 disables grouping
@@ -363,6 +365,8 @@ static int build_groups(blastp_query_table *t, const char *const *queries, const
   }
   const int32_t gap = t->p.window + 8;
   t->group_gap = gap;
+  int32_t budget = kGroupLen;  // knob: BLASTP_GROUP_LEN (combined length per group)
+  if (const char *v = std::getenv("BLASTP_GROUP_LEN")) budget = std::max(3, std::atoi(v));
   std::vector<int32_t> order(static_cast<size_t>(nq));
   for (int32_t i = 0; i < nq; ++i) order[static_cast<size_t>(i)] = i;
   std::stable_sort(order.begin(), order.end(),
@@ -372,7 +376,7 @@ static int build_groups(blastp_query_table *t, const char *const *queries, const
   for (int32_t i : order) {
     size_t b = 0;
     for (; b < bins.size(); ++b)
-      if (used[b] + gap + lens[i] <= kGroupLen) break;
+      if (used[b] + gap + lens[i] <= budget) break;
     if (b == bins.size()) {
       bins.push_back({});
       used.push_back(-gap);
