@@ -818,9 +818,9 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.nchunks = db->nchunks;
     a.long_items = db->items;
     a.nlong = db->nlong;
-    // STATEFUL's walk state at a segment start depends on the whole subject
-    // before it (extension ends), so long subjects are walked whole
-    a.nsegs = p->filter_mode == BLASTP_FILTER_STATEFUL ? 0 : db->nsegs;
+    // STATEFUL splits long subjects by diagonal range instead:
+    // the same segment plan, no segment lists
+    a.nsegs = db->nsegs;
     a.seg_item = db->seg_item;
     a.seg_list = db->seg_list;
     a.seg_count = db->seg_count;

@@ -409,6 +409,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
   int mode = 0;  // 0: take the next work item; 1: a walker is active
   for (;;) {
     int64_t wstart = 0, wend = 0, wemit = 0;
+    int64_t dlo = INT64_MIN, dhi = INT64_MAX;  // STATEFUL segment: its diagonals
     bool walk = false;
     bool retrace = false;  // fallback walk: its hits were traced by the segments
     int sg = -1;
@@ -423,11 +424,27 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       if (ci < nsegs) {
         sg = int(ci);
         const LongItem &it = a.long_items[a.seg_item[sg]];
-        wemit = it.c.start + int64_t(sg - it.seg0) * a.seg_len;
-        wend = min(it.c.end, wemit + a.seg_len);
-        // R6 looks back < A positions: a warm-up of A rounded up to whole
-        // windows (seg_len >= 256 >= A keeps it inside the chunk)
-        wstart = sg == it.seg0 ? it.c.start : wemit - warm;
+        if constexpr (kSt) {
+          // STATEFUL: segment j owns the diagonals (stream position - q) in
+          // [dlo, dhi); every hit of such a diagonal lies in [dlo, dhi + lq),
+          // so the segment walks that range, keeps the hits of its own
+          // diagonals and holds each diagonal's whole lasthit walk (R15)
+          // (segment 0 also owns the diagonals below the chunk start: hits
+          // at its first positions with large q)
+          const int j = sg - it.seg0;
+          const int64_t d0 = it.c.start + int64_t(j) * a.seg_len;
+          dlo = j == 0 ? INT64_MIN : d0;
+          dhi = j == it.nseg - 1 ? INT64_MAX : d0 + a.seg_len;
+          wstart = wemit = d0;
+          wend = j == it.nseg - 1 ? it.c.end : min(it.c.end, d0 + a.seg_len + lq);
+          sg = -1;  // extends and emits itself (no list, no walker)
+        } else {
+          wemit = it.c.start + int64_t(sg - it.seg0) * a.seg_len;
+          wend = min(it.c.end, wemit + a.seg_len);
+          // R6 looks back < A positions: a warm-up of A rounded up to whole
+          // windows (seg_len >= 256 >= A keeps it inside the chunk)
+          wstart = sg == it.seg0 ? it.c.start : wemit - warm;
+        }
         st.first_subj = it.c.first_subj;
         st.last_subj = it.c.last_subj;
         walk = true;
@@ -435,6 +452,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         const LongItem it = a.long_items[ci - nsegs];
         st.first_subj = it.c.first_subj;
         st.last_subj = it.c.last_subj;
+        if (kSt && it.nseg > 0) continue;  // covered by its diagonal segments
         if (it.nseg > 0 && !kSt) {
           st.spbase = it.c.start - frame;
           if (lane == 0) {
@@ -554,6 +572,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     }
     __syncwarp();
     st.spbase = wstart - frame;
+    // frame-relative diagonal range (P - q) of a STATEFUL segment
+    int dlo_f = INT_MIN, dhi_f = INT_MAX;
+    if (kSt && dlo != INT64_MIN) dlo_f = int(dlo - st.spbase);
+    if (kSt && dhi != INT64_MAX) dhi_f = int(dhi - st.spbase);
     int win = frame;                           // frame position of lane 0 of the window
     int lastsent = frame - 1;                  // the sentinel before the chunk
     int64_t end = wend - st.spbase;            // frame position of the chunk end (exclusive)
@@ -622,6 +644,8 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
         rebase_ring();
         win -= kFrameSpan;
         lastsent -= kFrameSpan;
+        if (kSt && dlo_f != INT_MIN) dlo_f -= kFrameSpan;
+        if (kSt && dhi_f != INT_MAX) dhi_f -= kFrameSpan;
         end -= kFrameSpan;
         emit_f -= kFrameSpan;
       }
@@ -676,9 +700,10 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
       if (Hn) locate(0u, nown, nq);
       for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
         const uint32_t k = k0 + uint32_t(lane);
-        const bool act = k < Hn;
         const int own = nown;
         int q = nq;
+        bool act = k < Hn;
+        if constexpr (kSt) act = act && win + own - q >= dlo_f && win + own - q < dhi_f;
         if (k0 + 32 < Hn) locate(k0 + 32u, nown, nq);
         const int ls = __shfl_sync(kFull, ls_lane, own);
         int slot = 0;

@@ -75,14 +75,22 @@ def test_adversarial_low_complexity(bp, orc):
                     trace=True)
 
 
-def test_long_subjects_walked_whole(bp, orc):
-    """Long subjects (> 2C residues, segmented in LEFT mode) are walked whole
-    by one warp in STATEFUL mode; one subject is longer than the 16-bit frame
-    (rebases with pending entries flushed first)."""
+@pytest.mark.parametrize("knobs", [{}, {"BLASTP_SEGLEN": "256"}, {"BLASTP_SEGMENTS": "0"}],
+                         ids=["default", "seglen256", "whole"])
+def test_long_subjects_diagonal_segments(bp, orc, monkeypatch, knobs):
+    """Long subjects are split by diagonal range in STATEFUL mode: segment j
+    owns the diagonals [d_j, d_j + seg_len) (segment 0 also those below the
+    chunk start), walks [d_j, d_j + seg_len + Lq) and holds each of its
+    diagonals' whole lasthit walk; with segments off they are walked whole.
+    Exact copies of the query are planted across segment boundaries, and
+    one subject is longer than the 16-bit frame (rebases with pending
+    entries flushed first)."""
+    for k, v in knobs.items():
+        monkeypatch.setenv(k, v)
     q = gen_query(21, 300).decode()
     ascii, off = _long_subject_db(q)
     d = bp.pack_db(ascii, off)
-    assert d.segments > 0
+    assert (d.segments == 0) == ("BLASTP_SEGMENTS" in knobs)
     for window in (40, 256):
         g, _ = assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=ST, window=window),
                            trace=True)
