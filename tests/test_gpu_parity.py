@@ -725,6 +725,31 @@ def test_bad_residue_reported(bp):
     assert e.value.status == bp.E_BAD_RESIDUE
 
 
+def test_formatted_db_and_groups_errors(bp):
+    """Error paths of the formatted host database and of query batches: a bad
+    residue or a decreasing offset fails the format with the pack's status,
+    a bad query in a batch fails the whole batch, NULL handles are rejected."""
+    import ctypes
+    bad = np.frombuffer(b"MKVLAGGQ-RST", dtype=np.uint8).copy()
+    with pytest.raises(bp.BlastpError) as e:
+        bp.format_host_db(bad, np.array([0, 6, 12], dtype=np.int64), num_parts=2)
+    assert e.value.status == bp.E_BAD_RESIDUE
+    ok = np.frombuffer(b"MKVLAGGQWRST", dtype=np.uint8).copy()
+    with pytest.raises(bp.BlastpError) as e:
+        bp.format_host_db(ok, np.array([0, 8, 6, 12], dtype=np.int64))
+    assert e.value.status == bp.E_INVALID_ARG
+    with pytest.raises(bp.BlastpError) as e:
+        bp.build_query_batch(["MKVLAGG", "MKV1LL", "WWWAAA"], bp.Params())
+    assert e.value.status == bp.E_BAD_RESIDUE
+    t = bp.build_query_table("MKVLAGGQ", bp.Params())
+    rc = bp.lib.blastp_search_formatted_db(t.handle, None, ctypes.byref(bp.Params().c()), None,
+                                           None, 0, None)
+    assert rc == bp.E_INVALID_ARG
+    assert bp.lib.blastp_query_table_groups(None, None, None, None) == bp.E_INVALID_ARG
+    assert bp.lib.blastp_host_db_info(None, None, None, None, None, None) == bp.E_INVALID_ARG
+    bp.lib.blastp_host_db_free(None)  # no-op
+
+
 def test_debug_stats_match_oracle_counts(bp, orc):
     """Event counters of the kernel agree with the oracle's lists (config 1)."""
     (q,), db = config_workload(1)
