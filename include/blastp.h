@@ -101,8 +101,10 @@ const char *blastp_version(void);
  * q in [0, len-3] the list of all 24^3 words v with
  * sum_i BLOSUM62[query[q+i]][v_i] >= p->threshold, stored as a CSR table
  * word -> ascending query positions (the function of the paper's DFA),
- * plus the query codes.  Built on the host, copied to `device` on
- * `cuda_stream`; the call returns after the copies complete.
+ * plus the query codes.  The codes are validated and encoded on the host,
+ * the table is built on `device` (one thread per word: count, scan, fill;
+ * BLASTP_TABLE_BUILD=host enumerates on the host instead) on `cuda_stream`;
+ * the call returns when the table is complete.
  * query_ascii: host, `len` bytes (3 <= len <= BLASTP_MAX_QUERY_LEN).
  * Errors: INVALID_ARG (NULL, len < 3, word_len != 3), BAD_RESIDUE,
  * TOO_LONG, NOMEM, CUDA. */
