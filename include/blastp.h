@@ -51,7 +51,7 @@ extern "C" {
                                     W <= h - lasthit < A: extend, lasthit <- HSP subject
                                     end; else no change.  Decides coverage itself, so it
                                     requires ext_mode BLASTP_EXT_DIAGONAL.  Warp kernel
-                                    only; long subjects are walked whole (no segments). */
+                                    only; long subjects are split by diagonal range. */
 #define BLASTP_EXT_DIAGONAL 0  /* Alg. 3: a passing hit covered by the
                                   previous extension of its diagonal is skipped (R10) */
 #define BLASTP_EXT_HIT 1       /* Alg. 4: every passing
