@@ -217,6 +217,22 @@ def test_config5_shard_sampled(bp, orc, kernel_variant):
         d = bp.pack_db(db.ascii, db.offsets - db.offsets[0])
         g = bp.search_ungapped(t, d, p)
         del d
+        if k == 7:
+            # the same shard streamed from its formatted host image (the e2e
+            # path) gives the identical list
+            import torch
+            h = bp.format_host_db(db.ascii, db.offsets - db.offsets[0])
+            cap = len(g) + 1024
+            out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+            cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+            bp.search_formatted_db(t, h, out.data_ptr(), cap, cnt.data_ptr(), p)
+            nf = int(cnt.item())
+            assert nf == len(g)
+            bp.sort_hsps_device(out.data_ptr(), nf)
+            fm = out[: nf * 7].view(nf, 7).cpu().numpy()
+            h.free()
+            del out
+            assert np.array_equal(fm, g.view(np.int32).reshape(-1, 7))
         g["subject_id"] += lo
         assert len(g) > 100000
         assert set(np.unique(g["query_id"])) == set(range(64))
