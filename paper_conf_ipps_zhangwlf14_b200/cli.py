@@ -1,0 +1,113 @@
+"""Command line: ungapped BLASTP search of FASTA queries against a FASTA database.
+
+    python -m paper_conf_ipps_zhangwlf14_b200.cli QUERIES.fa DB.fa [options] > hits.tsv
+
+Reads both files, packs the database onto the GPU (or streams it from a
+formatted host image with --stream), searches every query (a batch: short
+queries share one scan as query groups) and prints one tab-separated line per
+HSP in canonical order (R11):
+
+    query  subject  q_start  s_start  length  score  diagonal
+
+with FASTA identifiers (first word of the header) and 0-based starts.  All of
+the search runs in libblastp.so (include/blastp.h); this module only parses
+FASTA and formats the result.  Options map to blastp_params (P:L143-144 T,
+P:L1344-1351 A, Fig. 8 X; R3-R15).
+"""
+from __future__ import annotations
+
+import argparse
+import sys
+
+import numpy as np
+
+
+def read_fasta(path: str) -> tuple[list[str], bytes, np.ndarray]:
+    """(ids, concatenated residues, offsets[n+1]) of a FASTA file; residue
+    letters are kept as written (the library validates and encodes them)."""
+    ids: list[str] = []
+    seqs: list[bytes] = []
+    cur: list[bytes] = []
+    with open(path, "rb") as f:
+        for raw in f:
+            line = raw.strip()
+            if not line:
+                continue
+            if line.startswith(b">"):
+                if ids:
+                    seqs.append(b"".join(cur))
+                cur = []
+                head = line[1:].split()
+                ids.append(head[0].decode(errors="replace") if head else f"seq{len(ids)}")
+            else:
+                if not ids:
+                    raise ValueError(f"{path}: sequence data before the first '>' header")
+                cur.append(line)
+    if ids:
+        seqs.append(b"".join(cur))
+    lens = np.array([len(s) for s in seqs], dtype=np.int64)
+    off = np.zeros(len(seqs) + 1, dtype=np.int64)
+    np.cumsum(lens, out=off[1:])
+    return ids, b"".join(seqs), off
+
+
+def main(argv: list[str] | None = None) -> int:
+    ap = argparse.ArgumentParser(description=__doc__.split("\n\n")[0])
+    ap.add_argument("queries", help="query FASTA")
+    ap.add_argument("db", help="database FASTA")
+    ap.add_argument("--threshold", "-T", type=int, default=11)
+    ap.add_argument("--window", "-A", type=int, default=40)
+    ap.add_argument("--xdrop", "-X", type=int, default=16)
+    ap.add_argument("--cutoff", type=int, default=41)
+    ap.add_argument("--filter", choices=["left", "either", "stateful"], default="left")
+    ap.add_argument("--ext", choices=["diagonal", "hit", "window"], default="diagonal")
+    ap.add_argument("--stream", action="store_true",
+                    help="keep the database in pinned host memory (formatted image) and stream it")
+    ap.add_argument("--device", type=int, default=0)
+    args = ap.parse_args(argv)
+
+    import torch
+
+    from . import blastp as bp
+
+    qids, qres, qoff = read_fasta(args.queries)
+    sids, sres, soff = read_fasta(args.db)
+    if not qids:
+        print("no queries", file=sys.stderr)
+        return 1
+    queries = [qres[qoff[i]:qoff[i + 1]] for i in range(len(qids))]
+    p = bp.Params(threshold=args.threshold, window=args.window, xdrop=args.xdrop,
+                  cutoff=args.cutoff,
+                  filter_mode={"left": bp.FILTER_LEFT, "either": bp.FILTER_EITHER,
+                               "stateful": bp.FILTER_STATEFUL}[args.filter],
+                  ext_mode={"diagonal": bp.EXT_DIAGONAL, "hit": bp.EXT_HIT,
+                            "window": bp.EXT_WINDOW}[args.ext])
+    torch.cuda.set_device(args.device)
+    table = bp.build_query_batch(queries, p, device=args.device)
+    residues = np.frombuffer(sres, dtype=np.uint8)
+    if args.stream:
+        h = bp.format_host_db(residues, soff, device=args.device)
+        cap = max(1 << 16, len(residues) // 100 * len(queries))
+        while True:
+            out = torch.empty(cap * 7, dtype=torch.int32, device="cuda")
+            cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+            bp.search_formatted_db(table, h, out.data_ptr(), cap, cnt.data_ptr(), p)
+            n = int(cnt.item())
+            if n <= cap:
+                break
+            cap = n + 1024
+        bp.sort_hsps_device(out.data_ptr(), n)
+        hsps = out[: n * 7].view(n, 7).cpu().numpy()
+        h.free()
+    else:
+        db = bp.pack_db(residues, soff, device=args.device)
+        hsps = bp.search_ungapped(table, db, p).view(np.int32).reshape(-1, 7)
+        db.free()
+    w = sys.stdout.write
+    for qi, si, diag, qs, ss, ln, sc in hsps.tolist():
+        w(f"{qids[qi]}\t{sids[si]}\t{qs}\t{ss}\t{ln}\t{sc}\t{diag}\n")
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,60 @@
+"""The FASTA command line (paper_conf_ipps_zhangwlf14_b200/cli.py): FASTA parsing
+on CPU; on the GPU its TSV equals the oracle's HSPs (resident and streamed DB)."""
+import os
+
+import numpy as np
+import pytest
+
+from synth import gen_db, gen_query
+
+
+def _write_fasta(path, ids, seqs, width=60):
+    with open(path, "w") as f:
+        for i, s in zip(ids, seqs):
+            f.write(f">{i} description text\n")
+            for k in range(0, len(s), width):
+                f.write(s[k:k + width] + "\n")
+            f.write("\n")
+
+
+def test_read_fasta(tmp_path):
+    from paper_conf_ipps_zhangwlf14_b200.cli import read_fasta
+    p = tmp_path / "a.fa"
+    p.write_text(">q1 first\nMKVL\nAGG\n\n>q2\n>q3 x y\nWW\n")
+    ids, res, off = read_fasta(str(p))
+    assert ids == ["q1", "q2", "q3"]
+    assert res == b"MKVLAGGWW"
+    assert off.tolist() == [0, 7, 7, 9]
+    bad = tmp_path / "b.fa"
+    bad.write_text("MKV\n>q\nAA\n")
+    with pytest.raises(ValueError):
+        read_fasta(str(bad))
+
+
+@pytest.mark.gpu
+def test_cli_matches_oracle(tmp_path, capsys, orc):
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_ipps_zhangwlf14_b200 import cli
+    qs = [gen_query(900 + i, L).decode() for i, L in enumerate([127, 300, 60])]
+    db = gen_db(901, 902, n_subjects=200, mean_len=250.0, queries=[q.encode() for q in qs],
+                plant_frac=0.4)
+    subs = [db.ascii[db.offsets[i]:db.offsets[i + 1]].tobytes().decode()
+            for i in range(len(db.offsets) - 1)]
+    qids = [f"query{i}" for i in range(len(qs))]
+    sids = [f"subj{i}" for i in range(len(subs))]
+    _write_fasta(tmp_path / "q.fa", qids, qs)
+    _write_fasta(tmp_path / "d.fa", sids, subs)
+    codes = orc.encode(db.ascii.tobytes())
+    tuples = sorted(tuple(h) for i, q in enumerate(qs)
+                    for h in orc.search(orc.encode(q), codes, db.offsets, query_id=i).hsps.tolist())
+    exp_lines = [f"{qids[qi]}\t{sids[si]}\t{q0}\t{s0}\t{ln}\t{sc}\t{diag}"
+                 for qi, si, diag, q0, s0, ln, sc in tuples]
+    assert len(exp_lines) > 20
+    for extra in ([], ["--stream"]):
+        assert cli.main([str(tmp_path / "q.fa"), str(tmp_path / "d.fa"), *extra]) == 0
+        out = capsys.readouterr().out.strip().split("\n")
+        assert out == exp_lines, extra
+    assert cli.main([str(tmp_path / "q.fa"), str(tmp_path / "d.fa"), "--filter", "stateful"]) == 0
+    assert len(capsys.readouterr().out.strip().split("\n")) > 20
