@@ -64,11 +64,24 @@ def main(argv: list[str] | None = None) -> int:
     ap.add_argument("--stream", action="store_true",
                     help="keep the database in pinned host memory (formatted image) and stream it")
     ap.add_argument("--device", type=int, default=0)
+    ap.add_argument("--distributed", action="store_true",
+                    help="one process per GPU under torchrun: each rank searches a residue-"
+                         "balanced subject range, HSPs gathered to rank 0 (dist.py), which prints")
     args = ap.parse_args(argv)
+
+    import os
 
     import torch
 
     from . import blastp as bp
+    rank, world = 0, 1
+    if args.distributed:
+        import torch.distributed as dist
+        rank = int(os.environ.get("RANK", "0"))
+        world = int(os.environ.get("WORLD_SIZE", "1"))
+        args.device = int(os.environ.get("LOCAL_RANK", "0")) % max(1, torch.cuda.device_count())
+        torch.cuda.set_device(args.device)
+        dist.init_process_group(os.environ.get("BLASTP_DIST_BACKEND", "nccl"))
 
     qids, qres, qoff = read_fasta(args.queries)
     sids, sres, soff = read_fasta(args.db)
@@ -85,7 +98,24 @@ def main(argv: list[str] | None = None) -> int:
     torch.cuda.set_device(args.device)
     table = bp.build_query_batch(queries, p, device=args.device)
     residues = np.frombuffer(sres, dtype=np.uint8)
-    if args.stream:
+    if world > 1:
+        # this rank's shard (blastp_shard_range), HSPs with global subject ids,
+        # gathered in rank order (canonical per query; re-sorted on rank 0)
+        from .dist import gather_hsps
+        d = bp.pack_db(residues, soff, rank, world, device=args.device)
+        local = torch.from_numpy(bp.search_ungapped(table, d, p).view(np.int32).reshape(-1, 7)
+                                 .copy()).cuda()
+        d.free()
+        allh = gather_hsps(local)
+        import torch.distributed as dist
+        dist.destroy_process_group()
+        if rank != 0:
+            return 0
+        n = allh.shape[0]
+        flat = allh.contiguous().view(-1)
+        bp.sort_hsps_device(flat.data_ptr(), n)
+        hsps = flat.view(n, 7).cpu().numpy()
+    elif args.stream:
         h = bp.format_host_db(residues, soff, device=args.device)
         cap = max(1 << 16, len(residues) // 100 * len(queries))
         while True:

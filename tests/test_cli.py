@@ -58,3 +58,36 @@ def test_cli_matches_oracle(tmp_path, capsys, orc):
         assert out == exp_lines, extra
     assert cli.main([str(tmp_path / "q.fa"), str(tmp_path / "d.fa"), "--filter", "stateful"]) == 0
     assert len(capsys.readouterr().out.strip().split("\n")) > 20
+
+
+@pytest.mark.gpu
+def test_cli_distributed_two_ranks(tmp_path):
+    """--distributed under torchrun (2 ranks sharing the one GPU through the
+    gloo backend): rank 0 prints exactly the single-process table."""
+    import subprocess
+    import sys
+
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    qs = [gen_query(910 + i, L).decode() for i, L in enumerate([200, 90])]
+    db = gen_db(911, 912, n_subjects=300, mean_len=250.0, queries=[q.encode() for q in qs],
+                plant_frac=0.4)
+    subs = [db.ascii[db.offsets[i]:db.offsets[i + 1]].tobytes().decode()
+            for i in range(len(db.offsets) - 1)]
+    _write_fasta(tmp_path / "q.fa", [f"q{i}" for i in range(len(qs))], qs)
+    _write_fasta(tmp_path / "d.fa", [f"s{i}" for i in range(len(subs))], subs)
+    args = [str(tmp_path / "q.fa"), str(tmp_path / "d.fa")]
+    env = dict(os.environ, PYTHONPATH=root, BLASTP_DIST_BACKEND="gloo")
+    one = subprocess.run([sys.executable, "-m", "paper_conf_ipps_zhangwlf14_b200.cli", *args],
+                         capture_output=True, text=True, env=env, cwd=root, timeout=300)
+    assert one.returncode == 0, one.stderr
+    two = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+                          "--nproc-per-node", "2", "--master-addr", "127.0.0.1",
+                          "--master-port", "29561", "-m", "paper_conf_ipps_zhangwlf14_b200.cli",
+                          *args, "--distributed"],
+                         capture_output=True, text=True, env=env, cwd=root, timeout=300)
+    assert two.returncode == 0, two.stderr[-2000:]
+    assert one.stdout.count("\n") > 20
+    assert two.stdout == one.stdout
