@@ -185,7 +185,7 @@ class SearchResult:
 def search(query: np.ndarray, db: np.ndarray, offsets: np.ndarray, params: Params | None = None,
            *, query_id: int = 0, subject_base: int = 0, matrix: np.ndarray | None = None,
            table=None, nthreads: int = 1, want_hits: bool = False,
-           want_extensions: bool = True) -> SearchResult:
+           want_extensions: bool = True, cap_hint: int = 0) -> SearchResult:
     """Oracle search of one query (codes) against db codes with offsets[nseq+1]."""
     p = params or Params()
     q = np.ascontiguousarray(query, dtype=np.uint8)
@@ -208,7 +208,7 @@ def search(query: np.ndarray, db: np.ndarray, offsets: np.ndarray, params: Param
             hbufs = [np.zeros(cap_h, dtype=np.int32) for _ in range(6)]
             hl = _HitList(cap_h, 0, hbufs[0].ctypes.data, hbufs[1].ctypes.data, hbufs[2].ctypes.data)
             ps = _HitList(cap_h, 0, hbufs[3].ctypes.data, hbufs[4].ctypes.data, hbufs[5].ctypes.data)
-        cap = 1 << 12
+        cap = max(1 << 12, int(cap_hint))  # output buffer size only (a rerun if too small)
         for _ in range(8):
             out = np.zeros(cap, dtype=HSP_DTYPE)
             ext = np.zeros(cap * 8 if want_extensions else 1, dtype=HSP_DTYPE)

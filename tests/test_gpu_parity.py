@@ -85,12 +85,73 @@ def test_config1_full_trace(bp, orc, mode, ext_mode):
     assert len(g) > 10
 
 
-def test_config2_full(bp, orc):
-    """Config 2 (q517 vs 20M residues), complete HSP list."""
-    (q,), db = config_workload(2)
-    p = bp.Params()
-    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, p, trace=False,
-                       nthreads=os.cpu_count() or 8)
+# Complete oracle lists at full size, computed once per session on all host
+# cores and shared by the kernel-variant parametrisation: key -> canonical
+# HSP array of one query (query_id 0).
+_ORACLE_FULL = {}
+
+
+def oracle_full(orc, key, q_ascii, ascii, offsets, p):
+    """The oracle's complete HSP list of one query against a whole (shard of
+    a) database, all host cores, no sampling."""
+    k = (key, bytes(q_ascii if isinstance(q_ascii, bytes) else q_ascii.encode()), p.filter_mode,
+         1 if p.ext_mode == 1 else 0, p.window, p.min_gap)
+    if k not in _ORACLE_FULL:
+        codes = _ORACLE_FULL.get(("codes", key))
+        if codes is None:
+            codes = orc.encode(ascii.tobytes())
+            _ORACLE_FULL[("codes", key)] = codes
+        P = orc.Params(word_len=p.word_len, threshold=p.threshold, window=p.window,
+                       min_gap=p.min_gap, xdrop=p.xdrop, cutoff=p.cutoff,
+                       filter_mode=p.filter_mode, ext_mode=1 if p.ext_mode == 1 else 0)
+        off = np.asarray(offsets, dtype=np.int64)
+        r = orc.search(orc.encode(q_ascii), codes, off - off[0], P, nthreads=os.cpu_count() or 8,
+                       want_extensions=False, cap_hint=max(1 << 16, int(off[-1] - off[0]) // 2000))
+        _ORACLE_FULL[k] = r.hsps
+    return _ORACLE_FULL[k]
+
+
+def assert_lists_equal(got, exp, what):
+    """Element-by-element equality of two canonical HSP arrays; on a mismatch
+    report the first divergence."""
+    got = np.asarray(got)
+    exp = np.asarray(exp)
+    if len(got) == len(exp) and (got == exp).all():
+        return
+    n = min(len(got), len(exp))
+    bad = np.nonzero(got[:n] != exp[:n])[0]
+    i = int(bad[0]) if len(bad) else n
+    raise AssertionError(f"{what}: {len(got)} GPU vs {len(exp)} oracle HSPs; first divergence at "
+                         f"{i}: gpu {tuple(got[i]) if i < len(got) else None} oracle "
+                         f"{tuple(exp[i]) if i < len(exp) else None}")
+
+
+def _with_qid(a, qid):
+    a = a.copy()
+    a["query_id"] = qid
+    return a
+
+
+_CONFIG2 = {}
+
+
+def _config2():
+    if not _CONFIG2:
+        _CONFIG2["w"] = config_workload(2)
+    return _CONFIG2["w"]
+
+
+@pytest.mark.parametrize("mode,ext_mode", [(0, 0), (1, 0), (2, 0), (0, 1), (0, 2)],
+                         ids=["LEFT", "EITHER", "STATEFUL", "HIT", "WINDOW"])
+def test_config2_full(bp, orc, mode, ext_mode):
+    """Config 2 (q517 vs 20M residues): the complete HSP list identical to the
+    oracle's, every filter reading (R6 LEFT / EITHER, R15 STATEFUL) and every
+    extension strategy (Alg. 3 diagonal, Alg. 4 hit, Alg. 5 window)."""
+    (q,), db = _config2()
+    p = bp.Params(filter_mode=mode, ext_mode=ext_mode)
+    g = bp.search_ungapped(bp.build_query_table(q, p), bp.pack_db(db.ascii, db.offsets), p)
+    exp = oracle_full(orc, "config2", q, db.ascii, db.offsets, p)
+    assert_lists_equal(g, exp, f"config 2 {p}")
     assert len(g) > 1000
 
 
@@ -104,21 +165,85 @@ def _config3():
     return _CONFIG3["w"]
 
 
-def assert_sampled_parity(bp, orc, queries, ascii, offsets, g, p, blocks, subject_base=0,
-                          rescore=2000):
-    """Full-size parity where the oracle cannot redo the whole search: every
-    GPU HSP of a deterministic sample is re-scored from the sequences (P5),
-    and for each subject block [lo, hi) (global ids) the oracle re-searches
-    the block for every query and the GPU's HSPs on those subjects must be
-    identical."""
+def _config3_db(bp):
+    if "db" not in _CONFIG3:
+        (_,), db = _config3()
+        _CONFIG3["db"] = bp.pack_db(db.ascii, db.offsets)
+    return _CONFIG3["db"]
+
+
+def rescore(orc, queries, ascii, offsets, g, subject_base=0, n=2000):
+    """P5 on a deterministic sample of HSPs: score = the BLOSUM62 sum over the
+    segment, read from the sequences."""
     B = orc.blosum62()
     Qs = [orc.encode(q) for q in queries]
     rng = np.random.default_rng(0)
-    for h in g[rng.choice(len(g), size=min(rescore, len(g)), replace=False)]:
+    for h in g[rng.choice(len(g), size=min(n, len(g)), replace=False)]:
         a = offsets[h["subject_id"]] + h["s_start"] - offsets[subject_base]
         S = orc.encode(ascii[a:a + h["length"]].tobytes())
         Q = Qs[h["query_id"]]
         assert B[Q[h["q_start"]:h["q_start"] + h["length"]], S].sum() == h["score"]
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2], ids=["LEFT", "EITHER", "STATEFUL"])
+def test_config3_full(bp, orc, kernel_variant, mode):
+    """Config 3 at full size (q1054 vs 6.0M subjects / ~1.2G residues, the
+    bench launch): the complete HSP list identical to the oracle's complete
+    list (no sampling), both R6 readings and the STATEFUL walk."""
+    if kernel_variant == "cta" and mode == 2:
+        pytest.skip("STATEFUL runs on the warp variant only")
+    (q,), db = _config3()
+    p = bp.Params(filter_mode=mode)
+    g = bp.search_ungapped(bp.build_query_table(q, p), _config3_db(bp), p)
+    exp = oracle_full(orc, "config3", q, db.ascii, db.offsets, p)
+    assert len(exp) > 10000
+    assert_lists_equal(g, exp, f"config 3 {p}")
+    rescore(orc, [q], db.ascii, db.offsets, g)
+
+
+def test_config4_sharded_full(bp, orc, kernel_variant):
+    """Config 4: queries 127/517/1054 (one batch) against config 3's database
+    cut into 1, 2, 4 and 8 residue-balanced subject-range shards (one per GPU
+    in production; here shard by shard on one device).  The concatenation of
+    the shards' lists (dist.gather_hsps) is, for every shard count, exactly the
+    oracle's complete list of the three queries against the whole database."""
+    if kernel_variant == "cta":
+        pytest.skip("shard arithmetic is kernel-independent; the cta variant is covered "
+                    "by config 3")
+    from synth import CONFIGS, gen_query
+    (_,), db = _config3()
+    queries = [gen_query(CONFIGS[1]["query_seed"], 127), gen_query(CONFIGS[2]["query_seed"], 517),
+               gen_query(CONFIGS[3]["query_seed"], 1054)]
+    p = bp.Params()
+    exp = np.concatenate([_with_qid(oracle_full(orc, "config3", q, db.ascii, db.offsets, p), i)
+                          for i, q in enumerate(queries)])
+    exp = np.sort(exp, order=list(exp.dtype.names))
+    t = bp.build_query_batch(queries, p)
+    for n in (1, 2, 4, 8):
+        parts = []
+        for k in range(n):
+            d = _config3_db(bp) if n == 1 else bp.pack_db(db.ascii, db.offsets, k, n)
+            parts.append(bp.search_ungapped(t, d, p))
+            if n > 1:
+                d.free()
+        cat = np.concatenate(parts)
+        # per-shard canonical order; the gathered list sorted by query first
+        got = np.sort(cat, order=list(cat.dtype.names))
+        assert_lists_equal(got, exp, f"config 4, {n} shards")
+    assert len(exp) > 10000
+
+
+def assert_sampled_parity(bp, orc, queries, ascii, offsets, g, p, blocks, subject_base=0,
+                          rescore_n=2000):
+    """Full-size parity where the oracle cannot redo the whole search in the
+    default suite (config 5: 64 queries x 1.9G residues per shard): every GPU
+    HSP of a deterministic sample is re-scored from the sequences (P5), and
+    for each subject block [lo, hi) (global ids) the oracle re-searches the
+    block for every query and the GPU's HSPs on those subjects must be
+    identical.  test_config5_shard_full runs the complete comparison."""
+    rescore(orc, queries, ascii, offsets, g, subject_base, rescore_n)
+    B = orc.blosum62()
+    Qs = [orc.encode(q) for q in queries]
     P = orc.Params(word_len=p.word_len, threshold=p.threshold, window=p.window,
                    min_gap=p.min_gap, xdrop=p.xdrop, cutoff=p.cutoff, filter_mode=p.filter_mode,
                    ext_mode=1 if p.ext_mode == 1 else 0)
@@ -136,64 +261,6 @@ def assert_sampled_parity(bp, orc, queries, ascii, offsets, g, p, blocks, subjec
             exp += tuples(e)
         sel = g[(g["subject_id"] >= lo) & (g["subject_id"] < hi)]
         assert tuples(sel) == sorted(exp), (lo, hi)
-
-
-def test_config3_full_size_sampled(bp, orc):
-    """Config 3 at full size (q1054 vs ~1.2G residues, the bench launch):
-    the oracle re-searches a deterministic sample of subject blocks and the
-    GPU's HSPs restricted to those subjects must be identical; every GPU HSP
-    is re-scored from the sequences."""
-    (q,), db = _config3()
-    p = bp.Params()
-    t = bp.build_query_table(q, p)
-    d = bp.pack_db(db.ascii, db.offsets)
-    g = bp.search_ungapped(t, d, p)
-    assert len(g) > 10000
-    n = db.nseq
-    blocks = [(k, min(k + 3000, n)) for k in range(0, n, n // 12)][:12]
-    blocks.append((n // 2 - 5, n // 2 + 5))  # the 36,805-residue subject
-    assert_sampled_parity(bp, orc, [q], db.ascii, db.offsets, g, p, blocks)
-
-
-def test_config4_sharded_sampled(bp, orc, kernel_variant):
-    """Config 4: queries 127/517/1054 (one batch) against config 3's database
-    cut into 2, 4 and 8 residue-balanced subject-range shards (one per GPU in
-    production; here shard by shard on one device).  Every shard count gives
-    the whole-database list (contiguous ranges, canonical order per shard:
-    the NCCL gather is a plain concatenation, dist.gather_hsps), and that list
-    matches the oracle on sampled subject blocks, including the blocks that
-    straddle every 8-shard boundary."""
-    if kernel_variant == "cta":
-        pytest.skip("shard arithmetic is kernel-independent; the cta variant is covered "
-                    "by config 3")
-    from synth import CONFIGS, gen_query
-    (_,), db = _config3()
-    queries = [gen_query(CONFIGS[1]["query_seed"], 127), gen_query(CONFIGS[2]["query_seed"], 517),
-               gen_query(CONFIGS[3]["query_seed"], 1054)]
-    p = bp.Params()
-    t = bp.build_query_batch(queries, p)
-    whole = None
-    bounds = []
-    for n in (1, 2, 4, 8):
-        parts = []
-        for k in range(n):
-            d = bp.pack_db(db.ascii, db.offsets, k, n)
-            if n == 8 and k > 0:
-                bounds.append(d.subject_base)
-            parts.append(bp.search_ungapped(t, d, p))
-            del d
-        cat = np.concatenate(parts)
-        # per-shard canonical order; the gathered list sorted by query first
-        got = np.sort(cat, order=list(cat.dtype.names))
-        if whole is None:
-            whole = got
-            assert len(whole) > 10000
-        else:
-            assert tuples(got) == tuples(whole), n
-    nseq = db.nseq
-    blocks = [(max(0, b - 300), min(nseq, b + 300)) for b in bounds]
-    blocks += [(k, min(k + 1500, nseq)) for k in range(0, nseq, nseq // 5)][:5]
-    assert_sampled_parity(bp, orc, queries, db.ascii, db.offsets, whole, p, blocks)
 
 
 def test_config5_shard_sampled(bp, orc, kernel_variant):
@@ -239,6 +306,41 @@ def test_config5_shard_sampled(bp, orc, kernel_variant):
         n = hi - lo
         blocks = [(lo + j, lo + min(j + 600, n)) for j in range(0, n, n // 6)][:6]
         assert_sampled_parity(bp, orc, queries, db.ascii, off, g, p, blocks, subject_base=lo)
+
+
+
+
+@pytest.mark.skipif(os.environ.get("BLASTP_FULL_CONFIG5") != "1",
+                    reason="~10 min of oracle time on 16 cores: run once per round with "
+                           "BLASTP_FULL_CONFIG5=1 (log in profiles/)")
+def test_config5_shard_full(bp, orc, kernel_variant):
+    """Config 5, one full shard with no sampling: the 64 queries (len
+    U[100, 2000]) against shard 0 of 8 of the nr-shaped database (~1.9G
+    residues, ~5M subjects); the GPU list equals the oracle's complete list of
+    all 64 queries."""
+    if kernel_variant == "cta":
+        pytest.skip("the 64-query full-size shard runs on the default (warp) variant")
+    import time
+    from paper_conf_ipps_zhangwlf14_b200.dist import shard_subjects
+    from synth import config_offsets
+    off = config_offsets(5)
+    lo, hi = shard_subjects(off, 0, 8)
+    queries, db = config_workload(5, subject_range=(lo, hi))
+    p = bp.Params()
+    t0 = time.perf_counter()
+    g = bp.search_ungapped(bp.build_query_batch(queries, p),
+                           bp.pack_db(db.ascii, db.offsets - db.offsets[0]), p)
+    t_gpu = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    exp = np.concatenate([_with_qid(oracle_full(orc, "config5s0", q, db.ascii, db.offsets, p), i)
+                          for i, q in enumerate(queries)])
+    t_orc = time.perf_counter() - t0
+    exp = np.sort(exp, order=list(exp.dtype.names))
+    assert_lists_equal(g, exp, "config 5 shard 0 of 8")
+    print(f"config5 shard 0/8 full parity: {len(g)} HSPs, {hi - lo} subjects, "
+          f"{int(db.offsets[-1] - db.offsets[0])} residues, 64 queries; GPU search "
+          f"{t_gpu:.1f} s (incl. table build + pack), oracle {t_orc:.1f} s on "
+          f"{os.cpu_count()} threads")
 
 
 @pytest.mark.parametrize("T", [8, 11, 13])
@@ -592,7 +694,7 @@ def test_formatted_host_db_config3_full_size(bp):
     """Config 3 at full size (the bench's e2e path): the formatted image
     streamed in parts gives exactly the resident shard's HSP list (the
     resident list is itself pinned to the oracle by
-    test_config3_full_size_sampled)."""
+    test_config3_full)."""
     import torch
     (q,), db = _config3()
     p = bp.Params()

@@ -8,8 +8,7 @@ import numpy as np
 import pytest
 
 from synth import config_workload, gen_db, gen_query
-from test_gpu_parity import (_config3, _long_subject_db, _rand_db, assert_same,
-                             assert_sampled_parity, tuples, ALPHA)
+from test_gpu_parity import _long_subject_db, _rand_db, assert_same, ALPHA
 
 pytestmark = pytest.mark.gpu
 ST = 2  # BLASTP_FILTER_STATEFUL
@@ -40,11 +39,9 @@ def test_config1_full_trace(bp, orc):
     assert len(g) > 10 and len(r.passing) > 100
 
 
-def test_config2_full(bp, orc):
-    (q,), db = config_workload(2)
-    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=ST), trace=False,
-                       nthreads=os.cpu_count() or 8)
-    assert len(g) > 1000
+# Configs 2 and 3 in STATEFUL mode (complete lists vs the oracle, no
+# sampling): test_gpu_parity.py::test_config2_full[STATEFUL] and
+# ::test_config3_full[STATEFUL].
 
 
 def test_fuzz_small_random(bp, orc):
@@ -101,24 +98,6 @@ def test_long_query_2000(bp, orc):
     q = gen_query(2000, 2000)
     db = gen_db(7, 8, n_subjects=400, mean_len=375.0, queries=[q], plant_frac=0.2)
     assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=ST), trace=True)
-
-
-def test_config3_full_size_sampled(bp, orc, kernel_variant):
-    """Config 3 at full size in STATEFUL mode: sampled subject blocks re-searched
-    by the oracle, every sampled GPU HSP re-scored from the sequences."""
-    if kernel_variant == "cta":
-        pytest.skip("same kernel as the warp run")
-    (q,), db = _config3()
-    p = bp.Params(filter_mode=ST)
-    t = bp.build_query_table(q, p)
-    d = bp.pack_db(db.ascii, db.offsets)
-    g = bp.search_ungapped(t, d, p)
-    left = bp.search_ungapped(t, d, bp.Params())
-    assert len(g) > 10000 and len(g) != len(left)
-    n = db.nseq
-    blocks = [(k, min(k + 2000, n)) for k in range(0, n, n // 8)][:8]
-    blocks.append((n // 2 - 5, n // 2 + 5))  # the 36,805-residue subject
-    assert_sampled_parity(bp, orc, [q], db.ascii, db.offsets, g, p, blocks)
 
 
 def test_stateful_requires_diagonal_ext_mode(bp):
