@@ -101,6 +101,7 @@ int num_sms(int device) {
 
 struct QueryDev {
   uint32_t *woff = nullptr;
+  uint2 *wtab = nullptr;  // radix-32 view of woff (launch_table_radix32)
   uint16_t *qpos = nullptr;
   uint8_t *qcodes = nullptr;
   int32_t lq = 0;
@@ -202,6 +203,7 @@ static cudaError_t plan_long_items(blastp_db *db, int nlong, cudaStream_t s) {
 
 static void free_query_dev(QueryDev &d) {
   cudaFree(d.woff);
+  cudaFree(d.wtab);
   cudaFree(d.qpos);
   cudaFree(d.qcodes);
   cudaFree(d.sub);
@@ -259,6 +261,18 @@ static int encode_query(const char *ascii, int32_t len, std::vector<uint8_t> &Q)
 // Lookup table (R3) of the query codes Q (a query, or a group's members
 // separated by sentinel codes: a word touching a sentinel scores -1000 per
 // sentinel letter and neighbours nothing).
+// The radix-32 (start, count) view the block kernel reads (table.cu).
+static int finish_table(QueryDev &out, cudaStream_t s) {
+  if (cudaMallocAsync(&out.wtab, sizeof(uint2) * 32 * 32 * 32, s) != cudaSuccess) {
+    cudaGetLastError();
+    free_query_dev(out);
+    return fail(BLASTP_E_NOMEM, "device allocation for the query table failed");
+  }
+  CUDA_TRY(launch_table_radix32(out.woff, out.wtab, s));
+  CUDA_TRY(cudaStreamSynchronize(s));
+  return BLASTP_OK;
+}
+
 static int build_table(const std::vector<uint8_t> &Q, const blastp_params *p, QueryDev &out,
                        cudaStream_t s) {
   const int32_t len = static_cast<int32_t>(Q.size());
@@ -283,8 +297,7 @@ static int build_table(const std::vector<uint8_t> &Q, const blastp_params *p, Qu
       return fail(BLASTP_E_NOMEM, "device allocation for the query table failed");
     }
     CUDA_TRY(launch_table_fill(out.qcodes, len, p->threshold, out.woff, out.qpos, s));
-    CUDA_TRY(cudaStreamSynchronize(s));
-    return BLASTP_OK;
+    return finish_table(out, s);
   }
   // Neighbourhood words by pruned enumeration: for each query word, walk the
   // 24^3 words letter by letter and cut a branch as soon as even the best
@@ -334,8 +347,7 @@ static int build_table(const std::vector<uint8_t> &Q, const blastp_params *p, Qu
   CUDA_TRY(cudaMemcpyAsync(out.qpos, pos.data(), sizeof(uint16_t) * pos.size(),
                            cudaMemcpyHostToDevice, s));
   CUDA_TRY(cudaMemcpyAsync(out.qcodes, Q.data(), Q.size(), cudaMemcpyHostToDevice, s));
-  CUDA_TRY(cudaStreamSynchronize(s));  // host vectors die here
-  return BLASTP_OK;
+  return finish_table(out, s);  // synchronises: the host vectors die here
 }
 
 static int build_one_query(const char *ascii, int32_t len, const blastp_params *p, QueryDev &out,
@@ -829,6 +841,7 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.seg_cap = db->seg_cap;
     a.seq = ++const_cast<blastp_db *>(db)->seq;
     a.qv.woff = qd.woff;
+    a.qv.wtab = qd.wtab;
     a.qv.qpos = qd.qpos;
     a.qv.qcodes = qd.qcodes;
     a.qv.lq = qd.lq;

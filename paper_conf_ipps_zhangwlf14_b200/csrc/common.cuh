@@ -86,6 +86,7 @@ struct TraceRec {
 // Per-query device view of a lookup table (R3): CSR word -> query positions.
 struct QueryView {
   const uint32_t *woff;   // [kWords + 1]
+  const uint2 *wtab;      // [32^3] radix-32 code -> (woff, count) (table.cu)
   const uint16_t *qpos;   // [entries], ascending within a word
   const uint8_t *qcodes;  // [lq] query codes
   int32_t lq, query_id;
@@ -152,10 +153,15 @@ int search_ring_slots(int lq, int window);
 // variable BLASTP_KERNEL=warp|cta forces one (tests cover both).
 cudaError_t launch_search(const SearchArgs &a, int num_sms, cudaStream_t s);
 cudaError_t launch_search_warp(const SearchArgs &a, int num_sms, cudaStream_t s);
+// The block kernel (search_block.cu), default for filter_mode LEFT with
+// ext_mode DIAGONAL/HIT when window >= 31 + min_gap (block_kernel_eligible).
+bool block_kernel_eligible(const SearchArgs &a);
+cudaError_t launch_search_block(const SearchArgs &a, int num_sms, cudaStream_t s);
 // Query lookup table on the GPU (table.cu): woff (kWords + 1) from the query
 // codes, the entry count returned on the host (synchronises s), then qpos.
 cudaError_t launch_table_count(const uint8_t *qcodes, int lq, int T, uint32_t *woff,
                                int64_t *total, cudaStream_t s);
+cudaError_t launch_table_radix32(const uint32_t *woff, uint2 *wtab, cudaStream_t s);
 cudaError_t launch_table_fill(const uint8_t *qcodes, int lq, int T, const uint32_t *woff,
                               uint16_t *qpos, cudaStream_t s);
 cudaError_t launch_pack(const uint8_t *ascii, const int64_t *off, int64_t n,

@@ -1,0 +1,559 @@
+// search_block.cu -- the default search kernel of filter_mode LEFT (sm_100a):
+// hit detection, two-hit filter and X-drop ungapped extension fused per warp,
+// with a per-diagonal "block" two-hit state that makes every 32-hit round
+// conflict-free (no per-round loop over same-diagonal hits).
+//
+// Each warp owns a chunk of whole subjects at a time (work stealing) and
+// walks it in ascending subject position, 32 positions per window, lane =
+// position ("coalesced": one byte per lane, consecutive lanes,
+// consecutive positions).
+//
+//   hit detection   Alg. 2: lane v looks up the word at its
+//                   position in the query table (R3; radix-32 view, one
+//                   8-byte L2 load: (first entry, count)), the window's hits
+//                   are expanded in 32-hit rounds in s order.
+//   bins / sort     P:L967-1343: replaced by a per-warp ring indexed by the
+//                   diagonal (s - q) mod M, visited in ascending s -- the
+//                   order the paper's segmented sort establishes.
+//   two-hit filter  P:L1344-1351, reading R6 (LEFT): h passes iff a hit p on
+//                   its diagonal and subject has W <= h - p < A.
+//   extension       Alg. 3 + Fig. 8 (R7-R10): passing hits
+//                   not covered by ext_reach are queued; 32 at a time are
+//                   X-dropped lane-parallel and the ext_reach chain is
+//                   resolved per diagonal in queue (= s) order.
+//
+// Block state.  Positions are cut into record blocks of 32:
+// the window [b, b+32) of lanes is block k, split further at subject
+// boundaries (a sentinel starts a new block: bid = max(b, last sentinel+1)).
+// One 32-bit word per diagonal slot describes the hits recorded on it:
+//   bid (14 bits, frame position of its block start; 0 = none),
+//   min - bid, max - bid (5 bits each: the first and last hit of the block),
+//   bid - prev (8 bits: prev = the last hit before the block; 0 = none).
+// Test of a hit h at lane v, with L = W - 1:
+//   * v >= L: valid predecessors are the block's hits <= h - W, and every
+//     earlier hit (each is <= b - 1 <= h - W).  With A >= 32 + L every
+//     block hit lies within A of h, so "a block hit <= h - W exists" is
+//     "min <= h - W"; the earlier hits reduce to the largest (max of the
+//     older state, or prev).  Hits of the same block in this round count
+//     through the round's first member of the (slot, bid) group.
+//   * v < L: h - W falls before the block, so h is tested against the
+//     previous block's final state (the ring as the round starts): min of
+//     that block <= h - W, else its prev.
+// The state write is commutative per round: the group's first member gives
+// min, its last member max, and the last member alone stores the word.
+// Valid for filter LEFT when A >= 31 + W (block_kernel_eligible); other
+// parameters run the warp kernel (search.cu), which keeps exact per-hit
+// state (last / far / near) instead.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstdlib>
+#include <cstring>
+
+#include "search_common.cuh"
+
+namespace blastp {
+
+using namespace dev;
+
+namespace {
+
+constexpr int kBlkWarps = 32;        // warps per CTA (independent walkers)
+constexpr int kBlkQcap = 64;         // extension queue slots per warp
+constexpr int kBlkFrameMin = 512;    // first frame position (> A + 2 blocks)
+constexpr int kBlkFrameSpan = 8192;  // rebase step: frame positions < 2^14
+constexpr int kBlkFixed = 448;       // queue 256 B + flush / owner scratch 192 B
+
+__constant__ int8_t c_b62_blk[32 * 32];
+
+__device__ __forceinline__ int be_bid(uint32_t e) { return int(e & 0x3fffu); }
+__device__ __forceinline__ int be_minoff(uint32_t e) { return int((e >> 14) & 31u); }
+__device__ __forceinline__ int be_maxoff(uint32_t e) { return int((e >> 19) & 31u); }
+__device__ __forceinline__ int be_prevoff(uint32_t e) { return int(e >> 24); }
+
+// Per-warp shared memory: fixed parts first (every address is the warp's
+// base plus a constant), then ring[M] (block state) and reach[M] (ext_reach).
+struct BlkArea {
+  uint8_t *base;
+  int reach_off;
+  __device__ __forceinline__ uint32_t *queue() const { return reinterpret_cast<uint32_t *>(base); }
+  __device__ __forceinline__ uint32_t *scr() const { return reinterpret_cast<uint32_t *>(base + 256); }
+  __device__ __forceinline__ uint16_t *fs_p() const { return reinterpret_cast<uint16_t *>(base + 256); }
+  __device__ __forceinline__ uint16_t *fs_end() const { return fs_p() + 32; }
+  __device__ __forceinline__ uint16_t *fs_acc() const { return fs_p() + 64; }
+  __device__ __forceinline__ uint32_t *ring() const {
+    return reinterpret_cast<uint32_t *>(base + kBlkFixed);
+  }
+  __device__ __forceinline__ uint16_t *reach() const {
+    return reinterpret_cast<uint16_t *>(base + reach_off);
+  }
+};
+
+__host__ __device__ size_t blk_area_bytes(int ring) {
+  return kBlkFixed + align16(size_t(ring) * 4) + align16(size_t(ring) * 2);
+}
+
+struct BlkState {
+  int64_t spbase;  // stream position of frame position 0
+  int64_t first_subj, last_subj;
+  int qhead, qcount;
+  unsigned long long stat[kNumStats];  // tracing variant only
+};
+
+template <bool kStats>
+__device__ __forceinline__ void bstat(BlkState &st, int i, unsigned long long v) {
+  if (kStats) st.stat[i] += v;
+}
+
+// Extend up to 32 queued passing hits lane-parallel (R7-R9), then resolve the
+// ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order;
+// kHit: Alg. 4, every passing hit extended and kept (reading R14).
+template <bool kTrace, bool kHit>
+__device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w, BlkState &st,
+                                          int n, const uint8_t *qc, const int8_t *b62, int lane,
+                                          int slotc, int M) {
+  const bool act = lane < n;
+  uint32_t ent = 0;
+  if (act) ent = w.queue()[(st.qhead + lane) & (kBlkQcap - 1)];
+  const int P = int(ent & 0xffffu), q = int(ent >> 16);
+  int slot = (P - q + slotc) % M;
+  slot += slot < 0 ? M : 0;
+  const int64_t sp = st.spbase + P;
+  int total = 0, llen = 0, rlen = 0, scanned = 0;
+  if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen, scanned);
+  if (kTrace) {
+    bstat<kTrace>(st, kStatFlushes, 1);
+    bstat<kTrace>(st, kStatExtended, n);
+    bstat<kTrace>(st, kStatXdropSteps, __reduce_add_sync(kFull, unsigned(scanned)));
+    bstat<kTrace>(st, kStatXdropLaneSlots, 32ull * __reduce_max_sync(kFull, unsigned(scanned)));
+  }
+  bool acc = false;
+  if constexpr (kHit) {
+    acc = act;
+  } else {
+    // HSP subject end (inclusive); < 2^16: P < 2^14 and an extension never
+    // runs past the query (rlen < 16,000)
+    const int endp = P + 2 + rlen;
+    uint16_t *r16 = w.reach() + slot;
+    const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
+    const bool uniq = grp == (1u << lane);
+    if (__all_sync(kFull, uniq || !act)) {
+      if (act) {
+        acc = P > int(*r16);
+        if (acc) *r16 = uint16_t(endp);
+      }
+    } else {
+      w.fs_p()[lane] = uint16_t(P);
+      w.fs_end()[lane] = uint16_t(endp);
+      __syncwarp();
+      if (act) {
+        if (uniq) {
+          acc = P > int(*r16);
+          if (acc) *r16 = uint16_t(endp);
+        } else if (lane == __ffs(grp) - 1) {
+          int r = *r16;
+          unsigned g = grp;
+          while (g) {
+            const int j = __ffs(g) - 1;
+            g &= g - 1;
+            const bool aj = int(w.fs_p()[j]) > r;
+            if (aj) r = w.fs_end()[j];
+            w.fs_acc()[j] = aj;
+          }
+          *r16 = uint16_t(r);
+        }
+      }
+      __syncwarp();
+      if (act && !uniq) acc = w.fs_acc()[lane] != 0;
+    }
+  }
+  if (kTrace) {
+    bstat<kTrace>(st, kStatAccepted, __popc(__ballot_sync(kFull, acc)));
+    bstat<kTrace>(st, kStatEmitted, __popc(__ballot_sync(kFull, acc && total >= a.cutoff)));
+  }
+  if (acc) {
+    if (kTrace) trace_push(a, 2, sp, q, llen, rlen, total);
+    emit_hsp(a, sp, q, llen, rlen, total, st.first_subj, st.last_subj);
+  }
+  __syncwarp();
+  st.qhead = (st.qhead + n) & (kBlkQcap - 1);
+  st.qcount -= n;
+}
+
+// kW: min_gap fixed at compile time (3, the default) or 0 (runtime value);
+// kHit: ext_mode HIT (Alg. 4) instead of DIAGONAL (Alg. 3).
+template <bool kTrace, int kW, bool kHit>
+__global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const SearchArgs a) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int lq = a.qv.lq;
+  int8_t *b62 = reinterpret_cast<int8_t *>(smem);
+  uint8_t *qc = smem + 1024;
+  const size_t qc_bytes = align16(size_t(lq) + 2 * kQPad + 8);
+  for (int i = threadIdx.x; i < 1024; i += blockDim.x) b62[i] = c_b62_blk[i];
+  for (int i = threadIdx.x; i < int(qc_bytes); i += blockDim.x) {
+    const int k = i - kQPad;
+    qc[i] = (k >= 0 && k < lq) ? a.qv.qcodes[k] : uint8_t(kSentinel);
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int M = a.ring;
+  BlkArea w;
+  w.base = smem + 1024 + qc_bytes + size_t(warp) * blk_area_bytes(M);
+  w.reach_off = kBlkFixed + int(align16(size_t(M) * 4));
+  for (int i = lane; i < M; i += 32) {
+    w.ring()[i] = 0;
+    w.reach()[i] = 0;
+  }
+  __syncthreads();
+
+  const uint8_t *__restrict__ stream = a.stream;
+  const uint2 *__restrict__ wtab = a.qv.wtab;
+  const uint16_t *__restrict__ qpos = a.qv.qpos;
+  const int W = kW ? kW : a.min_gap;
+  const int L = W - 1;  // record lag: lanes v < L are tested against the previous block
+  const int A = a.window;
+  const unsigned ltmask = lanemask_lt(lane);
+  uint32_t *scr = w.scr();
+
+  BlkState st;
+  if (kTrace)
+    for (int i = 0; i < kNumStats; ++i) st.stat[i] = 0;
+  st.qhead = 0;
+  st.qcount = 0;
+  int frame = kBlkFrameMin;  // frame position of the next work item's first residue
+  int base_slot = 0;         // ring slot of (P, q) = base_slot + (P - b) - q (mod M)
+  const unsigned long long nsegs = (unsigned long long)a.nsegs;
+  const unsigned long long nitems = nsegs + (unsigned long long)a.nlong;
+  for (;;) {
+    unsigned long long ci = 0;
+    if (lane == 0) ci = atomicAdd(a.chunk_cursor, 1ull);
+    ci = __shfl_sync(kFull, ci, 0);
+    int64_t wstart, wend;
+    int64_t dlo = INT64_MIN, dhi = INT64_MAX;
+    if (ci < nsegs) {
+      // A long subject cut by diagonal range: segment j owns
+      // the diagonals (stream position - q) in [d_j, d_j + seg_len) --
+      // segment 0 also those below the chunk start -- and walks the positions
+      // [d_j, d_j + seg_len + Lq) where all of their hits lie, so each of its
+      // diagonals' whole R6 / R10 history stays inside the segment.
+      const LongItem it = a.long_items[a.seg_item[ci]];
+      const int j = int(ci) - it.seg0;
+      const int64_t d0 = it.c.start + int64_t(j) * a.seg_len;
+      dlo = j == 0 ? INT64_MIN : d0;
+      dhi = j == it.nseg - 1 ? INT64_MAX : d0 + a.seg_len;
+      wstart = d0;
+      wend = j == it.nseg - 1 ? it.c.end : min(it.c.end, d0 + a.seg_len + lq);
+      st.first_subj = it.c.first_subj;
+      st.last_subj = it.c.last_subj;
+    } else if (ci < nitems) {
+      const LongItem it = a.long_items[ci - nsegs];
+      if (it.nseg > 0) continue;  // covered by its diagonal segments
+      wstart = it.c.start;
+      wend = it.c.end;
+      st.first_subj = it.c.first_subj;
+      st.last_subj = it.c.last_subj;
+    } else {
+      const unsigned long long cj = ci - nitems;
+      if (cj >= (unsigned long long)a.nchunks) break;
+      const Chunk ch = a.chunks[cj];
+      wstart = ch.start;
+      wend = ch.end;
+      st.first_subj = ch.first_subj;
+      st.last_subj = ch.last_subj;
+    }
+
+    st.spbase = wstart - frame;
+    const bool seg = dlo != INT64_MIN || dhi != INT64_MAX;
+    int dlo_f = dlo != INT64_MIN ? int(dlo - st.spbase) : INT_MIN;
+    int dhi_f = dhi != INT64_MAX ? int(dhi - st.spbase) : INT_MAX;
+    int b = frame;             // frame position of lane 0 (block start)
+    int lastsent = frame - 1;  // the sentinel before the work item
+    int end = int(wend - st.spbase);
+    auto slotc = [&]() {  // ring slot of (P, q) = P - q + slotc (mod M)
+      int c = (base_slot - b) % M;
+      return c < 0 ? c + M : c;
+    };
+
+    // Software pipeline over windows: residues two windows ahead (one byte
+    // per lane + two of overlap), the table lookup one window ahead.
+    uint32_t pf_r = 0, pf_x = 0;
+    auto load_res = [&](int wn) {
+      const int64_t pp = st.spbase + wn;
+      pf_r = __ldg(stream + pp + lane);
+      pf_x = lane < 2 ? __ldg(stream + pp + 32 + lane) : 0u;
+    };
+    uint32_t nx_o = 0, nx_c = 0;
+    bool nx_s = false;
+    auto lookup = [&](int wn) {  // consumes pf_* (residues of window wn)
+      const uint32_t r0 = pf_r;
+      uint32_t r1 = __shfl_down_sync(kFull, pf_r, 1), r2 = __shfl_down_sync(kFull, pf_r, 2);
+      const uint32_t x0 = __shfl_sync(kFull, pf_x, 0), x1 = __shfl_sync(kFull, pf_x, 1);
+      if (lane == 31) {
+        r1 = x0;
+        r2 = x1;
+      }
+      if (lane == 30) r2 = x0;
+      load_res(wn + 32);
+      const bool in = wn + lane < end;
+      nx_s = in && r0 == uint32_t(kSentinel);
+      uint2 t = make_uint2(0u, 0u);
+      if (in) t = __ldg(wtab + ((r0 << 10) | (r1 << 5) | r2));
+      nx_o = t.x;
+      nx_c = t.y;
+    };
+    load_res(b);
+    lookup(b);
+
+    while (b < end) {
+      // ---- rebase the frame before positions outgrow 14 bits -------------
+      if (b >= kBlkFrameMin + kBlkFrameSpan) {
+        const int sc = slotc();
+        while (st.qcount > 0)
+          blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
+        for (int i = lane; i < M; i += 32) {
+          const uint32_t e = w.ring()[i];
+          // a state whose block starts before the new frame origin is older
+          // than any window A can reach back to: dropped
+          w.ring()[i] = be_bid(e) > kBlkFrameSpan ? e - uint32_t(kBlkFrameSpan) : 0u;
+          const uint32_t r = w.reach()[i];
+          w.reach()[i] = uint16_t(r > uint32_t(kBlkFrameSpan) ? r - kBlkFrameSpan : 0u);
+        }
+        __syncwarp();
+        st.spbase += kBlkFrameSpan;
+        b -= kBlkFrameSpan;
+        lastsent -= kBlkFrameSpan;
+        end -= kBlkFrameSpan;
+        if (dlo_f != INT_MIN) dlo_f -= kBlkFrameSpan;
+        if (dhi_f != INT_MAX) dhi_f -= kBlkFrameSpan;
+      }
+      bstat<kTrace>(st, kStatIterations, 1);
+      // ---- this window's lookup (issued last iteration); issue the next ---
+      const uint32_t o = nx_o, cnt = nx_c;
+      const unsigned sm = __ballot_sync(kFull, nx_s);
+      lookup(b + 32);
+      uint32_t incl = cnt;
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t t = __shfl_up_sync(kFull, incl, d);
+        if (lane >= d) incl += t;
+      }
+      const uint32_t excl = incl - cnt;
+      const uint32_t Hn = __shfl_sync(kFull, incl, 31);
+      // last sentinel at or before each lane (before the window: lastsent)
+      const unsigned prior = sm & ((lane == 31) ? kFull : ((2u << lane) - 1u));
+      const int ls_lane = prior ? (b + 31 - __clz(prior)) : lastsent;
+
+      if (Hn) {
+        // Owner lane and query position of hit kb + lane: each lane whose run
+        // of hits intersects [kb, kb + 32) stores (lane, table offset -
+        // excl) at the slot of its run's first hit in the round; a hit's
+        // owner is the last run start at or before it (OR-reduced mask).
+        auto locate = [&](uint32_t kb, uint32_t lim, int &own_out, int &q_out) {
+          const bool wr = cnt != 0u && excl < kb + 32u && incl > kb;
+          const int p0 = wr ? max(int(excl) - int(kb), 0) : 0;
+          if (wr) scr[p0] = uint32_t(lane) | ((o - excl) << 5);
+          const unsigned S = __reduce_or_sync(kFull, wr ? (1u << p0) : 0u);
+          __syncwarp();
+          const int src = 31 - __clz(S & (kFull >> (31 - lane)));
+          const uint32_t vv = scr[src];
+          own_out = int(vv & 31u);
+          const uint32_t k = kb + uint32_t(lane);
+          q_out = k < lim ? int(__ldg(qpos + (((vv >> 5) + k) & 0x7ffffffu))) : 0;
+          __syncwarp();
+        };
+        // hits of lanes v < L (tested against the previous block's state)
+        const uint32_t CL = L > 0 ? __shfl_sync(kFull, incl, L - 1) : 0u;
+        const bool pre_ok = CL <= 32u;  // all of them in the first round
+        const int sc = slotc();
+        auto enqueue = [&](bool enq, int P, int q) {
+          const unsigned bal = __ballot_sync(kFull, enq);
+          if (bal) {
+            if (enq)
+              w.queue()[(st.qhead + st.qcount + __popc(bal & ltmask)) & (kBlkQcap - 1)] =
+                  uint32_t(P) | (uint32_t(q) << 16);
+            st.qcount += __popc(bal);
+            __syncwarp();
+            if (st.qcount >= 32) blk_flush<kTrace, kHit>(a, w, st, 32, qc, b62, lane, sc, M);
+          }
+        };
+        if (!pre_ok) {
+          // rare (> 32 hits on the first L positions): test those hits
+          // before any of this window's records, in rounds of their own
+          for (uint32_t k0 = 0; k0 < CL; k0 += 32) {
+            int v, q;
+            locate(k0, CL, v, q);
+            const int P = b + v;
+            bool act = k0 + uint32_t(lane) < CL;
+            if (seg) act = act && P - q >= dlo_f && P - q < dhi_f;
+            int slot = base_slot + v - q;
+            slot += slot < 0 ? M : 0;
+            slot -= slot >= M ? M : 0;
+            const int lsv = __shfl_sync(kFull, ls_lane, v);
+            const uint32_t e = act ? w.ring()[slot] : 0u;
+            const int ebid = be_bid(e);
+            const int bt = max(b - 32, lsv + 1);
+            const int lo_ok = max(P - A + 1, lsv + 1);
+            int pv = ebid ? ebid + be_maxoff(e) : 0;
+            bool pin = false;
+            if (ebid == bt) {
+              pin = ebid + be_minoff(e) <= P - W;
+              pv = be_prevoff(e) ? ebid - be_prevoff(e) : 0;
+            }
+            const bool pass = act && (pin || pv >= lo_ok);
+            bool enq = pass;
+            if (!kHit && pass) enq = P > int(w.reach()[slot]);
+            if (kTrace) {
+              bstat<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
+              bstat<kTrace>(st, kStatEnqueued, __popc(__ballot_sync(kFull, enq)));
+              if (pass) trace_push(a, 1, st.spbase + P, q, 0, 0, 0);
+            }
+            enqueue(enq, P, q);
+            __syncwarp();
+          }
+        }
+        const bool multi_bid_possible = sm != 0u;
+        int nown = 0, nq = 0;
+        locate(0u, Hn, nown, nq);
+        for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
+          const int v = nown, q = nq;
+          if (k0 + 32 < Hn) locate(k0 + 32u, Hn, nown, nq);
+          const int P = b + v;
+          bool act = k0 + uint32_t(lane) < Hn;
+          if (seg) act = act && P - q >= dlo_f && P - q < dhi_f;
+          int slot = base_slot + v - q;
+          slot += slot < 0 ? M : 0;
+          slot -= slot >= M ? M : 0;
+          const int lsv = __shfl_sync(kFull, ls_lane, v);
+          const int bid = max(b, lsv + 1);  // record block (split at subject starts)
+          const unsigned G = __match_any_sync(
+              kFull, act ? (unsigned(slot) | (unsigned(bid) << 14)) : (0x80000000u | unsigned(lane)));
+          uint32_t e = 0;
+          if (act) e = w.ring()[slot];
+          const int Pf = __shfl_sync(kFull, P, __ffs(G) - 1);  // the group's first hit
+          const int ebid = be_bid(e);
+          const int emax = ebid + be_maxoff(e);
+          const bool pre = v < L;
+          const bool tst = act && (!pre || pre_ok);
+          const int bt = pre ? max(b - 32, lsv + 1) : bid;  // the block h is tested against
+          const bool same = ebid == bt;
+          const int mn = same ? ebid + be_minoff(e) : (pre ? INT_MAX : Pf);
+          const int po = be_prevoff(e);
+          const int pv = same ? (po ? ebid - po : 0) : (ebid ? emax : 0);
+          const int lo_ok = max(P - A + 1, lsv + 1);  // within A, same subject
+          const bool pass = tst && (mn <= P - W || pv >= lo_ok);
+          // the state write: the last member of the slot's group (of the
+          // slot's last group when a subject starts inside the round)
+          unsigned Gw = G;
+          if (multi_bid_possible && __any_sync(kFull, act && bid != b))
+            Gw = __match_any_sync(kFull, act ? slot : -1 - lane);
+          if (act && lane == 31 - __clz(Gw)) {
+            const bool sw = ebid == bid;
+            const int dp = bid - emax;
+            const uint32_t nmin = sw ? uint32_t(be_minoff(e)) : uint32_t(Pf - bid);
+            const uint32_t npo =
+                sw ? uint32_t(po) : ((ebid != 0 && dp <= 255) ? uint32_t(dp) : 0u);
+            w.ring()[slot] =
+                uint32_t(bid) | (nmin << 14) | (uint32_t(P - bid) << 19) | (npo << 24);
+          }
+          bool enq = pass;
+          if (!kHit && pass) enq = P > int(w.reach()[slot]);
+          if (kTrace) {
+            bstat<kTrace>(st, kStatRounds, 1);
+            bstat<kTrace>(st, kStatConflictRounds,
+                          __any_sync(kFull, act && __popc(G) > 1) ? 1 : 0);
+            bstat<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, act)));
+            bstat<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));
+            bstat<kTrace>(st, kStatEnqueued, __popc(__ballot_sync(kFull, enq)));
+            if (act) trace_push(a, 0, st.spbase + P, q, 0, 0, 0);
+            if (pass) trace_push(a, 1, st.spbase + P, q, 0, 0, 0);
+          }
+          enqueue(enq, P, q);
+          __syncwarp();
+        }
+      }
+      // ---- advance the window ---------------------------------------------
+      if (sm) lastsent = b + 31 - __clz(sm);
+      b += 32;
+      base_slot += 32;
+      if (base_slot >= M) base_slot -= M;
+    }
+    {
+      const int sc = slotc();
+      while (st.qcount > 0)
+        blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
+    }
+    // the next work item continues the frame after a gap (stale state ages out)
+    frame = b + 64;
+    base_slot = (base_slot + 64) % M;
+  }
+  if (kTrace && a.stats && lane == 0)
+    for (int i = 0; i < kNumStats; ++i)
+      if (st.stat[i]) atomicAdd(a.stats + i, st.stat[i]);
+}
+
+size_t blk_smem_bytes(int lq, int ring, int warps) {
+  return 1024 + align16(size_t(lq) + 2 * kQPad + 8) + size_t(warps) * blk_area_bytes(ring);
+}
+
+template <bool kTrace, int kW, bool kHit>
+cudaError_t blk_launch(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
+  void (*k)(const SearchArgs) = search_block_kernel<kTrace, kW, kHit>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  if (e != cudaSuccess) return e;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, warps * 32, smem);
+  if (e != cudaSuccess) return e;
+  if (per_sm < 1) return cudaErrorInvalidConfiguration;
+  int64_t grid = int64_t(num_sms) * per_sm;
+  const int64_t need = (int64_t(a.nchunks) + a.nlong + a.nsegs + warps - 1) / warps;
+  if (grid > need) grid = need < 1 ? 1 : need;
+  k<<<unsigned(grid), warps * 32, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+template <bool kTrace>
+cudaError_t blk_pick(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
+  const bool hit = a.ext_mode == BLASTP_EXT_HIT;
+  if (a.min_gap == 3)
+    return hit ? blk_launch<kTrace, 3, true>(a, warps, smem, num_sms, s)
+               : blk_launch<kTrace, 3, false>(a, warps, smem, num_sms, s);
+  return hit ? blk_launch<kTrace, 0, true>(a, warps, smem, num_sms, s)
+             : blk_launch<kTrace, 0, false>(a, warps, smem, num_sms, s);
+}
+
+}  // namespace
+
+bool block_kernel_eligible(const SearchArgs &a) {
+  return a.filter_mode == BLASTP_FILTER_LEFT &&
+         (a.ext_mode == BLASTP_EXT_DIAGONAL || a.ext_mode == BLASTP_EXT_HIT) &&
+         a.min_gap >= 1 && a.min_gap <= 8 && a.window >= 31 + a.min_gap && a.window <= 256 &&
+         a.qv.lq <= 16000 && a.qv.wtab != nullptr;
+}
+
+cudaError_t launch_search_block(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
+  static unsigned long long b62_ready = 0;  // one bit per device
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!(b62_ready >> dev & 1ull)) {
+    int8_t h[32 * 32];
+    fill_b62(h);
+    e = cudaMemcpyToSymbol(c_b62_blk, h, sizeof(h));
+    if (e != cudaSuccess) return e;
+    b62_ready |= 1ull << dev;
+  }
+  SearchArgs a = a_in;
+  a.ring = search_ring_slots(a.qv.lq, a.window);
+  int optin = 0;
+  e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+  if (e != cudaSuccess) return e;
+  const char *warps_env = std::getenv("BLASTP_WARPS");
+  int warps = warps_env ? std::max(1, std::min(kBlkWarps, std::atoi(warps_env))) : kBlkWarps;
+  while (warps > 0 && blk_smem_bytes(a.qv.lq, a.ring, warps) > size_t(optin)) --warps;
+  if (warps < 1) return cudaErrorInvalidConfiguration;
+  const size_t smem = blk_smem_bytes(a.qv.lq, a.ring, warps);
+  return a.trace[0] != nullptr ? blk_pick<true>(a, warps, smem, num_sms, s)
+                               : blk_pick<false>(a, warps, smem, num_sms, s);
+}
+
+}  // namespace blastp

@@ -751,15 +751,20 @@ int kernel_choice() {
   if (!v) return 0;
   if (!std::strcmp(v, "warp")) return 1;
   if (!std::strcmp(v, "cta")) return 2;
+  if (!std::strcmp(v, "block")) return 3;
   return 0;
 }
 
 }  // namespace
 
 cudaError_t launch_search(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
-  // The warp variant is the default (faster on B200, profiles/r01); the CTA
-  // variant runs when BLASTP_KERNEL=cta.
+  // Default: the block kernel (search_block.cu) where its state encoding
+  // applies (filter LEFT, ext_mode DIAGONAL/HIT, window >= 31 + min_gap),
+  // else the warp kernel; BLASTP_KERNEL=warp|cta|block forces a variant
+  // (block falls back to warp outside its domain; tests cover all three).
   const int choice = kernel_choice();
+  if ((choice == 0 || choice == 3) && block_kernel_eligible(a_in))
+    return launch_search_block(a_in, num_sms, s);
   if (choice != 2 || a_in.filter_mode == BLASTP_FILTER_STATEFUL)
     return launch_search_warp(a_in, num_sms, s);  // STATEFUL: warp variant only
   static unsigned long long b62_ready = 0;  // one bit per device

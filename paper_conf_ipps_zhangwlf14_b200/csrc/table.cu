@@ -65,7 +65,30 @@ __global__ void __launch_bounds__(kTableThreads)
   if (!kFill) woff[w + 1] = k;  // counts; scanned in place into offsets
 }
 
+// Radix-32 view of the CSR table for the block kernel (search_block.cu):
+// entry (r0 << 10 | r1 << 5 | r2) = (woff[w], count of w) for the word w of
+// letters r0 r1 r2 < 24, (0, 0) for any code with a sentinel or unused letter
+// -- a word touching a subject boundary neighbours nothing (R4), and the
+// kernel needs no letter check; one 8-byte load per subject position.
+__global__ void radix32_kernel(const uint32_t *__restrict__ woff, uint2 *__restrict__ wtab) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= 32 * 32 * 32) return;
+  const int r0 = c >> 10, r1 = (c >> 5) & 31, r2 = c & 31;
+  uint2 v = make_uint2(0u, 0u);
+  if (r0 < kNumLetters && r1 < kNumLetters && r2 < kNumLetters) {
+    const int w = (r0 * kNumLetters + r1) * kNumLetters + r2;
+    v.x = woff[w];
+    v.y = woff[w + 1] - woff[w];
+  }
+  wtab[c] = v;
+}
+
 }  // namespace
+
+cudaError_t launch_table_radix32(const uint32_t *woff, uint2 *wtab, cudaStream_t s) {
+  radix32_kernel<<<(32 * 32 * 32) / 256, 256, 0, s>>>(woff, wtab);
+  return cudaGetLastError();
+}
 
 // Builds woff (device, kWords + 1) and returns the entry count on the host;
 // then qpos must be allocated with max(total, 1) entries and filled by

@@ -23,9 +23,11 @@ def bp():
     return blastp
 
 
-@pytest.fixture(params=["cta", "warp"], autouse=True)
+@pytest.fixture(params=["cta", "warp", "block"], autouse=True)
 def kernel_variant(request, monkeypatch):
-    """Every parity test runs on both kernel variants (BLASTP_KERNEL)."""
+    """Every parity test runs on every kernel variant (BLASTP_KERNEL): the
+    block kernel (default where eligible: LEFT, window >= 31 + min_gap; the
+    warp kernel otherwise), the warp kernel and the CTA kernel."""
     monkeypatch.setenv("BLASTP_KERNEL", request.param)
     return request.param
 
@@ -192,6 +194,8 @@ def test_config3_full(bp, orc, kernel_variant, mode):
     list (no sampling), both R6 readings and the STATEFUL walk."""
     if kernel_variant == "cta" and mode == 2:
         pytest.skip("STATEFUL runs on the warp variant only")
+    if kernel_variant == "block" and mode != 0:
+        pytest.skip("EITHER and STATEFUL run on the warp kernel (the block kernel is LEFT only)")
     (q,), db = _config3()
     p = bp.Params(filter_mode=mode)
     g = bp.search_ungapped(bp.build_query_table(q, p), _config3_db(bp), p)
@@ -268,8 +272,8 @@ def test_config5_shard_sampled(bp, orc, kernel_variant):
     eighth of the nr-shaped 40M-subject database (~1.9G residues: the shard
     one of the 8 GPUs owns; first and last shard), full size, in one batched
     search.  Sampled oracle parity on subject blocks for all 64 queries."""
-    if kernel_variant == "cta":
-        pytest.skip("the 64-query full-size shard runs on the default (warp) variant")
+    if kernel_variant != "block":
+        pytest.skip("the 64-query full-size shard runs on the default (block) kernel")
     from paper_conf_ipps_zhangwlf14_b200.dist import shard_subjects
     from synth import config_offsets
     off = config_offsets(5)
@@ -318,8 +322,8 @@ def test_config5_shard_full(bp, orc, kernel_variant):
     U[100, 2000]) against shard 0 of 8 of the nr-shaped database (~1.9G
     residues, ~5M subjects); the GPU list equals the oracle's complete list of
     all 64 queries."""
-    if kernel_variant == "cta":
-        pytest.skip("the 64-query full-size shard runs on the default (warp) variant")
+    if kernel_variant != "block":
+        pytest.skip("the 64-query full-size shard runs on the default (block) kernel")
     import time
     from paper_conf_ipps_zhangwlf14_b200.dist import shard_subjects
     from synth import config_offsets
