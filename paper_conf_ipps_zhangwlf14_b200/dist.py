@@ -4,9 +4,8 @@ The database shards by contiguous subject ranges balanced by residues
 (blastp_shard_range); subjects are independent, so each rank
 searches its shard with no data-path communication.  The one exchange is the
 result: every rank's HSP list (int32 x 7 per HSP, device memory) is gathered
-to rank 0 with two collectives -- an all_gather of the counts, then an
-all_gather of the lists padded to the largest count -- and concatenated in
-rank order.  Because shards are contiguous in subject id and each rank's list
+to rank 0 -- one all_gather of the counts, then exact-size point-to-point
+transfers into rank 0's output (gather_hsps) -- in rank order.  Because shards are contiguous in subject id and each rank's list
 is canonical (R11), the concatenation is already canonical for one query;
 for query batches rank 0 re-sorts (query_id major) on the GPU.
 
@@ -42,33 +41,49 @@ def gather_hsps(local, group=None, dst: int = 0):
     """Gather [n_r, 7] int32 HSP tensors of every rank onto rank `dst`.
 
     Returns the concatenation in rank order on rank dst (None elsewhere).
-    Works for any torch.distributed backend; tensors stay on their device.
+    One collective for the counts (all_gather_into_tensor of one int64 per
+    rank, read back once), then exact-size point-to-point transfers batched
+    in one group (NCCL: one ncclGroupStart/End): rank dst receives each
+    rank's list straight into its slice of the output -- no padding, no
+    concatenation copy, and no rank receives lists it does not keep.  Works
+    for any torch.distributed backend; tensors stay on their device.
     """
     import torch
     import torch.distributed as dist
 
     world = dist.get_world_size(group)
     rank = dist.get_rank(group)
+    if world == 1:
+        return local
     if local.is_cuda and dist.get_backend(group) != "nccl":
         # gloo (functional multi-rank checks on one device): collectives on host
         out = gather_hsps(local.cpu(), group, dst)
         return None if out is None else out.to(local.device)
     dev = local.device
     n = torch.tensor([local.shape[0]], dtype=torch.int64, device=dev)
-    counts = [torch.zeros_like(n) for _ in range(world)]
-    dist.all_gather(counts, n, group=group)
-    counts = [int(c.item()) for c in counts]
-    maxn = max(counts) if counts else 0
-    if maxn == 0:
-        return local.new_zeros((0, HSP_FIELDS)) if rank == dst else None
-    padded = local.new_zeros((maxn, HSP_FIELDS))
-    if local.shape[0]:
-        padded[: local.shape[0]] = local
-    bufs = [local.new_empty((maxn, HSP_FIELDS)) for _ in range(world)]
-    dist.all_gather(bufs, padded, group=group)
-    if rank != dst:
-        return None
-    return torch.cat([b[:c] for b, c in zip(bufs, counts)], dim=0)
+    counts_t = torch.empty(world, dtype=torch.int64, device=dev)
+    dist.all_gather_into_tensor(counts_t, n, group=group)
+    counts = counts_t.tolist()  # the one host synchronisation of the gather
+    glob = (lambda r: r) if group is None else (lambda r: dist.get_global_rank(group, r))
+    ops = []
+    out = None
+    if rank == dst:
+        out = local.new_empty((sum(counts), HSP_FIELDS))
+        offs = np.concatenate([[0], np.cumsum(counts)]).astype(np.int64)
+        for r in range(world):
+            if counts[r] == 0:
+                continue
+            view = out[int(offs[r]): int(offs[r + 1])]
+            if r == rank:
+                view.copy_(local)
+            else:
+                ops.append(dist.P2POp(dist.irecv, view, glob(r), group))
+    elif counts[rank] > 0:
+        ops.append(dist.P2POp(dist.isend, local.contiguous(), glob(dst), group))
+    if ops:
+        for req in dist.batch_isend_irecv(ops):
+            req.wait()
+    return out
 
 
 def search_sharded(search_fn: Callable[[int, int], "object"], offsets: np.ndarray, group=None,
@@ -88,33 +103,37 @@ def search_sharded(search_fn: Callable[[int, int], "object"], offsets: np.ndarra
 def gpu_shard_search(table, residues_local: np.ndarray, offsets_full: np.ndarray, rank: int,
                      world: int, params=None, capacity: int | None = None, stream=None):
     """Pack this rank's shard -- only its bytes need to be resident on the
-    host -- and search it on the current CUDA device.  Returns a device
-    [n, 7] int32 tensor (global subject ids, canonical order)."""
+    host -- and search it on the current CUDA device, all on `stream` (torch's
+    current stream by default; the output buffers are allocated on it and the
+    count is read after the search on it).  Returns a device [n, 7] int32
+    tensor (global subject ids, canonical order)."""
     import torch
 
     from . import blastp as bp
 
     off = np.ascontiguousarray(offsets_full, dtype=np.int64)
     lo, hi = shard_subjects(off, rank, world)
-    # libblastp reads residues at base + offsets[i] for the shard's subjects
-    # only; hand it a base such that base + offsets[lo] is the local buffer.
-    base = residues_local.ctypes.data - int(off[lo])
-    db = bp.Database.from_pinned(base, off, rank, world, device=torch.cuda.current_device(),
-                                 stream=stream)
-    assert db.subject_base == lo
-    try:
-        cap = capacity or max(4096, db.residues // 1000 * max(1, table.num_queries))
-        while True:
-            out = torch.empty((cap, 7), dtype=torch.int32, device="cuda")
-            cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
-            bp.search_ungapped_device(table, db, out.data_ptr(), cap, cnt.data_ptr(), params,
-                                      stream)
-            n = int(cnt.item())
-            if n <= cap:
-                break
-            cap = n + n // 4 + 1024
-        res = out[:n]
-        bp.sort_hsps_device(res.data_ptr(), n, stream)
-        return res
-    finally:
-        db.free()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    with torch.cuda.stream(s):
+        # libblastp reads residues at base + offsets[i] for the shard's subjects
+        # only; hand it a base such that base + offsets[lo] is the local buffer.
+        base = residues_local.ctypes.data - int(off[lo])
+        db = bp.Database.from_pinned(base, off, rank, world, device=torch.cuda.current_device(),
+                                     stream=s)
+        assert db.subject_base == lo
+        try:
+            cap = capacity or max(4096, db.residues // 1000 * max(1, table.num_queries))
+            while True:
+                out = torch.empty((cap, 7), dtype=torch.int32, device="cuda")
+                cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+                bp.search_ungapped_device(table, db, out.data_ptr(), cap, cnt.data_ptr(), params,
+                                          s)
+                n = int(cnt.item())  # a copy on s, after the search
+                if n <= cap:
+                    break
+                cap = n + n // 4 + 1024
+            res = out[:n]
+            bp.sort_hsps_device(res.data_ptr(), n, s)
+            return res
+        finally:
+            db.free()
