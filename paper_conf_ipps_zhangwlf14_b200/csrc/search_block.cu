@@ -106,6 +106,11 @@ __device__ __forceinline__ void bstat(BlkState &st, int i, unsigned long long v)
   if (kStats) st.stat[i] += v;
 }
 
+// Query codes in shared memory with kBlkQPad sentinel codes on both sides
+// (the X-drop's word loads stay inside the array).
+constexpr int kBlkQPad = 16;
+
+// REGION: flush
 // Extend up to 32 queued passing hits lane-parallel (R7-R9), then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order;
 // kHit: Alg. 4, every passing hit extended and kept (reading R14).
@@ -121,7 +126,10 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
   slot += slot < 0 ? M : 0;
   const int64_t sp = st.spbase + P;
   int total = 0, llen = 0, rlen = 0, scanned = 0;
-  if (act) xdrop_extend(a.stream, sp, q, qc, b62, a.xdrop, total, llen, rlen, scanned);
+  // (a variant reading the query codes four per shared load measured 3%
+  // slower on config 3: DESIGN.md 5.9)
+  if (act) xdrop_extend(a.stream, sp, q, qc + (kBlkQPad - kQPad), b62, a.xdrop, total, llen, rlen,
+                        scanned);
   if (kTrace) {
     bstat<kTrace>(st, kStatFlushes, 1);
     bstat<kTrace>(st, kStatExtended, n);
@@ -181,18 +189,20 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
   st.qcount -= n;
 }
 
-// kW: min_gap fixed at compile time (3, the default) or 0 (runtime value);
-// kHit: ext_mode HIT (Alg. 4) instead of DIAGONAL (Alg. 3).
-template <bool kTrace, int kW, bool kHit>
+// REGION: setup
+// kDef: the default parameters (min_gap 3, window 40) as compile-time
+// constants, else read from the arguments; kHit: ext_mode HIT (Alg. 4)
+// instead of DIAGONAL (Alg. 3).
+template <bool kTrace, bool kDef, bool kHit>
 __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const SearchArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
   int8_t *b62 = reinterpret_cast<int8_t *>(smem);
   uint8_t *qc = smem + 1024;
-  const size_t qc_bytes = align16(size_t(lq) + 2 * kQPad + 8);
+  const size_t qc_bytes = align16(size_t(lq) + 2 * kBlkQPad);
   for (int i = threadIdx.x; i < 1024; i += blockDim.x) b62[i] = c_b62_blk[i];
   for (int i = threadIdx.x; i < int(qc_bytes); i += blockDim.x) {
-    const int k = i - kQPad;
+    const int k = i - kBlkQPad;
     qc[i] = (k >= 0 && k < lq) ? a.qv.qcodes[k] : uint8_t(kSentinel);
   }
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -209,9 +219,9 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
   const uint8_t *__restrict__ stream = a.stream;
   const uint2 *__restrict__ wtab = a.qv.wtab;
   const uint16_t *__restrict__ qpos = a.qv.qpos;
-  const int W = kW ? kW : a.min_gap;
+  const int W = kDef ? 3 : a.min_gap;
   const int L = W - 1;  // record lag: lanes v < L are tested against the previous block
-  const int A = a.window;
+  const int A = kDef ? 40 : a.window;
   const unsigned ltmask = lanemask_lt(lane);
   uint32_t *scr = w.scr();
 
@@ -222,6 +232,9 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
   st.qcount = 0;
   int frame = kBlkFrameMin;  // frame position of the next work item's first residue
   int base_slot = 0;         // ring slot of (P, q) = base_slot + (P - b) - q (mod M)
+  // ring slot of (P, q) = P - q + slotc (mod M): b and base_slot advance
+  // together, so slotc only changes when the frame is rebased
+  int slotc = (M - kBlkFrameMin % M) % M;
   const unsigned long long nsegs = (unsigned long long)a.nsegs;
   const unsigned long long nitems = nsegs + (unsigned long long)a.nlong;
   for (;;) {
@@ -269,11 +282,8 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
     int b = frame;             // frame position of lane 0 (block start)
     int lastsent = frame - 1;  // the sentinel before the work item
     int end = int(wend - st.spbase);
-    auto slotc = [&]() {  // ring slot of (P, q) = P - q + slotc (mod M)
-      int c = (base_slot - b) % M;
-      return c < 0 ? c + M : c;
-    };
 
+    // REGION: window
     // Software pipeline over windows: residues two windows ahead (one byte
     // per lane + two of overlap), the table lookup one window ahead.
     uint32_t pf_r = 0, pf_x = 0;
@@ -307,9 +317,9 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
     while (b < end) {
       // ---- rebase the frame before positions outgrow 14 bits -------------
       if (b >= kBlkFrameMin + kBlkFrameSpan) {
-        const int sc = slotc();
         while (st.qcount > 0)
-          blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
+          blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc, M);
+        slotc = (slotc + kBlkFrameSpan) % M;
         for (int i = lane; i < M; i += 32) {
           const uint32_t e = w.ring()[i];
           // a state whose block starts before the new frame origin is older
@@ -348,6 +358,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
         // of hits intersects [kb, kb + 32) stores (lane, table offset -
         // excl) at the slot of its run's first hit in the round; a hit's
         // owner is the last run start at or before it (OR-reduced mask).
+        // REGION: locate
         auto locate = [&](uint32_t kb, uint32_t lim, int &own_out, int &q_out) {
           const bool wr = cnt != 0u && excl < kb + 32u && incl > kb;
           const int p0 = wr ? max(int(excl) - int(kb), 0) : 0;
@@ -364,7 +375,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
         // hits of lanes v < L (tested against the previous block's state)
         const uint32_t CL = L > 0 ? __shfl_sync(kFull, incl, L - 1) : 0u;
         const bool pre_ok = CL <= 32u;  // all of them in the first round
-        const int sc = slotc();
+        // REGION: enqueue
         auto enqueue = [&](bool enq, int P, int q) {
           const unsigned bal = __ballot_sync(kFull, enq);
           if (bal) {
@@ -373,9 +384,10 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
                   uint32_t(P) | (uint32_t(q) << 16);
             st.qcount += __popc(bal);
             __syncwarp();
-            if (st.qcount >= 32) blk_flush<kTrace, kHit>(a, w, st, 32, qc, b62, lane, sc, M);
+            if (st.qcount >= 32) blk_flush<kTrace, kHit>(a, w, st, 32, qc, b62, lane, slotc, M);
           }
         };
+        // REGION: prepass
         if (!pre_ok) {
           // rare (> 32 hits on the first L positions): test those hits
           // before any of this window's records, in rounds of their own
@@ -412,34 +424,51 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
           }
         }
         const bool multi_bid_possible = sm != 0u;
-        int nown = 0, nq = 0;
-        locate(0u, Hn, nown, nq);
-        for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
-          const int v = nown, q = nq;
-          if (k0 + 32 < Hn) locate(k0 + 32u, Hn, nown, nq);
-          const int P = b + v;
+        // Round pipeline: round r's (v, q) are located at the start of round
+        // r - 1 (the query-position load, an L2 hit, overlaps a round), its
+        // MATCH (the (slot, bid) groups) is issued at the end of round r - 1
+        // and overlaps the next locate.
+        // REGION: prep
+        auto prep = [&](uint32_t k0, int v, int q, int &slot_o, int &lsv_o, bool &act_o) {
           bool act = k0 + uint32_t(lane) < Hn;
-          if (seg) act = act && P - q >= dlo_f && P - q < dhi_f;
+          if (seg) act = act && b + v - q >= dlo_f && b + v - q < dhi_f;
           int slot = base_slot + v - q;
           slot += slot < 0 ? M : 0;
           slot -= slot >= M ? M : 0;
-          const int lsv = __shfl_sync(kFull, ls_lane, v);
+          int lsv = lastsent;
+          if (multi_bid_possible) lsv = __shfl_sync(kFull, ls_lane, v);
           const int bid = max(b, lsv + 1);  // record block (split at subject starts)
-          const unsigned G = __match_any_sync(
+          slot_o = slot;
+          lsv_o = lsv;
+          act_o = act;
+          return __match_any_sync(
               kFull, act ? (unsigned(slot) | (unsigned(bid) << 14)) : (0x80000000u | unsigned(lane)));
+        };
+        int cv = 0, cq = 0, nv = 0, nq = 0, cslot = 0, clsv = 0;
+        bool cact = false;
+        locate(0u, Hn, cv, cq);
+        unsigned cG = prep(0u, cv, cq, cslot, clsv, cact);
+        if (32u < Hn) locate(32u, Hn, nv, nq);
+        // REGION: round
+        for (uint32_t k0 = 0; k0 < Hn; k0 += 32) {
+          const int v = cv, q = cq, slot = cslot, lsv = clsv;
+          const bool act = cact;
+          const unsigned G = cG;
+          const int P = b + v;
+          const int bid = max(b, lsv + 1);  // record block (split at subject starts)
           uint32_t e = 0;
           if (act) e = w.ring()[slot];
+          const bool pre = v < L;
+          const int lo_ok = max(P - A + 1, lsv + 1);  // within A, same subject
           const int Pf = __shfl_sync(kFull, P, __ffs(G) - 1);  // the group's first hit
           const int ebid = be_bid(e);
           const int emax = ebid + be_maxoff(e);
-          const bool pre = v < L;
           const bool tst = act && (!pre || pre_ok);
           const int bt = pre ? max(b - 32, lsv + 1) : bid;  // the block h is tested against
           const bool same = ebid == bt;
           const int mn = same ? ebid + be_minoff(e) : (pre ? INT_MAX : Pf);
           const int po = be_prevoff(e);
           const int pv = same ? (po ? ebid - po : 0) : (ebid ? emax : 0);
-          const int lo_ok = max(P - A + 1, lsv + 1);  // within A, same subject
           const bool pass = tst && (mn <= P - W || pv >= lo_ok);
           // the state write: the last member of the slot's group (of the
           // slot's last group when a subject starts inside the round)
@@ -455,8 +484,15 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
             w.ring()[slot] =
                 uint32_t(bid) | (nmin << 14) | (uint32_t(P - bid) << 19) | (npo << 24);
           }
-          bool enq = pass;
-          if (!kHit && pass) enq = P > int(w.reach()[slot]);
+          // every passing hit is queued: the flush's ext_reach chain (R10)
+          // rejects the covered ones (0.5% of passing hits are covered by an
+          // already resolved extension at this point on config 3; a reach
+          // load per round costs more)
+#ifdef BLK_ENQ_REACH  // A/B knob: skip passing hits already covered at enqueue
+          const bool enq = pass && (kHit || P > int(w.reach()[slot]));
+#else
+          const bool enq = pass;
+#endif
           if (kTrace) {
             bstat<kTrace>(st, kStatRounds, 1);
             bstat<kTrace>(st, kStatConflictRounds,
@@ -467,21 +503,28 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
             if (act) trace_push(a, 0, st.spbase + P, q, 0, 0, 0);
             if (pass) trace_push(a, 1, st.spbase + P, q, 0, 0, 0);
           }
+          // the queue first (a flush here keeps only the next round's
+          // (v, q) live across the X-drop), then the next round's MATCH and
+          // the locate of the one after
           enqueue(enq, P, q);
           __syncwarp();
+          if (k0 + 32u < Hn) {
+            cv = nv;
+            cq = nq;
+            cG = prep(k0 + 32u, cv, cq, cslot, clsv, cact);
+            if (k0 + 64u < Hn) locate(k0 + 64u, Hn, nv, nq);
+          }
         }
       }
+      // REGION: window
       // ---- advance the window ---------------------------------------------
       if (sm) lastsent = b + 31 - __clz(sm);
       b += 32;
       base_slot += 32;
       if (base_slot >= M) base_slot -= M;
     }
-    {
-      const int sc = slotc();
-      while (st.qcount > 0)
-        blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
-    }
+    while (st.qcount > 0)
+      blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc, M);
     // the next work item continues the frame after a gap (stale state ages out)
     frame = b + 64;
     base_slot = (base_slot + 64) % M;
@@ -491,13 +534,14 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
       if (st.stat[i]) atomicAdd(a.stats + i, st.stat[i]);
 }
 
+// REGION: host
 size_t blk_smem_bytes(int lq, int ring, int warps) {
-  return 1024 + align16(size_t(lq) + 2 * kQPad + 8) + size_t(warps) * blk_area_bytes(ring);
+  return 1024 + align16(size_t(lq) + 2 * kBlkQPad) + size_t(warps) * blk_area_bytes(ring);
 }
 
-template <bool kTrace, int kW, bool kHit>
+template <bool kTrace, bool kDef, bool kHit>
 cudaError_t blk_launch(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
-  void (*k)(const SearchArgs) = search_block_kernel<kTrace, kW, kHit>;
+  void (*k)(const SearchArgs) = search_block_kernel<kTrace, kDef, kHit>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
   int per_sm = 0;
@@ -514,11 +558,11 @@ cudaError_t blk_launch(const SearchArgs &a, int warps, size_t smem, int num_sms,
 template <bool kTrace>
 cudaError_t blk_pick(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
   const bool hit = a.ext_mode == BLASTP_EXT_HIT;
-  if (a.min_gap == 3)
-    return hit ? blk_launch<kTrace, 3, true>(a, warps, smem, num_sms, s)
-               : blk_launch<kTrace, 3, false>(a, warps, smem, num_sms, s);
-  return hit ? blk_launch<kTrace, 0, true>(a, warps, smem, num_sms, s)
-             : blk_launch<kTrace, 0, false>(a, warps, smem, num_sms, s);
+  if (a.min_gap == 3 && a.window == 40)
+    return hit ? blk_launch<kTrace, true, true>(a, warps, smem, num_sms, s)
+               : blk_launch<kTrace, true, false>(a, warps, smem, num_sms, s);
+  return hit ? blk_launch<kTrace, false, true>(a, warps, smem, num_sms, s)
+             : blk_launch<kTrace, false, false>(a, warps, smem, num_sms, s);
 }
 
 }  // namespace

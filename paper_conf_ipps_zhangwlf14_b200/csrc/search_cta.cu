@@ -748,6 +748,9 @@ cudaError_t launch_variant(const SearchArgs &a, const CtaConfig &c, size_t smem,
 // 0: pick automatically, 1: force the warp variant, 2: force the CTA variant
 int kernel_choice() {
   const char *v = std::getenv("BLASTP_KERNEL");
+#ifdef BLASTP_DEFAULT_WARP  // A/B builds: the warp kernel by default
+  if (!v) return 1;
+#endif
   if (!v) return 0;
   if (!std::strcmp(v, "warp")) return 1;
   if (!std::strcmp(v, "cta")) return 2;

@@ -64,3 +64,12 @@ print(f"instructions executed {tot_i:.3e}, samples {tot_s}")
 for key, n in inst.most_common(top):
     print(f"{key[0][:12]:12s}:{key[1]:4d} inst {100 * n / tot_i:5.1f}% samp "
           f"{100 * samp[key] / max(tot_s, 1):5.1f}%  {text(*key)}")
+if os.environ.get("TOP_INSTR"):
+    # the instructions with the most stall samples, with their source line
+    order = sorted(range(len(data)), key=lambda i: -int(data[i]["# Samples"] or 0))
+    print("--- top instructions by stall samples")
+    for i in order[:int(os.environ["TOP_INSTR"])]:
+        r = data[i]
+        key = line_of.get(i, ("?", 0))
+        print(f"{100 * int(r['# Samples'] or 0) / max(tot_s, 1):5.1f}%  {r['Source'][:44]:44s} "
+              f"{key[0][:12]}:{key[1]} {text(*key)[:60]}")
