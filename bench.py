@@ -43,7 +43,7 @@ sys.path.insert(0, ROOT)
 
 METRIC = "database residues/sec (hit detect + ungapped ext) at 1/2/4/8 B200; % HBM roofline"
 UNIT = "residues/s"
-CPU_SAMPLE_RESIDUES = 240_000_000  # oracle sample (first subjects of the DB)
+ORACLE_SAMPLE_RQ = 48_000_000  # oracle sample per step: residue-queries at q1054-equivalent
 
 
 def parse_args():
@@ -179,64 +179,82 @@ def ncu_capture():
         return json.load(f)
 
 
-# --------------------------------------------------------------- reference arm
+# --------------------------------------------------------------- oracle (CPU) legs
+
+def oracle_sample(queries, db):
+    """The one oracle sample definition (the --impl reference arm and the
+    cpu_baseline key): the first subjects of the workload's database holding
+    ORACLE_SAMPLE_RQ residue-queries (all queries), re-searched every step."""
+    # the oracle's work scales with residues x query length: the sample holds
+    # ORACLE_SAMPLE_RQ residue-queries of a 1054-residue query's worth
+    want = ORACLE_SAMPLE_RQ * 1054 // max(1, sum(len(q) for q in queries))
+    nsub = max(1, min(int(np.searchsorted(db.offsets, want)), db.nseq))
+    return nsub, db.offsets[: nsub + 1]
+
+
+def oracle_rate(queries, db, steps, warmup):
+    """Times the oracle (oracle/, as it stands) on the host's cores over the
+    sample: residue-queries per second, mean step time."""
+    from oracle import oracle as o
+    Qs = [o.encode(q) for q in queries]
+    tables = [o.neighbourhood(Q, o.blosum62(), 11) for Q in Qs]
+    nsub, sub_off = oracle_sample(queries, db)
+    codes = o.encode(db.ascii[: sub_off[-1]].tobytes())
+    cores = os.cpu_count() or 1
+    times = []
+    for i in range(warmup + steps):
+        t0 = time.perf_counter()
+        for Q, tab in zip(Qs, tables):
+            o.search(Q, codes, sub_off, table=tab, nthreads=cores, want_extensions=False)
+        if i >= warmup:
+            times.append(time.perf_counter() - t0)
+    res = int(sub_off[-1]) * len(Qs)
+    return {"value": res * len(times) / sum(times), "unit": UNIT, "cores": cores,
+            "kind": "oracle", "ms_per_step": 1e3 * sum(times) / len(times),
+            "sample": f"first {nsub} subjects ({int(sub_off[-1])} residues) of the workload's "
+                      f"database x {len(Qs)} quer{'y' if len(Qs) == 1 else 'ies'} per step "
+                      f"(scan + two-hit filter + extension; table prebuilt), {cores} pthreads, "
+                      f"{steps} steps after {warmup} warm-up"}
+
 
 def run_reference(args):
     rank, _, world = env_rank()
     if rank != 0:
         return  # rank 0 alone runs the CPU arm
-    from oracle import oracle as o
     queries, db, full_off, (lo, hi), desc = workload(args, 0, 1)
-    Qs = [o.encode(q) for q in queries]
-    tables = [o.neighbourhood(Q, o.blosum62(), 11) for Q in Qs]
-    budget = CPU_SAMPLE_RESIDUES * 1054 // max(1, sum(len(q) for q in queries))
-    nsub = int(np.searchsorted(db.offsets, budget // max(1, args.steps + args.warmup)))
-    nsub = max(1, min(nsub, db.nseq))
-    sub_off = db.offsets[: nsub + 1]
-    codes = o.encode(db.ascii[: sub_off[-1]].tobytes())
-    cores = os.cpu_count() or 1
-    times = []
-    for i in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        for Q, tab in zip(Qs, tables):
-            o.search(Q, codes, sub_off, table=tab, nthreads=cores, want_extensions=False)
-        if i >= args.warmup:
-            times.append(time.perf_counter() - t0)
-    res = int(sub_off[-1]) * len(Qs)
-    value = res * len(times) / sum(times)
+    r = oracle_rate(queries, db, args.steps, args.warmup)
+    value = r["value"]
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": 1e3 * sum(times) / len(times), "higher_is_better": True,
-            "scaling": "weak" if args.config == 5 else "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-            "config": {"workload": desc, "sample_subjects": nsub,
-                       "sample_residues": int(sub_off[-1])},
-            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
-                             "sample": f"first {nsub} subjects ({int(sub_off[-1])} residues) of "
-                                       f"the workload per step, {cores} pthreads"},
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": r["ms_per_step"],
+            "higher_is_better": True, "scaling": "weak" if args.config == 5 else "strong",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": desc, "sample": r["sample"]},
+            "cpu_baseline": r,
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0,
                     "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
-# --------------------------------------------------------------- our arm
+# --------------------------------------------------------------- roofline inputs
 
-def cpu_baseline(queries, db):
-    from oracle import oracle as o
-    Qs = [o.encode(q) for q in queries]
-    tables = [o.neighbourhood(Q, o.blosum62(), 11) for Q in Qs]
-    budget = CPU_SAMPLE_RESIDUES * 1054 // max(1, sum(len(q) for q in queries))
-    nsub = max(1, min(int(np.searchsorted(db.offsets, budget)), db.nseq))
-    sub_off = db.offsets[: nsub + 1]
-    codes = o.encode(db.ascii[: sub_off[-1]].tobytes())
-    cores = os.cpu_count() or 1
-    t0 = time.perf_counter()
-    for Q, tab in zip(Qs, tables):
-        o.search(Q, codes, sub_off, table=tab, nthreads=cores, want_extensions=False)
-    dt = time.perf_counter() - t0
-    return {"value": int(sub_off[-1]) * len(Qs) / dt, "unit": UNIT, "cores": cores,
-            "kind": "oracle", "seconds": dt,
-            "sample": f"first {nsub} subjects ({int(sub_off[-1])} residues) of the same DB, "
-                      f"scan+filter+extension only (table prebuilt), {cores} pthreads"}
+def csrc_hash():
+    """sha256 of the CUDA sources + header: ties a committed ncu capture to the
+    build it was taken on."""
+    import glob
+    import hashlib
+    h = hashlib.sha256()
+    pkg = os.path.join(ROOT, "paper_conf_ipps_zhangwlf14_b200", "csrc")
+    for f in sorted(glob.glob(os.path.join(pkg, "*.cu")) + glob.glob(os.path.join(pkg, "*.cuh"))
+                    + [os.path.join(ROOT, "include", "blastp.h")]):
+        with open(f, "rb") as fh:
+            h.update(os.path.basename(f).encode() + b"\0" + fh.read())
+    return h.hexdigest()[:16]
+
+
+# SURVEY.md 8(d)'s operation budget of the method itself (not of any kernel):
+# per DB residue scanned (word code + table probe), per hit (position load,
+# diagonal, key, bin append, sort share, two-hit test) and per X-drop step.
+OPS_PER_RESIDUE, OPS_PER_HIT, OPS_PER_XDROP_STEP = 10, 30, 5
 
 
 def main():
@@ -354,41 +372,58 @@ def main():
     total_residues = int(full_off[shard_subjects(full_off, world - 1, nshards)[1]] - full_off[0])
     value = total_residues * nq * args.steps / (elapsed_ms / 1e3)
 
-    # ---- roofline of the dominant kernel (search_kernel) --------------------
+    # ---- rooflines of the dominant kernel (the search kernel) --------------
+    # (1) HBM, the metric's roofline: algorithmic bytes = 1 B
+    # per residue per query pass + 28 B per HSP written, over the kernel's
+    # CUDA-event time; DRAM traffic from the committed ncu capture when it was
+    # taken on this very source tree (csrc hash), else null.
     peak, peak_src = peaks()
-    # algorithmic bytes per step on this rank: 1 B per residue per query pass
-    # + the HSP records written
     alg_bytes = gdb.residues * nq + n_hsp * 28
-    achieved = alg_bytes / (statistics.mean(kern_ms) / 1e3) / 1e9
-    # the committed capture is one config-3 launch over the whole DB; a rank's
-    # shard of it (N > 1) is credited its residue fraction of the counts
-    capt = ncu_capture() if (args.config == 3 and nq == 1) else {}
+    kern_s = kern_avg_ms / 1e3  # the mean search-kernel time, max over ranks
+    achieved = alg_bytes / kern_s / 1e9
+    capt = ncu_capture()
+    src_sha = csrc_hash()
+    fresh = bool(capt) and capt.get("csrc_sha") == src_sha and args.config == 3 and nq == 1
     frac_shard = gdb.residues / max(1, total_residues)
-    traffic = capt.get("dram_bytes_per_launch")
-    traffic = traffic * frac_shard if traffic is not None else None
-    traffic_src = capt.get("source")
-    if capt and world > 1:
-        traffic_src = f"{traffic_src}, x {frac_shard:.4f} (this rank's residue share)"
-
-    # issue-rate roofline: warp instructions of the captured launch / this
-    # run's kernel time vs 148 SMs x 4 issue slots x the sampled SM clock
-    issue = None
-    if capt.get("smsp__inst_executed.sum") and clk.get("sm_mhz"):
-        inst = float(capt["smsp__inst_executed.sum"]) * frac_shard
-        props = torch.cuda.get_device_properties(dev)
-        peak_i = props.multi_processor_count * 4 * clk["sm_mhz"] * 1e6
-        ach_i = inst / (kern_avg_ms / 1e3)
-        issue = {"bound": "alu", "achieved": ach_i, "peak": peak_i, "unit": "warp-inst/s",
-                 "frac": ach_i / peak_i, "inst_per_launch": inst,
-                 "peak_source": f"{props.multi_processor_count} SMs x 4 schedulers x 1 warp "
-                                f"instruction/cycle x sampled SM clock (B200_PROFILING.md unit "
-                                f"counts)", "source": traffic_src}
-
+    traffic = capt["dram_bytes_per_launch"] * frac_shard if fresh else None
+    capt_note = (f"{capt.get('source')} ({capt.get('kernel')}), csrc {capt.get('csrc_sha')}"
+                 + (f", x {frac_shard:.4f} (this rank's residue share)" if fresh and world > 1
+                    else "")) if fresh else \
+        (f"no capture of this build (csrc {src_sha}; committed capture is csrc "
+         f"{capt.get('csrc_sha')}, config 3 single query only)")
     hbm_roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "traffic": traffic,
-                "kernel": "search_kernel", "kernel_ms": kern_avg_ms,
-                "alg_bytes_per_launch": alg_bytes // nq,
-                "peak_source": peak_src, "traffic_source": traffic_src}
+                "frac": achieved / peak, "traffic": traffic, "kernel": "search kernel",
+                "kernel_ms": 1e3 * kern_s, "alg_bytes_per_launch": alg_bytes // nq,
+                "alg_bytes_per_unit": "1 B per residue per query pass + 28 B per HSP",
+                "peak_source": peak_src, "traffic_source": capt_note}
+    # (2) on chip: the METHOD's integer work (SURVEY 8(d) op budget x this
+    # search's event counts, blastp_debug_stats, one traced launch outside the
+    # timed region) per kernel second vs the measured integer-ALU roof of this
+    # device (blastp_debug_alu_peak); the kernel's own warp instructions per
+    # residue from the capture of this build beside it.
+    onchip = None
+    try:
+        st = bp.debug_stats(table, gdb, params, stream)
+        torch.cuda.synchronize()
+        alu_peak = bp.debug_alu_peak(local_rank)
+        ops = (OPS_PER_RESIDUE * gdb.residues * nq + OPS_PER_HIT * st["hits"]
+               + OPS_PER_XDROP_STEP * st["xdrop_residues"])
+        winst = (float(capt["smsp__inst_executed.sum"]) * frac_shard / max(1, gdb.residues * nq)
+                 if fresh else None)
+        onchip = {"bound": "alu", "achieved": ops / kern_s, "peak": alu_peak,
+                  "unit": "int lane-ops/s", "frac": ops / kern_s / alu_peak,
+                  "method_ops_per_residue": ops / max(1, gdb.residues * nq),
+                  "ops_model": f"SURVEY 8(d): {OPS_PER_RESIDUE}/residue scanned + "
+                               f"{OPS_PER_HIT}/hit + {OPS_PER_XDROP_STEP}/X-drop residue",
+                  "events_per_residue": {k: st[k] / max(1, gdb.residues * nq)
+                                         for k in ("hits", "passing", "extended", "accepted",
+                                                   "xdrop_residues")},
+                  "peak_source": "blastp_debug_alu_peak: measured integer add/xor lane-"
+                                 "instructions/s, 32 warps per SM, this device",
+                  "kernel_warp_inst_per_residue": winst,
+                  "warp_inst_source": capt_note}
+    except Exception as ex:  # noqa: BLE001 -- the roofline is a report, not the step
+        onchip = {"error": str(ex)}
 
     # the step's result lands in pinned host memory (an asynchronous copy)
     hsp_host = torch.empty(cap * 7, dtype=torch.int32, pin_memory=True)
@@ -512,7 +547,7 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(queries, db)
+        cpu = oracle_rate(queries, db, steps=3, warmup=1)
 
     if rank == 0:
         line = {
@@ -530,13 +565,9 @@ def main():
                        "hsps_per_step": n_hsp,
                        "parallelism": f"db-shard{world}" + (f" (of {nshards})" if nshards != world
                                                              else "")},
-            # the binding roof: instruction issue (integer ALU / LSU / shuffle
-            # work per hit) when the capture gives the count;
-            # the metric's HBM fraction stays beside it as hbm_roofline
-            "roofline": (dict(issue, bound="alu", traffic=traffic, kernel="search_kernel",
-                              kernel_ms=kern_avg_ms, traffic_source=traffic_src)
-                         if issue else hbm_roof),
-            "hbm_roofline": hbm_roof,
+            # the metric's roofline (HBM) and the on-chip one
+            "roofline": hbm_roof,
+            "onchip_roofline": onchip,
             "setup": {"query_table_ms": table_ms, "pack_db_ms": pack_ms,
                       "note": "outside the timed region: host table build (+ H2D) of all "
                               "queries; blastp_pack_db of the rank's shard from pinned host "

@@ -278,6 +278,14 @@ int blastp_debug_stats(const blastp_query_table *q, const blastp_db *db,
                        const blastp_params *p, void *cuda_stream, int64_t *stats,
                        int32_t nstats);
 
+/* The measured integer-ALU roof of `device` (synchronous, ~0.1 s): lane
+ * operations per second of independent integer add / logic / multiply-add
+ * chains on every SM at the search kernel's residency (32 warps per SM).
+ * bench.py divides the method's work (ops per residue scanned,
+ * per hit, per X-drop step, counted by blastp_debug_stats) by the search
+ * time and by this roof: the on-chip roofline beside the HBM one. */
+int blastp_debug_alu_peak(int device, double *lane_ops_per_s);
+
 void blastp_hsp_free(blastp_hsp *h);
 void blastp_query_table_free(blastp_query_table *q);
 void blastp_db_free(blastp_db *db);

@@ -1500,6 +1500,14 @@ int blastp_debug_stats(const blastp_query_table *q, const blastp_db *db, const b
                    nullptr, stats, nstats);
 }
 
+int blastp_debug_alu_peak(int device, double *lane_ops_per_s) {
+  if (!lane_ops_per_s) return fail(BLASTP_E_INVALID_ARG, "output is NULL");
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
+  CUDA_TRY(measure_alu_peak(lane_ops_per_s));
+  return BLASTP_OK;
+}
+
 int blastp_debug_hits(const blastp_query_table *q, const blastp_db *db, const blastp_params *p,
                       void *cuda_stream, blastp_hit *hits, int64_t cap, int64_t *n) {
   return blastp_debug_trace(q, db, p, cuda_stream, hits, cap, n, nullptr, 0, nullptr, nullptr, 0,

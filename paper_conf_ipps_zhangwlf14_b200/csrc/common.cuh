@@ -185,6 +185,7 @@ cudaError_t launch_layout(const int64_t *off, int64_t n, const ChunkPlan &plan, 
 constexpr int kSegLen = 2048;
 constexpr int kSegCap = 2048;
 constexpr int kMaxSegments = 32768;  // 256 MB of lists at most
+cudaError_t measure_alu_peak(double *lane_ops_per_s);  // micro.cu
 cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
 cudaError_t unique_hsps(blastp_hsp *d, int64_t n, int64_t *d_n_out, cudaStream_t s);
 void upload_encode_table();

@@ -29,6 +29,7 @@ def test_reference_arm_json_line():
     assert d["impl"] == "reference" and d["value"] > 0 and d["higher_is_better"] is True
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
+    assert "first" in d["cpu_baseline"]["sample"] and d["cpu_baseline"]["value"] == d["value"]
     assert d["config"]["workload"].startswith("config1")
 
 
@@ -45,9 +46,11 @@ def test_gpu_arm_json_line():
     d = run_bench("--config", "1", "--steps", "3", "--warmup", "3", "--e2e-steps", "1")
     for k in REQUIRED + ["roofline", "clocks", "e2e", "gpu_launches", "cpu_baseline"]:
         assert k in d, k
-    r = d["hbm_roofline"]
+    r = d["roofline"]
     assert r["bound"] == "hbm" and 0 < r["frac"] < 1 and r["peak"] > 1000
-    assert d["roofline"]["bound"] in ("hbm", "alu") and 0 < d["roofline"]["frac"] < 1
+    o = d["onchip_roofline"]
+    assert o["bound"] == "alu" and 0 < o["frac"] < 1 and o["peak"] > 1e12
+    assert o["events_per_residue"]["hits"] > 0 and o["method_ops_per_residue"] > 10
     assert d["gpu_launches"] == 3
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle"
