@@ -52,6 +52,14 @@ extern "C" {
                                     end; else no change.  Decides coverage itself, so it
                                     requires ext_mode BLASTP_EXT_DIAGONAL.  Warp kernel
                                     only; long subjects are split by diagonal range. */
+#define BLASTP_FILTER_STATEFUL_RB 3 /* STATEFUL plus Alg. 1 L13's second argument,
+                                    ungapped_ext(hit, lasthit), reading R16: an
+                                    extension is kept only if its subject start is at or
+                                    before the lasthit it pairs with (the two hits lie in
+                                    one ungapped alignment, NCBI/FSA BLAST's two-hit
+                                    method); otherwise it is dropped (no output) and
+                                    lasthit <- the hit (L19).  Same constraints as
+                                    STATEFUL. */
 #define BLASTP_EXT_DIAGONAL 0  /* Alg. 3: a passing hit covered by the
                                   previous extension of its diagonal is skipped (R10) */
 #define BLASTP_EXT_HIT 1       /* Alg. 4: every passing
@@ -70,7 +78,7 @@ typedef struct {
   int32_t min_gap;     /* non-overlap distance (R6), 1..8; default = word_len */
   int32_t xdrop;       /* X: stop when best - run >= X (Fig. 8, R8), 1..127   */
   int32_t cutoff;      /* emit an extension iff score >= cutoff (R10)         */
-  int32_t filter_mode; /* BLASTP_FILTER_LEFT, _EITHER or _STATEFUL            */
+  int32_t filter_mode; /* BLASTP_FILTER_LEFT, _EITHER, _STATEFUL, _STATEFUL_RB */
   int32_t ext_mode;    /* BLASTP_EXT_DIAGONAL (default), _HIT or _WINDOW       */
 } blastp_params;
 

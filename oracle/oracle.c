@@ -164,11 +164,18 @@ void oracle_two_hit(const int32_t *s, int32_t n, int32_t min_gap,
  * min_gap (an overlapping word, or a hit inside the last extension): no
  * change (FSA-BLAST's rule, R15).  end_of(ctx, k) returns the subject end of
  * the extension from hit k, which does not depend on the walk (R7). */
-typedef int32_t (*ext_end_fn)(void *ctx, int32_t k);
+typedef int32_t (*ext_end_fn)(void *ctx, int32_t k, int32_t *start);
 
+/* filter_mode 3 adds Alg. 1 L13's second argument, ungapped_ext(hit_k,
+ * lasthit) (reading R16): the extension from h is kept only if it
+ * reaches back to the last hit -- its subject start is at or before
+ * lasthit (the two-hit pair lies inside one ungapped alignment, as in
+ * NCBI/FSA BLAST's two-hit method).  An extension that does not reach back
+ * is dropped (no output) and h becomes the diagonal's last hit (L19).
+ * end_of also returns the extension's subject start through *start. */
 static void stateful_walk(const int32_t *s, int32_t n, int32_t min_gap,
-                          int32_t window, ext_end_fn end_of, void *ctx,
-                          uint8_t *trigger) {
+                          int32_t window, int reach_back, ext_end_fn end_of,
+                          void *ctx, uint8_t *trigger) {
   int32_t have = 0, lasthit = 0;
   for (int32_t k = 0; k < n; ++k) {
     trigger[k] = 0;
@@ -179,19 +186,40 @@ static void stateful_walk(const int32_t *s, int32_t n, int32_t min_gap,
       continue;
     }
     if (h - lasthit < min_gap) continue; /* R15 */
+    int32_t start = 0;
+    const int32_t end = end_of(ctx, k, &start); /* L13 */
+    if (reach_back && start > lasthit) {        /* R16: not reaching back */
+      lasthit = h;
+      continue;
+    }
     trigger[k] = 1;                      /* L11-14 */
-    lasthit = end_of(ctx, k);            /* L15-16 */
+    lasthit = end;                       /* L15-16 */
   }
 }
 
-static int32_t end_from_array(void *ctx, int32_t k) {
-  return ((const int32_t *)ctx)[k];
+typedef struct {
+  const int32_t *start, *end;
+} ext_arrays;
+
+static int32_t end_from_array(void *ctx, int32_t k, int32_t *start) {
+  const ext_arrays *a = (const ext_arrays *)ctx;
+  *start = a->start ? a->start[k] : 0;
+  return a->end[k];
 }
 
 void oracle_two_hit_stateful(const int32_t *s, int32_t n,
                              const int32_t *ext_end, int32_t min_gap,
                              int32_t window, uint8_t *trigger) {
-  stateful_walk(s, n, min_gap, window, end_from_array, (void *)ext_end, trigger);
+  ext_arrays a = {0, ext_end};
+  stateful_walk(s, n, min_gap, window, 0, end_from_array, &a, trigger);
+}
+
+void oracle_two_hit_stateful_rb(const int32_t *s, int32_t n,
+                                const int32_t *ext_start,
+                                const int32_t *ext_end, int32_t min_gap,
+                                int32_t window, uint8_t *trigger) {
+  ext_arrays a = {ext_start, ext_end};
+  stateful_walk(s, n, min_gap, window, 1, end_from_array, &a, trigger);
 }
 
 /* ---------------------------------------------------------- search, R4-R11 */
@@ -303,9 +331,11 @@ typedef struct {
   oracle_hsp scratch;
 } ext_ctx;
 
-static int32_t ext_end_of(void *ctx, int32_t k) {
+static int32_t ext_end_of(void *ctx, int32_t k, int32_t *start) {
   ext_ctx *X = (ext_ctx *)ctx;
-  return extend_hit(X->J, X->S, X->ls, X->d, X->H[k], &X->scratch);
+  const int32_t end = extend_hit(X->J, X->S, X->ls, X->d, X->H[k], &X->scratch);
+  *start = X->scratch.s_start;
+  return end;
 }
 
 static void search_range(range_job *J) {
@@ -371,11 +401,12 @@ static void search_range(range_job *J) {
       if (n == 0) continue;
       const int32_t d = di - (lq - w);
       const int32_t *H = hs + dstart[di];
-      if (p->filter_mode == 2) {
-        /* Alg. 1 L8-19 (STATEFUL, R15): the walk decides which hits are
-         * extended; each extension is the same R7-R9 extension as below. */
+      if (p->filter_mode == 2 || p->filter_mode == 3) {
+        /* Alg. 1 L8-19 (STATEFUL, R15; mode 3 with L13's reach-back, R16):
+         * the walk decides which hits are extended; each extension is the
+         * same R7-R9 extension as below. */
         ext_ctx X = {J, S, ls, d, H, {0, 0, 0, 0, 0, 0, 0}};
-        stateful_walk(H, n, p->min_gap, p->window, ext_end_of, &X, pass);
+        stateful_walk(H, n, p->min_gap, p->window, p->filter_mode == 3, ext_end_of, &X, pass);
         for (int32_t k = 0; k < n; ++k) {
           if (!pass[k]) continue;
           hitlist_push(J->passing, subj, H[k] - d, H[k]);

@@ -28,6 +28,9 @@
  *                                    alg1_stateful.json), = LEFT on diagonals of
  *                                    <= 2 hits, covering-extension special case,
  *                                    trigger spacing invariant
+ *   oracle_two_hit_stateful_rb  pinned: hand-walked reach-back examples
+ *                                    (tests/golden/alg1_reachback.json), = STATEFUL
+ *                                    when every extension reaches back, oracle-B
  *   oracle_search            pinned: P5-P9 invariants, independent oracle-B
  *                                    (oracle/oracle_b.py) on random tiny cases,
  *                                    planted exact copies, E[hits] closed form;
@@ -61,7 +64,9 @@ typedef struct {
   int32_t cutoff;      /* emit iff score >= cutoff (R10)                     */
   int32_t filter_mode; /* 0 = LEFT (R6 default), 1 = EITHER (Fig. 7 reading),
                           2 = STATEFUL: Alg. 1 L8-19's lasthit walk (R15),
-                          which also decides coverage (ext_mode ignored) */
+                          which also decides coverage (ext_mode ignored),
+                          3 = STATEFUL with L13's reach-back: an extension is
+                          kept only if it reaches back to lasthit (R16) */
   int32_t ext_mode;    /* 0 = DIAGONAL: Alg. 3 coverage chain (R10, default);
                           1 = HIT: Alg. 4, every
                           passing hit extended independently, duplicates kept */
@@ -121,6 +126,15 @@ void oracle_two_hit(const int32_t *s, int32_t n, int32_t min_gap,
 void oracle_two_hit_stateful(const int32_t *s, int32_t n,
                              const int32_t *ext_end, int32_t min_gap,
                              int32_t window, uint8_t *trigger);
+
+/* The same walk with Alg. 1 L13's reach-back (ungapped_ext(hit_k,
+ * lasthit); R16): ext_start[k] = subject start of the extension from hit k;
+ * an extension with ext_start[k] > lasthit is dropped (trigger[k] = 0) and
+ * lasthit <- s[k] instead. */
+void oracle_two_hit_stateful_rb(const int32_t *s, int32_t n,
+                                const int32_t *ext_start,
+                                const int32_t *ext_end, int32_t min_gap,
+                                int32_t window, uint8_t *trigger);
 
 /* Full search of one query against the subjects of `db` (codes,
  * concatenated; subject i is db[offsets[i] .. offsets[i+1]) ).

@@ -57,7 +57,8 @@ class Params:
     min_gap: int = 3
     xdrop: int = 16
     cutoff: int = 41
-    filter_mode: int = 0  # 0 LEFT, 1 EITHER, 2 STATEFUL (Alg. 1 lasthit walk, R15)
+    filter_mode: int = 0  # 0 LEFT, 1 EITHER, 2 STATEFUL (Alg. 1 lasthit walk, R15),
+    #                       3 STATEFUL + Alg. 1 L13's reach-back (R16)
     ext_mode: int = 0  # 0 DIAGONAL (Alg. 3 coverage chain), 1 HIT (Alg. 4)
 
     def _c(self) -> _Params:
@@ -88,6 +89,10 @@ def lib():
         L.oracle_two_hit.restype = None
         L.oracle_two_hit.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
                                      ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]
+        L.oracle_two_hit_stateful_rb.restype = None
+        L.oracle_two_hit_stateful_rb.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p,
+                                                 ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,
+                                                 ctypes.c_void_p]
         L.oracle_two_hit_stateful.restype = None
         L.oracle_two_hit_stateful.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p,
                                               ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]
@@ -171,6 +176,19 @@ def two_hit_stateful(s, ext_end, min_gap: int = 3, window: int = 40) -> np.ndarr
     assert len(e) == len(s)
     out = np.zeros(len(s), dtype=np.uint8)
     lib().oracle_two_hit_stateful(_ptr(s), len(s), _ptr(e), min_gap, window, _ptr(out))
+    return out.astype(bool)
+
+
+def two_hit_stateful_rb(s, ext_start, ext_end, min_gap: int = 3, window: int = 40) -> np.ndarray:
+    """Alg. 1 L8-19 walk with L13's reach-back (R16): an extension is kept only
+    if its subject start is at or before the lasthit it was triggered by."""
+    s = np.ascontiguousarray(s, dtype=np.int32)
+    a = np.ascontiguousarray(ext_start, dtype=np.int32)
+    e = np.ascontiguousarray(ext_end, dtype=np.int32)
+    assert len(a) == len(e) == len(s)
+    out = np.zeros(len(s), dtype=np.uint8)
+    lib().oracle_two_hit_stateful_rb(_ptr(s), len(s), _ptr(a), _ptr(e), min_gap, window,
+                                     _ptr(out))
     return out.astype(bool)
 
 

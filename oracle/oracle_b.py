@@ -12,7 +12,9 @@ with oracle.c except the definition of the method in PAPER.md:
 * coverage follows Alg. 3 L19-23 (R10); ext_mode=1 is Alg. 4
   (P:L1465-1486): every passing hit is extended, no coverage test;
 * mode=2 (STATEFUL, R15) is Alg. 1 L8-19 written as a scan of
-  the diagonal position by position with the lasthit register.
+  the diagonal position by position with the lasthit register; mode=3 adds
+  L13's reach-back (R16): an extension whose subject start lies after the
+  lasthit is dropped and the hit becomes the lasthit.
 
 Results are returned as a sorted list of 7-tuples (R11).
 """
@@ -58,7 +60,7 @@ def search_b(Q, subjects, M, *, T=11, w=3, A=40, W=3, X=16, cutoff=41, mode=0,
                     H.append(s)
             if not H:
                 continue
-            if mode == 2:
+            if mode in (2, 3):
                 # Alg. 1: one register per diagonal, updated at every hit
                 lasthit = None
                 for h in H:
@@ -71,6 +73,9 @@ def search_b(Q, subjects, M, *, T=11, w=3, A=40, W=3, X=16, cutoff=41, mode=0,
                         gr, rl = _extend_one_side(Q, S, q + w, h + w, +1, M, X)
                         gl, ll = _extend_one_side(Q, S, q - 1, h - 1, -1, M, X)
                         rec = (query_id, sid, d, q - ll, h - ll, ll + w + rl, seed + gl + gr)
+                        if mode == 3 and h - ll > lasthit:  # does not reach back
+                            lasthit = h
+                            continue
                         exts.append(rec)
                         if rec[6] >= cutoff:
                             hsps.append(rec)

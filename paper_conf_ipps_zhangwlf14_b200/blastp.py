@@ -22,7 +22,7 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("BLASTP_LIB") or os.path.join(_PKG, "libblastp.so")
 
 OK, E_INVALID_ARG, E_BAD_RESIDUE, E_TOO_LONG, E_NOMEM, E_CUDA, E_CAPACITY = 0, -1, -2, -3, -4, -5, -6
-FILTER_LEFT, FILTER_EITHER, FILTER_STATEFUL = 0, 1, 2
+FILTER_LEFT, FILTER_EITHER, FILTER_STATEFUL, FILTER_STATEFUL_RB = 0, 1, 2, 3
 EXT_DIAGONAL, EXT_HIT, EXT_WINDOW = 0, 1, 2
 
 HSP_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("diagonal", "<i4"),

@@ -59,7 +59,7 @@ def main(argv: list[str] | None = None) -> int:
     ap.add_argument("--window", "-A", type=int, default=40)
     ap.add_argument("--xdrop", "-X", type=int, default=16)
     ap.add_argument("--cutoff", type=int, default=41)
-    ap.add_argument("--filter", choices=["left", "either", "stateful"], default="left")
+    ap.add_argument("--filter", choices=["left", "either", "stateful", "stateful_rb"], default="left")
     ap.add_argument("--ext", choices=["diagonal", "hit", "window"], default="diagonal")
     ap.add_argument("--stream", action="store_true",
                     help="keep the database in pinned host memory (formatted image) and stream it")
@@ -92,7 +92,8 @@ def main(argv: list[str] | None = None) -> int:
     p = bp.Params(threshold=args.threshold, window=args.window, xdrop=args.xdrop,
                   cutoff=args.cutoff,
                   filter_mode={"left": bp.FILTER_LEFT, "either": bp.FILTER_EITHER,
-                               "stateful": bp.FILTER_STATEFUL}[args.filter],
+                               "stateful": bp.FILTER_STATEFUL,
+                               "stateful_rb": bp.FILTER_STATEFUL_RB}[args.filter],
                   ext_mode={"diagonal": bp.EXT_DIAGONAL, "hit": bp.EXT_HIT,
                             "window": bp.EXT_WINDOW}[args.ext])
     torch.cuda.set_device(args.device)

@@ -76,9 +76,10 @@ int validate_params(const blastp_params *p) {
   if (p->threshold < -100 || p->threshold > 100)
     return fail(BLASTP_E_INVALID_ARG, "threshold %d outside [-100, 100]", p->threshold);
   if (p->filter_mode != BLASTP_FILTER_LEFT && p->filter_mode != BLASTP_FILTER_EITHER &&
-      p->filter_mode != BLASTP_FILTER_STATEFUL)
+      p->filter_mode != BLASTP_FILTER_STATEFUL && p->filter_mode != BLASTP_FILTER_STATEFUL_RB)
     return fail(BLASTP_E_INVALID_ARG, "filter_mode %d unknown", p->filter_mode);
-  if (p->filter_mode == BLASTP_FILTER_STATEFUL && p->ext_mode != BLASTP_EXT_DIAGONAL)
+  if ((p->filter_mode == BLASTP_FILTER_STATEFUL || p->filter_mode == BLASTP_FILTER_STATEFUL_RB) &&
+      p->ext_mode != BLASTP_EXT_DIAGONAL)
     return fail(BLASTP_E_INVALID_ARG, "filter_mode STATEFUL decides coverage itself: ext_mode "
                 "must be DIAGONAL (got %d)", p->ext_mode);
   if (p->ext_mode != BLASTP_EXT_DIAGONAL && p->ext_mode != BLASTP_EXT_HIT &&

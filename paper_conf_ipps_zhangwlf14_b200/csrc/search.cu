@@ -251,6 +251,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
     uint32_t cur = e & 0xffffu;
     const int gmax = __reduce_max_sync(kFull, act ? __popc(grp) : 0);
     const uint32_t fl = ent >> 30;
+    const int sst = P - llen;  // the extension's subject start (frame), for R16
     unsigned rem = act ? grp : 0u;
     for (int it = 0; it < gmax; ++it) {
       const int src = rem ? __ffs(rem) - 1 : lane;
@@ -259,6 +260,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
       const int Pj = __shfl_sync(kFull, P, src);
       const int Ej = __shfl_sync(kFull, endp, src);
       const uint32_t fj = __shfl_sync(kFull, fl, src);
+      const int Sj = kSt == 2 ? __shfl_sync(kFull, sst, src) : 0;
       if (valid) {
         bool aj;
         if (fj & 2u) {
@@ -269,6 +271,13 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
           aj = false;
           if (cur == 0 || d >= a.window) cur = uint32_t(Pj);
           else if (d >= a.min_gap) aj = true;
+        }
+        // R16 (filter_mode STATEFUL_RB, Alg. 1 L13 ungapped_ext(hit, lasthit)):
+        // an extension not reaching back to the lasthit is dropped and the hit
+        // becomes the lasthit (L19)
+        if (kSt == 2 && aj && Sj > int(cur)) {
+          aj = false;
+          cur = uint32_t(Pj);
         }
         if (aj) cur = uint32_t(Ej);
         if (src == lane) acc = aj;
@@ -335,7 +344,8 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
 template <bool kTrace, int kF, typename OffT, int kW, bool kWin>
 __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const SearchArgs a) {
   constexpr bool kEither = kF == BLASTP_FILTER_EITHER;
-  constexpr int kSt = kF == BLASTP_FILTER_STATEFUL;
+  // 1: STATEFUL (R15); 2: STATEFUL_RB (R15 + R16's reach-back)
+  constexpr int kSt = kF == BLASTP_FILTER_STATEFUL ? 1 : kF == BLASTP_FILTER_STATEFUL_RB ? 2 : 0;
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
   int8_t *b62 = reinterpret_cast<int8_t *>(smem);
@@ -893,7 +903,7 @@ template <bool kTrace, int kF, typename OffT>
 cudaError_t launch_variant(const SearchArgs &a, int warps, size_t smem, int num_sms,
                            cudaStream_t s) {
   void (*k)(const SearchArgs) = search_warp_kernel<kTrace, kF, OffT, 0, false>;
-  if constexpr (kF != BLASTP_FILTER_STATEFUL) {
+  if constexpr (kF != BLASTP_FILTER_STATEFUL && kF != BLASTP_FILTER_STATEFUL_RB) {
     if (a.ext_mode == BLASTP_EXT_WINDOW) k = search_warp_kernel<kTrace, kF, OffT, 0, true>;
     else if (a.min_gap == 3) k = search_warp_kernel<kTrace, kF, OffT, 3, false>;
   }
@@ -964,10 +974,12 @@ cudaError_t launch_search_warp(const SearchArgs &a_in, int num_sms, cudaStream_t
     if (trace) {
       if (fm == BLASTP_FILTER_EITHER) return launch_variant<true, 1, OffT>(a, warps, smem, num_sms, s);
       if (fm == BLASTP_FILTER_STATEFUL) return launch_variant<true, 2, OffT>(a, warps, smem, num_sms, s);
+      if (fm == BLASTP_FILTER_STATEFUL_RB) return launch_variant<true, 3, OffT>(a, warps, smem, num_sms, s);
       return launch_variant<true, 0, OffT>(a, warps, smem, num_sms, s);
     }
     if (fm == BLASTP_FILTER_EITHER) return launch_variant<false, 1, OffT>(a, warps, smem, num_sms, s);
     if (fm == BLASTP_FILTER_STATEFUL) return launch_variant<false, 2, OffT>(a, warps, smem, num_sms, s);
+    if (fm == BLASTP_FILTER_STATEFUL_RB) return launch_variant<false, 3, OffT>(a, warps, smem, num_sms, s);
     return launch_variant<false, 0, OffT>(a, warps, smem, num_sms, s);
   };
   return use_s ? pick(uint16_t{}) : pick(uint32_t{});

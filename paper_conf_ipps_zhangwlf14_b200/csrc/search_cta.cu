@@ -768,7 +768,8 @@ cudaError_t launch_search(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
   const int choice = kernel_choice();
   if ((choice == 0 || choice == 3) && block_kernel_eligible(a_in))
     return launch_search_block(a_in, num_sms, s);
-  if (choice != 2 || a_in.filter_mode == BLASTP_FILTER_STATEFUL)
+  if (choice != 2 || a_in.filter_mode == BLASTP_FILTER_STATEFUL ||
+      a_in.filter_mode == BLASTP_FILTER_STATEFUL_RB)
     return launch_search_warp(a_in, num_sms, s);  // STATEFUL: warp variant only
   static unsigned long long b62_ready = 0;  // one bit per device
   int dev = 0;

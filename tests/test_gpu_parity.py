@@ -143,8 +143,8 @@ def _config2():
     return _CONFIG2["w"]
 
 
-@pytest.mark.parametrize("mode,ext_mode", [(0, 0), (1, 0), (2, 0), (0, 1), (0, 2)],
-                         ids=["LEFT", "EITHER", "STATEFUL", "HIT", "WINDOW"])
+@pytest.mark.parametrize("mode,ext_mode", [(0, 0), (1, 0), (2, 0), (3, 0), (0, 1), (0, 2)],
+                         ids=["LEFT", "EITHER", "STATEFUL", "STATEFUL_RB", "HIT", "WINDOW"])
 def test_config2_full(bp, orc, mode, ext_mode):
     """Config 2 (q517 vs 20M residues): the complete HSP list identical to the
     oracle's, every filter reading (R6 LEFT / EITHER, R15 STATEFUL) and every
@@ -187,12 +187,12 @@ def rescore(orc, queries, ascii, offsets, g, subject_base=0, n=2000):
         assert B[Q[h["q_start"]:h["q_start"] + h["length"]], S].sum() == h["score"]
 
 
-@pytest.mark.parametrize("mode", [0, 1, 2], ids=["LEFT", "EITHER", "STATEFUL"])
+@pytest.mark.parametrize("mode", [0, 1, 2, 3], ids=["LEFT", "EITHER", "STATEFUL", "STATEFUL_RB"])
 def test_config3_full(bp, orc, kernel_variant, mode):
     """Config 3 at full size (q1054 vs 6.0M subjects / ~1.2G residues, the
     bench launch): the complete HSP list identical to the oracle's complete
     list (no sampling), both R6 readings and the STATEFUL walk."""
-    if kernel_variant == "cta" and mode == 2:
+    if kernel_variant == "cta" and mode >= 2:
         pytest.skip("STATEFUL runs on the warp variant only")
     if kernel_variant == "block" and mode != 0:
         pytest.skip("EITHER and STATEFUL run on the warp kernel (the block kernel is LEFT only)")

@@ -11,7 +11,12 @@ from synth import config_workload, gen_db, gen_query
 from test_gpu_parity import _long_subject_db, _rand_db, assert_same, ALPHA
 
 pytestmark = pytest.mark.gpu
-ST = 2  # BLASTP_FILTER_STATEFUL
+
+
+@pytest.fixture(params=[2, 3], ids=["STATEFUL", "STATEFUL_RB"])
+def st(request):
+    """BLASTP_FILTER_STATEFUL (R15) and _STATEFUL_RB (R15 + R16 reach-back)."""
+    return request.param
 
 
 @pytest.fixture(scope="module")
@@ -22,7 +27,7 @@ def bp():
     from paper_conf_ipps_zhangwlf14_b200 import build
     build.build()
     from paper_conf_ipps_zhangwlf14_b200 import blastp
-    assert blastp.FILTER_STATEFUL == ST
+    assert blastp.FILTER_STATEFUL == 2 and blastp.FILTER_STATEFUL_RB == 3
     return blastp
 
 
@@ -33,9 +38,9 @@ def kernel_variant(request, monkeypatch):
     return request.param
 
 
-def test_config1_full_trace(bp, orc):
+def test_config1_full_trace(bp, orc, st):
     (q,), db = config_workload(1)
-    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=ST))
+    g, r = assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=st))
     assert len(g) > 10 and len(r.passing) > 100
 
 
@@ -44,7 +49,7 @@ def test_config1_full_trace(bp, orc):
 # ::test_config3_full[STATEFUL].
 
 
-def test_fuzz_small_random(bp, orc):
+def test_fuzz_small_random(bp, orc, st):
     rng = np.random.default_rng(1515)
     for case in range(80):
         lq = int(rng.choice([3, 5, 17, 64, 127, 300, 517]))
@@ -54,11 +59,11 @@ def test_fuzz_small_random(bp, orc):
                       window=int(rng.choice([40, 40, 10, 80, 3])),
                       min_gap=int(rng.choice([3, 3, 1, 2, 5])),
                       xdrop=int(rng.choice([16, 16, 5, 30])),
-                      cutoff=int(rng.choice([41, 20, 0])), filter_mode=ST)
+                      cutoff=int(rng.choice([41, 20, 0])), filter_mode=st)
         assert_same(bp, orc, q, ascii, off, p, trace=True)
 
 
-def test_adversarial_low_complexity(bp, orc):
+def test_adversarial_low_complexity(bp, orc, st):
     """Every (q, s) a hit: long runs of hits per diagonal inside one round and
     across flushes (many conditional entries per diagonal, chains split over
     two flushes), fresh-subject entries on a still-pending diagonal."""
@@ -68,13 +73,13 @@ def test_adversarial_low_complexity(bp, orc):
     ascii = np.frombuffer("".join(subs).encode(), dtype=np.uint8).copy()
     off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
     for window, W in ((40, 3), (10, 3), (80, 1), (3, 2)):
-        assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=ST, window=window, min_gap=W),
+        assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=st, window=window, min_gap=W),
                     trace=True)
 
 
 @pytest.mark.parametrize("knobs", [{}, {"BLASTP_SEGLEN": "256"}, {"BLASTP_SEGMENTS": "0"}],
                          ids=["default", "seglen256", "whole"])
-def test_long_subjects_diagonal_segments(bp, orc, monkeypatch, knobs):
+def test_long_subjects_diagonal_segments(bp, orc, st, monkeypatch, knobs):
     """Long subjects are split by diagonal range in STATEFUL mode: segment j
     owns the diagonals [d_j, d_j + seg_len) (segment 0 also those below the
     chunk start), walks [d_j, d_j + seg_len + Lq) and holds each of its
@@ -89,22 +94,22 @@ def test_long_subjects_diagonal_segments(bp, orc, monkeypatch, knobs):
     d = bp.pack_db(ascii, off)
     assert (d.segments == 0) == ("BLASTP_SEGMENTS" in knobs)
     for window in (40, 256):
-        g, _ = assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=ST, window=window),
+        g, _ = assert_same(bp, orc, q, ascii, off, bp.Params(filter_mode=st, window=window),
                            trace=True)
         assert len(g) > 10
 
 
-def test_long_query_2000(bp, orc):
+def test_long_query_2000(bp, orc, st):
     q = gen_query(2000, 2000)
     db = gen_db(7, 8, n_subjects=400, mean_len=375.0, queries=[q], plant_frac=0.2)
-    assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=ST), trace=True)
+    assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params(filter_mode=st), trace=True)
 
 
-def test_stateful_requires_diagonal_ext_mode(bp):
+def test_stateful_requires_diagonal_ext_mode(bp, st):
     q = gen_query(3, 100).decode()
     for ext in (1, 2):
         with pytest.raises(bp.BlastpError) as e:
             t = bp.build_query_table(q, bp.Params())
             d = bp.pack_db(np.frombuffer(q.encode(), np.uint8).copy(), np.array([0, len(q)]))
-            bp.search_ungapped(t, d, bp.Params(filter_mode=ST, ext_mode=ext))
+            bp.search_ungapped(t, d, bp.Params(filter_mode=st, ext_mode=ext))
         assert e.value.status == -1  # BLASTP_E_INVALID_ARG

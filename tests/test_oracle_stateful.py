@@ -154,3 +154,84 @@ def test_stateful_search_invariants(orc, B62):
         assert [bool(x) for x in want] == [(subj, d, s_) in trig for s_ in ss]
         n_checked += 1
     assert n_checked > 200
+
+
+# ---------------------------------------------------------------------------
+# filter_mode 3: STATEFUL with Alg. 1 L13's reach-back (reading R16)
+# ---------------------------------------------------------------------------
+
+def test_reachback_hand_walked_examples(orc):
+    with open(os.path.join(GOLD, "alg1_reachback.json")) as f:
+        g = json.load(f)
+    for c in g["cases"]:
+        got = orc.two_hit_stateful_rb(c["s"], c["ext_start"], c["ext_end"], c["W"], c["A"])
+        assert list(got) == c["trigger"], c["name"]
+        assert list(orc.two_hit_stateful(c["s"], c["ext_end"], c["W"], c["A"])) == \
+            c["stateful"], c["name"]
+
+
+def test_reachback_limits(orc):
+    """Extensions that always reach back (start before every hit) give the
+    STATEFUL walk (R15) exactly; extensions that never do (start after every
+    hit) give no extension at all, whatever the hits."""
+    rng = np.random.default_rng(18)
+    for _ in range(2000):
+        s, ext = _random_diagonal(rng, int(rng.integers(1, 16)), span=int(rng.integers(16, 150)))
+        W, A = int(rng.integers(1, 5)), int(rng.integers(2, 60))
+        always = np.full(len(s), -1, dtype=np.int32)
+        never = np.full(len(s), 10 ** 6, dtype=np.int32)
+        assert list(orc.two_hit_stateful_rb(s, always, ext, W, A)) == \
+            list(orc.two_hit_stateful(s, ext, W, A))
+        assert not orc.two_hit_stateful_rb(s, never, ext, W, A).any()
+
+
+def test_reachback_kept_extensions_reach_back(orc):
+    """Every kept extension starts at or before the last hit (or extension
+    end) the walk pairs it with, and a dropped one makes its hit the
+    lasthit: replaying the walk by hand reproduces the triggers."""
+    rng = np.random.default_rng(19)
+    for _ in range(2000):
+        n = int(rng.integers(1, 14))
+        s, ext = _random_diagonal(rng, n)
+        start = (s - rng.integers(0, 20, size=n)).astype(np.int32)
+        trig = orc.two_hit_stateful_rb(s, start, ext, 3, 40)
+        last = None
+        for k in range(n):
+            h = int(s[k])
+            if last is None or h - last >= 40:
+                assert not trig[k]
+                last = h
+            elif h - last < 3:
+                assert not trig[k]
+            elif start[k] <= last:
+                assert trig[k]
+                last = int(ext[k])
+            else:
+                assert not trig[k]
+                last = h
+
+
+def test_oracle_b_agrees_reachback(orc, B62):
+    """oracle.c's STATEFUL_RB search == oracle-B's (Alg. 1 as a position scan with
+    direct word scoring and the reach-back test) on random tiny cases."""
+    al = orc.alphabet()
+    rng = np.random.default_rng(2026)
+    M = B62.tolist()
+    n_ext = n_diff = 0
+    for i, (Q, subs) in enumerate(_oracle_b_cases(rng, al, 300)):
+        T = 11 if i % 5 else 9
+        X = int(rng.choice([16, 16, 5, 30]))
+        cutoff = int(rng.choice([41, 20]))
+        offs = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+        db = np.concatenate(subs).astype(np.uint8) if offs[-1] else np.zeros(0, np.uint8)
+        p = orc.Params(threshold=T, xdrop=X, cutoff=cutoff, filter_mode=3)
+        r = orc.search(Q, db, offs, p, query_id=3, subject_base=10)
+        hb, eb = search_b(Q, subs, M, T=T, X=X, cutoff=cutoff, mode=3, query_id=3,
+                          subject_base=10)
+        assert [tuple(x) for x in r.hsps.tolist()] == hb, i
+        assert [tuple(x) for x in r.extensions.tolist()] == eb, i
+        _, e2 = search_b(Q, subs, M, T=T, X=X, cutoff=cutoff, mode=2, query_id=3,
+                         subject_base=10)
+        n_ext += len(eb)
+        n_diff += eb != e2
+    assert n_ext > 50 and n_diff > 10  # the reach-back changes real searches
