@@ -68,6 +68,17 @@ extern "C" {
                                   each extension a warp-wide window scan (prefix sum,
                                   running max, drop flag over 32 positions at a time);
                                   results identical to DIAGONAL                       */
+#define BLASTP_EXT_HIT_DEDUP 3 /* Alg. 4 followed by the de-duplication step the paper
+                                  puts after it (reading R17): every
+                                  passing hit is extended independently (Alg. 4), then
+                                  each diagonal's extensions, in seed order, are reduced
+                                  by Alg. 3's coverage rule (a seed covered by the last
+                                  kept extension's subject end is dropped) -- exactly
+                                  DIAGONAL's list.  blastp_search_ungapped applies the
+                                  step itself; blastp_search_ungapped_device returns the
+                                  SEED RECORDS of every extension (q_start = the seed's
+                                  query position, s_start = llen; see
+                                  blastp_dedup_covered_device) for the caller to reduce */
 
 /* Search parameters.  Defaults (blastp_params_default) are the BASELINE.json
  * configuration: w = 3, T = 11, A = 40, X = 7 bits -> 16 raw, cutoff 41. */
@@ -243,6 +254,19 @@ int blastp_search_ungapped_device(const blastp_query_table *q,
                                   const blastp_db *db, const blastp_params *p,
                                   void *cuda_stream, blastp_hsp *d_out,
                                   int64_t capacity, int64_t *d_count);
+
+/* The coverage-aware de-duplication of ext_mode HIT_DEDUP (R17), on the
+ * device, in place: d_rec[0..n) are seed records {query_id, subject_id,
+ * diagonal, q_seed, llen, length, score} of every extension (one per passing
+ * hit; the HSP starts at q_seed - llen); they are sorted, each diagonal's
+ * records are walked in seed order keeping a record iff its seed's subject
+ * position exceeds the subject end of the last kept one (Alg. 3 L19-23), and
+ * the kept ones with score >= cutoff are written back as canonical HSPs
+ * (R11).  *d_n_out (device int64) receives their count; runs on cuda_stream
+ * and synchronises it (the kept count sizes the final sort).  Errors:
+ * INVALID_ARG, NOMEM, CUDA. */
+int blastp_dedup_covered_device(blastp_hsp *d_rec, int64_t n, int32_t cutoff, int64_t *d_n_out,
+                                void *cuda_stream);
 
 /* Canonical order (R11) of n device HSPs, in place, on the GPU. */
 int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream);

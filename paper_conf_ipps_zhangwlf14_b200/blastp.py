@@ -23,7 +23,7 @@ LIB_PATH = os.environ.get("BLASTP_LIB") or os.path.join(_PKG, "libblastp.so")
 
 OK, E_INVALID_ARG, E_BAD_RESIDUE, E_TOO_LONG, E_NOMEM, E_CUDA, E_CAPACITY = 0, -1, -2, -3, -4, -5, -6
 FILTER_LEFT, FILTER_EITHER, FILTER_STATEFUL, FILTER_STATEFUL_RB = 0, 1, 2, 3
-EXT_DIAGONAL, EXT_HIT, EXT_WINDOW = 0, 1, 2
+EXT_DIAGONAL, EXT_HIT, EXT_WINDOW, EXT_HIT_DEDUP = 0, 1, 2, 3
 
 HSP_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("diagonal", "<i4"),
                       ("q_start", "<i4"), ("s_start", "<i4"), ("length", "<i4"),
@@ -99,6 +99,8 @@ def _load():
         L.blastp_host_db_free.restype = None
     L.blastp_sort_hsps_device.argtypes = [vp, i64, vp]
     L.blastp_unique_hsps_device.argtypes = [vp, i64, vp, vp]
+    if hasattr(L, "blastp_dedup_covered_device"):  # absent in older builds (A/B timing)
+        L.blastp_dedup_covered_device.argtypes = [vp, i64, i32, vp, vp]
     L.blastp_debug_trace.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64), vp, i64, P(i64),
                                      vp, i64, P(i64)]
     L.blastp_debug_hits.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
@@ -121,7 +123,7 @@ EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "bl
             "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_search_host_db",
             "blastp_format_host_db", "blastp_search_formatted_db", "blastp_host_db_info",
             "blastp_host_db_free",
-            "blastp_sort_hsps_device", "blastp_unique_hsps_device",
+            "blastp_sort_hsps_device", "blastp_unique_hsps_device", "blastp_dedup_covered_device",
             "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
             "blastp_debug_alu_peak",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
@@ -403,6 +405,14 @@ def unique_hsps_device(ptr: int, n: int, count_ptr: int, stream=None):
     the new count is written to the device int64 at count_ptr."""
     _check(lib.blastp_unique_hsps_device(ptr, n, count_ptr, _stream_handle(stream)),
            "blastp_unique_hsps_device")
+
+
+def dedup_covered_device(ptr: int, n: int, cutoff: int, count_ptr: int, stream=None):
+    """ext_mode HIT_DEDUP's de-duplication step on device seed records (R17):
+    the kept HSPs (canonical order) replace the records; the count is written
+    to the device int64 at count_ptr."""
+    _check(lib.blastp_dedup_covered_device(ptr, n, cutoff, count_ptr, _stream_handle(stream)),
+           "blastp_dedup_covered_device")
 
 
 STAT_NAMES = ["windows", "rounds", "conflict_rounds", "hits", "passing", "enqueued", "flushes",

@@ -83,7 +83,7 @@ int validate_params(const blastp_params *p) {
     return fail(BLASTP_E_INVALID_ARG, "filter_mode STATEFUL decides coverage itself: ext_mode "
                 "must be DIAGONAL (got %d)", p->ext_mode);
   if (p->ext_mode != BLASTP_EXT_DIAGONAL && p->ext_mode != BLASTP_EXT_HIT &&
-      p->ext_mode != BLASTP_EXT_WINDOW)
+      p->ext_mode != BLASTP_EXT_WINDOW && p->ext_mode != BLASTP_EXT_HIT_DEDUP)
     return fail(BLASTP_E_INVALID_ARG, "ext_mode %d unknown", p->ext_mode);
   return BLASTP_OK;
 }
@@ -856,7 +856,10 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.xdrop = p->xdrop;
     a.cutoff = p->cutoff;
     a.filter_mode = p->filter_mode;
-    a.ext_mode = p->ext_mode;
+    // HIT_DEDUP searches as Alg. 4 and writes every extension's seed record
+    // (R17); the de-duplication step runs after the search
+    a.ext_mode = p->ext_mode == BLASTP_EXT_HIT_DEDUP ? BLASTP_EXT_HIT : p->ext_mode;
+    a.emit_seed = p->ext_mode == BLASTP_EXT_HIT_DEDUP ? 1 : 0;
     a.ring = search_ring_slots(qd.lq, p->window);
     a.table_entries = qd.entries;
     a.out = out;
@@ -1348,7 +1351,18 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
 
 int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream) {
   if (n < 0 || (n > 0 && !d_hsps)) return fail(BLASTP_E_INVALID_ARG, "bad HSP buffer");
-  CUDA_TRY(sort_hsps(d_hsps, n, static_cast<cudaStream_t>(cuda_stream)));
+  const cudaError_t e = sort_hsps(d_hsps, n, static_cast<cudaStream_t>(cuda_stream));
+  if (e == cudaErrorMemoryAllocation) return fail(BLASTP_E_NOMEM, "sort scratch");
+  CUDA_TRY(e);
+  return BLASTP_OK;
+}
+
+int blastp_dedup_covered_device(blastp_hsp *d_rec, int64_t n, int32_t cutoff, int64_t *d_n_out,
+                                void *cuda_stream) {
+  if (n < 0 || (n > 0 && !d_rec) || !d_n_out) return fail(BLASTP_E_INVALID_ARG, "bad buffers");
+  const cudaError_t e = dedup_covered(d_rec, n, cutoff, d_n_out, static_cast<cudaStream_t>(cuda_stream));
+  if (e == cudaErrorMemoryAllocation) return fail(BLASTP_E_NOMEM, "de-duplication scratch");
+  CUDA_TRY(e);
   return BLASTP_OK;
 }
 
@@ -1356,7 +1370,9 @@ int blastp_unique_hsps_device(blastp_hsp *d_hsps, int64_t n, int64_t *d_n_out,
                               void *cuda_stream) {
   if (n < 0 || (n > 0 && !d_hsps) || !d_n_out)
     return fail(BLASTP_E_INVALID_ARG, "bad HSP buffer");
-  CUDA_TRY(unique_hsps(d_hsps, n, d_n_out, static_cast<cudaStream_t>(cuda_stream)));
+  const cudaError_t e = unique_hsps(d_hsps, n, d_n_out, static_cast<cudaStream_t>(cuda_stream));
+  if (e == cudaErrorMemoryAllocation) return fail(BLASTP_E_NOMEM, "unique scratch");
+  CUDA_TRY(e);
   return BLASTP_OK;
 }
 
@@ -1393,8 +1409,19 @@ int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
       return fail(BLASTP_E_NOMEM, "device HSP buffer (%lld)", static_cast<long long>(want));
     mdb->out_cap = want;
   }
-  const int64_t n = static_cast<int64_t>(h_count);
-  CUDA_TRY(sort_hsps(mdb->out, n, s));
+  int64_t n = static_cast<int64_t>(h_count);
+  if (p->ext_mode == BLASTP_EXT_HIT_DEDUP) {
+    // Alg. 4's de-duplication step (R17): every extension's seed record ->
+    // the coverage chain per diagonal -> canonical HSPs (synchronises s)
+    const cudaError_t e = dedup_covered(mdb->out, n, p->cutoff,
+                                        reinterpret_cast<int64_t *>(mdb->counters + 2), s);
+    if (e == cudaErrorMemoryAllocation) return fail(BLASTP_E_NOMEM, "de-duplication scratch");
+    CUDA_TRY(e);
+    CUDA_TRY(cudaMemcpyAsync(&n, mdb->counters + 2, sizeof(n), cudaMemcpyDeviceToHost, s));
+    CUDA_TRY(cudaStreamSynchronize(s));
+  } else {
+    CUDA_TRY(sort_hsps(mdb->out, n, s));
+  }
   auto *h = static_cast<blastp_hsp *>(malloc(sizeof(blastp_hsp) * static_cast<size_t>(std::max<int64_t>(n, 1))));
   if (!h) return fail(BLASTP_E_NOMEM, "host HSP array");
   if (n > 0) CUDA_TRY(cudaMemcpyAsync(h, mdb->out, sizeof(blastp_hsp) * static_cast<size_t>(n),

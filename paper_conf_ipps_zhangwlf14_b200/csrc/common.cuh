@@ -128,6 +128,7 @@ struct SearchArgs {
   int64_t trace_cap[3];
   unsigned long long *trace_count;   // [3]
   unsigned long long *stats;         // [kNumStats] event counters (trace runs only)
+  int32_t emit_seed;                 // ext_mode HIT_DEDUP: every extension as a seed record
 };
 
 // Event counters collected by the tracing kernel variant (blastp_debug_stats).
@@ -188,6 +189,8 @@ constexpr int kMaxSegments = 32768;  // 256 MB of lists at most
 cudaError_t measure_alu_peak(double *lane_ops_per_s);  // micro.cu
 cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
 cudaError_t unique_hsps(blastp_hsp *d, int64_t n, int64_t *d_n_out, cudaStream_t s);
+cudaError_t dedup_covered(blastp_hsp *d, int64_t n, int32_t cutoff, int64_t *d_n_out,
+                          cudaStream_t s);
 void upload_encode_table();
 
 }  // namespace blastp

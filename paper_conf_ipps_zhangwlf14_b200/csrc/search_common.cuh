@@ -220,7 +220,7 @@ __device__ __forceinline__ void trace_push(const SearchArgs &a, int which, int64
 // is found by binary search over [lo, hi) of the shard's subject starts.
 __device__ __forceinline__ bool emit_hsp(const SearchArgs &a, int64_t sp, int q, int llen,
                                          int rlen, int total, int64_t lo, int64_t hi) {
-  if (total < a.cutoff) return false;
+  if (total < a.cutoff && !a.emit_seed) return false;
   hi -= 1;
   while (lo < hi) {
     const int64_t mid = (lo + hi + 1) >> 1;
@@ -246,6 +246,10 @@ __device__ __forceinline__ bool emit_hsp(const SearchArgs &a, int64_t sp, int q,
   h.diagonal = h.s_start - h.q_start;
   h.length = llen + 3 + rlen;
   h.score = total;
+  if (a.emit_seed) {  // ext_mode HIT_DEDUP: the seed record (blastp_dedup_covered_device)
+    h.q_start = q;
+    h.s_start = llen;
+  }
   const unsigned long long idx = atomicAdd(a.hsp_count, 1ull);
   if ((long long)idx < a.out_cap) a.out[idx] = h;
   return true;

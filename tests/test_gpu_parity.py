@@ -602,6 +602,49 @@ def test_hit_mode_dedup_device(bp, orc):
             assert m == n
 
 
+def test_hit_dedup_equals_diagonal(bp, orc):
+    """ext_mode HIT_DEDUP (R17): Alg. 4 extends every passing hit, then the
+    de-duplication step walks each diagonal's extensions in seed
+    order with Alg. 3's coverage rule -- the result is exactly the oracle's
+    DIAGONAL list (config 1, a long-subject DB, random small cases); the
+    device variant's seed records reduce to the same list through
+    blastp_dedup_covered_device."""
+    import torch
+    cases = []
+    (q,), db = config_workload(1)
+    cases.append((q, db.ascii, db.offsets, bp.Params()))
+    q2 = gen_query(21, 300).decode()
+    a2, o2 = _long_subject_db(q2)
+    cases.append((q2, a2, o2, bp.Params(window=80)))
+    rng = np.random.default_rng(4)
+    for _ in range(20):
+        lq = int(rng.choice([17, 64, 300]))
+        qq = "".join(rng.choice(list(ALPHA[:20]), size=lq))
+        a3, o3 = _rand_db(rng, int(rng.integers(1, 40)), 0, 400, qq, plant=0.6)
+        cases.append((qq, a3, o3, bp.Params(window=int(rng.choice([40, 10])),
+                                            cutoff=int(rng.choice([41, 20])))))
+    n_hit_extra = 0
+    for qq, aa, oo, p in cases:
+        pd = bp.Params(**{**p.__dict__, "ext_mode": bp.EXT_HIT_DEDUP})
+        t = bp.build_query_table(qq, pd)
+        d = bp.pack_db(aa, oo)
+        got = tuples(bp.search_ungapped(t, d, pd))
+        exp = tuples(oracle_run(orc, qq, aa, oo, p).hsps)
+        assert got == exp
+        hit = tuples(bp.search_ungapped(t, d, bp.Params(**{**p.__dict__, "ext_mode": 1})))
+        n_hit_extra += len(hit) - len(exp)
+        cap = 1 << 16
+        out = torch.zeros(cap * 7, dtype=torch.int32, device="cuda")
+        cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+        bp.search_ungapped_device(t, d, out.data_ptr(), cap, cnt.data_ptr(), pd)
+        n = int(cnt.item())
+        assert n <= cap
+        bp.dedup_covered_device(out.data_ptr(), n, pd.cutoff, cnt.data_ptr())
+        m = int(cnt.item())
+        assert [tuple(x) for x in out[: m * 7].view(m, 7).cpu().numpy().tolist()] == exp
+    assert n_hit_extra > 0  # Alg. 4 alone returns more (duplicates / covered seeds)
+
+
 def _host_db_search(bp, t, ascii, off, p, **kw):
     import torch
     cap = 1 << 16
