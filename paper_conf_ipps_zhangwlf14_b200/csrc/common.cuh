@@ -129,6 +129,7 @@ struct SearchArgs {
   unsigned long long *trace_count;   // [3]
   unsigned long long *stats;         // [kNumStats] event counters (trace runs only)
   int32_t emit_seed;                 // ext_mode HIT_DEDUP: every extension as a seed record
+  const int8_t *pssm;                // block kernel, BLASTP_SCORE=pssm_global: the PSSM
 };
 
 // Event counters collected by the tracing kernel variant (blastp_debug_stats).

@@ -110,14 +110,82 @@ __device__ __forceinline__ void bstat(BlkState &st, int i, unsigned long long v)
 // (the X-drop's word loads stay inside the array).
 constexpr int kBlkQPad = 16;
 
+// PSSM: one row of 32 int8 scores per query
+// position, row r = query position r - kBlkQPad (sentinel rows and codes
+// score -128), PSSM[q][a] = BLOSUM62[query[q]][a] -- a perf-only switch
+// (BLASTP_SCORE=pssm|pssm_global), the scores are identical.
+__global__ void pssm_fill_kernel(const uint8_t *__restrict__ qcodes, int lq, int8_t *pssm) {
+  const int rows = lq + 2 * kBlkQPad;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < rows * 32; i += gridDim.x * blockDim.x) {
+    const int r = i >> 5, c = i & 31, k = r - kBlkQPad;
+    const int qcode = (k >= 0 && k < lq) ? qcodes[k] : kSentinel;
+    pssm[i] = c_b62_blk[qcode * 32 + c];
+  }
+}
+
+// R7/R8 X-drop as xdrop_extend (search_common.cuh), the score of query
+// position i against subject code c read as pssm[row(i)][c]: one load per
+// residue instead of a query-code load and a matrix load.
+__device__ __forceinline__ void xdrop_pssm(const uint8_t *__restrict__ stream, int64_t sp, int q,
+                                           const int8_t *pssm, int X, int &total, int &llen,
+                                           int &rlen, int &scanned) {
+  const int8_t *pq = pssm + (q + kBlkQPad) * 32;
+  const int seed = pq[__ldg(stream + sp)] + pq[32 + __ldg(stream + sp + 1)] +
+                   pq[64 + __ldg(stream + sp + 2)];
+  int run = 0, best = 0, bl = 0;
+  {  // right, from (q+3, sp+3)
+    const int64_t a = sp + 3;
+    const uint8_t *base = stream + (a & ~int64_t(3));
+    const uint32_t sh = uint32_t(a & 3) * 8;
+    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
+    const int8_t *pr = pq + 96;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      lo = hi;
+      hi = ldg32(base + t + 8);
+      const int8_t *row = pr + t * 32;
+      xdrop_group4(row[w & 0xffu], row[32 + ((w >> 8) & 0xffu)], row[64 + ((w >> 16) & 0xffu)],
+                   row[96 + (w >> 24)], X, t, run, best, bl, stop);
+    }
+    scanned = t;
+  }
+  const int best_r = best;
+  rlen = bl;
+  run = 0;
+  best = 0;
+  bl = 0;
+  {  // left, from (q-1, sp-1) downwards
+    const int64_t a3 = sp - 4;
+    const uint8_t *base = stream + (a3 & ~int64_t(3));
+    const uint32_t sh = uint32_t(a3 & 3) * 8;
+    uint32_t lo = ldg32(base), hi = ldg32(base + 4);
+    const int8_t *pl = pq - 32;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      hi = lo;
+      lo = ldg32(base - t - 4);
+      const int8_t *row = pl - t * 32;
+      xdrop_group4(row[w >> 24], row[-32 + ((w >> 16) & 0xffu)], row[-64 + ((w >> 8) & 0xffu)],
+                   row[-96 + (w & 0xffu)], X, t, run, best, bl, stop);
+    }
+    scanned += t;
+  }
+  llen = bl;
+  total = seed + best_r + best;
+}
+
 // REGION: flush
 // Extend up to 32 queued passing hits lane-parallel (R7-R9), then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order;
 // kHit: Alg. 4, every passing hit extended and kept (reading R14).
-template <bool kTrace, bool kHit>
+template <bool kTrace, bool kHit, bool kPssm>
 __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w, BlkState &st,
                                           int n, const uint8_t *qc, const int8_t *b62, int lane,
-                                          int slotc, int M) {
+                                          int slotc, int M, const int8_t *pssm) {
   const bool act = lane < n;
   uint32_t ent = 0;
   if (act) ent = w.queue()[(st.qhead + lane) & (kBlkQcap - 1)];
@@ -128,8 +196,12 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
   int total = 0, llen = 0, rlen = 0, scanned = 0;
   // (a variant reading the query codes four per shared load measured 3%
   // slower on config 3: DESIGN.md 5.9)
-  if (act) xdrop_extend(a.stream, sp, q, qc + (kBlkQPad - kQPad), b62, a.xdrop, total, llen, rlen,
-                        scanned);
+  if constexpr (kPssm) {
+    if (act) xdrop_pssm(a.stream, sp, q, pssm, a.xdrop, total, llen, rlen, scanned);
+  } else {
+    if (act) xdrop_extend(a.stream, sp, q, qc + (kBlkQPad - kQPad), b62, a.xdrop, total, llen,
+                          rlen, scanned);
+  }
   if (kTrace) {
     bstat<kTrace>(st, kStatFlushes, 1);
     bstat<kTrace>(st, kStatExtended, n);
@@ -192,8 +264,9 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
 // REGION: setup
 // kDef: the default parameters (min_gap 3, window 40) as compile-time
 // constants, else read from the arguments; kHit: ext_mode HIT (Alg. 4)
-// instead of DIAGONAL (Alg. 3).
-template <bool kTrace, bool kDef, bool kHit>
+// instead of DIAGONAL (Alg. 3); kPssm: X-drop scores from a PSSM (in shared
+// memory when a.pssm is null -- built here --, else a.pssm in global memory).
+template <bool kTrace, bool kDef, bool kHit, bool kPssm>
 __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const SearchArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
@@ -205,10 +278,25 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
     const int k = i - kBlkQPad;
     qc[i] = (k >= 0 && k < lq) ? a.qv.qcodes[k] : uint8_t(kSentinel);
   }
+  uint8_t *areas = smem + 1024 + qc_bytes;
+  const int8_t *pssm = a.pssm;
+  if constexpr (kPssm) {
+    if (!pssm) {  // the PSSM in shared memory (hierarchical buffering)
+      int8_t *ps = reinterpret_cast<int8_t *>(areas);
+      const int rows = lq + 2 * kBlkQPad;
+      for (int i = threadIdx.x; i < rows * 32; i += blockDim.x) {
+        const int r = i >> 5, c = i & 31, k = r - kBlkQPad;
+        const int qcode = (k >= 0 && k < lq) ? a.qv.qcodes[k] : kSentinel;
+        ps[i] = c_b62_blk[qcode * 32 + c];
+      }
+      pssm = ps;
+      areas += align16(size_t(rows) * 32);
+    }
+  }
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int M = a.ring;
   BlkArea w;
-  w.base = smem + 1024 + qc_bytes + size_t(warp) * blk_area_bytes(M);
+  w.base = areas + size_t(warp) * blk_area_bytes(M);
   w.reach_off = kBlkFixed + int(align16(size_t(M) * 4));
   for (int i = lane; i < M; i += 32) {
     w.ring()[i] = 0;
@@ -318,7 +406,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
       // ---- rebase the frame before positions outgrow 14 bits -------------
       if (b >= kBlkFrameMin + kBlkFrameSpan) {
         while (st.qcount > 0)
-          blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc, M);
+          blk_flush<kTrace, kHit, kPssm>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc, M, pssm);
         slotc = (slotc + kBlkFrameSpan) % M;
         for (int i = lane; i < M; i += 32) {
           const uint32_t e = w.ring()[i];
@@ -384,7 +472,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
                   uint32_t(P) | (uint32_t(q) << 16);
             st.qcount += __popc(bal);
             __syncwarp();
-            if (st.qcount >= 32) blk_flush<kTrace, kHit>(a, w, st, 32, qc, b62, lane, slotc, M);
+            if (st.qcount >= 32) blk_flush<kTrace, kHit, kPssm>(a, w, st, 32, qc, b62, lane, slotc, M, pssm);
           }
         };
         // REGION: prepass
@@ -524,7 +612,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
       if (base_slot >= M) base_slot -= M;
     }
     while (st.qcount > 0)
-      blk_flush<kTrace, kHit>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc, M);
+      blk_flush<kTrace, kHit, kPssm>(a, w, st, min(st.qcount, 32), qc, b62, lane, slotc, M, pssm);
     // the next work item continues the frame after a gap (stale state ages out)
     frame = b + 64;
     base_slot = (base_slot + 64) % M;
@@ -535,13 +623,15 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
 }
 
 // REGION: host
-size_t blk_smem_bytes(int lq, int ring, int warps) {
-  return 1024 + align16(size_t(lq) + 2 * kBlkQPad) + size_t(warps) * blk_area_bytes(ring);
+size_t blk_smem_bytes(int lq, int ring, int warps, bool pssm_smem) {
+  return 1024 + align16(size_t(lq) + 2 * kBlkQPad) +
+         (pssm_smem ? align16(size_t(lq + 2 * kBlkQPad) * 32) : 0) +
+         size_t(warps) * blk_area_bytes(ring);
 }
 
-template <bool kTrace, bool kDef, bool kHit>
+template <bool kTrace, bool kDef, bool kHit, bool kPssm>
 cudaError_t blk_launch(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
-  void (*k)(const SearchArgs) = search_block_kernel<kTrace, kDef, kHit>;
+  void (*k)(const SearchArgs) = search_block_kernel<kTrace, kDef, kHit, kPssm>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
   if (e != cudaSuccess) return e;
   int per_sm = 0;
@@ -555,14 +645,14 @@ cudaError_t blk_launch(const SearchArgs &a, int warps, size_t smem, int num_sms,
   return cudaGetLastError();
 }
 
-template <bool kTrace>
+template <bool kTrace, bool kPssm>
 cudaError_t blk_pick(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
   const bool hit = a.ext_mode == BLASTP_EXT_HIT;
   if (a.min_gap == 3 && a.window == 40)
-    return hit ? blk_launch<kTrace, true, true>(a, warps, smem, num_sms, s)
-               : blk_launch<kTrace, true, false>(a, warps, smem, num_sms, s);
-  return hit ? blk_launch<kTrace, false, true>(a, warps, smem, num_sms, s)
-             : blk_launch<kTrace, false, false>(a, warps, smem, num_sms, s);
+    return hit ? blk_launch<kTrace, true, true, kPssm>(a, warps, smem, num_sms, s)
+               : blk_launch<kTrace, true, false, kPssm>(a, warps, smem, num_sms, s);
+  return hit ? blk_launch<kTrace, false, true, kPssm>(a, warps, smem, num_sms, s)
+             : blk_launch<kTrace, false, false, kPssm>(a, warps, smem, num_sms, s);
 }
 
 }  // namespace
@@ -588,16 +678,36 @@ cudaError_t launch_search_block(const SearchArgs &a_in, int num_sms, cudaStream_
   }
   SearchArgs a = a_in;
   a.ring = search_ring_slots(a.qv.lq, a.window);
+  a.pssm = nullptr;
   int optin = 0;
   e = cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (e != cudaSuccess) return e;
+  // X-drop scores (perf only, identical results; paper E2, Fig. 15):
+  // BLASTP_SCORE=pssm (PSSM in shared memory, fewer warps if it costs room),
+  // pssm_global (PSSM in global memory, L1/L2), default: BLOSUM62 + query codes
+  const char *score_env = std::getenv("BLASTP_SCORE");
+  const bool pssm = score_env && !std::strncmp(score_env, "pssm", 4);
+  const bool pssm_smem = pssm && std::strcmp(score_env, "pssm_global") != 0;
   const char *warps_env = std::getenv("BLASTP_WARPS");
   int warps = warps_env ? std::max(1, std::min(kBlkWarps, std::atoi(warps_env))) : kBlkWarps;
-  while (warps > 0 && blk_smem_bytes(a.qv.lq, a.ring, warps) > size_t(optin)) --warps;
+  while (warps > 0 && blk_smem_bytes(a.qv.lq, a.ring, warps, pssm_smem) > size_t(optin)) --warps;
   if (warps < 1) return cudaErrorInvalidConfiguration;
-  const size_t smem = blk_smem_bytes(a.qv.lq, a.ring, warps);
-  return a.trace[0] != nullptr ? blk_pick<true>(a, warps, smem, num_sms, s)
-                               : blk_pick<false>(a, warps, smem, num_sms, s);
+  const size_t smem = blk_smem_bytes(a.qv.lq, a.ring, warps, pssm_smem);
+  const bool trace = a.trace[0] != nullptr;
+  if (!pssm)
+    return trace ? blk_pick<true, false>(a, warps, smem, num_sms, s)
+                 : blk_pick<false, false>(a, warps, smem, num_sms, s);
+  int8_t *g = nullptr;
+  if (!pssm_smem) {
+    const size_t bytes = size_t(a.qv.lq + 2 * kBlkQPad) * 32;
+    if ((e = cudaMallocAsync(reinterpret_cast<void **>(&g), bytes, s)) != cudaSuccess) return e;
+    pssm_fill_kernel<<<int((bytes + 255) / 256), 256, 0, s>>>(a.qv.qcodes, a.qv.lq, g);
+    a.pssm = g;
+  }
+  e = trace ? blk_pick<true, true>(a, warps, smem, num_sms, s)
+            : blk_pick<false, true>(a, warps, smem, num_sms, s);
+  if (g) cudaFreeAsync(g, s);
+  return e;
 }
 
 }  // namespace blastp

@@ -27,6 +27,7 @@
 // per-diagonal ext_reach array.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdlib>
 #include <cstring>
 
@@ -782,8 +783,14 @@ cudaError_t launch_search(const SearchArgs &a_in, int num_sms, cudaStream_t s) {
   CtaConfig c{};
   c.np = 24;
   c.nc = 8;
+  // E1 knobs (the paper's bins-per-warp sweep):
+  // producer / consumer warps; a window of 32 * np positions is binned into
+  // 32 * np + Lq diagonal bins, i.e. (32 * np + Lq) / np bins per producer warp
+  if (const char *v = std::getenv("BLASTP_CTA_NP")) c.np = std::max(1, std::min(31, std::atoi(v)));
+  if (const char *v = std::getenv("BLASTP_CTA_NC")) c.nc = std::max(1, std::min(32 - c.np, std::atoi(v)));
+  if (c.np + c.nc > 32) c.nc = 32 - c.np;
   c.nmax = 32 * c.np;
-  c.cap = 4096;
+  c.cap = std::max(4096, 4096 * c.np / 24);
   c.nb = c.nmax + a.qv.lq;
   c.M = ((a.qv.lq + c.nmax + a.window + 64) + 31) & ~31;
   c.qcap = 256;

@@ -645,6 +645,41 @@ def test_hit_dedup_equals_diagonal(bp, orc):
     assert n_hit_extra > 0  # Alg. 4 alone returns more (duplicates / covered seeds)
 
 
+@pytest.mark.parametrize("score", ["pssm", "pssm_global"])
+def test_pssm_scores_identical(bp, orc, monkeypatch, kernel_variant, score):
+    """The PSSM switch (paper E2; BLASTP_SCORE) is perf-only: the
+    X-drop reads PSSM[q][a] = BLOSUM62[query[q]][a] instead of the matrix and
+    the query code -- every hit, passing hit, extension and HSP identical to
+    the oracle (config 1 traced, config 2 complete, long subjects)."""
+    if kernel_variant != "block":
+        pytest.skip("the PSSM switch is the block kernel's")
+    monkeypatch.setenv("BLASTP_SCORE", score)
+    (q,), db = config_workload(1)
+    assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params())
+    q2 = gen_query(21, 300).decode()
+    a2, o2 = _long_subject_db(q2)
+    assert_same(bp, orc, q2, a2, o2, bp.Params(ext_mode=1))
+    (q3,), db3 = _config2()
+    p = bp.Params()
+    g = bp.search_ungapped(bp.build_query_table(q3, p), bp.pack_db(db3.ascii, db3.offsets), p)
+    assert_lists_equal(g, oracle_full(orc, "config2", q3, db3.ascii, db3.offsets, p), "config 2")
+
+
+@pytest.mark.parametrize("np_nc", [(8, 8), (16, 16), (28, 4)])
+def test_cta_bins_per_warp_knobs(bp, orc, monkeypatch, kernel_variant, np_nc):
+    """The E1 knobs of the CTA variant (producer / consumer warps: bins per
+    warp) leave results unchanged (config 1 traced, long subjects)."""
+    if kernel_variant != "cta":
+        pytest.skip("CTA-variant knobs")
+    monkeypatch.setenv("BLASTP_CTA_NP", str(np_nc[0]))
+    monkeypatch.setenv("BLASTP_CTA_NC", str(np_nc[1]))
+    (q,), db = config_workload(1)
+    assert_same(bp, orc, q, db.ascii, db.offsets, bp.Params())
+    q2 = gen_query(21, 300).decode()
+    a2, o2 = _long_subject_db(q2)
+    assert_same(bp, orc, q2, a2, o2, bp.Params(filter_mode=1))
+
+
 def _host_db_search(bp, t, ascii, off, p, **kw):
     import torch
     cap = 1 << 16
