@@ -130,8 +130,8 @@ __device__ __forceinline__ void xdrop_pssm(const uint8_t *__restrict__ stream, i
                                            const int8_t *pssm, int X, int &total, int &llen,
                                            int &rlen, int &scanned) {
   const int8_t *pq = pssm + (q + kBlkQPad) * 32;
-  const int seed = pq[__ldg(stream + sp)] + pq[32 + __ldg(stream + sp + 1)] +
-                   pq[64 + __ldg(stream + sp + 2)];
+  const int seed = pq[int(__ldg(stream + sp))] + pq[32 + int(__ldg(stream + sp + 1))] +
+                   pq[64 + int(__ldg(stream + sp + 2))];
   int run = 0, best = 0, bl = 0;
   {  // right, from (q+3, sp+3)
     const int64_t a = sp + 3;
@@ -146,8 +146,9 @@ __device__ __forceinline__ void xdrop_pssm(const uint8_t *__restrict__ stream, i
       lo = hi;
       hi = ldg32(base + t + 8);
       const int8_t *row = pr + t * 32;
-      xdrop_group4(row[w & 0xffu], row[32 + ((w >> 8) & 0xffu)], row[64 + ((w >> 16) & 0xffu)],
-                   row[96 + (w >> 24)], X, t, run, best, bl, stop);
+      xdrop_group4(row[int(w & 0xffu)], row[32 + int((w >> 8) & 0xffu)],
+                   row[64 + int((w >> 16) & 0xffu)], row[96 + int(w >> 24)], X, t, run, best, bl,
+                   stop);
     }
     scanned = t;
   }
@@ -169,8 +170,9 @@ __device__ __forceinline__ void xdrop_pssm(const uint8_t *__restrict__ stream, i
       hi = lo;
       lo = ldg32(base - t - 4);
       const int8_t *row = pl - t * 32;
-      xdrop_group4(row[w >> 24], row[-32 + ((w >> 16) & 0xffu)], row[-64 + ((w >> 8) & 0xffu)],
-                   row[-96 + (w & 0xffu)], X, t, run, best, bl, stop);
+      xdrop_group4(row[int(w >> 24)], row[-32 + int((w >> 16) & 0xffu)],
+                   row[-64 + int((w >> 8) & 0xffu)], row[-96 + int(w & 0xffu)], X, t, run, best,
+                   bl, stop);
     }
     scanned += t;
   }
