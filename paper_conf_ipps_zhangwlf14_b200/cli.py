@@ -62,7 +62,9 @@ def main(argv: list[str] | None = None) -> int:
     ap.add_argument("--filter", choices=["left", "either", "stateful", "stateful_rb"], default="left")
     ap.add_argument("--ext", choices=["diagonal", "hit", "window"], default="diagonal")
     ap.add_argument("--stream", action="store_true",
-                    help="keep the database in pinned host memory (formatted image) and stream it")
+                    help="keep the database in pinned host memory (formatted image) and stream it "
+                         "(each part's copy overlaps the previous part's search; the shard's "
+                         "device image must fit in HBM)")
     ap.add_argument("--device", type=int, default=0)
     ap.add_argument("--distributed", action="store_true",
                     help="one process per GPU under torchrun: each rank searches a residue-"
@@ -89,6 +91,17 @@ def main(argv: list[str] | None = None) -> int:
         print("no queries", file=sys.stderr)
         return 1
     queries = [qres[qoff[i]:qoff[i + 1]] for i in range(len(qids))]
+    # a query shorter than one word (3 residues) has no hits: skipped with a
+    # warning, the others keep their ids
+    keep = [i for i, q in enumerate(queries) if len(q) >= 3]
+    for i in range(len(queries)):
+        if i not in keep:
+            print(f"warning: query {qids[i]} shorter than 3 residues: skipped", file=sys.stderr)
+    if not keep:
+        print("no searchable queries", file=sys.stderr)
+        return 1
+    qids = [qids[i] for i in keep]
+    queries = [queries[i] for i in keep]
     p = bp.Params(threshold=args.threshold, window=args.window, xdrop=args.xdrop,
                   cutoff=args.cutoff,
                   filter_mode={"left": bp.FILTER_LEFT, "either": bp.FILTER_EITHER,
@@ -102,13 +115,29 @@ def main(argv: list[str] | None = None) -> int:
     if world > 1:
         # this rank's shard (blastp_shard_range), HSPs with global subject ids,
         # gathered in rank order (canonical per query; re-sorted on rank 0)
-        from .dist import gather_hsps
-        d = bp.pack_db(residues, soff, rank, world, device=args.device)
-        local = torch.from_numpy(bp.search_ungapped(table, d, p).view(np.int32).reshape(-1, 7)
-                                 .copy()).cuda()
-        d.free()
-        allh = gather_hsps(local)
         import torch.distributed as dist
+
+        from .dist import gather_hsps
+        # an error on one rank (e.g. a bad residue in its shard only) is agreed
+        # on by all ranks before the gather, so none waits forever in it
+        err = None
+        local = torch.zeros((0, 7), dtype=torch.int32, device="cuda")
+        try:
+            d = bp.pack_db(residues, soff, rank, world, device=args.device)
+            local = torch.from_numpy(bp.search_ungapped(table, d, p).view(np.int32)
+                                     .reshape(-1, 7).copy()).cuda()
+            d.free()
+        except bp.BlastpError as ex:
+            err = ex
+        flag = torch.tensor([1 if err else 0], dtype=torch.int32,
+                            device="cuda" if dist.get_backend() == "nccl" else "cpu")
+        dist.all_reduce(flag, op=dist.ReduceOp.MAX)
+        if int(flag.item()):
+            dist.destroy_process_group()
+            if err:
+                print(f"rank {rank}: {err}", file=sys.stderr)
+            return 1
+        allh = gather_hsps(local)
         dist.destroy_process_group()
         if rank != 0:
             return 0
@@ -118,7 +147,7 @@ def main(argv: list[str] | None = None) -> int:
         hsps = flat.view(n, 7).cpu().numpy()
     elif args.stream:
         h = bp.format_host_db(residues, soff, device=args.device)
-        cap = max(1 << 16, len(residues) // 100 * len(queries))
+        cap = max(1 << 16, len(residues) // 1000 * len(queries))  # grown below if short
         while True:
             out = torch.empty(cap * 7, dtype=torch.int32, device="cuda")
             cnt = torch.zeros(1, dtype=torch.int64, device="cuda")

@@ -185,11 +185,11 @@ static cudaError_t plan_long_items(blastp_db *db, int nlong, cudaStream_t s) {
   db->nlong = nlong;
   db->nsegs = static_cast<int32_t>(seg_item.size());
   const size_t ns = std::max<size_t>(seg_item.size(), 1);
-  if ((e = cudaMallocAsync(&db->items, sizeof(LongItem) * items.size(), s)) != cudaSuccess) return e;
-  if ((e = cudaMallocAsync(&db->seg_item, sizeof(int32_t) * ns, s)) != cudaSuccess) return e;
-  if ((e = cudaMallocAsync(&db->seg_count, sizeof(int32_t) * ns, s)) != cudaSuccess) return e;
-  if ((e = cudaMallocAsync(&db->seg_done, sizeof(unsigned) * ns, s)) != cudaSuccess) return e;
-  if ((e = cudaMallocAsync(&db->seg_list, sizeof(uint32_t) * ns * size_t(db->seg_cap), s)) != cudaSuccess)
+  if ((e = pool_malloc_async(&db->items, sizeof(LongItem) * items.size(), s)) != cudaSuccess) return e;
+  if ((e = pool_malloc_async(&db->seg_item, sizeof(int32_t) * ns, s)) != cudaSuccess) return e;
+  if ((e = pool_malloc_async(&db->seg_count, sizeof(int32_t) * ns, s)) != cudaSuccess) return e;
+  if ((e = pool_malloc_async(&db->seg_done, sizeof(unsigned) * ns, s)) != cudaSuccess) return e;
+  if ((e = pool_malloc_async(&db->seg_list, sizeof(uint32_t) * ns * size_t(db->seg_cap), s)) != cudaSuccess)
     return e;
   if ((e = cudaMemcpyAsync(db->items, items.data(), sizeof(LongItem) * items.size(),
                            cudaMemcpyHostToDevice, s)) != cudaSuccess)
@@ -264,7 +264,7 @@ static int encode_query(const char *ascii, int32_t len, std::vector<uint8_t> &Q)
 // sentinel letter and neighbours nothing).
 // The radix-32 (start, count) view the block kernel reads (table.cu).
 static int finish_table(QueryDev &out, cudaStream_t s) {
-  if (cudaMallocAsync(&out.wtab, sizeof(uint2) * 32 * 32 * 32, s) != cudaSuccess) {
+  if (pool_malloc_async(&out.wtab, sizeof(uint2) * 32 * 32 * 32, s) != cudaSuccess) {
     cudaGetLastError();
     free_query_dev(out);
     return fail(BLASTP_E_NOMEM, "device allocation for the query table failed");
@@ -281,8 +281,8 @@ static int build_table(const std::vector<uint8_t> &Q, const blastp_params *p, Qu
   const char *how = std::getenv("BLASTP_TABLE_BUILD");  // "host": the host enumeration below
   if (!(how && !std::strcmp(how, "host"))) {
     // GPU build (table.cu): one thread per word counts, scans, fills
-    if (cudaMallocAsync(&out.woff, sizeof(uint32_t) * (kWords + 1), s) != cudaSuccess ||
-        cudaMallocAsync(&out.qcodes, static_cast<size_t>(len) + 16, s) != cudaSuccess) {
+    if (pool_malloc_async(&out.woff, sizeof(uint32_t) * (kWords + 1), s) != cudaSuccess ||
+        pool_malloc_async(&out.qcodes, static_cast<size_t>(len) + 16, s) != cudaSuccess) {
       cudaGetLastError();
       free_query_dev(out);
       return fail(BLASTP_E_NOMEM, "device allocation for the query table failed");
@@ -291,7 +291,7 @@ static int build_table(const std::vector<uint8_t> &Q, const blastp_params *p, Qu
     int64_t total = 0;
     CUDA_TRY(launch_table_count(out.qcodes, len, p->threshold, out.woff, &total, s));
     out.entries = total;
-    if (cudaMallocAsync(&out.qpos, sizeof(uint16_t) * size_t(std::max<int64_t>(total, 1)), s) !=
+    if (pool_malloc_async(&out.qpos, sizeof(uint16_t) * size_t(std::max<int64_t>(total, 1)), s) !=
         cudaSuccess) {
       cudaGetLastError();
       free_query_dev(out);
@@ -606,15 +606,8 @@ static int pack_range(const char *residues_ascii, const int64_t *offsets, int64_
   db->nchunks = static_cast<int32_t>(nchunks);
   db->carved = arena != nullptr;
 
-  // stream-ordered allocations from a pool that keeps its memory (repeated
-  // pack calls, e.g. the e2e benchmark, do not pay cudaMalloc again)
-  {
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
-      uint64_t thr = ~uint64_t(0);
-      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
-  }
+  // stream-ordered allocations from the library's pool, which keeps its
+  // memory (repeated pack calls do not pay cudaMalloc again; common.cuh)
   uint8_t *d_ascii = staging ? staging->ascii : nullptr;
   int64_t *d_off = staging ? staging->off : nullptr;
   int *d_err = staging ? staging->err : nullptr;
@@ -635,7 +628,7 @@ static int pack_range(const char *residues_ascii, const int64_t *offsets, int64_
       *p = static_cast<std::remove_pointer_t<decltype(p)>>(arena->take(bytes));
       return *p != nullptr;
     }
-    return cudaMallocAsync(reinterpret_cast<void **>(p), bytes, s) == cudaSuccess;
+    return pool_malloc_async(reinterpret_cast<void **>(p), bytes, s) == cudaSuccess;
   };
   if (!dalloc(&db->stream, static_cast<size_t>(db->stream_len)) ||
       !dalloc(&db->sstart, sizeof(int64_t) * static_cast<size_t>(std::max<int64_t>(n, 1))) ||
@@ -643,9 +636,9 @@ static int pack_range(const char *residues_ascii, const int64_t *offsets, int64_
       !dalloc(&db->long_chunks, sizeof(Chunk) * static_cast<size_t>(std::max<int64_t>(nchunks, 1))) ||
       !dalloc(&db->counters, 64) ||
       (!staging &&
-       (cudaMallocAsync(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1)), s) != cudaSuccess ||
-        cudaMallocAsync(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1), s) != cudaSuccess ||
-        cudaMallocAsync(&d_err, sizeof(int), s) != cudaSuccess))) {
+       (pool_malloc_async(&d_ascii, static_cast<size_t>(std::max<int64_t>(nres, 1)), s) != cudaSuccess ||
+        pool_malloc_async(&d_off, sizeof(int64_t) * static_cast<size_t>(n + 1), s) != cudaSuccess ||
+        pool_malloc_async(&d_err, sizeof(int), s) != cudaSuccess))) {
     cudaGetLastError();
     return cleanup(fail(BLASTP_E_NOMEM, "device allocation for the database failed"));
   }
@@ -986,15 +979,8 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
   }
   const auto al = [](size_t b) { return (b + 255) & ~size_t(255); };
   total_bytes += al(size_t(std::max<int64_t>(max_res, 1))) + al(8 * size_t(max_n + 1)) + al(4);
-  {
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, q->device) == cudaSuccess) {
-      uint64_t thr = ~uint64_t(0);
-      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
-  }
   Arena arena;
-  if (cudaMallocAsync(reinterpret_cast<void **>(&arena.base), total_bytes, cs) != cudaSuccess) {
+  if (pool_malloc_async(reinterpret_cast<void **>(&arena.base), total_bytes, cs) != cudaSuccess) {
     cudaGetLastError();
     cudaStreamDestroy(cs);
     return fail(BLASTP_E_NOMEM, "device arena of %zu bytes for the host-db search", total_bytes);
@@ -1252,13 +1238,6 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
     scratch_off[k] = bytes;
     bytes += al256(64) + al256(4 * ns) + al256(4 * ns) + al256(4 * ns * size_t(hp.seg_cap));
   }
-  {
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, q->device) == cudaSuccess) {
-      uint64_t thr = ~uint64_t(0);
-      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
-  }
   cudaStream_t cs = nullptr, s2 = nullptr;
   CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
   if (cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking) != cudaSuccess) {
@@ -1269,7 +1248,7 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
   bytes = std::max<size_t>(bytes, 256);
   uint8_t *dev = nullptr;
   // the arena is allocated in s's order; the copies on cs wait for that
-  if (cudaMallocAsync(reinterpret_cast<void **>(&dev), bytes, s) != cudaSuccess) {
+  if (pool_malloc_async(reinterpret_cast<void **>(&dev), bytes, s) != cudaSuccess) {
     cudaGetLastError();
     cudaStreamDestroy(cs);
     cudaStreamDestroy(s2);

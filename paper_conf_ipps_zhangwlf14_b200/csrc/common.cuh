@@ -5,6 +5,7 @@
 #pragma once
 
 #include <cstdint>
+#include <mutex>
 
 #include <cuda_runtime.h>
 
@@ -148,6 +149,37 @@ enum StatIndex {
   kStatXdropLaneSlots,   // lanes x steps of the X-drop loops (utilisation)
   kNumStats = 16
 };
+
+// Stream-ordered device allocations of the library come from its own memory
+// pool per device (created on first use, release threshold = keep
+// everything), so repeated pack / search / format calls do not pay cudaMalloc
+// again -- without changing the device's default pool, which belongs to the
+// caller (PyTorch and others allocate from it).  Freed with cudaFreeAsync.
+inline cudaError_t pool_malloc_async(void **ptr, size_t bytes, cudaStream_t s) {
+  static cudaMemPool_t pools[64] = {};
+  static std::mutex mu;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaMallocAsync(ptr, bytes, s);
+  std::lock_guard<std::mutex> lock(mu);
+  if (!pools[dev]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t pool;
+    if ((e = cudaMemPoolCreate(&pool, &props)) != cudaSuccess) return e;
+    uint64_t thr = ~uint64_t(0);
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    pools[dev] = pool;
+  }
+  return cudaMallocFromPoolAsync(ptr, bytes, pools[dev], s);
+}
+template <typename T>
+inline cudaError_t pool_malloc_async(T **ptr, size_t bytes, cudaStream_t s) {
+  return pool_malloc_async(reinterpret_cast<void **>(ptr), bytes, s);
+}
 
 // Launch helpers implemented in search.cu / pack.cu / sort.cu.
 int search_ring_slots(int lq, int window);

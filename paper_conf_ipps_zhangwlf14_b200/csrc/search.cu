@@ -1,16 +1,19 @@
 // search.cu -- "warp" variant of the fused BLASTP ungapped hot path (sm_100a).
 //
-// Used for long queries (the CTA variant in search_cta.cu needs a
-// per-CTA diagonal ring of ~Lq + window slots plus the hit buckets).  Each
-// warp owns a chunk of whole subjects at a time (work-stealing over chunks)
-// and walks it in ascending subject position:
+// The general kernel: every filter reading (LEFT, EITHER, STATEFUL,
+// STATEFUL_RB) and extension strategy (DIAGONAL, HIT, WINDOW), any window A;
+// the block kernel (search_block.cu) replaces it for LEFT with A >= 31 + W.
+// Each warp owns a chunk of whole subjects at a time (work-stealing over
+// chunks) and walks it in ascending subject position:
 //
 //   hit detection     Alg. 2: a 32-lane window of consecutive
-//                     word positions, residues staged per warp in shared
-//                     memory by cp.async ("coalesced"), lookup
-//                     table (R3) in shared memory when it fits (P:L1702-1730
-//                     hierarchical buffering).  The window advances by just
-//                     enough positions that all their hits fit one round.
+//                     word positions, one residue byte per lane per load
+//                     (coalesced) plus two of overlap, prefetched
+//                     two windows ahead; the lookup table (R3) is read through
+//                     L1/L2, or from shared memory when it fits beside the
+//                     rings without costing resident warps (P:L1702-1730
+//                     hierarchical buffering).  Every window is 32 positions;
+//                     its hits are processed in 32-hit rounds.
 //   binning/sorting   P:L967-1343: replaced by a per-warp diagonal ring in
 //                     shared memory indexed by (s - q) mod M.  Positions are
 //                     visited in ascending s, so each diagonal's hits arrive
@@ -18,7 +21,8 @@
 //                     Hits of one round on the same diagonal are grouped by
 //                     __match_any_sync and ordered by lane (= s).
 //   two-hit filter    P:L1344-1351 (R6): exists p on the same diagonal and
-//                     subject with W <= h - p < A (ring state: last, far, near).
+//                     subject with W <= h - p < A (ring state: last, far, near);
+//                     Alg. 1's lasthit walk for STATEFUL (R15, R16).
 //   extension         Alg. 3/5 + Fig. 8 (R7-R10): passing hits
 //                     not covered by ext_reach are queued; 32 at a time are
 //                     X-dropped lane-parallel and the ext_reach chain is
@@ -885,7 +889,6 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
     while (st.qcount > 0)
       flush_queue<kTrace, kWin, kSt>(a, w, st, min(st.qcount, 32), qc, b62, lane, sc, M);
   }
-  cp_async_wait_all();
   if (kTrace && a.stats && lane == 0)
     for (int i = 0; i < kNumStats; ++i)
       if (st.stat[i]) atomicAdd(a.stats + i, st.stat[i]);

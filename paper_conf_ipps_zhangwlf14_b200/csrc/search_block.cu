@@ -702,7 +702,7 @@ cudaError_t launch_search_block(const SearchArgs &a_in, int num_sms, cudaStream_
   int8_t *g = nullptr;
   if (!pssm_smem) {
     const size_t bytes = size_t(a.qv.lq + 2 * kBlkQPad) * 32;
-    if ((e = cudaMallocAsync(reinterpret_cast<void **>(&g), bytes, s)) != cudaSuccess) return e;
+    if ((e = pool_malloc_async(reinterpret_cast<void **>(&g), bytes, s)) != cudaSuccess) return e;
     pssm_fill_kernel<<<int((bytes + 255) / 256), 256, 0, s>>>(a.qv.qcodes, a.qv.lq, g);
     a.pssm = g;
   }

@@ -1,6 +1,7 @@
-// search_common.cuh -- device helpers shared by the two search kernels
-// (search.cu: warp-private diagonal rings; search_cta.cu: CTA windows with
-// per-diagonal buckets and warp-specialised extension).
+// search_common.cuh -- device helpers shared by the search kernels
+// (search_block.cu: block two-hit state; search.cu: warp-private diagonal
+// rings; search_cta.cu: CTA windows with per-diagonal buckets and
+// warp-specialised extension).
 #pragma once
 
 #include <cuda_runtime.h>
@@ -32,18 +33,6 @@ __device__ __forceinline__ int score(const int8_t *b62, uint32_t qcode, uint32_t
 __device__ __forceinline__ uint32_t ldg32(const uint8_t *p) {
   return __ldg(reinterpret_cast<const uint32_t *>(p));
 }
-
-__device__ __forceinline__ void cp_async16(void *smem, const void *gmem) {
-  const unsigned s = static_cast<unsigned>(__cvta_generic_to_shared(smem));
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
-}
-__device__ __forceinline__ void cp_async8(void *smem, const void *gmem) {
-  const unsigned s = static_cast<unsigned>(__cvta_generic_to_shared(smem));
-  asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(gmem));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;\n"); }
-__device__ __forceinline__ void cp_async_wait_1() { asm volatile("cp.async.wait_group 1;\n"); }
 
 // Work item ci of the chunk cursor without the segment pipeline: the long
 // items whole (their single warp must not start last), then the regular

@@ -63,12 +63,12 @@ cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s) {
   const size_t bytes = size_t(n) * sizeof(uint32_t);
   // every allocation checked: a failed one frees the others and returns
   // cudaErrorMemoryAllocation (the C-ABI maps it to BLASTP_E_NOMEM)
-  if ((e = cudaMallocAsync(&idx, bytes, s)) == cudaSuccess &&
-      (e = cudaMallocAsync(&idx2, bytes, s)) == cudaSuccess &&
-      (e = cudaMallocAsync(&key, bytes, s)) == cudaSuccess &&
-      (e = cudaMallocAsync(&key2, bytes, s)) == cudaSuccess &&
-      (e = cudaMallocAsync(&tmp, size_t(n) * sizeof(blastp_hsp), s)) == cudaSuccess &&
-      (e = cudaMallocAsync(&temp, temp_bytes, s)) == cudaSuccess) {
+  if ((e = pool_malloc_async(&idx, bytes, s)) == cudaSuccess &&
+      (e = pool_malloc_async(&idx2, bytes, s)) == cudaSuccess &&
+      (e = pool_malloc_async(&key, bytes, s)) == cudaSuccess &&
+      (e = pool_malloc_async(&key2, bytes, s)) == cudaSuccess &&
+      (e = pool_malloc_async(&tmp, size_t(n) * sizeof(blastp_hsp), s)) == cudaSuccess &&
+      (e = pool_malloc_async(&temp, temp_bytes, s)) == cudaSuccess) {
     const int blocks = int((n + 255) / 256 > 4096 ? 4096 : (n + 255) / 256);
     iota_kernel<<<blocks, 256, 0, s>>>(idx, n);
     const int fields[5] = {5, 3, 2, 1, 0};  // length, q_start, diagonal, subject_id, query_id
@@ -103,8 +103,8 @@ cudaError_t unique_hsps(blastp_hsp *d, int64_t n, int64_t *d_n_out, cudaStream_t
   size_t temp_bytes = 0;
   cudaError_t e = cub::DeviceSelect::Unique(nullptr, temp_bytes, d, tmp, d_n_out, n, s);
   if (e != cudaSuccess) return e;
-  if ((e = cudaMallocAsync(&tmp, size_t(n) * sizeof(blastp_hsp), s)) == cudaSuccess &&
-      (e = cudaMallocAsync(&temp, temp_bytes, s)) == cudaSuccess) {
+  if ((e = pool_malloc_async(&tmp, size_t(n) * sizeof(blastp_hsp), s)) == cudaSuccess &&
+      (e = pool_malloc_async(&temp, temp_bytes, s)) == cudaSuccess) {
     e = cub::DeviceSelect::Unique(temp, temp_bytes, d, tmp, d_n_out, n, s);
     if (e == cudaSuccess)
       e = cudaMemcpyAsync(d, tmp, size_t(n) * sizeof(blastp_hsp), cudaMemcpyDeviceToDevice, s);
@@ -162,7 +162,7 @@ cudaError_t dedup_covered(blastp_hsp *d, int64_t n, int32_t cutoff, int64_t *d_n
   // (query, subject, diagonal, q_seed, ...) lexicographic = seed order per diagonal
   if ((e = sort_hsps(d, n, s)) != cudaSuccess) return e;
   blastp_hsp *tmp = nullptr;
-  if ((e = cudaMallocAsync(&tmp, size_t(n) * sizeof(blastp_hsp), s)) != cudaSuccess) {
+  if ((e = pool_malloc_async(&tmp, size_t(n) * sizeof(blastp_hsp), s)) != cudaSuccess) {
     cudaGetLastError();
     return e;
   }

@@ -105,7 +105,7 @@ cudaError_t launch_table_count(const uint8_t *qcodes, int lq, int T, uint32_t *w
   e = cub::DeviceScan::InclusiveSum(nullptr, temp_bytes, woff + 1, woff + 1, kWords, s);
   if (e != cudaSuccess) return e;
   void *temp = nullptr;
-  if ((e = cudaMallocAsync(&temp, temp_bytes, s)) != cudaSuccess) return e;
+  if ((e = pool_malloc_async(&temp, temp_bytes, s)) != cudaSuccess) return e;
   e = cub::DeviceScan::InclusiveSum(temp, temp_bytes, woff + 1, woff + 1, kWords, s);
   cudaFreeAsync(temp, s);
   if (e != cudaSuccess) return e;
