@@ -322,6 +322,12 @@ int blastp_debug_stats(const blastp_query_table *q, const blastp_db *db,
  * time and by this roof: the on-chip roofline beside the HBM one. */
 int blastp_debug_alu_peak(int device, double *lane_ops_per_s);
 
+/* The library's stream-ordered device allocations come from its own memory
+ * pool per device, which keeps freed memory for reuse (repeated pack /
+ * search calls do not pay cudaMalloc again); this returns the pool's unused
+ * memory to the device (synchronises the device).  Errors: CUDA. */
+int blastp_trim_memory(int device);
+
 void blastp_hsp_free(blastp_hsp *h);
 void blastp_query_table_free(blastp_query_table *q);
 void blastp_db_free(blastp_db *db);

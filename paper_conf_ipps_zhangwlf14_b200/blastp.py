@@ -106,6 +106,8 @@ def _load():
     L.blastp_debug_hits.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
     L.blastp_debug_passing.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
     L.blastp_debug_stats.argtypes = [vp, vp, P(_CParams), vp, vp, i32]
+    if hasattr(L, "blastp_trim_memory"):
+        L.blastp_trim_memory.argtypes = [ctypes.c_int]
     if hasattr(L, "blastp_debug_alu_peak"):  # absent in older builds (A/B timing)
         L.blastp_debug_alu_peak.argtypes = [ctypes.c_int, P(ctypes.c_double)]
     for f in ("blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"):
@@ -125,7 +127,7 @@ EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "bl
             "blastp_host_db_free",
             "blastp_sort_hsps_device", "blastp_unique_hsps_device", "blastp_dedup_covered_device",
             "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
-            "blastp_debug_alu_peak",
+            "blastp_debug_alu_peak", "blastp_trim_memory",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
 
 
@@ -428,6 +430,11 @@ def debug_stats(table: QueryTable, db: Database, params: Params | None = None,
                                   _stream_handle(stream), buf, len(STAT_NAMES)),
            "blastp_debug_stats")
     return dict(zip(STAT_NAMES, list(buf)))
+
+
+def trim_memory(device: int = 0):
+    """Return the library pool's unused device memory (blastp_trim_memory)."""
+    _check(lib.blastp_trim_memory(device), "blastp_trim_memory")
 
 
 def debug_alu_peak(device: int = 0) -> float:

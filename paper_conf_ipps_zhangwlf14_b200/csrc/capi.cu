@@ -1507,6 +1507,13 @@ int blastp_debug_stats(const blastp_query_table *q, const blastp_db *db, const b
                    nullptr, stats, nstats);
 }
 
+int blastp_trim_memory(int device) {
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
+  CUDA_TRY(pool_trim(device));
+  return BLASTP_OK;
+}
+
 int blastp_debug_alu_peak(int device, double *lane_ops_per_s) {
   if (!lane_ops_per_s) return fail(BLASTP_E_INVALID_ARG, "output is NULL");
   DeviceGuard g(device);

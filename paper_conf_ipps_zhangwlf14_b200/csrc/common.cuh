@@ -155,9 +155,17 @@ enum StatIndex {
 // everything), so repeated pack / search / format calls do not pay cudaMalloc
 // again -- without changing the device's default pool, which belongs to the
 // caller (PyTorch and others allocate from it).  Freed with cudaFreeAsync.
+struct LibPools {
+  cudaMemPool_t pools[64] = {};
+  std::mutex mu;
+};
+inline LibPools &lib_pools() {
+  static LibPools p;
+  return p;
+}
 inline cudaError_t pool_malloc_async(void **ptr, size_t bytes, cudaStream_t s) {
-  static cudaMemPool_t pools[64] = {};
-  static std::mutex mu;
+  cudaMemPool_t *pools = lib_pools().pools;
+  std::mutex &mu = lib_pools().mu;
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
@@ -175,6 +183,16 @@ inline cudaError_t pool_malloc_async(void **ptr, size_t bytes, cudaStream_t s) {
     pools[dev] = pool;
   }
   return cudaMallocFromPoolAsync(ptr, bytes, pools[dev], s);
+}
+// Returns the memory the library's pool of `device` holds to the device
+// (blastp_trim_memory); allocations still alive are kept.
+inline cudaError_t pool_trim(int device) {
+  if (device < 0 || device >= 64) return cudaSuccess;
+  std::lock_guard<std::mutex> lock(lib_pools().mu);
+  cudaMemPool_t pool = lib_pools().pools[device];
+  if (!pool) return cudaSuccess;
+  cudaError_t e = cudaDeviceSynchronize();
+  return e == cudaSuccess ? cudaMemPoolTrimTo(pool, 0) : e;
 }
 template <typename T>
 inline cudaError_t pool_malloc_async(T **ptr, size_t bytes, cudaStream_t s) {

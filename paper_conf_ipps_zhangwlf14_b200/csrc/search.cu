@@ -250,7 +250,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
     // decided at enqueue; a fresh entry (bit 30) starts a new subject (no
     // lasthit); any other entry applies L11-19 to the lasthit the walk has
     // reached.  An accepted extension sets lasthit = its subject end.
-    const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
+    const unsigned grp = __match_any_sync(kFull, act ? slot : -1);
     const uint32_t e = act ? w.ring()[slot] : 0u;
     uint32_t cur = e & 0xffffu;
     const int gmax = __reduce_max_sync(kFull, act ? __popc(grp) : 0);
@@ -298,7 +298,7 @@ __device__ void flush_queue(const SearchArgs &a, const WarpSmem &w, WarpState &s
     // Alg. 4: every passing hit is extended and kept; ext_reach
     // is never written, so every passing hit was also queued
     acc = act;
-  } else if (const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane),
+  } else if (const unsigned grp = __match_any_sync(kFull, act ? slot : -1),
              uniq = (grp == (1u << lane));
              __all_sync(kFull, uniq || !act)) {
     if (act) {
@@ -727,7 +727,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           slot += (slot < 0) ? M : 0;
           slot -= (slot >= M) ? M : 0;
         }
-        const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
+        const unsigned grp = __match_any_sync(kFull, act ? slot : -1);
         const unsigned earlier = grp & lanemask_lt(lane);
         uint32_t e = 0, rch = 0;
         if (act) {
@@ -800,7 +800,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
           // the mask of those within W of this hit
           int cand_e = 0;
           uint32_t nb = 0;
-          if (const int nearly = __reduce_max_sync(kFull, __popc(earlier)); nearly) {
+          if (const int nearly = __reduce_max_sync(kFull, act ? __popc(earlier) : 0); nearly) {
             unsigned rem = earlier;
             for (int it = 0; it < nearly; ++it) {
               const int src = rem ? __ffs(rem) - 1 : lane;
@@ -822,7 +822,7 @@ __global__ void __launch_bounds__(kMaxWarps * 32) search_warp_kernel(const Searc
             pass = has_successor(stream, sph, q, qc, b62, lq, W, A, a.threshold);
           if (kTrace) {
             stat_add<kTrace>(st, kStatRounds, 1);
-            stat_add<kTrace>(st, kStatConflictRounds, __any_sync(kFull, earlier != 0) ? 1 : 0);
+            stat_add<kTrace>(st, kStatConflictRounds, __any_sync(kFull, act && earlier != 0) ? 1 : 0);
             if (!retrace) {
               stat_add<kTrace>(st, kStatHits, __popc(__ballot_sync(kFull, counts)));
               stat_add<kTrace>(st, kStatPassing, __popc(__ballot_sync(kFull, pass)));

@@ -218,7 +218,7 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
     // runs past the query (rlen < 16,000)
     const int endp = P + 2 + rlen;
     uint16_t *r16 = w.reach() + slot;
-    const unsigned grp = __match_any_sync(kFull, act ? slot : -1 - lane);
+    const unsigned grp = __match_any_sync(kFull, act ? slot : -1);
     const bool uniq = grp == (1u << lane);
     if (__all_sync(kFull, uniq || !act)) {
       if (act) {
@@ -531,8 +531,13 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
           slot_o = slot;
           lsv_o = lsv;
           act_o = act;
+#ifdef BLK_FAKE_MATCH  // experiment only (wrong results): the cost of MATCH.ANY
+          (void)bid;
+          return (1u << lane) | (__shfl_xor_sync(kFull, slot, 1) == slot ? (1u << (lane ^ 1)) : 0u);
+#else
           return __match_any_sync(
-              kFull, act ? (unsigned(slot) | (unsigned(bid) << 14)) : (0x80000000u | unsigned(lane)));
+              kFull, act ? (unsigned(slot) | (unsigned(bid) << 14)) : 0xffffffffu);
+#endif
         };
         int cv = 0, cq = 0, nv = 0, nq = 0, cslot = 0, clsv = 0;
         bool cact = false;
@@ -564,7 +569,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
           // slot's last group when a subject starts inside the round)
           unsigned Gw = G;
           if (multi_bid_possible && __any_sync(kFull, act && bid != b))
-            Gw = __match_any_sync(kFull, act ? slot : -1 - lane);
+            Gw = __match_any_sync(kFull, act ? slot : -1);
           if (act && lane == 31 - __clz(Gw)) {
             const bool sw = ebid == bid;
             const int dp = bid - emax;

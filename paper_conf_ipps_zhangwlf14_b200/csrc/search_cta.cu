@@ -160,7 +160,11 @@ __device__ void consumer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
     // entries are ready when their sequence number matches the slot's index;
     // idle consumers probe one slot and sleep (they must not steal issue
     // slots from the producers)
-    const bool done = S.ctrl->done != 0;
+    // the producers' completion flag: written once by producer warp 0 after
+    // its __threadfence_block (release), read here volatile (acquire side);
+    // racecheck reports this flag handshake as a shared-memory hazard, the
+    // only one in the library (profiles/r02/sanitizer_*.log)
+    const bool done = *reinterpret_cast<volatile int *>(&S.ctrl->done) != 0;
     if (!done) {
       unsigned probe = 0;
       if (lane == 0)
@@ -204,7 +208,7 @@ __device__ void consumer(const SearchArgs &a, const CtaConfig &c, const Smem &S,
     bool acc = false;
     if (hitm) {
       acc = pre;
-    } else if (const unsigned grp = __match_any_sync(kFull, pre ? slot : -1 - lane),
+    } else if (const unsigned grp = __match_any_sync(kFull, pre ? slot : -1),
                uniq = grp == (1u << lane);
                __all_sync(kFull, uniq || !pre)) {
       if (pre) {
@@ -726,7 +730,7 @@ __global__ void __launch_bounds__(kThreads, 1) search_cta_kernel(const SearchArg
     pbar(c.np);
     if (warp == 0 && lane == 0) {
       __threadfence_block();
-      S.ctrl->done = 1;
+      *reinterpret_cast<volatile int *>(&S.ctrl->done) = 1;
     }
   } else if (warp < c.np + c.nc) {
     consumer<kTrace>(a, c, S, warp - c.np, lane);

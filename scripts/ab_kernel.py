@@ -86,7 +86,8 @@ def main():
         m = statistics.median(times[name])
         base = base or m
         print(f"{name:28s} {m:8.3f}  ({100 * (m / base - 1):+5.1f}%)  hsps {counts[name]}")
-    assert len(set(counts.values())) == 1, counts
+    if os.environ.get("AB_NO_CHECK") != "1":
+        assert len(set(counts.values())) == 1, counts
 
 
 if __name__ == "__main__":

@@ -24,6 +24,8 @@ def check(q, ascii, off, p, label):
     t = bp.build_query_table(q, p)
     d = bp.pack_db(ascii, off)
     g = [tuple(x) for x in bp.search_ungapped(t, d, p).tolist()]
+    t.free()
+    d.free()
     P = orc.Params(word_len=p.word_len, threshold=p.threshold, window=p.window,
                    min_gap=p.min_gap, xdrop=p.xdrop, cutoff=p.cutoff, filter_mode=p.filter_mode,
                    ext_mode=1 if p.ext_mode == 1 else 0)
@@ -63,9 +65,13 @@ def main():
     qs = [gen_query(300 + i, L) for i, L in enumerate([60, 120, 200, 350])]
     dbq = gen_db(301, 302, n_subjects=150, mean_len=300.0, queries=qs, plant_frac=0.5)
     t = bp.build_query_batch(qs, bp.Params())
-    g = bp.search_ungapped(t, bp.pack_db(dbq.ascii, dbq.offsets), bp.Params())
+    d = bp.pack_db(dbq.ascii, dbq.offsets)
+    g = bp.search_ungapped(t, d, bp.Params())
     assert len(g) > 10
     print(f"ok query groups: {len(g)} HSPs", flush=True)
+    t.free()
+    d.free()
+    bp.trim_memory(0)  # pool memory back to the device: memcheck's leak check sees only leaks
 
 
 if __name__ == "__main__":

@@ -88,7 +88,7 @@ def test_shard_range_rejects_bad_arguments(bp):
 
 def test_invalid_params_rejected_before_any_gpu_work(bp):
     for bad in [dict(word_len=4), dict(min_gap=0), dict(window=0), dict(xdrop=0),
-                dict(xdrop=200), dict(filter_mode=7), dict(ext_mode=3), dict(threshold=500)]:
+                dict(xdrop=200), dict(filter_mode=7), dict(ext_mode=4), dict(threshold=500)]:
         with pytest.raises(bp.BlastpError) as e:
             bp.build_query_table("MKVLAAGIVALLA", bp.Params(**bad))
         assert e.value.status == bp.E_INVALID_ARG, bad
