@@ -180,6 +180,69 @@ __device__ __forceinline__ void xdrop_pssm(const uint8_t *__restrict__ stream, i
   total = seed + best_r + best;
 }
 
+// R7/R8 X-drop, the same scan as search_common.cuh's xdrop_extend (Fig. 8's
+// running sum / best / drop rule in branch-free groups of four), with the
+// subject read as 32-bit words by a 32-bit word index from the stream base
+// (one IMAD.WIDE per load): inside the round loop's register pressure the
+// compiler otherwise rebuilds the 64-bit byte address every iteration.
+__device__ __forceinline__ void blk_xdrop(const uint8_t *__restrict__ stream, int64_t sp, int q,
+                                          const uint8_t *qc, const int8_t *b62, int X, int &total,
+                                          int &llen, int &rlen, int &scanned) {
+  const uint32_t *__restrict__ sw = reinterpret_cast<const uint32_t *>(stream);
+  const uint8_t *qq = qc + kQPad;
+  const int seed = score(b62, qq[q], __ldg(stream + sp)) +
+                   score(b62, qq[q + 1], __ldg(stream + sp + 1)) +
+                   score(b62, qq[q + 2], __ldg(stream + sp + 2));
+  int run = 0, best = 0, bl = 0;
+  {  // right, from (q+3, sp+3)
+    const int64_t a = sp + 3;
+    uint32_t wi = uint32_t(a >> 2);
+    const uint32_t sh = uint32_t(a & 3) * 8;
+    uint32_t lo = __ldg(sw + wi), hi = __ldg(sw + wi + 1);
+    wi += 2;
+    const uint8_t *qp = qq + q + 3;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      lo = hi;
+      hi = __ldg(sw + wi);
+      ++wi;
+      xdrop_group4(score(b62, qp[t], w & 0xffu), score(b62, qp[t + 1], (w >> 8) & 0xffu),
+                   score(b62, qp[t + 2], (w >> 16) & 0xffu), score(b62, qp[t + 3], w >> 24), X,
+                   t, run, best, bl, stop);
+    }
+    scanned = t;
+  }
+  const int best_r = best;
+  rlen = bl;
+  run = 0;
+  best = 0;
+  bl = 0;
+  {  // left, from (q-1, sp-1) downwards
+    const int64_t a3 = sp - 4;  // bytes a3 .. a3+3 = positions sp-4 .. sp-1
+    uint32_t wi = uint32_t(a3 >> 2);
+    const uint32_t sh = uint32_t(a3 & 3) * 8;
+    uint32_t lo = __ldg(sw + wi), hi = __ldg(sw + wi + 1);
+    --wi;
+    const uint8_t *qp = qq + q - 1;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      hi = lo;
+      lo = __ldg(sw + wi);
+      --wi;
+      xdrop_group4(score(b62, qp[-t], w >> 24), score(b62, qp[-(t + 1)], (w >> 16) & 0xffu),
+                   score(b62, qp[-(t + 2)], (w >> 8) & 0xffu), score(b62, qp[-(t + 3)], w & 0xffu),
+                   X, t, run, best, bl, stop);
+    }
+    scanned += t;
+  }
+  llen = bl;
+  total = seed + best_r + best;
+}
+
 // REGION: flush
 // Extend up to 32 queued passing hits lane-parallel (R7-R9), then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order;
@@ -201,8 +264,13 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
   if constexpr (kPssm) {
     if (act) xdrop_pssm(a.stream, sp, q, pssm, a.xdrop, total, llen, rlen, scanned);
   } else {
+#ifdef BLK_OLD_XDROP  // A/B knob
     if (act) xdrop_extend(a.stream, sp, q, qc + (kBlkQPad - kQPad), b62, a.xdrop, total, llen,
                           rlen, scanned);
+#else
+    if (act) blk_xdrop(a.stream, sp, q, qc + (kBlkQPad - kQPad), b62, a.xdrop, total, llen, rlen,
+                       scanned);
+#endif
   }
   if (kTrace) {
     bstat<kTrace>(st, kStatFlushes, 1);
