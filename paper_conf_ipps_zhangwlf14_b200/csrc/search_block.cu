@@ -381,6 +381,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
   const int L = W - 1;  // record lag: lanes v < L are tested against the previous block
   const int A = kDef ? 40 : a.window;
   const unsigned ltmask = lanemask_lt(lane);
+  const unsigned lemask = kFull >> (31 - lane);  // lanes <= lane
   uint32_t *scr = w.scr();
 
   BlkState st;
@@ -520,14 +521,16 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
         auto locate = [&](uint32_t kb, uint32_t lim, int &own_out, int &q_out) {
           const bool wr = cnt != 0u && excl < kb + 32u && incl > kb;
           const int p0 = wr ? max(int(excl) - int(kb), 0) : 0;
+          // (table offset - excl) << 5 | lane: the offset difference is
+          // signed and fits 27 bits (tables < 2^26 entries)
           if (wr) scr[p0] = uint32_t(lane) | ((o - excl) << 5);
           const unsigned S = __reduce_or_sync(kFull, wr ? (1u << p0) : 0u);
           __syncwarp();
-          const int src = 31 - __clz(S & (kFull >> (31 - lane)));
-          const uint32_t vv = scr[src];
-          own_out = int(vv & 31u);
+          const int src = 31 - __clz(S & lemask);
+          const int vv = int(scr[src]);
+          own_out = vv & 31;
           const uint32_t k = kb + uint32_t(lane);
-          q_out = k < lim ? int(__ldg(qpos + (((vv >> 5) + k) & 0x7ffffffu))) : 0;
+          q_out = k < lim ? int(__ldg(qpos + ((vv >> 5) + int(k)))) : 0;
           __syncwarp();
         };
         // hits of lanes v < L (tested against the previous block's state)
