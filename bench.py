@@ -60,6 +60,9 @@ def parse_args():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--gather", choices=["p2p", "nccl"], default="p2p",
+                    help="N > 1: HSPs appended by the search kernels into rank 0's buffer over "
+                         "NVLink (CUDA IPC), or per-rank lists gathered with NCCL")
     ap.add_argument("--scale", type=float, default=1.0, help="DB scale (tests only)")
     return ap.parse_args()
 
@@ -324,11 +327,26 @@ def main():
     out = torch.empty((cap, 7), dtype=torch.int32, device=dev)
     cnt = torch.zeros(1, dtype=torch.int64, device=dev)
 
+    # N > 1: the search kernels append into rank 0's buffer over NVLink
+    # (dist.PeerHspBuffer, CUDA IPC) -- the gather fused into the search;
+    # --gather nccl: per-rank buffers + the NCCL count/point-to-point gather
+    peer = None
+    if world > 1 and args.gather == "p2p":
+        from paper_conf_ipps_zhangwlf14_b200.dist import PeerHspBuffer
+        peer = PeerHspBuffer(cap * world)
+
     def search():
         bp.search_ungapped_device(table, gdb, out.data_ptr(), cap, cnt.data_ptr(), params, stream)
 
-    def step():
+    def step(events=None):
+        if peer is not None:
+            peer.search(table, gdb, params, canonical=False, events=events)
+            return
+        if events:
+            events[0].record(stream)
         search()
+        if events:
+            events[1].record(stream)
         if world > 1:
             n = int(cnt.item())
             gather_hsps(out[: min(n, cap)])
@@ -338,6 +356,10 @@ def main():
     torch.cuda.synchronize()
     n_hsp = int(cnt.item())
     assert n_hsp <= cap, "HSP buffer too small"
+    if peer is not None:
+        search()  # this rank's own count (n_hsp) for the roofline's HSP bytes
+        torch.cuda.synchronize()
+        n_hsp = int(cnt.item())
 
     # ---- timed region -------------------------------------------------------
     clocks = ClockSampler(local_rank)
@@ -352,11 +374,7 @@ def main():
     t_end = torch.cuda.Event(enable_timing=True)
     t_start.record(stream)
     for k in range(args.steps):
-        ev[k][0].record(stream)
-        search()
-        ev[k][1].record(stream)
-        if world > 1:
-            gather_hsps(out[: min(int(cnt.item()), cap)])
+        step(ev[k])
     t_end.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -564,7 +582,11 @@ def main():
                        "l2": "inputs larger than L2 (DB shard >> 126 MB), no flush",
                        "hsps_per_step": n_hsp,
                        "parallelism": f"db-shard{world}" + (f" (of {nshards})" if nshards != world
-                                                             else "")},
+                                                             else ""),
+                       "gather": None if world == 1 else (
+                           "p2p: every rank's search kernel appends its HSPs into rank 0's "
+                           "buffer over NVLink (CUDA IPC, blastp_search_ungapped_append)"
+                           if peer is not None else "NCCL count all_gather + point-to-point")},
             # the metric's roofline (HBM) and the on-chip one
             "roofline": hbm_roof,
             "onchip_roofline": onchip,
@@ -584,6 +606,8 @@ def main():
             "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
+    if peer is not None:
+        peer.free()
     if world > 1:
         dist.destroy_process_group()
 

@@ -259,6 +259,38 @@ int blastp_search_ungapped_device(const blastp_query_table *q,
                                   void *cuda_stream, blastp_hsp *d_out,
                                   int64_t capacity, int64_t *d_count);
 
+/* APPEND variant for multi-GPU result collection, asynchronous:
+ * as blastp_search_ungapped_device, except that *d_count is NOT reset -- each
+ * HSP takes the next index of the shared counter (device atomics) -- and
+ * d_out / d_count may be another GPU's memory mapped with blastp_ipc_open:
+ * the search kernel then stores its HSPs straight into that GPU's buffer over
+ * NVLink / NVSwitch (no separate gather), each record performed at system
+ * scope (__threadfence_system) before the kernel completes.  Several ranks
+ * append to one buffer; the order is unspecified (sort with
+ * blastp_sort_hsps_device) and a count above capacity means records were
+ * dropped (retry larger).  The caller orders the counter reset before every
+ * rank's append and every rank's completion before reading (stream order
+ * plus a collective, see dist.py PeerHspBuffer).  Errors: as
+ * blastp_search_ungapped_device. */
+int blastp_search_ungapped_append(const blastp_query_table *q, const blastp_db *db,
+                                  const blastp_params *p, void *cuda_stream, blastp_hsp *d_out,
+                                  int64_t capacity, int64_t *d_count);
+
+/* Exported device buffers (CUDA IPC) for blastp_search_ungapped_append.
+ * blastp_ipc_alloc: `bytes` of device memory on `device` (cudaMalloc) and
+ * its IPC handle (BLASTP_IPC_HANDLE_BYTES bytes written to handle_out, to be
+ * sent to the other processes); free with blastp_ipc_free in the allocating
+ * process after every opener closed it.  blastp_ipc_open: maps a handle from
+ * another process into this one's address space for `device` (peer access
+ * enabled on demand); unmap with blastp_ipc_close.  A handle cannot be
+ * opened by the process that allocated it.  Errors: INVALID_ARG, NOMEM,
+ * CUDA. */
+#define BLASTP_IPC_HANDLE_BYTES 64
+int blastp_ipc_alloc(int device, int64_t bytes, void **d_ptr, void *handle_out);
+int blastp_ipc_open(int device, const void *handle, void **d_ptr);
+int blastp_ipc_close(void *d_ptr);
+int blastp_ipc_free(void *d_ptr);
+
 /* The coverage-aware de-duplication of ext_mode HIT_DEDUP (R17), on the
  * device, in place: d_rec[0..n) are seed records {query_id, subject_id,
  * diagonal, q_seed, llen, length, score} of every extension (one per passing

@@ -106,6 +106,12 @@ def _load():
     L.blastp_debug_hits.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
     L.blastp_debug_passing.argtypes = [vp, vp, P(_CParams), vp, vp, i64, P(i64)]
     L.blastp_debug_stats.argtypes = [vp, vp, P(_CParams), vp, vp, i32]
+    if hasattr(L, "blastp_search_ungapped_append"):  # absent in older builds (A/B timing)
+        L.blastp_search_ungapped_append.argtypes = [vp, vp, P(_CParams), vp, vp, i64, vp]
+        L.blastp_ipc_alloc.argtypes = [ctypes.c_int, i64, P(vp), vp]
+        L.blastp_ipc_open.argtypes = [ctypes.c_int, vp, P(vp)]
+        L.blastp_ipc_close.argtypes = [vp]
+        L.blastp_ipc_free.argtypes = [vp]
     if hasattr(L, "blastp_trim_memory"):
         L.blastp_trim_memory.argtypes = [ctypes.c_int]
     if hasattr(L, "blastp_debug_alu_peak"):  # absent in older builds (A/B timing)
@@ -122,7 +128,9 @@ EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "bl
             "blastp_build_query_table", "blastp_build_query_batch", "blastp_pack_db",
             "blastp_shard_range", "blastp_db_info", "blastp_db_long_info", "blastp_query_table_info",
             "blastp_query_table_groups",
-            "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_search_host_db",
+            "blastp_search_ungapped", "blastp_search_ungapped_device", "blastp_search_ungapped_append",
+            "blastp_ipc_alloc", "blastp_ipc_open", "blastp_ipc_close", "blastp_ipc_free",
+            "blastp_search_host_db",
             "blastp_format_host_db", "blastp_search_formatted_db", "blastp_host_db_info",
             "blastp_host_db_free",
             "blastp_sort_hsps_device", "blastp_unique_hsps_device", "blastp_dedup_covered_device",
@@ -322,6 +330,45 @@ def search_ungapped_device(table: QueryTable, db: Database, out_ptr: int, capaci
     _check(lib.blastp_search_ungapped_device(table.handle, db.handle, ctypes.byref(c),
                                              _stream_handle(stream), out_ptr, capacity,
                                              count_ptr), "blastp_search_ungapped_device")
+
+
+def search_ungapped_append(table: QueryTable, db: Database, out_ptr: int, capacity: int,
+                           count_ptr: int, params: Params | None = None, stream=None):
+    """Append variant (async; blastp_search_ungapped_append): the count at
+    count_ptr is not reset, HSPs take the next indices of it; out_ptr /
+    count_ptr may be another GPU's buffer mapped with ipc_open (the kernel
+    stores its HSPs there over NVLink)."""
+    c = (params or table.params).c()
+    _check(lib.blastp_search_ungapped_append(table.handle, db.handle, ctypes.byref(c),
+                                             _stream_handle(stream), out_ptr, capacity,
+                                             count_ptr), "blastp_search_ungapped_append")
+
+
+IPC_HANDLE_BYTES = 64
+
+
+def ipc_alloc(device: int, nbytes: int) -> tuple[int, bytes]:
+    """(device pointer, IPC handle) of a new exported buffer (blastp_ipc_alloc)."""
+    ptr = ctypes.c_void_p()
+    h = ctypes.create_string_buffer(IPC_HANDLE_BYTES)
+    _check(lib.blastp_ipc_alloc(device, nbytes, ctypes.byref(ptr), h), "blastp_ipc_alloc")
+    return int(ptr.value), h.raw
+
+
+def ipc_open(device: int, handle: bytes) -> int:
+    """Map another process's exported buffer (blastp_ipc_open); its pointer."""
+    ptr = ctypes.c_void_p()
+    h = ctypes.create_string_buffer(bytes(handle), IPC_HANDLE_BYTES)
+    _check(lib.blastp_ipc_open(device, h, ctypes.byref(ptr)), "blastp_ipc_open")
+    return int(ptr.value)
+
+
+def ipc_close(ptr: int):
+    _check(lib.blastp_ipc_close(ptr), "blastp_ipc_close")
+
+
+def ipc_free(ptr: int):
+    _check(lib.blastp_ipc_free(ptr), "blastp_ipc_free")
 
 
 def search_host_db(table: QueryTable, residues, offsets: np.ndarray, out_ptr: int, capacity: int,

@@ -788,7 +788,7 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
                           const blastp_params *p, cudaStream_t s, blastp_hsp *out, int64_t cap,
                           unsigned long long *count, TraceRec *const trace[3],
                           const int64_t trace_cap[3], unsigned long long *trace_count,
-                          bool reset_count = true) {
+                          bool reset_count = true, bool out_fence = false) {
   if (reset_count) CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
   if (trace_count)  // [0..3): trace record counts, [3..3+kNumStats): event counters
     CUDA_TRY(cudaMemsetAsync(trace_count, 0, (3 + kNumStats) * sizeof(unsigned long long), s));
@@ -858,6 +858,7 @@ static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
     a.out = out;
     a.out_cap = cap;
     a.hsp_count = count;
+    a.out_fence = out_fence ? 1 : 0;
     a.chunk_cursor = db->counters + 1;
     for (int k = 0; k < 3; ++k) {
       a.trace[k] = trace ? trace[k] : nullptr;
@@ -881,6 +882,79 @@ int blastp_search_ungapped_device(const blastp_query_table *q, const blastp_db *
   DeviceGuard g(db->device);
   return enqueue_search(q, db, p, static_cast<cudaStream_t>(cuda_stream), d_out, capacity,
                         reinterpret_cast<unsigned long long *>(d_count), nullptr, nullptr, nullptr);
+}
+
+int blastp_search_ungapped_append(const blastp_query_table *q, const blastp_db *db,
+                                  const blastp_params *p, void *cuda_stream, blastp_hsp *d_out,
+                                  int64_t capacity, int64_t *d_count) {
+  int rc = check_pair(q, db, p);
+  if (rc) return rc;
+  if (!d_count || capacity < 0 || (capacity > 0 && !d_out))
+    return fail(BLASTP_E_INVALID_ARG, "bad output buffer");
+  DeviceGuard g(db->device);
+  return enqueue_search(q, db, p, static_cast<cudaStream_t>(cuda_stream), d_out, capacity,
+                        reinterpret_cast<unsigned long long *>(d_count), nullptr, nullptr, nullptr,
+                        /*reset_count=*/false, /*out_fence=*/true);
+}
+
+// Exported device buffers (CUDA IPC).  cudaMalloc'd (not from the stream
+// pool: pool memory cannot be exported with cudaIpcGetMemHandle).
+static_assert(sizeof(cudaIpcMemHandle_t) <= BLASTP_IPC_HANDLE_BYTES, "IPC handle size");
+
+int blastp_ipc_alloc(int device, int64_t bytes, void **d_ptr, void *handle_out) {
+  if (!d_ptr || !handle_out || bytes <= 0) return fail(BLASTP_E_INVALID_ARG, "bad arguments");
+  *d_ptr = nullptr;
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess)
+    return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
+  void *ptr = nullptr;
+  if (cudaMalloc(&ptr, size_t(bytes)) != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BLASTP_E_NOMEM, "cudaMalloc(%lld) for an exported buffer failed",
+                static_cast<long long>(bytes));
+  }
+  cudaIpcMemHandle_t h;
+  const cudaError_t e = cudaIpcGetMemHandle(&h, ptr);
+  if (e != cudaSuccess) {
+    cudaFree(ptr);
+    return fail(BLASTP_E_CUDA, "cudaIpcGetMemHandle: %s", cudaGetErrorString(e));
+  }
+  std::memset(handle_out, 0, BLASTP_IPC_HANDLE_BYTES);
+  std::memcpy(handle_out, &h, sizeof(h));
+  *d_ptr = ptr;
+  return BLASTP_OK;
+}
+
+int blastp_ipc_open(int device, const void *handle, void **d_ptr) {
+  if (!d_ptr || !handle) return fail(BLASTP_E_INVALID_ARG, "bad arguments");
+  *d_ptr = nullptr;
+  DeviceGuard g(device);
+  if (g.err != cudaSuccess)
+    return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  void *ptr = nullptr;
+  const cudaError_t e = cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(BLASTP_E_CUDA, "cudaIpcOpenMemHandle: %s", cudaGetErrorString(e));
+  }
+  *d_ptr = ptr;
+  return BLASTP_OK;
+}
+
+int blastp_ipc_close(void *d_ptr) {
+  if (!d_ptr) return BLASTP_OK;
+  const cudaError_t e = cudaIpcCloseMemHandle(d_ptr);
+  if (e != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaIpcCloseMemHandle: %s", cudaGetErrorString(e));
+  return BLASTP_OK;
+}
+
+int blastp_ipc_free(void *d_ptr) {
+  if (!d_ptr) return BLASTP_OK;
+  const cudaError_t e = cudaFree(d_ptr);
+  if (e != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaFree: %s", cudaGetErrorString(e));
+  return BLASTP_OK;
 }
 
 // Stream-ordered release of a database (its buffers come from the pool):

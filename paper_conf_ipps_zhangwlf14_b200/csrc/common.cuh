@@ -130,6 +130,7 @@ struct SearchArgs {
   unsigned long long *trace_count;   // [3]
   unsigned long long *stats;         // [kNumStats] event counters (trace runs only)
   int32_t emit_seed;                 // ext_mode HIT_DEDUP: every extension as a seed record
+  int32_t out_fence;                 // blastp_search_ungapped_append: out may be peer memory
   const int8_t *pssm;                // block kernel, BLASTP_SCORE=pssm_global: the PSSM
 };
 

@@ -381,7 +381,6 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
   const int L = W - 1;  // record lag: lanes v < L are tested against the previous block
   const int A = kDef ? 40 : a.window;
   const unsigned ltmask = lanemask_lt(lane);
-  const unsigned lemask = kFull >> (31 - lane);  // lanes <= lane
   uint32_t *scr = w.scr();
 
   BlkState st;
@@ -522,15 +521,15 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
           const bool wr = cnt != 0u && excl < kb + 32u && incl > kb;
           const int p0 = wr ? max(int(excl) - int(kb), 0) : 0;
           // (table offset - excl) << 5 | lane: the offset difference is
-          // signed and fits 27 bits (tables < 2^26 entries)
+          // taken mod 2^27 (tables < 2^27 entries)
           if (wr) scr[p0] = uint32_t(lane) | ((o - excl) << 5);
           const unsigned S = __reduce_or_sync(kFull, wr ? (1u << p0) : 0u);
           __syncwarp();
-          const int src = 31 - __clz(S & lemask);
-          const int vv = int(scr[src]);
-          own_out = vv & 31;
+          const int src = 31 - __clz(S & (kFull >> (31 - lane)));
+          const uint32_t vv = scr[src];
+          own_out = int(vv & 31u);
           const uint32_t k = kb + uint32_t(lane);
-          q_out = k < lim ? int(__ldg(qpos + ((vv >> 5) + int(k)))) : 0;
+          q_out = k < lim ? int(__ldg(qpos + (((vv >> 5) + k) & 0x7ffffffu))) : 0;
           __syncwarp();
         };
         // hits of lanes v < L (tested against the previous block's state)
@@ -739,7 +738,8 @@ bool block_kernel_eligible(const SearchArgs &a) {
   return a.filter_mode == BLASTP_FILTER_LEFT &&
          (a.ext_mode == BLASTP_EXT_DIAGONAL || a.ext_mode == BLASTP_EXT_HIT) &&
          a.min_gap >= 1 && a.min_gap <= 8 && a.window >= 31 + a.min_gap && a.window <= 256 &&
-         a.qv.lq <= 16000 && a.qv.wtab != nullptr;
+         a.qv.lq <= 16000 && a.qv.wtab != nullptr &&
+         a.table_entries < (int64_t(1) << 27);  // the owner lookup's 27-bit offsets
 }
 
 cudaError_t launch_search_block(const SearchArgs &a_in, int num_sms, cudaStream_t s) {

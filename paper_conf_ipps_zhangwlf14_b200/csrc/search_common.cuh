@@ -241,6 +241,9 @@ __device__ __forceinline__ bool emit_hsp(const SearchArgs &a, int64_t sp, int q,
   }
   const unsigned long long idx = atomicAdd(a.hsp_count, 1ull);
   if ((long long)idx < a.out_cap) a.out[idx] = h;
+  // a record stored into another GPU's memory over NVLink is performed at
+  // system scope before the kernel can complete (blastp_search_ungapped_append)
+  if (a.out_fence) __threadfence_system();
   return true;
 }
 

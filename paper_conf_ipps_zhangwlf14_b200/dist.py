@@ -10,6 +10,13 @@ is canonical (R11), the concatenation is already canonical for one query;
 for query batches rank 0 re-sorts (query_id major) on the GPU.
 
 The collective code is backend-agnostic (NCCL on GPUs, gloo in the CPU tests).
+
+PeerHspBuffer fuses the gather into the search instead: rank dst exports one
+HSP buffer (CUDA IPC), every rank maps it, and every rank's search kernel
+appends its HSPs straight into it over NVLink / NVSwitch
+(blastp_search_ungapped_append) -- no gather step, the transfer overlaps the
+search record by record; two tiny collectives order the count reset before
+and every rank's kernel completion after.
 """
 from __future__ import annotations
 
@@ -137,3 +144,134 @@ def gpu_shard_search(table, residues_local: np.ndarray, offsets_full: np.ndarray
             return res
         finally:
             db.free()
+
+
+class _DevMem:
+    """A raw device range as a torch tensor (zero-copy, __cuda_array_interface__)."""
+
+    def __init__(self, ptr: int, shape: tuple, typestr: str):
+        self.__cuda_array_interface__ = {"shape": shape, "typestr": typestr, "data": (ptr, False),
+                                         "strides": None, "version": 2}
+
+
+class PeerHspBuffer:
+    """One HSP buffer in rank `dst`'s device memory that the search kernels of
+    every rank write into directly (blastp_search_ungapped_append over a CUDA
+    IPC mapping: NVLink / NVSwitch stores between GPUs; ranks sharing one
+    device, as in the 1-GPU tests, map it on that device).
+
+    Layout: the int64 count at offset 0, `capacity` blastp_hsp records from
+    offset HEADER.  search() returns the canonical [n, 7] int32 list on rank
+    dst (a view of the buffer, valid until the next search) and None on the
+    other ranks; a count above capacity re-runs the search with a buffer
+    grown to fit (every rank reads the shared count, so all agree).
+    """
+
+    HEADER = 256
+
+    def __init__(self, capacity: int, group=None, dst: int = 0):
+        import torch
+        import torch.distributed as dist
+
+        from . import blastp as bp
+        self._bp = bp
+        self.group = group
+        self.dst = dst
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        self.nccl = dist.get_backend(group) == "nccl"
+        self.device = torch.cuda.current_device()
+        self.ptr = 0
+        self.capacity = 0
+        self._alloc(max(1, int(capacity)))
+
+    def _glob(self, r: int) -> int:
+        import torch.distributed as dist
+        return r if self.group is None else dist.get_global_rank(self.group, r)
+
+    def _alloc(self, capacity: int):
+        import torch
+        import torch.distributed as dist
+        bp = self._bp
+        nbytes = self.HEADER + capacity * bp.HSP_BYTES
+        h = bytes(bp.IPC_HANDLE_BYTES)
+        if self.rank == self.dst:
+            self.ptr, h = bp.ipc_alloc(self.device, nbytes)
+        ht = torch.frombuffer(bytearray(h), dtype=torch.uint8)
+        if self.nccl:
+            ht = ht.cuda()
+        dist.broadcast(ht, src=self._glob(self.dst), group=self.group)
+        if self.rank != self.dst:
+            self.ptr = bp.ipc_open(self.device, bytes(ht.cpu().numpy()))
+        self.capacity = capacity
+        self.count = torch.as_tensor(_DevMem(self.ptr, (1,), "<i8"), device="cuda")
+        self.out = torch.as_tensor(_DevMem(self.ptr + self.HEADER, (capacity, HSP_FIELDS), "<i4"),
+                                   device="cuda")
+
+    def _sync(self):
+        """Every rank's preceding work on its current stream is complete
+        before any rank's following work: a stream-ordered all_reduce under
+        NCCL; a host synchronisation + barrier under gloo."""
+        import torch
+        import torch.distributed as dist
+        if self.nccl:
+            dist.all_reduce(torch.ones(1, device="cuda"), group=self.group)
+        else:
+            torch.cuda.synchronize()
+            dist.barrier(group=self.group)
+
+    def free(self):
+        import torch.distributed as dist
+        if not self.ptr:
+            return
+        self.count = self.out = None
+        self._sync()  # nobody still writes or reads
+        if self.rank != self.dst:
+            self._bp.ipc_close(self.ptr)
+        dist.barrier(group=self.group)  # every mapping closed before the free
+        if self.rank == self.dst:
+            self._bp.ipc_free(self.ptr)
+        self.ptr = 0
+
+    def search(self, table, db, params=None, canonical: bool = True, events=None):
+        """This rank's shard `db` searched into the shared buffer.  canonical:
+        rank dst sorts the list (R11; HIT_DEDUP: de-duplicates it), else it is
+        returned in append order.  events: optional (start, end) CUDA events
+        recorded around this rank's search launch (kernel timing)."""
+        bp = self._bp
+        while True:
+            if self.rank == self.dst:
+                self.count.zero_()
+            self._sync()  # the reset precedes every append
+            if events:
+                events[0].record()
+            bp.search_ungapped_append(table, db, self.out.data_ptr(), self.capacity,
+                                      self.count.data_ptr(), params)
+            if events:
+                events[1].record()
+            self._sync()  # every rank's kernel (and its NVLink stores) completed
+            n = int(self.count.item())
+            if n <= self.capacity:
+                break
+            self._sync()  # every rank read the count before the buffer goes
+            old = self.ptr
+            self.count = self.out = None
+            if self.rank != self.dst:
+                bp.ipc_close(old)
+            self._sync()
+            if self.rank == self.dst:
+                bp.ipc_free(old)
+            self._alloc(n + n // 4 + 1024)
+        if self.rank != self.dst:
+            return None
+        res = self.out[:n]
+        if not canonical:
+            return res
+        p = params or table.params
+        if p.ext_mode == bp.EXT_HIT_DEDUP:
+            import torch
+            kept = torch.zeros(1, dtype=torch.int64, device="cuda")
+            bp.dedup_covered_device(res.data_ptr(), n, p.cutoff, kept.data_ptr())
+            return res[: int(kept.item())]
+        bp.sort_hsps_device(res.data_ptr(), n)
+        return res
