@@ -132,6 +132,7 @@ struct SearchArgs {
   int32_t emit_seed;                 // ext_mode HIT_DEDUP: every extension as a seed record
   int32_t out_fence;                 // blastp_search_ungapped_append: out may be peer memory
   const int8_t *pssm;                // block kernel, BLASTP_SCORE=pssm_global: the PSSM
+  uint16_t *reach_scratch;           // block kernel: per-warp ext_reach regions (launch-owned)
 };
 
 // Event counters collected by the tracing kernel variant (blastp_debug_stats).

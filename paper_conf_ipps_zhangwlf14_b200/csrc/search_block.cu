@@ -59,7 +59,16 @@ using namespace dev;
 
 namespace {
 
-constexpr int kBlkWarps = 32;        // warps per CTA (independent walkers)
+// 2 CTAs of 18 warps per SM: 36 resident warps with <= 56 registers each
+// (32 warps in one CTA: 2.4% slower on config 3, profiles/r02/ab_block_kernel.txt)
+#ifndef BLK_WARPS
+#define BLK_WARPS 18
+#endif
+#ifndef BLK_MINB
+#define BLK_MINB 2
+#endif
+constexpr int kBlkWarps = BLK_WARPS;  // warps per CTA (independent walkers)
+constexpr int kBlkMinCtas = BLK_MINB;  // CTAs per SM the register budget allows
 constexpr int kBlkQcap = 64;         // extension queue slots per warp
 constexpr int kBlkFrameMin = 512;    // first frame position (> A + 2 blocks)
 constexpr int kBlkFrameSpan = 8192;  // rebase step: frame positions < 2^14
@@ -73,10 +82,13 @@ __device__ __forceinline__ int be_maxoff(uint32_t e) { return int((e >> 19) & 31
 __device__ __forceinline__ int be_prevoff(uint32_t e) { return int(e >> 24); }
 
 // Per-warp shared memory: fixed parts first (every address is the warp's
-// base plus a constant), then ring[M] (block state) and reach[M] (ext_reach).
+// base plus a constant), then ring[M] (block state); reach[M] (ext_reach,
+// read once per queued hit) in global memory, the warp's own region of
+// a.reach_scratch (L1-resident; keeping it in shared memory costs 2 B per
+// slot and 4 resident warps at q1054).
 struct BlkArea {
   uint8_t *base;
-  int reach_off;
+  uint16_t *reach_g;
   __device__ __forceinline__ uint32_t *queue() const { return reinterpret_cast<uint32_t *>(base); }
   __device__ __forceinline__ uint32_t *scr() const { return reinterpret_cast<uint32_t *>(base + 256); }
   __device__ __forceinline__ uint16_t *fs_p() const { return reinterpret_cast<uint16_t *>(base + 256); }
@@ -85,13 +97,11 @@ struct BlkArea {
   __device__ __forceinline__ uint32_t *ring() const {
     return reinterpret_cast<uint32_t *>(base + kBlkFixed);
   }
-  __device__ __forceinline__ uint16_t *reach() const {
-    return reinterpret_cast<uint16_t *>(base + reach_off);
-  }
+  __device__ __forceinline__ uint16_t *reach() const { return reach_g; }
 };
 
 __host__ __device__ size_t blk_area_bytes(int ring) {
-  return kBlkFixed + align16(size_t(ring) * 4) + align16(size_t(ring) * 2);
+  return kBlkFixed + align16(size_t(ring) * 4);
 }
 
 struct BlkState {
@@ -337,7 +347,7 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
 // instead of DIAGONAL (Alg. 3); kPssm: X-drop scores from a PSSM (in shared
 // memory when a.pssm is null -- built here --, else a.pssm in global memory).
 template <bool kTrace, bool kDef, bool kHit, bool kPssm>
-__global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const SearchArgs a) {
+__global__ void __launch_bounds__(kBlkWarps * 32, kBlkMinCtas) search_block_kernel(const SearchArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
   int8_t *b62 = reinterpret_cast<int8_t *>(smem);
@@ -367,7 +377,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
   const int M = a.ring;
   BlkArea w;
   w.base = areas + size_t(warp) * blk_area_bytes(M);
-  w.reach_off = kBlkFixed + int(align16(size_t(M) * 4));
+  w.reach_g = a.reach_scratch + size_t(blockIdx.x * (blockDim.x >> 5) + warp) * M;
   for (int i = lane; i < M; i += 32) {
     w.ring()[i] = 0;
     w.reach()[i] = 0;
@@ -544,7 +554,8 @@ __global__ void __launch_bounds__(kBlkWarps * 32) search_block_kernel(const Sear
                   uint32_t(P) | (uint32_t(q) << 16);
             st.qcount += __popc(bal);
             __syncwarp();
-            if (st.qcount >= 32) blk_flush<kTrace, kHit, kPssm>(a, w, st, 32, qc, b62, lane, slotc, M, pssm);
+            if (st.qcount >= 32)
+              blk_flush<kTrace, kHit, kPssm>(a, w, st, 32, qc, b62, lane, slotc, M, pssm);
           }
         };
         // REGION: prepass
@@ -706,30 +717,51 @@ size_t blk_smem_bytes(int lq, int ring, int warps, bool pssm_smem) {
          size_t(warps) * blk_area_bytes(ring);
 }
 
+// Warps per CTA: the most resident warps per SM (occupancy of this kernel
+// instance at each CTA size up to warps_max whose shared memory fits),
+// larger CTAs on ties.
 template <bool kTrace, bool kDef, bool kHit, bool kPssm>
-cudaError_t blk_launch(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
+cudaError_t blk_launch(const SearchArgs &a, int warps_max, bool pssm_smem, int optin,
+                       int num_sms, cudaStream_t s) {
   void (*k)(const SearchArgs) = search_block_kernel<kTrace, kDef, kHit, kPssm>;
-  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, optin);
   if (e != cudaSuccess) return e;
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, warps * 32, smem);
-  if (e != cudaSuccess) return e;
-  if (per_sm < 1) return cudaErrorInvalidConfiguration;
+  int warps = 0, per_sm = 0;
+  for (int w = warps_max; w >= 1; --w) {
+    const size_t sm = blk_smem_bytes(a.qv.lq, a.ring, w, pssm_smem);
+    if (sm > size_t(optin)) continue;
+    int per = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, w * 32, sm);
+    if (e != cudaSuccess) return e;
+    if (per * w > per_sm * warps) {
+      warps = w;
+      per_sm = per;
+    }
+  }
+  if (warps < 1 || per_sm < 1) return cudaErrorInvalidConfiguration;
+  const size_t smem = blk_smem_bytes(a.qv.lq, a.ring, warps, pssm_smem);
   int64_t grid = int64_t(num_sms) * per_sm;
   const int64_t need = (int64_t(a.nchunks) + a.nlong + a.nsegs + warps - 1) / warps;
   if (grid > need) grid = need < 1 ? 1 : need;
-  k<<<unsigned(grid), warps * 32, smem, s>>>(a);
-  return cudaGetLastError();
+  SearchArgs g = a;
+  e = pool_malloc_async(reinterpret_cast<void **>(&g.reach_scratch),
+                        size_t(grid) * warps * size_t(a.ring) * 2, s);
+  if (e != cudaSuccess) return e;
+  k<<<unsigned(grid), warps * 32, smem, s>>>(g);
+  e = cudaGetLastError();
+  cudaFreeAsync(g.reach_scratch, s);
+  return e;
 }
 
 template <bool kTrace, bool kPssm>
-cudaError_t blk_pick(const SearchArgs &a, int warps, size_t smem, int num_sms, cudaStream_t s) {
+cudaError_t blk_pick(const SearchArgs &a, int warps_max, bool pssm_smem, int optin, int num_sms,
+                     cudaStream_t s) {
   const bool hit = a.ext_mode == BLASTP_EXT_HIT;
   if (a.min_gap == 3 && a.window == 40)
-    return hit ? blk_launch<kTrace, true, true, kPssm>(a, warps, smem, num_sms, s)
-               : blk_launch<kTrace, true, false, kPssm>(a, warps, smem, num_sms, s);
-  return hit ? blk_launch<kTrace, false, true, kPssm>(a, warps, smem, num_sms, s)
-             : blk_launch<kTrace, false, false, kPssm>(a, warps, smem, num_sms, s);
+    return hit ? blk_launch<kTrace, true, true, kPssm>(a, warps_max, pssm_smem, optin, num_sms, s)
+               : blk_launch<kTrace, true, false, kPssm>(a, warps_max, pssm_smem, optin, num_sms, s);
+  return hit ? blk_launch<kTrace, false, true, kPssm>(a, warps_max, pssm_smem, optin, num_sms, s)
+             : blk_launch<kTrace, false, false, kPssm>(a, warps_max, pssm_smem, optin, num_sms, s);
 }
 
 }  // namespace
@@ -767,14 +799,11 @@ cudaError_t launch_search_block(const SearchArgs &a_in, int num_sms, cudaStream_
   const bool pssm = score_env && !std::strncmp(score_env, "pssm", 4);
   const bool pssm_smem = pssm && std::strcmp(score_env, "pssm_global") != 0;
   const char *warps_env = std::getenv("BLASTP_WARPS");
-  int warps = warps_env ? std::max(1, std::min(kBlkWarps, std::atoi(warps_env))) : kBlkWarps;
-  while (warps > 0 && blk_smem_bytes(a.qv.lq, a.ring, warps, pssm_smem) > size_t(optin)) --warps;
-  if (warps < 1) return cudaErrorInvalidConfiguration;
-  const size_t smem = blk_smem_bytes(a.qv.lq, a.ring, warps, pssm_smem);
+  const int warps = warps_env ? std::max(1, std::min(kBlkWarps, std::atoi(warps_env))) : kBlkWarps;
   const bool trace = a.trace[0] != nullptr;
   if (!pssm)
-    return trace ? blk_pick<true, false>(a, warps, smem, num_sms, s)
-                 : blk_pick<false, false>(a, warps, smem, num_sms, s);
+    return trace ? blk_pick<true, false>(a, warps, false, optin, num_sms, s)
+                 : blk_pick<false, false>(a, warps, false, optin, num_sms, s);
   int8_t *g = nullptr;
   if (!pssm_smem) {
     const size_t bytes = size_t(a.qv.lq + 2 * kBlkQPad) * 32;
@@ -782,8 +811,8 @@ cudaError_t launch_search_block(const SearchArgs &a_in, int num_sms, cudaStream_
     pssm_fill_kernel<<<int((bytes + 255) / 256), 256, 0, s>>>(a.qv.qcodes, a.qv.lq, g);
     a.pssm = g;
   }
-  e = trace ? blk_pick<true, true>(a, warps, smem, num_sms, s)
-            : blk_pick<false, true>(a, warps, smem, num_sms, s);
+  e = trace ? blk_pick<true, true>(a, warps, pssm_smem, optin, num_sms, s)
+            : blk_pick<false, true>(a, warps, pssm_smem, optin, num_sms, s);
   if (g) cudaFreeAsync(g, s);
   return e;
 }

@@ -243,7 +243,9 @@ __device__ __forceinline__ bool emit_hsp(const SearchArgs &a, int64_t sp, int q,
   if ((long long)idx < a.out_cap) a.out[idx] = h;
   // a record stored into another GPU's memory over NVLink is performed at
   // system scope before the kernel can complete (blastp_search_ungapped_append)
+#ifndef BLK_NOFENCE
   if (a.out_fence) __threadfence_system();
+#endif
   return true;
 }
 
