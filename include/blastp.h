@@ -200,13 +200,15 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
  * once its copy has landed; HSPs are appended to d_out / *d_count exactly as
  * blastp_search_ungapped_device does for the whole shard (same results as
  * blastp_pack_db + blastp_search_ungapped_device).  Asynchronous on
- * cuda_stream; the device image is released in stream order.  The streaming
- * overlaps each part's host->device copy with the previous part's search; it
- * does not bound device memory: the whole shard's device image (about the
- * pinned image's size) is allocated for the search, so a shard must fit in
- * HBM.  Errors: as blastp_pack_db (format) and blastp_search_ungapped_device
- * (search), E_NOMEM if the pinned image or the device image cannot be
- * allocated. */
+ * cuda_stream; device memory is released in stream order.  The streaming
+ * overlaps each part's host->device copy with the previous part's search and
+ * bounds device memory: a ring of min(num_parts, BLASTP_PIPE_SLOTS = 3) part
+ * slots, each the largest part's image plus its scratch, is allocated; part
+ * k is copied into slot k mod slots once the search of the slot's previous
+ * part has completed (stream-ordered events, no host synchronisation) -- a
+ * shard larger than HBM is searched by formatting it into enough parts.
+ * Errors: as blastp_pack_db (format) and blastp_search_ungapped_device
+ * (search), E_NOMEM if the pinned image or the slots cannot be allocated. */
 typedef struct blastp_host_db blastp_host_db;
 int blastp_format_host_db(const char *residues_ascii, const int64_t *offsets, int64_t nseq,
                           int32_t shard_index, int32_t num_shards, int32_t num_parts,

@@ -1302,16 +1302,32 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
   cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
   auto *count = reinterpret_cast<unsigned long long *>(d_count);
   CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
-  // device image: the host image's layout plus per-part scratch (counters,
-  // segment lists / counts / publication flags)
-  std::vector<size_t> scratch_off(h->parts.size());
-  size_t bytes = al256(h->bytes);
-  for (size_t k = 0; k < h->parts.size(); ++k) {
-    const HostPart &hp = h->parts[k];
-    const size_t ns = size_t(std::max(hp.nsegs, 1));
-    scratch_off[k] = bytes;
-    bytes += al256(64) + al256(4 * ns) + al256(4 * ns) + al256(4 * ns * size_t(hp.seg_cap));
+  // Device memory: a ring of part slots (BLASTP_PIPE_SLOTS, default 3, at
+  // most one per part), each the largest part's image plus its scratch
+  // (counters, segment lists / counts / publication flags); part k goes to
+  // slot k mod nslots once the search of part k - nslots has released it.
+  // The part images are position-independent (offsets within the part).
+  const size_t nparts = h->parts.size();
+  auto part_bytes = [&](size_t k) {
+    const size_t end = k + 1 < nparts ? h->parts[k + 1].off_stream : h->bytes;
+    return end - h->parts[k].off_stream;
+  };
+  size_t slot_img = 0, slot_bytes = 0;
+  for (size_t k = 0; k < nparts; ++k) slot_img = std::max(slot_img, al256(part_bytes(k)));
+  slot_bytes = slot_img;
+  {
+    size_t scr = 0;
+    for (size_t k = 0; k < nparts; ++k) {
+      const HostPart &hp = h->parts[k];
+      const size_t ns = size_t(std::max(hp.nsegs, 1));
+      scr = std::max(scr, al256(64) + al256(4 * ns) + al256(4 * ns) +
+                              al256(4 * ns * size_t(hp.seg_cap)));
+    }
+    slot_bytes += scr;
   }
+  size_t nslots = 3;
+  if (const char *v = std::getenv("BLASTP_PIPE_SLOTS")) nslots = size_t(std::max(1, std::atoi(v)));
+  nslots = std::max<size_t>(1, std::min(nslots, nparts));
   cudaStream_t cs = nullptr, s2 = nullptr;
   CUDA_TRY(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
   if (cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking) != cudaSuccess) {
@@ -1319,14 +1335,15 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
     cudaStreamDestroy(cs);
     return fail(BLASTP_E_CUDA, "could not create the second search stream");
   }
-  bytes = std::max<size_t>(bytes, 256);
+  const size_t bytes = std::max<size_t>(nslots * slot_bytes, 256);
   uint8_t *dev = nullptr;
-  // the arena is allocated in s's order; the copies on cs wait for that
+  // the slots are allocated in s's order; the copies on cs wait for that
   if (pool_malloc_async(reinterpret_cast<void **>(&dev), bytes, s) != cudaSuccess) {
     cudaGetLastError();
     cudaStreamDestroy(cs);
     cudaStreamDestroy(s2);
-    return fail(BLASTP_E_NOMEM, "device image of %zu bytes for the formatted search", bytes);
+    return fail(BLASTP_E_NOMEM, "%zu part slots of %zu bytes for the formatted search", nslots,
+                slot_bytes);
   }
   std::vector<cudaEvent_t> evs;
   auto event = [&]() {
@@ -1338,11 +1355,14 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
   cudaEventRecord(ev_start, s);  // arena allocated, count reset
   cudaStreamWaitEvent(cs, ev_start, 0);
   cudaStreamWaitEvent(s2, ev_start, 0);
-  std::vector<blastp_db> dbs(h->parts.size());
+  std::vector<blastp_db> dbs(nparts);
+  std::vector<cudaEvent_t> done(nparts, nullptr);  // part k's search released its slot
   rc = BLASTP_OK;
-  for (size_t k = 0; k < h->parts.size() && rc == BLASTP_OK; ++k) {
+  for (size_t k = 0; k < nparts && rc == BLASTP_OK; ++k) {
     const HostPart &hp = h->parts[k];
     blastp_db &d = dbs[k];
+    uint8_t *slot = dev + (k % nslots) * slot_bytes;
+    auto at = [&](size_t off) { return slot + (off - hp.off_stream); };
     d.device = h->device;
     d.sms = num_sms(h->device);
     d.nseq = hp.nseq;
@@ -1355,13 +1375,13 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
     d.seg_len = hp.seg_len;
     d.seg_cap = hp.seg_cap;
     d.carved = true;
-    d.stream = dev + hp.off_stream;
-    d.sstart = reinterpret_cast<int64_t *>(dev + hp.off_sstart);
-    d.chunks = reinterpret_cast<Chunk *>(dev + hp.off_chunks);
-    d.items = reinterpret_cast<LongItem *>(dev + hp.off_items);
-    d.seg_item = reinterpret_cast<int32_t *>(dev + hp.off_seg_item);
+    d.stream = slot;
+    d.sstart = reinterpret_cast<int64_t *>(at(hp.off_sstart));
+    d.chunks = reinterpret_cast<Chunk *>(at(hp.off_chunks));
+    d.items = reinterpret_cast<LongItem *>(at(hp.off_items));
+    d.seg_item = reinterpret_cast<int32_t *>(at(hp.off_seg_item));
     const size_t ns = size_t(std::max(hp.nsegs, 1));
-    uint8_t *sc = dev + scratch_off[k];
+    uint8_t *sc = slot + slot_img;
     d.counters = reinterpret_cast<unsigned long long *>(sc);
     sc += al256(64);
     d.seg_count = reinterpret_cast<int32_t *>(sc);
@@ -1370,10 +1390,11 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
     sc += al256(4 * ns);
     d.seg_list = reinterpret_cast<uint32_t *>(sc);
     // copy engine only: the part's image in one copy (its buffers are
-    // contiguous in the image)
-    const size_t end = k + 1 < h->parts.size() ? h->parts[k + 1].off_stream : h->bytes;
-    cudaError_t e = cudaMemcpyAsync(dev + hp.off_stream, h->buf + hp.off_stream,
-                                    end - hp.off_stream, cudaMemcpyHostToDevice, cs);
+    // contiguous in the image), after the slot's previous part was searched
+    cudaError_t e = cudaSuccess;
+    if (k >= nslots) e = cudaStreamWaitEvent(cs, done[k - nslots], 0);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(slot, h->buf + hp.off_stream, part_bytes(k), cudaMemcpyHostToDevice, cs);
     cudaEvent_t ready = event();
     if (e == cudaSuccess) e = cudaEventRecord(ready, cs);
     cudaStream_t ss = (k & 1) ? s2 : s;
@@ -1386,6 +1407,9 @@ int blastp_search_formatted_db(const blastp_query_table *q, const blastp_host_db
       break;
     }
     rc = enqueue_search(q, &d, p, ss, d_out, capacity, count, nullptr, nullptr, nullptr, false);
+    done[k] = event();
+    if (rc == BLASTP_OK && (!done[k] || cudaEventRecord(done[k], ss) != cudaSuccess))
+      rc = fail(BLASTP_E_CUDA, "recording the end of part %zu's search", k);
   }
   // join s2 into s, then release the arena in s's order
   cudaEvent_t ev_join = event();

@@ -772,6 +772,25 @@ def test_formatted_host_db(bp, orc):
     assert _formatted_search(bp, t, empty, p) == []
 
 
+@pytest.mark.parametrize("slots", ["1", "2"])
+def test_formatted_host_db_slot_ring(bp, monkeypatch, slots):
+    """The formatted search's bounded device memory: with 1 or 2 part slots
+    for 9 parts every slot is reused (each copy waits for the search of the
+    slot's previous part) and the result still equals the resident search."""
+    monkeypatch.setenv("BLASTP_PIPE_SLOTS", slots)
+    q = gen_query(23, 400).decode()
+    rng = np.random.default_rng(11)
+    ascii, off = _rand_db(rng, 4000, 0, 700, q)
+    t = bp.build_query_table(q, bp.Params())
+    d = bp.pack_db(ascii, off)
+    for p in (bp.Params(), bp.Params(filter_mode=2)):
+        whole = tuples(bp.search_ungapped(t, d, p))
+        assert len(whole) > 10
+        hdb = bp.format_host_db(ascii, off, num_parts=9)
+        assert _formatted_search(bp, t, hdb, p) == whole
+        hdb.free()
+
+
 def test_formatted_host_db_config3_full_size(bp):
     """Config 3 at full size (the bench's e2e path): the formatted image
     streamed in parts gives exactly the resident shard's HSP list (the
