@@ -69,6 +69,9 @@ def main(argv: list[str] | None = None) -> int:
     ap.add_argument("--distributed", action="store_true",
                     help="one process per GPU under torchrun: each rank searches a residue-"
                          "balanced subject range, HSPs gathered to rank 0 (dist.py), which prints")
+    ap.add_argument("--gather", choices=["p2p", "nccl"], default="p2p",
+                    help="--distributed: the search kernels append into rank 0's buffer over "
+                         "NVLink (CUDA IPC), or per-rank lists gathered with NCCL")
     args = ap.parse_args(argv)
 
     import os
@@ -121,12 +124,15 @@ def main(argv: list[str] | None = None) -> int:
         # an error on one rank (e.g. a bad residue in its shard only) is agreed
         # on by all ranks before the gather, so none waits forever in it
         err = None
+        d = None
         local = torch.zeros((0, 7), dtype=torch.int32, device="cuda")
         try:
             d = bp.pack_db(residues, soff, rank, world, device=args.device)
-            local = torch.from_numpy(bp.search_ungapped(table, d, p).view(np.int32)
-                                     .reshape(-1, 7).copy()).cuda()
-            d.free()
+            if args.gather == "nccl":
+                local = torch.from_numpy(bp.search_ungapped(table, d, p).view(np.int32)
+                                         .reshape(-1, 7).copy()).cuda()
+                d.free()
+                d = None
         except bp.BlastpError as ex:
             err = ex
         flag = torch.tensor([1 if err else 0], dtype=torch.int32,
@@ -137,14 +143,26 @@ def main(argv: list[str] | None = None) -> int:
             if err:
                 print(f"rank {rank}: {err}", file=sys.stderr)
             return 1
-        allh = gather_hsps(local)
-        dist.destroy_process_group()
-        if rank != 0:
-            return 0
-        n = allh.shape[0]
-        flat = allh.contiguous().view(-1)
-        bp.sort_hsps_device(flat.data_ptr(), n)
-        hsps = flat.view(n, 7).cpu().numpy()
+        if args.gather == "p2p":
+            # every rank's search kernel stores its HSPs into rank 0's buffer
+            from .dist import PeerHspBuffer
+            buf = PeerHspBuffer(max(1 << 16, len(residues) // 1000 * len(queries)))
+            res = buf.search(table, d, p)  # canonical on rank 0
+            hsps = None if res is None else res.cpu().numpy()
+            buf.free()
+            d.free()
+            dist.destroy_process_group()
+            if rank != 0:
+                return 0
+        else:
+            allh = gather_hsps(local)
+            dist.destroy_process_group()
+            if rank != 0:
+                return 0
+            n = allh.shape[0]
+            flat = allh.contiguous().view(-1)
+            bp.sort_hsps_device(flat.data_ptr(), n)
+            hsps = flat.view(n, 7).cpu().numpy()
     elif args.stream:
         h = bp.format_host_db(residues, soff, device=args.device)
         cap = max(1 << 16, len(residues) // 1000 * len(queries))  # grown below if short

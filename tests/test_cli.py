@@ -61,7 +61,8 @@ def test_cli_matches_oracle(tmp_path, capsys, orc):
 
 
 @pytest.mark.gpu
-def test_cli_distributed_two_ranks(tmp_path):
+@pytest.mark.parametrize("gather,port", [("p2p", 29561), ("nccl", 29562)])
+def test_cli_distributed_two_ranks(tmp_path, gather, port):
     """--distributed under torchrun (2 ranks sharing the one GPU through the
     gloo backend): rank 0 prints exactly the single-process table."""
     import subprocess
@@ -85,8 +86,8 @@ def test_cli_distributed_two_ranks(tmp_path):
     assert one.returncode == 0, one.stderr
     two = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
                           "--nproc-per-node", "2", "--master-addr", "127.0.0.1",
-                          "--master-port", "29561", "-m", "paper_conf_ipps_zhangwlf14_b200.cli",
-                          *args, "--distributed"],
+                          "--master-port", str(port), "-m", "paper_conf_ipps_zhangwlf14_b200.cli",
+                          *args, "--distributed", "--gather", gather],
                          capture_output=True, text=True, env=env, cwd=root, timeout=300)
     assert two.returncode == 0, two.stderr[-2000:]
     assert one.stdout.count("\n") > 20

@@ -24,7 +24,8 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, queries, ascii, offsets, result_path, cap, ext_mode, repeats):
+def _worker(rank, world, port, queries, ascii, offsets, result_path, cap, ext_mode, repeats,
+            filter_mode=0):
     sys.path.insert(0, ROOT)
     import torch
     import torch.distributed as dist
@@ -36,7 +37,7 @@ def _worker(rank, world, port, queries, ascii, offsets, result_path, cap, ext_mo
     dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank,
                             world_size=world)
     try:
-        p = bp.Params(ext_mode=ext_mode)
+        p = bp.Params(ext_mode=ext_mode, filter_mode=filter_mode)
         table = bp.build_query_batch(queries, p)
         db = bp.pack_db(ascii, offsets, rank, world)
         buf = PeerHspBuffer(cap)
@@ -59,10 +60,11 @@ def _worker(rank, world, port, queries, ascii, offsets, result_path, cap, ext_mo
         dist.destroy_process_group()
 
 
-def _oracle_hsps(orc, queries, db):
+def _oracle_hsps(orc, queries, db, filter_mode=0):
     parts = []
     for qi, q in enumerate(queries):
-        r = orc.search(orc.encode(q), orc.encode(db.ascii.tobytes()), db.offsets)
+        r = orc.search(orc.encode(q), orc.encode(db.ascii.tobytes()), db.offsets,
+                       orc.Params(filter_mode=filter_mode))
         h = r.hsps.view(np.int32).reshape(-1, 7).copy()
         h[:, 0] = qi
         parts.append(h)
@@ -70,20 +72,45 @@ def _oracle_hsps(orc, queries, db):
     return allh[np.lexsort(allh.T[::-1])]
 
 
-@pytest.mark.parametrize("world,cap,ext", [(2, 1 << 16, "diagonal"), (3, 7, "diagonal"),
-                                            (2, 1 << 16, "hit_dedup")])
-def test_peer_append_equals_oracle(orc, tmp_path, world, cap, ext):
+@pytest.mark.parametrize("world,cap,ext,filt", [(2, 1 << 16, "diagonal", 0),
+                                                 (3, 7, "diagonal", 0),
+                                                 (2, 1 << 16, "hit_dedup", 0),
+                                                 (3, 1 << 16, "diagonal", 2),
+                                                 (2, 100, "diagonal", 3)])
+def test_peer_append_equals_oracle(orc, tmp_path, world, cap, ext, filt):
+    """filt: 0 LEFT (block kernel), 2 STATEFUL / 3 STATEFUL_RB (warp kernel)."""
     from paper_conf_ipps_zhangwlf14_b200 import blastp as bp
     from synth import config_workload
     (q,), db = config_workload(1)
     queries = [q, q[:60]]
-    exp = _oracle_hsps(orc, queries, db)
+    exp = _oracle_hsps(orc, queries, db, filt)
     path = str(tmp_path / "out.npy")
     ext_mode = {"diagonal": bp.EXT_DIAGONAL, "hit_dedup": bp.EXT_HIT_DEDUP}[ext]
     mp.spawn(_worker, args=(world, _free_port(), queries, db.ascii, db.offsets, path, cap,
-                            ext_mode, 2), nprocs=world, join=True)
+                            ext_mode, 2, filt), nprocs=world, join=True)
     got = np.load(path)
     assert len(exp) > 10
     assert got.shape == exp.shape and (got == exp).all()
     if cap < len(exp):  # the overflow path grew the buffer
         assert int(np.load(path + ".cap.npy")[0]) >= len(exp)
+
+
+def test_peer_append_empty_rank(orc, tmp_path):
+    """More ranks than subjects: some ranks search an empty shard and append
+    nothing; rank 0's list is still the oracle's."""
+    from synth import config_workload
+    (q,), db = config_workload(1)
+    keep = 2
+    off = db.offsets[: keep + 1].copy()
+    ascii = db.ascii[: int(off[-1])].copy()
+
+    class _Db:
+        pass
+    small = _Db()
+    small.ascii, small.offsets = ascii, off
+    exp = _oracle_hsps(orc, [q], small)
+    path = str(tmp_path / "out.npy")
+    mp.spawn(_worker, args=(4, _free_port(), [q], ascii, off, path, 1 << 12, 0, 1),
+             nprocs=4, join=True)
+    got = np.load(path)
+    assert got.shape == exp.shape and (got == exp).all()
