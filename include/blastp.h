@@ -171,7 +171,7 @@ int blastp_db_info(const blastp_db *db, int64_t *nseq, int64_t *residues,
 /* End-to-end search of a HOST-resident database shard (no blastp_db kept):
  * the shard's subjects (blastp_shard_range) are cut into parts of whole
  * subjects (num_parts > 0: that many residue-balanced parts; 0: automatic,
- * growing 1.5x from ~1/64 of the shard) and each part is packed (H2D copy
+ * growing 1.25x from ~1/64 of the shard) and each part is packed (H2D copy
  * + encode, as blastp_pack_db, on an internal stream) while the previous
  * part is searched on `cuda_stream` -- the copy overlaps the search (not in
  * the paper, whose database is resident; DESIGN.md "Host-resident
@@ -190,7 +190,7 @@ int blastp_search_host_db(const blastp_query_table *q, const char *residues_asci
 
 /* Formatted host database (the makeblastdb step): the shard `shard_index`
  * of `num_shards` (as blastp_pack_db) is packed on `device` in parts
- * (num_parts > 0: that many residue-balanced parts; 0: parts growing 1.5x
+ * (num_parts > 0: that many residue-balanced parts; 0: parts growing 1.25x
  * from a small first one, as blastp_search_host_db) and each part's device
  * image -- code stream, subject starts, chunk plan, long-item plan -- is
  * copied back into one pinned host buffer owned by the handle.  Synchronous.

@@ -9,6 +9,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <limits>
 #include <string>
 #include <type_traits>
 #include <vector>
@@ -975,26 +976,30 @@ static void db_free_async(blastp_db *db, cudaStream_t s) {
 }
 
 // Part boundaries of a streamed shard [lo, hi) (whole subjects, by
-// residues): num_parts equal parts, or (num_parts = 0) sizes growing 1.5x
+// residues): num_parts equal parts, or (num_parts = 0) sizes growing 1.25x
 // from a small first part -- its copy is the only one not hidden behind a
-// search, and each part copies faster than the previous one is searched.
+// search, and at 1.25x a part's H2D copy (~52 GB/s) takes about as long as
+// the previous part's search (~41 G residues/s at q1054): config 3 e2e
+// 30.4 ms at 1.2-1.3x vs 31.7 ms at 1.5x (profiles/r02/pipe_e2e_sweep.txt).
 static std::vector<int64_t> part_cuts(const int64_t *offsets, int64_t lo, int64_t hi,
-                                      int32_t num_parts, int growth = 150) {
+                                      int32_t num_parts, int growth = 125) {
   const int64_t total = offsets[hi] - offsets[lo];
   std::vector<int64_t> cut{lo};
   // knobs (tuning): BLASTP_PIPE_FIRST residues of the first part,
   // BLASTP_PIPE_GROWTH percent growth per part
   int64_t want = std::max<int64_t>(int64_t(1) << 24, total / 64);
+  int64_t cap = std::numeric_limits<int64_t>::max();
   if (const char *v = std::getenv("BLASTP_PIPE_FIRST")) want = std::max<int64_t>(1, std::atoll(v));
   if (const char *v = std::getenv("BLASTP_PIPE_GROWTH")) growth = std::max(101, std::atoi(v));
+  if (const char *v = std::getenv("BLASTP_PIPE_MAXPART")) cap = std::max<int64_t>(1, std::atoll(v));
   int64_t done = 0;
   for (int k = 0; cut.back() < hi; ++k) {
     int64_t size;
     if (num_parts > 0)
       size = (total * (k + 1)) / num_parts - done;
     else {
-      size = want;
-      want = want * growth / 100;
+      size = std::min(want, cap);
+      want = std::min(want * growth / 100, cap);
     }
     const int64_t target = offsets[lo] + done + std::max<int64_t>(size, 1);
     // first subject starting at or after target
