@@ -68,6 +68,11 @@ namespace {
 #define BLK_MINB 2
 #endif
 constexpr int kBlkWarps = BLK_WARPS;  // warps per CTA (independent walkers)
+#ifdef BLK_PRMT  // A/B knob: X-drop scores from a [qcode][256] matrix indexed by one PRMT
+constexpr int kBlkTab = 1024 + 8192;  // BLOSUM62 32x32 + the 32x256 X-drop matrix
+#else
+constexpr int kBlkTab = 1024;         // BLOSUM62 32x32
+#endif
 constexpr int kBlkMinCtas = BLK_MINB;  // CTAs per SM the register budget allows
 constexpr int kBlkQcap = 64;         // extension queue slots per warp
 constexpr int kBlkFrameMin = 512;    // first frame position (> A + 2 blocks)
@@ -253,6 +258,100 @@ __device__ __forceinline__ void blk_xdrop(const uint8_t *__restrict__ stream, in
   total = seed + best_r + best;
 }
 
+#ifdef BLK_PRMT
+// prmt.b32 in its default mode: a selector nibble with bit 3 set replicates
+// the sign of the selected byte (codes < 32: zero)
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
+  uint32_t d;
+  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(sel));
+  return d;
+}
+// byte k of the subject word | byte k of the query-code word << 8
+template <int k>
+__device__ __forceinline__ int xsc(const int8_t *bx, uint32_t w, uint32_t qw) {
+  constexpr uint32_t sel = uint32_t(k) | (uint32_t(4 + k) << 4) | (uint32_t(8 | k) << 8) |
+                           (uint32_t(8 | k) << 12);
+  return bx[prmt(w, qw, sel)];
+}
+
+// blk_xdrop with the query codes read four per shared load (funnel-shifted
+// like the subject) and each score one PRMT + one shared load from the
+// [qcode][256] matrix bx (bx[(qcode << 8) | scode] = BLOSUM62[qcode][scode]).
+__device__ __forceinline__ void blk_xdrop_prmt(const uint8_t *__restrict__ stream, int64_t sp,
+                                               int q, const uint8_t *qcb, const int8_t *b62,
+                                               const int8_t *bx, int X, int &total, int &llen,
+                                               int &rlen, int &scanned) {
+  const uint32_t *__restrict__ sw = reinterpret_cast<const uint32_t *>(stream);
+  const uint32_t *qw = reinterpret_cast<const uint32_t *>(qcb);  // 16-byte aligned
+  const uint8_t *qq = qcb + kBlkQPad;
+  const int seed = score(b62, qq[q], __ldg(stream + sp)) +
+                   score(b62, qq[q + 1], __ldg(stream + sp + 1)) +
+                   score(b62, qq[q + 2], __ldg(stream + sp + 2));
+  int run = 0, best = 0, bl = 0;
+  {  // right, from (q+3, sp+3)
+    const int64_t a = sp + 3;
+    uint32_t wi = uint32_t(a >> 2);
+    const uint32_t sh = uint32_t(a & 3) * 8;
+    uint32_t lo = __ldg(sw + wi), hi = __ldg(sw + wi + 1);
+    wi += 2;
+    const uint32_t qa = uint32_t(kBlkQPad + q + 3);
+    uint32_t qi = qa >> 2;
+    const uint32_t qsh = (qa & 3u) * 8;
+    uint32_t qlo = qw[qi], qhi = qw[qi + 1];
+    qi += 2;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      const uint32_t qv = __funnelshift_r(qlo, qhi, qsh);
+      lo = hi;
+      hi = __ldg(sw + wi);
+      ++wi;
+      qlo = qhi;
+      qhi = qw[qi];
+      ++qi;
+      xdrop_group4(xsc<0>(bx, w, qv), xsc<1>(bx, w, qv), xsc<2>(bx, w, qv), xsc<3>(bx, w, qv), X,
+                   t, run, best, bl, stop);
+    }
+    scanned = t;
+  }
+  const int best_r = best;
+  rlen = bl;
+  run = 0;
+  best = 0;
+  bl = 0;
+  {  // left, from (q-1, sp-1) downwards
+    const int64_t a3 = sp - 4;  // bytes a3 .. a3+3 = positions sp-4 .. sp-1
+    uint32_t wi = uint32_t(a3 >> 2);
+    const uint32_t sh = uint32_t(a3 & 3) * 8;
+    uint32_t lo = __ldg(sw + wi), hi = __ldg(sw + wi + 1);
+    --wi;
+    const uint32_t qa = uint32_t(kBlkQPad + q - 4);  // query positions q-4 .. q-1
+    uint32_t qi = qa >> 2;
+    const uint32_t qsh = (qa & 3u) * 8;
+    uint32_t qlo = qw[qi], qhi = qw[qi + 1];
+    --qi;
+    bool stop = false;
+    int t = 0;
+    for (; !stop; t += 4) {
+      const uint32_t w = __funnelshift_r(lo, hi, sh);
+      const uint32_t qv = __funnelshift_r(qlo, qhi, qsh);
+      hi = lo;
+      lo = __ldg(sw + wi);
+      --wi;
+      qhi = qlo;
+      qlo = qw[qi];
+      --qi;
+      xdrop_group4(xsc<3>(bx, w, qv), xsc<2>(bx, w, qv), xsc<1>(bx, w, qv), xsc<0>(bx, w, qv), X,
+                   t, run, best, bl, stop);
+    }
+    scanned += t;
+  }
+  llen = bl;
+  total = seed + best_r + best;
+}
+#endif
+
 // REGION: flush
 // Extend up to 32 queued passing hits lane-parallel (R7-R9), then resolve the
 // ext_reach chain (Alg. 3 L19-23, R10) per diagonal in queue (= s) order;
@@ -277,6 +376,9 @@ __device__ __forceinline__ void blk_flush(const SearchArgs &a, const BlkArea &w,
 #ifdef BLK_OLD_XDROP  // A/B knob
     if (act) xdrop_extend(a.stream, sp, q, qc + (kBlkQPad - kQPad), b62, a.xdrop, total, llen,
                           rlen, scanned);
+#elif defined(BLK_PRMT)
+    if (act) blk_xdrop_prmt(a.stream, sp, q, qc, b62, b62 + 1024, a.xdrop, total, llen, rlen,
+                            scanned);
 #else
     if (act) blk_xdrop(a.stream, sp, q, qc + (kBlkQPad - kQPad), b62, a.xdrop, total, llen, rlen,
                        scanned);
@@ -351,14 +453,18 @@ __global__ void __launch_bounds__(kBlkWarps * 32, kBlkMinCtas) search_block_kern
   extern __shared__ __align__(16) uint8_t smem[];
   const int lq = a.qv.lq;
   int8_t *b62 = reinterpret_cast<int8_t *>(smem);
-  uint8_t *qc = smem + 1024;
+  uint8_t *qc = smem + kBlkTab;
   const size_t qc_bytes = align16(size_t(lq) + 2 * kBlkQPad);
   for (int i = threadIdx.x; i < 1024; i += blockDim.x) b62[i] = c_b62_blk[i];
+#ifdef BLK_PRMT
+  for (int i = threadIdx.x; i < 8192; i += blockDim.x)
+    b62[1024 + i] = (i & 255) < 32 ? c_b62_blk[((i >> 8) << 5) | (i & 255)] : int8_t(0);
+#endif
   for (int i = threadIdx.x; i < int(qc_bytes); i += blockDim.x) {
     const int k = i - kBlkQPad;
     qc[i] = (k >= 0 && k < lq) ? a.qv.qcodes[k] : uint8_t(kSentinel);
   }
-  uint8_t *areas = smem + 1024 + qc_bytes;
+  uint8_t *areas = smem + kBlkTab + qc_bytes;
   const int8_t *pssm = a.pssm;
   if constexpr (kPssm) {
     if (!pssm) {  // the PSSM in shared memory (hierarchical buffering)
@@ -712,7 +818,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32, kBlkMinCtas) search_block_kern
 
 // REGION: host
 size_t blk_smem_bytes(int lq, int ring, int warps, bool pssm_smem) {
-  return 1024 + align16(size_t(lq) + 2 * kBlkQPad) +
+  return kBlkTab + align16(size_t(lq) + 2 * kBlkQPad) +
          (pssm_smem ? align16(size_t(lq + 2 * kBlkQPad) * 32) : 0) +
          size_t(warps) * blk_area_bytes(ring);
 }
