@@ -399,6 +399,21 @@ def test_fuzz_small_random(bp, orc):
         assert_same(bp, orc, q, ascii, off, p, trace=True)
 
 
+@pytest.mark.parametrize("W,A", [(1, 32), (3, 34), (3, 35), (8, 39), (8, 40), (3, 255),
+                                 (8, 256), (2, 100)])
+def test_block_state_window_limits(bp, orc, kernel_variant, W, A):
+    """The block kernel's validity edge (A >= 31 + W, A <= 256): every window
+    / min_gap pair at and next to it, on hit-dense planted data with long runs
+    of hits per diagonal, compared at trace level (hits, passing hits,
+    extensions) with the oracle; every kernel variant takes the same pairs."""
+    rng = np.random.default_rng(1000 + 7 * W + A)
+    q = gen_query(31 + W, 400).decode()
+    ascii, off = _rand_db(rng, 40, 50, 900, q, plant=0.8)
+    for ext in (0, 1):
+        assert_same(bp, orc, q, ascii, off,
+                    bp.Params(window=A, min_gap=W, threshold=9, ext_mode=ext), trace=True)
+
+
 def test_adversarial_low_complexity(bp, orc):
     """Poly-W query vs poly-W subjects: every (q, s) is a hit (the hit-dense
     slow path), plus runs of mixed low-complexity residues."""
