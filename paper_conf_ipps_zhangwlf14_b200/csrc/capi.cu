@@ -1193,11 +1193,11 @@ int blastp_format_host_db(const char *residues_ascii, const int64_t *offsets, in
   DeviceGuard g(device);
   if (g.err != cudaSuccess) return fail(BLASTP_E_CUDA, "cudaSetDevice(%d): %s", device, cudaGetErrorString(g.err));
   cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
-  // growth 1.4x: a part's copy (~55 GB/s from pinned memory) must not take
-  // longer than the previous part's search (~38 G residues/s at q1054):
-  // measured 33.1 ms vs 33.7 (1.5x), 38.5 (2x) on config 3
-  // (profiles/r01/fmt_sweep_v2.txt)
-  const std::vector<int64_t> cut = part_cuts(offsets, lo, hi, num_parts, 140);
+  // growth 1.25x (part_cuts' default): a part's copy (~52 GB/s from pinned
+  // memory) must not take longer than the previous part's search (~41 G
+  // residues/s at q1054): config 3 e2e 30.4 ms vs 31.7 at 1.4x
+  // (profiles/r02/pipe_e2e_sweep.txt; r01: profiles/r01/fmt_sweep_v2.txt)
+  const std::vector<int64_t> cut = part_cuts(offsets, lo, hi, num_parts);
   auto *h = new (std::nothrow) blastp_host_db;
   if (!h) return fail(BLASTP_E_NOMEM, "host allocation failed");
   h->device = device;

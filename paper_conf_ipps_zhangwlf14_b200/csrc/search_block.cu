@@ -649,8 +649,13 @@ __global__ void __launch_bounds__(kBlkWarps * 32, kBlkMinCtas) search_block_kern
           __syncwarp();
         };
         // hits of lanes v < L (tested against the previous block's state)
+#ifdef BLK_LAST3  // exact recent positions: no lag, no prepass
+        const uint32_t CL = 0u;
+        const bool pre_ok = true;
+#else
         const uint32_t CL = L > 0 ? __shfl_sync(kFull, incl, L - 1) : 0u;
         const bool pre_ok = CL <= 32u;  // all of them in the first round
+#endif
         // REGION: enqueue
         auto enqueue = [&](bool enq, int P, int q) {
           const unsigned bal = __ballot_sync(kFull, enq);
@@ -740,6 +745,56 @@ __global__ void __launch_bounds__(kBlkWarps * 32, kBlkMinCtas) search_block_kern
           const int bid = max(b, lsv + 1);  // record block (split at subject starts)
           uint32_t e = 0;
           if (act) e = w.ring()[slot];
+#ifdef BLK_LAST3
+          // The diagonal's three most recent hits p1 > p2 > p3 (p1 a frame
+          // position, g1 = p1 - p2, g2 = p2 - p3; 255: none or farther than
+          // A): the largest of them <= h - W, or an earlier member of h's
+          // round group (its first, >= h - 31 >= h - A + 1), decides R6.
+          const int lo_ok = max(P - A + 1, lsv + 1);  // within A, same subject
+          const int hiP = P - W;
+          const int Pf = __shfl_sync(kFull, P, __ffs(G) - 1);  // the group's first hit
+          const int p1 = int(e & 0x3fffu), g1 = int((e >> 14) & 0xffu);
+          int pq = p1;
+          if (pq > hiP) {
+            if (g1 == 255) {
+              pq = 0;
+            } else {
+              pq -= g1;
+              if (pq > hiP) {
+                const int g2 = int(e >> 22);
+                pq = g2 == 255 ? 0 : pq - g2;
+              }
+            }
+          }
+          const bool pass = act && ((pq >= lo_ok && pq <= hiP) || Pf <= hiP);
+          unsigned Gw = G;
+          if (multi_bid_possible && __any_sync(kFull, act && bid != b))
+            Gw = __match_any_sync(kFull, act ? slot : -1);
+          // the state write: the slot's last member, with its two
+          // predecessors in the round (else the old state's)
+          const bool wrl = act && lane == 31 - __clz(Gw);
+          const int d1 = p1 ? min(P - p1, 255) : 255;
+          if (__any_sync(kFull, act && (Gw & ltmask) != 0u)) {
+            const unsigned bef = Gw & ltmask;
+            const int j1 = bef ? 31 - __clz(bef) : lane;
+            const unsigned bef2 = bef & ~(0xffffffffu << j1);
+            const int j2 = bef2 ? 31 - __clz(bef2) : lane;
+            const int x1 = __shfl_sync(kFull, P, j1), x2 = __shfl_sync(kFull, P, j2);
+            if (wrl) {
+              int n1 = d1, n2 = g1;
+              if (bef2) {
+                n1 = P - x1;
+                n2 = x1 - x2;
+              } else if (bef) {
+                n1 = P - x1;
+                n2 = p1 ? min(x1 - p1, 255) : 255;
+              }
+              w.ring()[slot] = uint32_t(P) | (uint32_t(n1) << 14) | (uint32_t(n2) << 22);
+            }
+          } else if (wrl) {
+            w.ring()[slot] = uint32_t(P) | (uint32_t(d1) << 14) | (uint32_t(g1) << 22);
+          }
+#else
           const bool pre = v < L;
           const int lo_ok = max(P - A + 1, lsv + 1);  // within A, same subject
           const int Pf = __shfl_sync(kFull, P, __ffs(G) - 1);  // the group's first hit
@@ -766,6 +821,7 @@ __global__ void __launch_bounds__(kBlkWarps * 32, kBlkMinCtas) search_block_kern
             w.ring()[slot] =
                 uint32_t(bid) | (nmin << 14) | (uint32_t(P - bid) << 19) | (npo << 24);
           }
+#endif
           // every passing hit is queued: the flush's ext_reach chain (R10)
           // rejects the covered ones (0.5% of passing hits are covered by an
           // already resolved extension at this point on config 3; a reach
@@ -875,7 +931,11 @@ cudaError_t blk_pick(const SearchArgs &a, int warps_max, bool pssm_smem, int opt
 bool block_kernel_eligible(const SearchArgs &a) {
   return a.filter_mode == BLASTP_FILTER_LEFT &&
          (a.ext_mode == BLASTP_EXT_DIAGONAL || a.ext_mode == BLASTP_EXT_HIT) &&
+#ifdef BLK_LAST3
+         a.min_gap >= 1 && a.min_gap <= 3 && a.window >= 32 && a.window <= 255 &&
+#else
          a.min_gap >= 1 && a.min_gap <= 8 && a.window >= 31 + a.min_gap && a.window <= 256 &&
+#endif
          a.qv.lq <= 16000 && a.qv.wtab != nullptr &&
          a.table_entries < (int64_t(1) << 27);  // the owner lookup's 27-bit offsets
 }
