@@ -2,8 +2,8 @@
 on this implementation): kernel variant (warp rings / CTA bins, BLASTP_KERNEL)
 x extension strategy (diagonal-based Alg. 3 / hit-based Alg. 4 / window-based
 Alg. 5, warp variant; the CTA variant runs Alg. 3 for WINDOW) x two-hit
-reading (LEFT / EITHER / STATEFUL = Alg. 1's lasthit walk, DIAGONAL and warp
-only) on configs 1-3.  Device time per search (CUDA events
+reading (LEFT / EITHER / STATEFUL = Alg. 1's lasthit walk / STATEFUL_RB, DIAGONAL and
+warp only; the block kernel: LEFT with DIAGONAL / HIT) on configs 1-3.  Device time per search (CUDA events
 on the launch stream, median of `reps` after 2 warm-ups), residues/s and the
 HSP/extension counts of each cell.
 
@@ -31,11 +31,15 @@ for cfg in (1, 2, 3):
     cap = max(1 << 20, db.residues // 50)
     out = torch.empty((cap, 7), dtype=torch.int32, device="cuda")
     cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
-    for kernel in ("warp", "cta"):
+    for kernel in ("block", "warp", "cta"):
         os.environ["BLASTP_KERNEL"] = kernel
-        for ext_mode in (0, 1, 2):
-            for filt in (0, 1, 2):
-                if filt == 2 and (ext_mode != 0 or kernel != "warp"):
+        for ext_mode in (0, 1, 2, 3):
+            for filt in (0, 1, 2, 3):
+                if filt >= 2 and (ext_mode != 0 or kernel != "warp"):
+                    continue
+                if kernel == "block" and (filt != 0 or ext_mode == 2):
+                    continue  # the block kernel runs LEFT with DIAGONAL / HIT (/ HIT_DEDUP)
+                if kernel == "cta" and ext_mode == 3:
                     continue
                 p = bp.Params(filter_mode=filt, ext_mode=ext_mode)
                 t = bp.build_query_table(q, p, stream=stream)
@@ -52,8 +56,9 @@ for cfg in (1, 2, 3):
                 n = int(cnt.item())
                 med = statistics.median(ms)
                 row = {"config": cfg, "query_len": len(q), "residues": db.residues,
-                       "kernel": kernel, "ext_mode": ["DIAGONAL", "HIT", "WINDOW"][ext_mode],
-                       "filter": ["LEFT", "EITHER", "STATEFUL"][filt], "ms": med,
+                       "kernel": kernel,
+                       "ext_mode": ["DIAGONAL", "HIT", "WINDOW", "HIT_DEDUP(search)"][ext_mode],
+                       "filter": ["LEFT", "EITHER", "STATEFUL", "STATEFUL_RB"][filt], "ms": med,
                        "residues_per_s": db.residues / (med / 1e3), "hsps": n}
                 rows.append(row)
                 print(f"config {cfg} {kernel:4s} {row['ext_mode']:8s} {row['filter']:6s} "
