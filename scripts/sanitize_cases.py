@@ -71,6 +71,33 @@ def main():
     print(f"ok query groups: {len(g)} HSPs", flush=True)
     t.free()
     d.free()
+    # the append entry (peer-buffer protocol, here into a local buffer; the
+    # system-scope fence per HSP) and the formatted DB streamed through one
+    # reused part slot
+    import torch
+    t = bp.build_query_table(q1, bp.Params())
+    d = bp.pack_db(db1.ascii, db1.offsets)
+    cap = 1 << 16
+    out = torch.empty((cap, 7), dtype=torch.int32, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+    for _ in range(2):  # appends accumulate
+        bp.search_ungapped_append(t, d, out.data_ptr(), cap, cnt.data_ptr())
+    n = int(cnt.item())
+    exp = len(bp.search_ungapped(t, d))
+    assert n == 2 * exp, (n, exp)
+    print(f"ok append: {n} HSPs (2 x {exp})", flush=True)
+    os.environ["BLASTP_PIPE_SLOTS"] = "1"
+    h = bp.format_host_db(db1.ascii, db1.offsets, num_parts=5)
+    cnt.zero_()
+    bp.search_formatted_db(t, h, out.data_ptr(), cap, cnt.data_ptr())
+    assert int(cnt.item()) == exp
+    print(f"ok formatted, 1 slot x 5 parts: {exp} HSPs", flush=True)
+    os.environ.pop("BLASTP_PIPE_SLOTS")
+    h.free()
+    t.free()
+    d.free()
+    del out, cnt
+    torch.cuda.empty_cache()
     bp.trim_memory(0)  # pool memory back to the device: memcheck's leak check sees only leaks
 
 
