@@ -98,6 +98,7 @@ def main():
     d.free()
     del out, cnt
     torch.cuda.empty_cache()
+    torch._C._host_emptyCache()  # the pinned staging buffer of .item()
     bp.trim_memory(0)  # pool memory back to the device: memcheck's leak check sees only leaks
 
 
