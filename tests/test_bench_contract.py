@@ -54,3 +54,24 @@ def test_gpu_arm_json_line():
     assert d["gpu_launches"] == 3
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle"
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("gather,port", [("p2p", 29571), ("nccl", 29572)])
+def test_gpu_arm_two_ranks_one_gpu(gather, port):
+    """The N > 1 path of bench.py under torchrun (2 ranks sharing the one GPU,
+    gloo host collectives): rank 0 alone prints one line with n_gpus 2 and
+    the gather it timed (the fused peer append or the NCCL-style gather)."""
+    out = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+                          "--nproc-per-node", "2", "--master-addr", "127.0.0.1",
+                          "--master-port", str(port), os.path.join(ROOT, "bench.py"),
+                          "--gpus", "2", "--config", "1", "--steps", "3", "--warmup", "3",
+                          "--no-e2e", "--no-cpu-baseline", "--gather", gather],
+                         capture_output=True, text=True, timeout=600, cwd=ROOT,
+                         env={**os.environ, "BLASTP_DIST_BACKEND": "gloo"})
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0
+    assert d["config"]["gather"].startswith("p2p" if gather == "p2p" else "NCCL")
