@@ -172,18 +172,42 @@ __device__ __forceinline__ void xdrop_extend(const uint8_t *__restrict__ stream,
 __device__ __forceinline__ bool has_successor(const uint8_t *__restrict__ stream, int64_t sp,
                                               int q, const uint8_t *qc, const int8_t *b62, int lq,
                                               int W, int A, int T) {
-  const uint8_t *qq = qc + kQPad;
+  // EITHER (R6): a later hit h' = h + k, W <= k < A, on h's diagonal and
+  // subject -- the word pair at offset k scores >= T.  Residue scores r(j) =
+  // B62[Q[q+j]][S[sp+j]], word(k) = r(k) + r(k+1) + r(k+2); the subject is
+  // read four residues per 32-bit load (one sentinel test per load: a word
+  // reaching the next subject is never a successor).
+  const uint8_t *qq = qc + kQPad + q;
   const int kmax = min(A - 1, lq - 3 - q);
   if (kmax < W) return false;
-  int s1 = score(b62, qq[q + 1], __ldg(stream + sp + 1));
-  int s2 = score(b62, qq[q + 2], __ldg(stream + sp + 2));
-  for (int j = 3; j <= kmax + 2; ++j) {
-    const uint32_t c = __ldg(stream + sp + j);
-    if (c == uint32_t(kSentinel)) return false;  // the subject ends: no later word
-    const int s3 = score(b62, qq[q + j], c);
-    if (j - 2 >= W && s1 + s2 + s3 >= T) return true;
-    s1 = s2;
-    s2 = s3;
+  const uint32_t *__restrict__ sw = reinterpret_cast<const uint32_t *>(stream);
+  const int64_t a0 = sp + 1;  // residues sp+1, sp+2, ... (r(1), r(2), ...)
+  uint32_t wi = uint32_t(a0 >> 2);
+  const uint32_t sh = uint32_t(a0 & 3) * 8;
+  uint32_t lo = __ldg(sw + wi), hi = __ldg(sw + wi + 1);
+  wi += 2;
+  int s1 = 0, s2 = 0;  // r(j-2), r(j-1)
+  const int jend = kmax + 2;  // last residue of the last word
+  for (int j = 1; j <= jend; j += 4) {
+    const uint32_t w = __funnelshift_r(lo, hi, sh);
+    lo = hi;
+    hi = __ldg(sw + wi);
+    ++wi;
+    // a sentinel byte (code 31) among the four: stop there (the words before
+    // it were tested, the ones through it belong to no subject pair)
+    const uint32_t x = w ^ 0x1f1f1f1fu;
+    const uint32_t z = (x - 0x01010101u) & ~x & 0x80808080u;
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const int jj = j + b;
+      if (jj > jend) return false;
+      if ((z >> (8 * b + 7)) & 1u) return false;
+      const int r = score(b62, qq[jj], (w >> (8 * b)) & 0xffu);
+      const int k = jj - 2;
+      if (k >= W && s1 + s2 + r >= T) return true;
+      s1 = s2;
+      s2 = r;
+    }
   }
   return false;
 }
