@@ -36,6 +36,7 @@
  *                                    planted exact copies, E[hits] closed form;
  *                                    HIT mode: oracle-B, one extension per
  *                                    passing hit, Alg. 3 chain of HIT = DIAGONAL.
+ *   oracle_gapped_dir / oracle_gapped_hsps (gapped.c): see gapped.c's header
  *   Whole HSP list vs FSA-BLAST: parity unpinned (FSA-BLAST's rules are not
  *   in the paper); see DESIGN.md.
  */
@@ -156,6 +157,30 @@ int64_t oracle_search(const uint8_t *query, int32_t lq, int32_t query_id,
                       oracle_hsp *out, int64_t cap, oracle_hsp *ext_out,
                       int64_t ext_cap, int64_t *ext_count,
                       oracle_hitlist *hits, oracle_hitlist *passing);
+
+/* ---- gapped extension of the HSP hand-off (gapped.c; R18-R22) ---- */
+
+/* One gapped alignment: query [q_start, q_end) x subject [s_start, s_end),
+ * score, and its traceback path's identities, gaps opened and gap residues. */
+typedef struct {
+  int32_t query_id, subject_id, q_start, q_end, s_start, s_end, score, ident, gap_opens, gap_len;
+} oracle_gapped;
+
+/* R19/R22: one direction from the seed corner over a[0..la) x b[0..lb). */
+int32_t oracle_gapped_dir(const uint8_t *a, int32_t la, const uint8_t *b, int32_t lb,
+                          const int32_t *matrix, int32_t nalpha, int32_t gap_open,
+                          int32_t gap_extend, int32_t xdrop, int32_t *bi, int32_t *bj,
+                          int32_t *ident, int32_t *gopen, int32_t *glen);
+
+/* R20/R21 over a canonical HSP list (query k's codes queries[k]/qlens[k];
+ * subject i - subject_base at db[offsets[i] .. offsets[i+1])).  Returns the
+ * number of reported alignments (canonical order, first `cap` written). */
+int64_t oracle_gapped_hsps(const uint8_t *const *queries, const int32_t *qlens, int32_t nq,
+                           const uint8_t *db, const int64_t *offsets, int64_t nseq,
+                           int64_t subject_base, const oracle_hsp *hsps, int64_t n,
+                           const int32_t *matrix, int32_t nalpha, int32_t gap_open,
+                           int32_t gap_extend, int32_t xdrop, int32_t cutoff,
+                           oracle_gapped *out, int64_t cap);
 
 #ifdef __cplusplus
 }

@@ -23,15 +23,18 @@ HSP_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("diagonal", "
                       ("score", "<i4")])
 
 
+_SRC_GAPPED = os.path.join(_HERE, "gapped.c")
+
+
 def build(force: bool = False) -> str:
-    """Compile oracle.c into liboracle.so (plain gcc, no CUDA)."""
+    """Compile oracle.c + gapped.c into liboracle.so (plain gcc, no CUDA)."""
+    deps = [_SRC, _SRC_GAPPED, os.path.join(_HERE, "oracle.h")]
     if (not force and os.path.exists(_LIB_PATH)
-            and os.path.getmtime(_LIB_PATH) >= max(os.path.getmtime(_SRC),
-                                                    os.path.getmtime(os.path.join(_HERE, "oracle.h")))):
+            and os.path.getmtime(_LIB_PATH) >= max(os.path.getmtime(d) for d in deps)):
         return _LIB_PATH
     tmp = _LIB_PATH + f".tmp{os.getpid()}"
     subprocess.check_call(["gcc", "-O2", "-std=c99", "-Wall", "-Wextra", "-shared", "-fPIC",
-                           "-pthread", _SRC, "-o", tmp])
+                           "-pthread", _SRC, _SRC_GAPPED, "-o", tmp])
     os.replace(tmp, _LIB_PATH)
     return _LIB_PATH
 
@@ -96,6 +99,19 @@ def lib():
         L.oracle_two_hit_stateful.restype = None
         L.oracle_two_hit_stateful.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p,
                                               ctypes.c_int32, ctypes.c_int32, ctypes.c_void_p]
+        L.oracle_gapped_dir.restype = ctypes.c_int32
+        L.oracle_gapped_dir.argtypes = [ctypes.c_void_p, ctypes.c_int32, ctypes.c_void_p,
+                                        ctypes.c_int32, ctypes.c_void_p, ctypes.c_int32,
+                                        ctypes.c_int32, ctypes.c_int32, ctypes.c_int32] + \
+            [ctypes.POINTER(ctypes.c_int32)] * 5
+        L.oracle_gapped_hsps.restype = ctypes.c_int64
+        L.oracle_gapped_hsps.argtypes = [
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32,  # queries, qlens, nq
+            ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64,  # db, off, nseq, base
+            ctypes.c_void_p, ctypes.c_int64,  # hsps, n
+            ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
+            ctypes.c_int32,  # matrix, na, gap_open, gap_extend, xdrop, cutoff
+            ctypes.c_void_p, ctypes.c_int64]
         L.oracle_search.restype = ctypes.c_int64
         L.oracle_search.argtypes = [
             ctypes.c_void_p, ctypes.c_int32, ctypes.c_int32,  # query, lq, qid
@@ -254,3 +270,60 @@ def search(query: np.ndarray, db: np.ndarray, offsets: np.ndarray, params: Param
         passing = np.stack([hbufs[3][:ps.count], hbufs[4][:ps.count], hbufs[5][:ps.count]], axis=1)
     exts = ext[:ext_n.value].copy() if want_extensions else np.zeros(0, dtype=HSP_DTYPE)
     return SearchResult(out[:n].copy(), exts, hits, passing)
+
+
+# ---- gapped extension of the HSP hand-off (gapped.c; R18-R22) ----
+
+GAPPED_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("q_start", "<i4"),
+                         ("q_end", "<i4"), ("s_start", "<i4"), ("s_end", "<i4"),
+                         ("score", "<i4"), ("ident", "<i4"), ("gap_opens", "<i4"),
+                         ("gap_len", "<i4")])
+
+
+@dataclass
+class GappedParams:
+    """R18/R19/R21 (BLASTP defaults: gap cost 11 + 1 per residue, gapped X-drop
+    15 bits = 38 raw at the gapped lambda 0.267, report cutoff 41)."""
+    gap_open: int = 11
+    gap_extend: int = 1
+    xdrop: int = 38
+    cutoff: int = 41
+
+
+def gapped_dir(a: np.ndarray, b: np.ndarray, matrix: np.ndarray, gp: GappedParams | None = None):
+    """One direction (R19/R22): (score, bi, bj, ident, gap_opens, gap_len)."""
+    gp = gp or GappedParams()
+    a = np.ascontiguousarray(a, dtype=np.uint8)
+    b = np.ascontiguousarray(b, dtype=np.uint8)
+    m = np.ascontiguousarray(matrix, dtype=np.int32)
+    outs = [ctypes.c_int32() for _ in range(5)]
+    sc = lib().oracle_gapped_dir(_ptr(a), len(a), _ptr(b), len(b), _ptr(m), m.shape[0],
+                                 gp.gap_open, gp.gap_extend, gp.xdrop,
+                                 *[ctypes.byref(o) for o in outs])
+    if sc < 0:
+        raise MemoryError("oracle_gapped_dir")
+    return (int(sc), *[int(o.value) for o in outs])
+
+
+def gapped_hsps(queries, db: np.ndarray, offsets: np.ndarray, hsps: np.ndarray,
+                gp: GappedParams | None = None, subject_base: int = 0,
+                matrix: np.ndarray | None = None) -> np.ndarray:
+    """R20/R21 over a canonical HSP list; queries = list of code arrays
+    (index = query_id).  Returns GAPPED_DTYPE records in canonical order."""
+    gp = gp or GappedParams()
+    qs = [np.ascontiguousarray(q, dtype=np.uint8) for q in queries]
+    qptr = (ctypes.c_void_p * max(1, len(qs)))(*[q.ctypes.data for q in qs])
+    qlen = np.array([len(q) for q in qs] or [0], dtype=np.int32)
+    d = np.ascontiguousarray(db, dtype=np.uint8)
+    off = np.ascontiguousarray(offsets, dtype=np.int64)
+    h = np.ascontiguousarray(hsps).view(HSP_DTYPE) if len(hsps) else np.zeros(0, HSP_DTYPE)
+    m = np.ascontiguousarray(blosum62() if matrix is None else matrix, dtype=np.int32)
+    cap = max(1, len(h))
+    out = np.zeros(cap, dtype=GAPPED_DTYPE)
+    n = lib().oracle_gapped_hsps(ctypes.cast(qptr, ctypes.c_void_p), _ptr(qlen), len(qs),
+                                 _ptr(d), _ptr(off), len(off) - 1, subject_base, _ptr(h), len(h),
+                                 _ptr(m), m.shape[0], gp.gap_open, gp.gap_extend, gp.xdrop,
+                                 gp.cutoff, _ptr(out), cap)
+    if n < 0:
+        raise ValueError("oracle_gapped_hsps: bad HSP (query / subject id) or allocation failure")
+    return out[:n].copy()
