@@ -318,6 +318,73 @@ int blastp_sort_hsps_device(blastp_hsp *d_hsps, int64_t n, void *cuda_stream);
 int blastp_unique_hsps_device(blastp_hsp *d_hsps, int64_t n, int64_t *d_n_out,
                               void *cuda_stream);
 
+/* ---- Gapped-extension consumer of the HSP hand-off ----
+ * PAPER.md 3.6: "only the high-scoring seeds from ungapped
+ * extension can be passed to the gapped-extension stage", which the paper
+ * runs on the CPU, overlapped with the GPU search (Fig. 12).
+ * The paper prints no algorithm; R18-R22 fix it:
+ *  R18 a gap of k residues costs gap_open + gap_extend * k;
+ *  R19 per direction one Gotoh DP anchored at the seed corner, cells in
+ *      row-major order, a cell dead iff H < best - xdrop (best = the largest
+ *      H so far, from 0), the first maximum wins, a row without live cells
+ *      ends the direction;
+ *  R20 the seed of an HSP is its middle pair (q_start + length/2,
+ *      s_start + length/2): right = forward from it, left = backward from
+ *      the pair before;
+ *  R21 per (query, subject) the HSPs in descending score (ties: canonical
+ *      order); an HSP whose seed lies in the box [q_start, q_end) x
+ *      [s_start, s_end) of an alignment already made for the pair is
+ *      skipped; an alignment is reported iff score >= cutoff; the list is in
+ *      canonical order (lexicographic on all 10 fields);
+ *  R22 traceback from the best cell preferring the diagonal, then a gap in
+ *      the query, then a gap in the subject; a gap opening over its
+ *      extension.  ident / gap_opens / gap_len count the path's identical
+ *      pairs, gaps and gap residues. */
+typedef struct {
+  int32_t gap_open;   /* default 11 */
+  int32_t gap_extend; /* default 1, >= 1 */
+  int32_t xdrop;      /* raw score, default 38 (15 bits at the gapped lambda 0.267) */
+  int32_t cutoff;     /* report iff score >= cutoff, default 41 */
+} blastp_gapped_params;
+
+/* One gapped alignment: query [q_start, q_end) against subject
+ * [s_start, s_end) (subject_id global, as in blastp_hsp).  40 bytes. */
+typedef struct {
+  int32_t query_id, subject_id, q_start, q_end, s_start, s_end, score, ident, gap_opens,
+      gap_len;
+} blastp_gapped;
+
+void blastp_gapped_params_default(blastp_gapped_params *gp);
+
+/* Gapped extension of n ungapped HSPs on the GPU.  d_hsps: DEVICE records of
+ * THIS shard (subject ids global = the shard base + local index) for the
+ * queries of `q` (query_id = batch index), in canonical order (R11, e.g.
+ * from blastp_sort_hsps_device; any order with each (query, subject) pair's
+ * records contiguous and pairs ascending works).  The reported alignments
+ * (R21) are written to d_out (device, `capacity` records) in canonical
+ * order; *out_count (HOST) receives their number.  Synchronous on
+ * cuda_stream (it reads the traceback store size back).  Errors: INVALID_ARG
+ * (NULL pointers, bad params, an id outside the table / shard, pairs not
+ * contiguous, a seed outside its sequences), CAPACITY (count > capacity:
+ * the first `capacity` records are written, *out_count is the full count),
+ * NOMEM, CUDA. */
+int blastp_gapped_extend_device(const blastp_query_table *q, const blastp_db *db,
+                                const blastp_hsp *d_hsps, int64_t n,
+                                const blastp_gapped_params *gp, void *cuda_stream,
+                                blastp_gapped *d_out, int64_t capacity, int64_t *out_count);
+
+/* The two stages in one call: the ungapped search (as blastp_search_ungapped)
+ * and the gapped extension of its HSP list on the GPU; *out_host
+ * (library-malloc'd, free with blastp_gapped_free) receives *out_count
+ * alignments in canonical order.  If ungapped_host / ungapped_count are not
+ * NULL the canonical ungapped list is returned too (free with
+ * blastp_hsp_free).  Synchronous.  Errors: as the two stages. */
+int blastp_search_gapped(const blastp_query_table *q, const blastp_db *db,
+                         const blastp_params *p, const blastp_gapped_params *gp,
+                         void *cuda_stream, blastp_gapped **out_host, int64_t *out_count,
+                         blastp_hsp **ungapped_host, int64_t *ungapped_count);
+void blastp_gapped_free(blastp_gapped *g);
+
 /* Debug / parity entry points (synchronous, host buffers).  They run the
  * same kernel as the search with tracing enabled and return:
  *  hits:    every hit (R4) as (query_id, subject_id, q, s), unordered;

@@ -30,6 +30,11 @@ HSP_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("diagonal", "
                       ("score", "<i4")])
 HIT_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("q", "<i4"), ("s", "<i4")])
 HSP_BYTES = 28
+GAPPED_DTYPE = np.dtype([("query_id", "<i4"), ("subject_id", "<i4"), ("q_start", "<i4"),
+                         ("q_end", "<i4"), ("s_start", "<i4"), ("s_end", "<i4"),
+                         ("score", "<i4"), ("ident", "<i4"), ("gap_opens", "<i4"),
+                         ("gap_len", "<i4")])
+GAPPED_BYTES = 40
 
 
 class BlastpError(RuntimeError):
@@ -59,6 +64,23 @@ class Params:
     def c(self) -> _CParams:
         return _CParams(self.word_len, self.threshold, self.window, self.min_gap, self.xdrop,
                         self.cutoff, self.filter_mode, self.ext_mode)
+
+
+class _CGappedParams(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in ("gap_open", "gap_extend", "xdrop", "cutoff")]
+
+
+@dataclass
+class GappedParams:
+    """blastp_gapped_params (R18-R21): BLASTP defaults, gap cost 11 + 1 per
+    residue, gapped X-drop 38 raw (15 bits at lambda 0.267), cutoff 41."""
+    gap_open: int = 11
+    gap_extend: int = 1
+    xdrop: int = 38
+    cutoff: int = 41
+
+    def c(self) -> _CGappedParams:
+        return _CGappedParams(self.gap_open, self.gap_extend, self.xdrop, self.cutoff)
 
 
 def _load():
@@ -116,6 +138,15 @@ def _load():
         L.blastp_trim_memory.argtypes = [ctypes.c_int]
     if hasattr(L, "blastp_debug_alu_peak"):  # absent in older builds (A/B timing)
         L.blastp_debug_alu_peak.argtypes = [ctypes.c_int, P(ctypes.c_double)]
+    if hasattr(L, "blastp_gapped_extend_device"):  # absent in older builds (A/B timing)
+        L.blastp_gapped_params_default.argtypes = [P(_CGappedParams)]
+        L.blastp_gapped_params_default.restype = None
+        L.blastp_gapped_extend_device.argtypes = [vp, vp, vp, i64, P(_CGappedParams), vp, vp, i64,
+                                                  P(i64)]
+        L.blastp_search_gapped.argtypes = [vp, vp, P(_CParams), P(_CGappedParams), vp, P(vp),
+                                           P(i64), P(vp), P(i64)]
+        L.blastp_gapped_free.argtypes = [vp]
+        L.blastp_gapped_free.restype = None
     for f in ("blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"):
         getattr(L, f).argtypes = [vp]
         getattr(L, f).restype = None
@@ -136,6 +167,8 @@ EXPORTED = ["blastp_params_default", "blastp_strerror", "blastp_last_error", "bl
             "blastp_sort_hsps_device", "blastp_unique_hsps_device", "blastp_dedup_covered_device",
             "blastp_debug_trace", "blastp_debug_hits", "blastp_debug_passing", "blastp_debug_stats",
             "blastp_debug_alu_peak", "blastp_trim_memory",
+            "blastp_gapped_params_default", "blastp_gapped_extend_device", "blastp_search_gapped",
+            "blastp_gapped_free",
             "blastp_hsp_free", "blastp_query_table_free", "blastp_db_free"]
 
 
@@ -342,6 +375,51 @@ def search_ungapped_append(table: QueryTable, db: Database, out_ptr: int, capaci
     _check(lib.blastp_search_ungapped_append(table.handle, db.handle, ctypes.byref(c),
                                              _stream_handle(stream), out_ptr, capacity,
                                              count_ptr), "blastp_search_ungapped_append")
+
+
+def gapped_extend_device(table: QueryTable, db: Database, hsps_ptr: int, n: int, out_ptr: int,
+                         capacity: int, gparams: GappedParams | None = None, stream=None) -> int:
+    """Gapped extension (blastp_gapped_extend_device, synchronous) of n device
+    HSPs of this shard in canonical order at hsps_ptr; alignments written to
+    out_ptr (capacity records of 40 B).  Returns their count."""
+    g = (gparams or GappedParams()).c()
+    cnt = ctypes.c_int64()
+    _check(lib.blastp_gapped_extend_device(table.handle, db.handle, hsps_ptr, n, ctypes.byref(g),
+                                           _stream_handle(stream), out_ptr, capacity,
+                                           ctypes.byref(cnt)), "blastp_gapped_extend_device")
+    return int(cnt.value)
+
+
+def search_gapped(table: QueryTable, db: Database, params: Params | None = None,
+                  gparams: GappedParams | None = None, stream=None, want_ungapped: bool = False):
+    """Ungapped search + gapped extension on the GPU (blastp_search_gapped):
+    GAPPED_DTYPE array in canonical order (and the canonical ungapped list if
+    want_ungapped)."""
+    c = (params or table.params).c()
+    g = (gparams or GappedParams()).c()
+    out, n = ctypes.c_void_p(), ctypes.c_int64()
+    uout, un = ctypes.c_void_p(), ctypes.c_int64()
+    _check(lib.blastp_search_gapped(table.handle, db.handle, ctypes.byref(c), ctypes.byref(g),
+                                    _stream_handle(stream), ctypes.byref(out), ctypes.byref(n),
+                                    ctypes.byref(uout) if want_ungapped else None,
+                                    ctypes.byref(un) if want_ungapped else None),
+           "blastp_search_gapped")
+    try:
+        res = np.zeros(0, dtype=GAPPED_DTYPE)
+        if n.value:
+            buf = (ctypes.c_char * (n.value * GAPPED_BYTES)).from_address(out.value)
+            res = np.frombuffer(bytes(buf), dtype=GAPPED_DTYPE).copy()
+        if not want_ungapped:
+            return res
+        u = np.zeros(0, dtype=HSP_DTYPE)
+        if un.value:
+            buf = (ctypes.c_char * (un.value * HSP_BYTES)).from_address(uout.value)
+            u = np.frombuffer(bytes(buf), dtype=HSP_DTYPE).copy()
+        return res, u
+    finally:
+        lib.blastp_gapped_free(out)
+        if want_ungapped:
+            lib.blastp_hsp_free(uout)
 
 
 IPC_HANDLE_BYTES = 64

@@ -1458,16 +1458,11 @@ int blastp_unique_hsps_device(blastp_hsp *d_hsps, int64_t n, int64_t *d_n_out,
   return BLASTP_OK;
 }
 
-int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
-                           const blastp_params *p, void *cuda_stream, blastp_hsp **out_host,
-                           int64_t *out_count) {
-  if (!out_host || !out_count) return fail(BLASTP_E_INVALID_ARG, "output pointers are NULL");
-  *out_host = nullptr;
-  *out_count = 0;
-  int rc = check_pair(q, db, p);
-  if (rc) return rc;
-  DeviceGuard g(db->device);
-  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+// The search into the db's device buffer (grown and re-run on overflow), then
+// the canonical order (or Alg. 4's de-duplication, R17); *n = the HSP count.
+// Synchronises s.
+static int search_sorted_device(const blastp_query_table *q, const blastp_db *db,
+                                const blastp_params *p, cudaStream_t s, int64_t *n_out) {
   auto *mdb = const_cast<blastp_db *>(db);
   if (mdb->out_cap == 0) {
     const int64_t want = std::max<int64_t>(4096, (db->residues / 1000 + 1) * int64_t(q->q.size()));
@@ -1477,8 +1472,8 @@ int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
   }
   unsigned long long h_count = 0;
   for (int attempt = 0; attempt < 2; ++attempt) {
-    rc = enqueue_search(q, db, p, s, mdb->out, mdb->out_cap, mdb->counters, nullptr, nullptr,
-                        nullptr);
+    const int rc = enqueue_search(q, db, p, s, mdb->out, mdb->out_cap, mdb->counters, nullptr,
+                                  nullptr, nullptr);
     if (rc) return rc;
     CUDA_TRY(cudaMemcpyAsync(&h_count, mdb->counters, sizeof(h_count), cudaMemcpyDeviceToHost, s));
     CUDA_TRY(cudaStreamSynchronize(s));
@@ -1504,13 +1499,179 @@ int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
   } else {
     CUDA_TRY(sort_hsps(mdb->out, n, s));
   }
+  *n_out = n;
+  return BLASTP_OK;
+}
+
+int blastp_search_ungapped(const blastp_query_table *q, const blastp_db *db,
+                           const blastp_params *p, void *cuda_stream, blastp_hsp **out_host,
+                           int64_t *out_count) {
+  if (!out_host || !out_count) return fail(BLASTP_E_INVALID_ARG, "output pointers are NULL");
+  *out_host = nullptr;
+  *out_count = 0;
+  int rc = check_pair(q, db, p);
+  if (rc) return rc;
+  DeviceGuard g(db->device);
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  int64_t n = 0;
+  if ((rc = search_sorted_device(q, db, p, s, &n))) return rc;
   auto *h = static_cast<blastp_hsp *>(malloc(sizeof(blastp_hsp) * static_cast<size_t>(std::max<int64_t>(n, 1))));
   if (!h) return fail(BLASTP_E_NOMEM, "host HSP array");
-  if (n > 0) CUDA_TRY(cudaMemcpyAsync(h, mdb->out, sizeof(blastp_hsp) * static_cast<size_t>(n),
+  if (n > 0) CUDA_TRY(cudaMemcpyAsync(h, db->out, sizeof(blastp_hsp) * static_cast<size_t>(n),
                                       cudaMemcpyDeviceToHost, s));
   CUDA_TRY(cudaStreamSynchronize(s));
   *out_host = h;
   *out_count = n;
+  return BLASTP_OK;
+}
+
+// ------------------------------------------------------------ gapped stage
+
+void blastp_gapped_params_default(blastp_gapped_params *gp) {
+  if (!gp) return;
+  gp->gap_open = 11;
+  gp->gap_extend = 1;
+  gp->xdrop = 38;
+  gp->cutoff = 41;
+}
+
+void blastp_gapped_free(blastp_gapped *g) { free(g); }
+
+static int validate_gapped(const blastp_gapped_params *gp) {
+  if (!gp) return fail(BLASTP_E_INVALID_ARG, "gapped params are NULL");
+  if (gp->gap_open < 0 || gp->gap_open > 1000)
+    return fail(BLASTP_E_INVALID_ARG, "gap_open %d outside [0, 1000]", gp->gap_open);
+  if (gp->gap_extend < 1 || gp->gap_extend > 1000)
+    return fail(BLASTP_E_INVALID_ARG, "gap_extend %d outside [1, 1000]", gp->gap_extend);
+  if (gp->xdrop < 0 || gp->xdrop > 100000)
+    return fail(BLASTP_E_INVALID_ARG, "xdrop %d outside [0, 100000]", gp->xdrop);
+  return BLASTP_OK;
+}
+
+// The gapped stage over a device list of this shard (synchronous on s).
+static int gapped_device(const blastp_query_table *q, const blastp_db *db, const blastp_hsp *d_hsps,
+                         int64_t n, const blastp_gapped_params *gp, cudaStream_t s,
+                         blastp_gapped *d_out, int64_t capacity, int64_t *count) {
+  *count = 0;
+  if (n == 0) return BLASTP_OK;
+  const int32_t nq = static_cast<int32_t>(q->q.size());
+  std::vector<const uint8_t *> qp(static_cast<size_t>(nq));
+  std::vector<int32_t> ql(static_cast<size_t>(nq));
+  for (int32_t k = 0; k < nq; ++k) {
+    qp[k] = q->q[k].qcodes;
+    ql[k] = q->q[k].lq;
+  }
+  int64_t maxlen = 0;
+  const std::vector<int64_t> &st = host_sstart(db);
+  for (int64_t i = 0; i < db->nseq; ++i) {
+    const int64_t en = i + 1 < db->nseq ? st[i + 1] - 1 : kStreamPadFront + db->residues + db->nseq - 1;
+    maxlen = std::max(maxlen, en - st[i]);
+  }
+  const uint8_t **d_qp = nullptr;
+  int32_t *d_ql = nullptr;
+  if (pool_malloc_async(&d_qp, sizeof(void *) * static_cast<size_t>(nq), s) != cudaSuccess ||
+      pool_malloc_async(&d_ql, sizeof(int32_t) * static_cast<size_t>(nq), s) != cudaSuccess) {
+    if (d_qp) cudaFreeAsync(d_qp, s);
+    return fail(BLASTP_E_NOMEM, "gapped query arrays");
+  }
+  CUDA_TRY(cudaMemcpyAsync(d_qp, qp.data(), sizeof(void *) * qp.size(), cudaMemcpyHostToDevice, s));
+  CUDA_TRY(cudaMemcpyAsync(d_ql, ql.data(), sizeof(int32_t) * ql.size(), cudaMemcpyHostToDevice, s));
+  GappedArgs a{};
+  a.hsps = d_hsps;
+  a.n = n;
+  a.qcodes = d_qp;
+  a.qlens = d_ql;
+  a.nq = nq;
+  a.stream = db->stream;
+  a.sstart = db->sstart;
+  a.nseq = db->nseq;
+  a.subject_base = db->subject_base;
+  a.stream_end = kStreamPadFront + db->residues + db->nseq - 1;
+  a.max_subject_len = maxlen;
+  a.gap_open = gp->gap_open;
+  a.gap_extend = gp->gap_extend;
+  a.xdrop = gp->xdrop;
+  a.cutoff = gp->cutoff;
+  int err = 0;
+  const cudaError_t e = launch_gapped(a, db->sms, d_out, capacity, count, &err, s);
+  cudaFreeAsync(d_qp, s);
+  cudaFreeAsync(d_ql, s);
+  if (e == cudaErrorMemoryAllocation) return fail(BLASTP_E_NOMEM, "gapped scratch");
+  CUDA_TRY(e);
+  if (err & 1)
+    return fail(BLASTP_E_INVALID_ARG, "HSP list: an id outside the table / shard, or pairs not "
+                "in canonical order");
+  if (err & 2) return fail(BLASTP_E_INVALID_ARG, "HSP list: a seed outside its sequences");
+  if (*count > capacity)
+    return fail(BLASTP_E_CAPACITY, "%lld gapped alignments, capacity %lld",
+                static_cast<long long>(*count), static_cast<long long>(capacity));
+  return BLASTP_OK;
+}
+
+int blastp_gapped_extend_device(const blastp_query_table *q, const blastp_db *db,
+                                const blastp_hsp *d_hsps, int64_t n,
+                                const blastp_gapped_params *gp, void *cuda_stream,
+                                blastp_gapped *d_out, int64_t capacity, int64_t *out_count) {
+  if (!q || !db || !out_count || n < 0 || (n > 0 && !d_hsps) || capacity < 0 ||
+      (capacity > 0 && !d_out))
+    return fail(BLASTP_E_INVALID_ARG, "bad arguments");
+  *out_count = 0;
+  int rc = validate_gapped(gp);
+  if (rc) return rc;
+  if (q->device != db->device)
+    return fail(BLASTP_E_INVALID_ARG, "table on device %d, db on device %d", q->device, db->device);
+  DeviceGuard g(db->device);
+  return gapped_device(q, db, d_hsps, n, gp, static_cast<cudaStream_t>(cuda_stream), d_out,
+                       capacity, out_count);
+}
+
+int blastp_search_gapped(const blastp_query_table *q, const blastp_db *db,
+                         const blastp_params *p, const blastp_gapped_params *gp,
+                         void *cuda_stream, blastp_gapped **out_host, int64_t *out_count,
+                         blastp_hsp **ungapped_host, int64_t *ungapped_count) {
+  if (!out_host || !out_count) return fail(BLASTP_E_INVALID_ARG, "output pointers are NULL");
+  *out_host = nullptr;
+  *out_count = 0;
+  if (ungapped_host) *ungapped_host = nullptr;
+  if (ungapped_count) *ungapped_count = 0;
+  int rc = check_pair(q, db, p);
+  if (rc) return rc;
+  if ((rc = validate_gapped(gp))) return rc;
+  DeviceGuard g(db->device);
+  cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  int64_t n = 0;
+  if ((rc = search_sorted_device(q, db, p, s, &n))) return rc;
+  blastp_gapped *d_out = nullptr;
+  if (pool_malloc_async(&d_out, sizeof(blastp_gapped) * static_cast<size_t>(std::max<int64_t>(n, 1)), s) !=
+      cudaSuccess)
+    return fail(BLASTP_E_NOMEM, "gapped output");
+  int64_t m = 0;
+  rc = gapped_device(q, db, db->out, n, gp, s, d_out, n, &m);  // one alignment per HSP at most
+  blastp_gapped *h = nullptr;
+  blastp_hsp *u = nullptr;
+  if (!rc) {
+    h = static_cast<blastp_gapped *>(malloc(sizeof(blastp_gapped) * static_cast<size_t>(std::max<int64_t>(m, 1))));
+    if (ungapped_host)
+      u = static_cast<blastp_hsp *>(malloc(sizeof(blastp_hsp) * static_cast<size_t>(std::max<int64_t>(n, 1))));
+    if (!h || (ungapped_host && !u)) rc = fail(BLASTP_E_NOMEM, "host result arrays");
+  }
+  cudaError_t e = cudaSuccess;
+  if (!rc && m > 0)
+    e = cudaMemcpyAsync(h, d_out, sizeof(blastp_gapped) * static_cast<size_t>(m), cudaMemcpyDeviceToHost, s);
+  if (!rc && e == cudaSuccess && u && n > 0)
+    e = cudaMemcpyAsync(u, db->out, sizeof(blastp_hsp) * static_cast<size_t>(n), cudaMemcpyDeviceToHost, s);
+  cudaFreeAsync(d_out, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (!rc && e != cudaSuccess) rc = fail(BLASTP_E_CUDA, "gapped result copy: %s", cudaGetErrorString(e));
+  if (rc) {
+    free(h);
+    free(u);
+    return rc;
+  }
+  *out_host = h;
+  *out_count = m;
+  if (ungapped_host) *ungapped_host = u;
+  if (ungapped_count) *ungapped_count = n;
   return BLASTP_OK;
 }
 

@@ -239,6 +239,20 @@ cudaError_t launch_layout(const int64_t *off, int64_t n, const ChunkPlan &plan, 
 constexpr int kSegLen = 2048;
 constexpr int kSegCap = 2048;
 constexpr int kMaxSegments = 32768;  // 256 MB of lists at most
+// Gapped-extension consumer (gapped.cu, R18-R22).
+struct GappedArgs {
+  const blastp_hsp *hsps;  // canonical order (R11), n records
+  int64_t n;
+  const uint8_t *const *qcodes;  // device: codes of batch query k
+  const int32_t *qlens;          // device
+  int32_t nq;
+  const uint8_t *stream;  // packed shard: subject i at stream[sstart[i]]
+  const int64_t *sstart;
+  int64_t nseq, subject_base, stream_end, max_subject_len;
+  int32_t gap_open, gap_extend, xdrop, cutoff;
+};
+cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out, int64_t cap,
+                          int64_t *h_count, int *h_err, cudaStream_t s);
 cudaError_t measure_alu_peak(double *lane_ops_per_s);  // micro.cu
 cudaError_t sort_hsps(blastp_hsp *d, int64_t n, cudaStream_t s);
 cudaError_t unique_hsps(blastp_hsp *d, int64_t n, int64_t *d_n_out, cudaStream_t s);

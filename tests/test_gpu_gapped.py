@@ -1,0 +1,214 @@
+"""GPU parity of the gapped-extension consumer (DESIGN.md
+R18-R22): blastp_search_gapped / blastp_gapped_extend_device through the
+C-ABI vs the oracle's gapped stage (oracle/gapped.c) run on the oracle's own
+ungapped list, record by record (bit-exact: integer arithmetic)."""
+import os
+
+import numpy as np
+import pytest
+
+from synth import config_workload, gen_db, gen_query
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def bp():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_ipps_zhangwlf14_b200 import build
+    build.build()
+    from paper_conf_ipps_zhangwlf14_b200 import blastp
+    return blastp
+
+
+def assert_same(got, exp, what):
+    got, exp = np.asarray(got), np.asarray(exp)
+    if len(got) == len(exp) and (got.view(np.int32).reshape(-1, 10) ==
+                                 exp.view(np.int32).reshape(-1, 10)).all():
+        return
+    n = min(len(got), len(exp))
+    g = got.view(np.int32).reshape(-1, 10)[:n]
+    e = exp.view(np.int32).reshape(-1, 10)[:n]
+    bad = np.nonzero((g != e).any(axis=1))[0]
+    i = int(bad[0]) if len(bad) else n
+    raise AssertionError(f"{what}: {len(got)} GPU vs {len(exp)} oracle alignments; first "
+                         f"divergence at {i}: gpu {tuple(got[i]) if i < len(got) else None} "
+                         f"oracle {tuple(exp[i]) if i < len(exp) else None}")
+
+
+def oracle_gapped(orc, queries, ascii, offsets, gp, p=None, nthreads=None):
+    """The oracle's ungapped list of every query (its own search), then its
+    gapped stage over that list."""
+    codes = orc.encode(ascii.tobytes())
+    off = np.asarray(offsets, dtype=np.int64)
+    off = off - off[0]
+    P = orc.Params() if p is None else p
+    lists = []
+    for k, q in enumerate(queries):
+        r = orc.search(orc.encode(q), codes, off, P, nthreads=nthreads or os.cpu_count() or 8,
+                       want_extensions=False, query_id=k,
+                       cap_hint=max(1 << 16, int(off[-1]) // 2000))
+        lists.append(r.hsps)
+    u = np.concatenate(lists) if lists else np.zeros(0, orc.HSP_DTYPE)
+    u = np.sort(u, order=list(u.dtype.names))
+    OG = orc.GappedParams(gap_open=gp.gap_open, gap_extend=gp.gap_extend, xdrop=gp.xdrop,
+                          cutoff=gp.cutoff)
+    return u, orc.gapped_hsps([orc.encode(q) for q in queries], codes, off, u, OG)
+
+
+def check(bp, orc, queries, ascii, offsets, gp=None, what="", min_count=1):
+    gp = gp or bp.GappedParams()
+    t = bp.build_query_batch(queries) if len(queries) > 1 else bp.build_query_table(queries[0])
+    d = bp.pack_db(ascii, offsets)
+    got, ung = bp.search_gapped(t, d, gparams=gp, want_ungapped=True)
+    u, exp = oracle_gapped(orc, queries, ascii, offsets, gp)
+    assert (ung.view(np.int32).reshape(-1, 7) == u.view(np.int32).reshape(-1, 7)).all()
+    assert_same(got, exp, what)
+    assert len(exp) >= min_count
+    return got
+
+
+def test_config1_gapped(bp, orc):
+    """Config 1 (q127 vs 1,000 subjects, 5% planted homologs)."""
+    (q,), db = config_workload(1)
+    g = check(bp, orc, [q], db.ascii, db.offsets, what="config 1", min_count=20)
+    assert (g["gap_opens"] > 0).any() or len(g) < 50
+
+
+def test_config2_gapped(bp, orc):
+    """Config 2 (q517 vs 20M residues): every alignment identical."""
+    (q,), db = config_workload(2)
+    g = check(bp, orc, [q], db.ascii, db.offsets, what="config 2", min_count=1000)
+    assert (g["gap_opens"] > 0).sum() > 100
+
+
+def test_config3_gapped_full(bp, orc):
+    """Config 3 at full size (q1054 vs 1.2G residues): the gapped stage over
+    the complete ungapped list (~286K HSPs), every alignment identical."""
+    (q,), db = config_workload(3)
+    check(bp, orc, [q], db.ascii, db.offsets, what="config 3", min_count=10000)
+
+
+@pytest.mark.parametrize("knobs", [{"BLASTP_GAPPED_RING": "16"}, {"BLASTP_GAPPED_RING": "64"},
+                                   {"BLASTP_GAPPED_STORE": "4096"}],
+                         ids=["ring16", "ring64", "store4k"])
+def test_ring_overflow_and_store_windows(bp, orc, monkeypatch, knobs):
+    """Pairs whose DP rows outgrow the per-thread ring are redone with
+    subject-sized rings; traceback stores split into several windows: same
+    results."""
+    for k, v in knobs.items():
+        monkeypatch.setenv(k, v)
+    (q,), db = config_workload(1)
+    check(bp, orc, [q], db.ascii, db.offsets, what=str(knobs), min_count=20)
+
+
+def test_batch_and_shard_device_entry(bp, orc):
+    """A three-query batch against the shards of a database with long subjects:
+    blastp_gapped_extend_device over each shard's sorted device list
+    (global subject ids) equals the oracle's shard-by-shard result."""
+    import torch
+    queries = [gen_query(11, 160), gen_query(12, 700), gen_query(13, 1500)]
+    db = gen_db(31, 32, n_subjects=3000, mean_len=300.0, queries=queries, plant_frac=0.1)
+    # one long subject holding copies of every query (long alignments, big rows)
+    t = bp.build_query_batch(queries)
+    for k in range(3):
+        lo, hi = bp.shard_range(db.offsets, k, 3)
+        sub_off = db.offsets[lo:hi + 1]
+        d = bp.pack_db(db.ascii, db.offsets, k, 3)
+        u = bp.search_ungapped(t, d)
+        assert len(u) > 0
+        dev = torch.from_numpy(u.view(np.int32).reshape(-1, 7).copy()).cuda()
+        out = torch.zeros((len(u), 10), dtype=torch.int32, device="cuda")
+        n = bp.gapped_extend_device(t, d, dev.data_ptr(), len(u), out.data_ptr(), len(u))
+        got = out[:n].cpu().numpy().view(bp.GAPPED_DTYPE).ravel()
+        codes = orc.encode(db.ascii[sub_off[0]:sub_off[-1]].tobytes())
+        OG = orc.GappedParams()
+        exp = orc.gapped_hsps([orc.encode(q) for q in queries], codes, sub_off - sub_off[0],
+                              u.view(orc.HSP_DTYPE), OG, subject_base=lo)
+        assert_same(got, exp, f"shard {k}")
+
+
+def test_long_subjects_and_copies(bp, orc):
+    """Subjects of 8K-36,805 residues with planted query copies and indels:
+    long gapped alignments (rows far from the seed, big traceback stores)."""
+    rng = np.random.default_rng(77)
+    q = gen_query(4040, 1200)
+    alpha = np.frombuffer(b"ARNDCQEGHILKMFPSTWYV", dtype=np.uint8)
+    subs = []
+    for k in range(12):
+        L = int(rng.integers(8192, 36806))
+        s = alpha[rng.integers(0, 20, size=L)].copy()
+        for _ in range(4):  # copies of query segments with a few indels
+            a = int(rng.integers(0, 1000))
+            ln = int(rng.integers(60, 200))
+            seg = np.frombuffer(q[a:a + ln], dtype=np.uint8).copy()
+            for _ in range(int(rng.integers(0, 4))):
+                c = int(rng.integers(1, len(seg) - 1))
+                seg = np.delete(seg, c) if rng.random() < 0.5 else np.insert(seg, c, alpha[rng.integers(0, 20)])
+            pos = int(rng.integers(0, L - len(seg)))
+            s[pos:pos + len(seg)] = seg
+        subs.append(s)
+    ascii = np.concatenate(subs)
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    g = check(bp, orc, [q], ascii, off, what="long subjects", min_count=20)
+    assert (g["gap_opens"] > 0).any()
+    assert (g["q_end"] - g["q_start"]).max() >= 60
+
+
+@pytest.mark.parametrize("go,ge,x,cut", [(11, 1, 38, 41), (5, 2, 20, 30), (0, 1, 10, 20),
+                                         (11, 1, 0, 41), (11, 1, 200, 60)])
+def test_gapped_params(bp, orc, go, ge, x, cut):
+    """Gap costs, X-drop and cutoff variations (X = 0: only cells at the best
+    survive) on random planted databases."""
+    q = gen_query(99, 300)
+    db = gen_db(101, 102, n_subjects=800, mean_len=250.0, queries=[q], plant_frac=0.2)
+    check(bp, orc, [q], db.ascii, db.offsets, bp.GappedParams(go, ge, x, cut),
+          what=f"params {go}/{ge}/{x}/{cut}")
+
+
+def test_hit_dedup_list_gaps_like_diagonal(bp, orc):
+    """ext_mode HIT_DEDUP hands off DIAGONAL's list (R17): same gapped result."""
+    (q,), db = config_workload(1)
+    t = bp.build_query_table(q)
+    d = bp.pack_db(db.ascii, db.offsets)
+    a = bp.search_gapped(t, d, bp.Params(ext_mode=bp.EXT_HIT_DEDUP))
+    b = bp.search_gapped(t, d, bp.Params())
+    assert_same(a, b, "HIT_DEDUP vs DIAGONAL")
+
+
+def test_errors_and_capacity(bp, orc):
+    import torch
+    (q,), db = config_workload(1)
+    t = bp.build_query_table(q)
+    d = bp.pack_db(db.ascii, db.offsets)
+    u = bp.search_ungapped(t, d)
+    assert len(u) > 10
+    dev = torch.from_numpy(u.view(np.int32).reshape(-1, 7).copy()).cuda()
+    out = torch.zeros((len(u), 10), dtype=torch.int32, device="cuda")
+    n = bp.gapped_extend_device(t, d, dev.data_ptr(), len(u), out.data_ptr(), len(u))
+    assert n > 2
+    # capacity too small: CAPACITY, the first records written, the count reported
+    with pytest.raises(bp.BlastpError) as ei:
+        bp.gapped_extend_device(t, d, dev.data_ptr(), len(u), out.data_ptr(), 2)
+    assert ei.value.status == bp.E_CAPACITY
+    # pairs out of order, a query id outside the table, a seed outside the query
+    rev = torch.flip(dev, dims=[0]).contiguous()
+    with pytest.raises(bp.BlastpError) as ei:
+        bp.gapped_extend_device(t, d, rev.data_ptr(), len(u), out.data_ptr(), len(u))
+    assert ei.value.status == bp.E_INVALID_ARG
+    bad = dev.clone()
+    bad[0, 0] = 5
+    with pytest.raises(bp.BlastpError) as ei:
+        bp.gapped_extend_device(t, d, bad.data_ptr(), len(u), out.data_ptr(), len(u))
+    assert ei.value.status == bp.E_INVALID_ARG
+    bad = dev.clone()
+    bad[0, 3] = 10 ** 6
+    with pytest.raises(bp.BlastpError) as ei:
+        bp.gapped_extend_device(t, d, bad.data_ptr(), len(u), out.data_ptr(), len(u))
+    assert ei.value.status == bp.E_INVALID_ARG
+    with pytest.raises(bp.BlastpError):
+        bp.gapped_extend_device(t, d, dev.data_ptr(), len(u), out.data_ptr(), len(u),
+                                bp.GappedParams(gap_extend=0))
+    assert bp.gapped_extend_device(t, d, dev.data_ptr(), 0, out.data_ptr(), len(u)) == 0
