@@ -38,6 +38,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -49,18 +50,15 @@ namespace {
 constexpr int32_t kNeg = INT32_MIN / 4;  // -infinity that survives a few subtractions
 
 // counters[]
-enum { kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kNumCounters = 8 };
+enum { kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kNumCounters = 8 };
 
+// a reported direction for pass 2: its best cell, widest span, and whether
+// pass 1 logged its codes (then at nib_off / hdr_off of the logs)
 struct DirInfo {
-  int32_t bi, bj, maxspan, pad;
+  int32_t bi, bj, maxspan, logged;
+  int64_t nib_off, hdr_off;
 };
 
-struct DirResult {
-  int32_t score, bi, bj;
-  int32_t maxspan;  // widest computed span among rows 0..bi
-  int64_t cells;    // cells of those rows' spans
-  bool overflow;
-};
 
 __device__ __forceinline__ int32_t imax(int32_t a, int32_t b) { return a > b ? a : b; }
 
@@ -74,152 +72,208 @@ __host__ __device__ inline int32_t pow2_at_least(int32_t x) {
 // cell} (int2 per row), the cells' nibbles, then the DP ring (pow2 >= the
 // widest span, int2 per column).
 __host__ __device__ inline int64_t slab_hdr_bytes(int32_t rows) { return align16(int64_t(rows) * 8); }
-__host__ __device__ inline int64_t slab_nib_bytes(int64_t cells) { return align16((cells + 1) / 2); }
+__host__ __device__ inline int64_t slab_nib_bytes(int64_t cells) { return align16((cells + 7) / 8 * 4); }
+__host__ __device__ inline int32_t slab_ring_cols(int32_t maxspan) {
+  return pow2_at_least(maxspan < 2 ? 2 : maxspan);
+}
 __host__ __device__ inline int64_t slab_bytes(int32_t rows, int64_t cells, int32_t maxspan) {
-  return slab_hdr_bytes(rows) + slab_nib_bytes(cells) + int64_t(pow2_at_least(maxspan)) * 8;
+  return slab_hdr_bytes(rows) + slab_nib_bytes(cells) + int64_t(slab_ring_cols(maxspan)) * 8;
 }
 
-__device__ __forceinline__ void put_nib(uint8_t *nib, int64_t c, uint8_t code) {
-  if (c & 1) nib[c >> 1] |= uint8_t(code << 4);
-  else nib[c >> 1] = code;
+
+// One direction of the DP (R19) as a state machine advanced one cell per
+// dir_step(): a thread's cells run in lock-step with its warp's other lanes
+// whatever row, direction or pair each lane is in (the nested row / direction
+// / pair loops written directly leave ~3 of 32 lanes active: every lane sits
+// at another loop level).  a[i] = A[i * step] (i < la), b[j] = B[j * step]
+// (j < lb); ring: mask + 1 int2 cells {H, F} indexed by column.  With
+// nibw set, every computed cell's 4-bit code goes to the nibble stream (8 per
+// 32-bit word, cells numbered row after row) and each row's {start column,
+// first cell} to hdr[i]: bits 0-1 where H came from (0 diagonal, 1 E,
+// 2 F: R22's order of preference), bit 2 E opened here, bit 3 F opened here.
+// cap_cells / cap_rows bound the stream (a row that might not fit stops it:
+// nibw = nullptr).  Row 0 is the generic row under a dead row -1 (its F
+// values are -inf minus a gap cost instead of -inf: a live cell's H never
+// comes from such an F, so nothing observable differs).
+struct Dir {
+  const uint8_t *A, *B;
+  const int8_t *mrow;
+  uint32_t *nibw;
+  int2 *hdr;
+  int64_t cum, r_cells, nc, cap_cells;  // cells of the rows done / of rows 0..best; next nibble
+  uint32_t nword;
+  int32_t cap_rows;
+  int32_t step, la, lb, stop_row;
+  int32_t i, j, start, phi, lo, hi;  // phi: last live cell of the previous row
+  int32_t lh, le, dh;                // left H / E, previous row's H at j - 1
+  int32_t best, best_row, bi, bj, maxspan_all, r_maxspan;
+  bool done, overflow;
+};
+
+__device__ __forceinline__ void dir_finish(Dir &d) {
+  if (d.nibw && (d.nc & 7)) d.nibw[d.nc >> 3] = d.nword;
+  d.done = true;
 }
 
-// One direction (R19): a[i] = A[i * step] (i < la), b[j] = B[j * step]
-// (j < lb).  ring: mask + 1 int2 cells {H, F}.  Pass 2 passes nib/hdr and
-// stop_row (the best row found by pass 1): the rows 0..stop_row are stored.
-// Cell codes (pass 2): bits 0-1 where H came from (0 diagonal, 1 E, 2 F, in
-// R22's order of preference), bit 2 E opened here, bit 3 F opened here.
-__device__ DirResult gapped_dir(const uint8_t *A, const uint8_t *B, int step, int32_t la,
-                                int32_t lb, const int8_t (*M)[32], int32_t go, int32_t ge,
-                                int32_t X, int2 *ring, int32_t mask, uint8_t *nib, int2 *hdr,
-                                int32_t stop_row) {
-  DirResult r{0, 0, 0, 0, 0, false};
-  const int32_t goe = go + ge;
-  int32_t best = 0, best_row = 0, maxspan_all = 0;
-  int64_t cum = 0;  // cells of the rows computed so far
-  int32_t plo = 0, phi = 0;  // live range of the previous row
-  // row 0: the origin, then a leading gap in b (E only)
-  {
-    int32_t lh = 0, le = kNeg, j = 1;
-    ring[0] = make_int2(0, kNeg);
-    if (nib) {
-      hdr[0] = make_int2(0, 0);
-      put_nib(nib, 0, 1);
-    }
-    for (; j <= lb; ++j) {
-      int32_t e = imax(le - ge, lh - goe);
-      const uint8_t code = uint8_t(1 | (e == lh - goe ? 4 : 0));
-      int32_t h = e;                      // no diagonal, no F in row 0
-      if (h < best - X) h = e = kNeg;     // (h > best is impossible: best = 0)
-      if (j > mask) {
-        r.overflow = true;
-        return r;
-      }
-      ring[j & mask] = make_int2(h, kNeg);
-      if (nib) put_nib(nib, j, code);
-      lh = h;
-      le = e;
-      if (h > kNeg) phi = j;
-      else break;  // dead at j >= up_end (= 1): nothing to its right is reachable
-    }
-    const int32_t span = (j <= lb ? j : lb) + 1;
-    cum = span;
-    maxspan_all = span;
-    r.maxspan = span;
-    r.cells = span;
+__device__ __forceinline__ void dir_end_row(Dir &d, const int8_t (*M)[32], const int2 *ring,
+                                            int32_t mask) {
+  if (d.lo < 0) {  // a row without live cells ends the extension
+    dir_finish(d);
+    return;
   }
-  for (int32_t i = 1; i <= la && stop_row >= i; ++i) {
-    const int8_t *mrow = M[A[int64_t(i - 1) * step]];
-    int32_t lh = kNeg, le = kNeg, dh = kNeg;  // cell plo - 1 of both rows is dead
-    int32_t lo = -1, hi = -1, j = plo;
-    const int32_t start = plo;
-    if (nib) hdr[i] = make_int2(start, int32_t(cum));
-    for (;; ++j) {
-      const int2 up = (j <= phi) ? ring[j & mask] : make_int2(kNeg, kNeg);
-      const int32_t e = j > 0 ? imax(le - ge, lh - goe) : kNeg;
-      const int32_t f = imax(up.y - ge, up.x - goe);
-      const int32_t d = (j > 0 && dh > kNeg) ? dh + mrow[B[int64_t(j - 1) * step]] : kNeg;
-      int32_t h = imax(d, imax(e, f)), ee = e, ff = f;
-      const uint8_t code = uint8_t((h == d ? 0 : (h == e ? 1 : 2)) | (e == lh - goe ? 4 : 0) |
-                                   (f == up.x - goe ? 8 : 0));
-      if (h < best - X) {
-        h = ee = ff = kNeg;  // dead
-      } else if (h > best) {
-        best = h;
-        best_row = i;
-        r.bi = i;
-        r.bj = j;
-      }
-      if (j - start > mask) {
-        r.overflow = true;
-        return r;
-      }
-      dh = up.x;
-      ring[j & mask] = make_int2(h, ff);
-      if (nib) put_nib(nib, cum + (j - start), code);
-      lh = h;
-      le = ee;
-      if (h > kNeg) {
-        if (lo < 0) lo = j;
-        hi = j;
-      } else if (j > phi && j > 0) {
-        break;  // dead and beyond the previous row's live cells: the row ends
-      }
-      if (j == lb) break;
-    }
-    if (lo < 0) break;  // a row without live cells ends the extension
-    const int32_t span = j - start + 1;
-    cum += span;
-    maxspan_all = imax(maxspan_all, span);
-    if (best_row == i) {
-      r.cells = cum;
-      r.maxspan = maxspan_all;
-    }
-    plo = lo;
-    phi = hi;
+  const int32_t span = d.j - d.start + 1;
+  d.cum += span;
+  d.maxspan_all = imax(d.maxspan_all, span);
+  if (d.best_row == d.i) {
+    d.r_cells = d.cum;
+    d.r_maxspan = d.maxspan_all;
   }
-  r.score = best;
-  return r;
-}
-
-// R22 traceback from (bi, bj) over the pass-2 store: identities, gap opens,
-// gap residues.
-__device__ void traceback(const uint8_t *A, const uint8_t *B, int step, int32_t bi, int32_t bj,
-                          const uint8_t *nib, const int2 *hdr, int32_t *ident, int32_t *gopen,
-                          int32_t *glen) {
-  int32_t i = bi, j = bj, state = 0, idn = 0, go = 0, gl = 0;
-  while (i > 0 || j > 0) {
-    const int2 h = hdr[i];
-    const int64_t c = int64_t(h.y) + (j - h.x);
-    const int code = (nib[c >> 1] >> ((c & 1) * 4)) & 15;
-    if (state == 0) {
-      const int src = code & 3;
-      if (src == 0) {
-        idn += A[int64_t(i - 1) * step] == B[int64_t(j - 1) * step];
-        --i;
-        --j;
-      } else {
-        state = src;  // 1: in E (gap in a), 2: in F (gap in b)
-      }
-    } else if (state == 1) {
-      ++gl;
-      if (code & 4) {
-        ++go;
-        state = 0;
-      }
-      --j;
+  d.phi = d.hi;
+  d.start = d.j = d.lo;  // cells left of the previous row's first live one are dead
+  d.i += 1;
+  if (d.i > d.la || d.i > d.stop_row) {
+    dir_finish(d);
+    return;
+  }
+  d.lo = d.hi = -1;
+  d.lh = d.le = d.dh = kNeg;
+  d.mrow = M[d.A[int64_t(d.i - 1) * d.step]];
+  if (d.nibw) {
+    if (d.cum + mask + 1 > d.cap_cells || d.i >= d.cap_rows) {
+      d.nibw = nullptr;  // this row might not fit: no traceback store for this direction
     } else {
-      ++gl;
-      if (code & 8) {
-        ++go;
-        state = 0;
-      }
-      --i;
+      d.hdr[d.i] = make_int2(d.start, int32_t(d.cum));
     }
   }
-  *ident = idn;
-  *gopen = go;
-  *glen = gl;
+}
+
+__device__ __forceinline__ void dir_begin(Dir &d, const uint8_t *A, const uint8_t *B, int step,
+                                          int32_t la, int32_t lb, int32_t stop_row,
+                                          const int8_t (*M)[32], int2 *ring, int32_t mask,
+                                          uint32_t *nibw, int2 *hdr, int64_t cap_cells,
+                                          int32_t cap_rows) {
+  d.A = A;
+  d.B = B;
+  d.step = step;
+  d.la = la;
+  d.lb = lb;
+  d.stop_row = stop_row;
+  d.mrow = M[0];
+  d.cum = d.r_cells = 0;
+  d.i = d.j = d.start = 0;
+  d.phi = -1;
+  d.lo = d.hi = 0;  // the origin H(0,0) = 0 is live
+  d.lh = 0;
+  d.le = d.dh = kNeg;
+  d.best = d.best_row = d.bi = d.bj = 0;
+  d.maxspan_all = d.r_maxspan = 0;
+  d.done = d.overflow = false;
+  d.hdr = hdr;
+  d.cap_cells = cap_cells;
+  d.cap_rows = cap_rows;
+  d.nibw = (nibw && mask + 1 <= cap_cells && cap_rows >= 1) ? nibw : nullptr;
+  d.nc = 0;
+  d.nword = 0;
+  ring[0] = make_int2(0, kNeg);
+  if (d.nibw) {
+    hdr[0] = make_int2(0, 0);
+    d.nword = 1;  // the origin's code (never read)
+    d.nc = 1;
+  }
+  if (lb == 0) {
+    dir_end_row(d, M, ring, mask);
+  } else {
+    d.j = 1;
+  }
+}
+
+__device__ __forceinline__ void dir_step(Dir &d, const int8_t (*M)[32], int2 *ring, int32_t mask,
+                                         int32_t ge, int32_t goe, int32_t X) {
+  const int32_t j = d.j;
+  // (loading the next cell's ring entry and residue one step ahead, carried
+  // in registers, measured 5x slower: 300 vs 62 ms at config 3)
+  const int2 up = (j <= d.phi) ? ring[j & mask] : make_int2(kNeg, kNeg);
+  const int32_t bres = j > 0 ? d.B[int64_t(j - 1) * d.step] : 0;
+  const int32_t e = j > 0 ? imax(d.le - ge, d.lh - goe) : kNeg;
+  const int32_t f = imax(up.y - ge, up.x - goe);
+  const int32_t dg = (j > 0 && d.dh > kNeg) ? d.dh + d.mrow[bres] : kNeg;
+  const int32_t hraw = imax(dg, imax(e, f));
+  int32_t h = hraw, ee = e, ff = f;
+  if (h < d.best - X) {
+    h = ee = ff = kNeg;  // dead
+  } else if (h > d.best) {
+    d.best = h;
+    d.best_row = d.i;
+    d.bi = d.i;
+    d.bj = j;
+  }
+  if (j - d.start > mask) {
+    d.overflow = true;
+    d.nibw = nullptr;
+    d.done = true;
+    return;
+  }
+  d.dh = up.x;
+  ring[j & mask] = make_int2(h, ff);
+  if (d.nibw) {
+    const uint32_t code = uint32_t((hraw == dg ? 0 : (hraw == e ? 1 : 2)) |
+                                   (e == d.lh - goe ? 4 : 0) | (f == up.x - goe ? 8 : 0));
+    d.nword |= code << ((d.nc & 7) * 4);
+    if ((d.nc & 7) == 7) {
+      d.nibw[d.nc >> 3] = d.nword;
+      d.nword = 0;
+    }
+    ++d.nc;
+  }
+  d.lh = h;
+  d.le = ee;
+  bool row_end = (j == d.lb);
+  if (h > kNeg) {
+    if (d.lo < 0) d.lo = j;
+    d.hi = j;
+  } else if (j > d.phi && j > 0) {
+    row_end = true;  // dead and beyond the previous row's live cells: the row ends
+  }
+  if (row_end) dir_end_row(d, M, ring, mask);
+  else d.j = j + 1;
+}
+
+// R22 traceback from (bi, bj) over a direction's stored codes, one move per
+// step.
+struct Trace {
+  int32_t i, j, state, ident, gopen, glen;
+};
+__device__ __forceinline__ bool trace_step(Trace &t, const uint8_t *A, const uint8_t *B, int step,
+                                           const uint32_t *nibw, const int2 *hdr) {
+  if (t.i == 0 && t.j == 0) return true;
+  const int2 h = hdr[t.i];
+  const int64_t c = int64_t(h.y) + (t.j - h.x);
+  const int code = (nibw[c >> 3] >> ((c & 7) * 4)) & 15;
+  if (t.state == 0) {
+    const int src = code & 3;
+    if (src == 0) {
+      t.ident += A[int64_t(t.i - 1) * step] == B[int64_t(t.j - 1) * step];
+      --t.i;
+      --t.j;
+    } else {
+      t.state = src;  // 1: in E (gap in a), 2: in F (gap in b)
+    }
+  } else if (t.state == 1) {
+    ++t.glen;
+    if (code & 4) {
+      ++t.gopen;
+      t.state = 0;
+    }
+    --t.j;
+  } else {
+    ++t.glen;
+    if (code & 8) {
+      ++t.gopen;
+      t.state = 0;
+    }
+    --t.i;
+  }
+  return false;
 }
 
 // BLOSUM62 (R18: the search's matrix), passed by value to the kernels
@@ -289,118 +343,224 @@ __global__ void gapped_keys_kernel(GappedArgs a, const int32_t *flag, const int3
 }
 
 // pass 1: one thread per pair (work counter), or per pair of the overflow
-// list (big rings).
+// list (big rings).  The thread's pairs, their HSPs (R21 order) and both
+// directions of each run as one flat loop, one DP cell per turn.  The codes
+// of each direction are appended to the thread's logs (nibbles: nlog_words
+// 32-bit words; row headers: hlog_rows) and kept if the alignment is
+// reported; pass 2 traces them back.  A direction that no longer fits is
+// re-run by pass 2 into a store of its own (its need > 0).
 __global__ void __launch_bounds__(128) gapped_score_kernel(
     GappedArgs a, Matrix32 mat, const uint32_t *perm, const int32_t *gstart, blastp_gapped *rec,
     uint8_t *status, DirInfo *dinfo, int64_t *need, int2 *scratch, int32_t ring_cols,
-    int32_t *over_list, bool big, unsigned long long *counters) {
+    uint32_t *nlog, int32_t nlog_words, int2 *hlog, int32_t hlog_rows, int32_t *over_list,
+    bool big, unsigned long long *counters) {
   __shared__ int8_t M[32][32];
   load_matrix(M, mat);
   const int64_t tid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
   int2 *ring = scratch + tid * ring_cols;
-  const int32_t mask = ring_cols - 1;
+  const int64_t nbase = tid * nlog_words, hbase = tid * hlog_rows;
+  int32_t ncur = 0, hcur = 0;  // the logs' fill
+  const int32_t mask = ring_cols - 1, ge = a.gap_extend, goe = a.gap_open + a.gap_extend;
   const unsigned long long ngroups = big ? counters[kNumOver] : counters[kNumGroups];
+  Dir d;
+  d.done = true;
+  int phase = 0;  // 0 fetch, 1 DP
+  int32_t g = 0, g0 = 0, g1 = 0, k = 0, cur = 0, side = 0;
+  int32_t qm = 0, sm = 0, lq = 0, ls = 0;
+  const uint8_t *Q = nullptr, *S = nullptr;
+  int32_t r_score = 0, r_bi = 0, r_bj = 0, r_span = 0, n0 = 0, h0 = 0, r_n = 0, r_h = 0;
+  int64_t r_cells = 0;
+  bool r_logged = false;
   for (;;) {
-    const unsigned long long w = atomicAdd(&counters[big ? kCurBig : kCurPass1], 1ull);
-    if (w >= ngroups) break;
-    const int32_t g = big ? over_list[w] : int32_t(w);
-    const int32_t g0 = gstart[g], g1 = gstart[g + 1];
-    bool over = false;
-    for (int32_t k = g0; k < g1 && !over; ++k) {
-      status[k] = 0;
-      need[2 * k] = need[2 * k + 1] = 0;
-      const blastp_hsp h = a.hsps[perm[k]];
-      const uint8_t *Q = a.qcodes[h.query_id];
-      const int32_t lq = a.qlens[h.query_id];
+    if (phase == 1 && !d.done) dir_step(d, M, ring, mask, ge, goe, a.xdrop);
+    if (phase == 1 && d.done) {
+      if (d.overflow) {  // redo the whole pair with big rings
+        for (int32_t t = g0; t < g1; ++t) {
+          status[t] = 0;
+          need[2 * t] = need[2 * t + 1] = 0;
+          dinfo[2 * t].logged = dinfo[2 * t + 1].logged = 0;
+        }
+        over_list[atomicAdd(&counters[kNumOver], 1ull)] = g;
+        k = g1;
+        ncur = n0;
+        hcur = h0;
+        phase = 0;
+      } else {
+        const bool logged = d.nibw != nullptr;
+        const int32_t used_n = logged ? int32_t((d.nc + 7) >> 3) : 0, used_h = logged ? d.i + 1 : 0;
+        if (side == 0) {  // right done: the left direction from the pair before
+          r_score = d.best;
+          r_bi = d.bi;
+          r_bj = d.bj;
+          r_cells = d.r_cells;
+          r_span = d.r_maxspan;
+          r_logged = logged;
+          r_n = ncur;
+          r_h = hcur;
+          ncur += used_n;
+          hcur += used_h;
+          side = 1;
+          dir_begin(d, Q + qm - 1, S + sm - 1, -1, qm, sm, INT32_MAX, M, ring, mask,
+                    nlog + nbase + ncur, hlog + hbase + hcur, int64_t(nlog_words - ncur) * 8,
+                    hlog_rows - hcur);
+          continue;
+        }
+        blastp_gapped o;
+        o.query_id = rec[cur].query_id;
+        o.subject_id = rec[cur].subject_id;
+        o.q_start = qm - d.bi;
+        o.q_end = qm + r_bi;
+        o.s_start = sm - d.bj;
+        o.s_end = sm + r_bj;
+        o.score = d.best + r_score;
+        o.ident = o.gap_opens = o.gap_len = 0;
+        rec[cur] = o;
+        status[cur] = 1;
+        if (o.score >= a.cutoff) {  // reported: traced by pass 2 from the logs or re-run
+          dinfo[2 * cur] = DirInfo{r_bi, r_bj, r_span, r_logged ? 1 : 0, nbase + r_n, hbase + r_h};
+          dinfo[2 * cur + 1] = DirInfo{d.bi, d.bj, d.r_maxspan, logged ? 1 : 0, nbase + ncur,
+                                       hbase + hcur};
+          if (!r_logged) need[2 * cur] = slab_bytes(r_bi + 1, r_cells, r_span);
+          if (!logged) need[2 * cur + 1] = slab_bytes(d.bi + 1, d.r_cells, d.r_maxspan);
+          ncur += used_n;
+          hcur += used_h;
+        } else {  // not reported: the logs forget both directions
+          ncur = n0;
+          hcur = h0;
+        }
+        phase = 0;
+      }
+    }
+    if (phase != 0) continue;
+    bool finished = false;
+    while (phase == 0) {  // the next HSP to extend
+      if (k >= g1) {
+        const unsigned long long w = atomicAdd(&counters[big ? kCurBig : kCurPass1], 1ull);
+        if (w >= ngroups) {
+          finished = true;
+          break;
+        }
+        g = big ? over_list[w] : int32_t(w);
+        g0 = k = gstart[g];
+        g1 = gstart[g + 1];
+        n0 = ncur;  // the pair's first log position (a redo rewinds to it)
+        h0 = hcur;
+        continue;
+      }
+      cur = k++;
+      status[cur] = 0;
+      need[2 * cur] = need[2 * cur + 1] = 0;
+      dinfo[2 * cur].logged = dinfo[2 * cur + 1].logged = 0;
+      const blastp_hsp h = a.hsps[perm[cur]];
+      Q = a.qcodes[h.query_id];
+      lq = a.qlens[h.query_id];
       const Subject sub = subject_of(a, int64_t(h.subject_id) - a.subject_base);
-      const int32_t qm = h.q_start + h.length / 2, sm = h.s_start + h.length / 2;  // R20
-      if (qm > lq || sm > sub.ls) {
+      S = sub.S;
+      ls = sub.ls;
+      qm = h.q_start + h.length / 2;  // R20
+      sm = h.s_start + h.length / 2;
+      if (qm > lq || sm > ls) {
         atomicOr(&counters[kErr], 2ull);
         continue;
       }
       bool inside = false;  // R21: the seed inside an earlier alignment's box
-      for (int32_t t = g0; t < k && !inside; ++t)
+      for (int32_t t = g0; t < cur && !inside; ++t)
         if (status[t]) {
           const blastp_gapped &b = rec[t];
           inside = b.q_start <= qm && qm < b.q_end && b.s_start <= sm && sm < b.s_end;
         }
       if (inside) continue;
-      const DirResult R = gapped_dir(Q + qm, sub.S + sm, 1, lq - qm, sub.ls - sm, M, a.gap_open,
-                                     a.gap_extend, a.xdrop, ring, mask, nullptr, nullptr, INT32_MAX);
-      if (R.overflow) {
-        over = true;
-        break;
-      }
-      const DirResult L = gapped_dir(Q + qm - 1, sub.S + sm - 1, -1, qm, sm, M, a.gap_open,
-                                     a.gap_extend, a.xdrop, ring, mask, nullptr, nullptr,
-                                     INT32_MAX);
-      if (L.overflow) {
-        over = true;
-        break;
-      }
-      blastp_gapped o;
-      o.query_id = h.query_id;
-      o.subject_id = h.subject_id;
-      o.q_start = qm - L.bi;
-      o.q_end = qm + R.bi;
-      o.s_start = sm - L.bj;
-      o.s_end = sm + R.bj;
-      o.score = L.score + R.score;
-      o.ident = o.gap_opens = o.gap_len = 0;
-      rec[k] = o;
-      status[k] = 1;
-      dinfo[2 * k] = DirInfo{R.bi, R.bj, R.maxspan, 0};
-      dinfo[2 * k + 1] = DirInfo{L.bi, L.bj, L.maxspan, 0};
-      if (o.score >= a.cutoff) {  // reported: its traceback is needed
-        need[2 * k] = slab_bytes(R.bi + 1, R.cells, R.maxspan);
-        need[2 * k + 1] = slab_bytes(L.bi + 1, L.cells, L.maxspan);
-      }
+      rec[cur].query_id = h.query_id;
+      rec[cur].subject_id = h.subject_id;
+      side = 0;
+      n0 = ncur;  // this HSP's first log position (forgotten if not reported)
+      h0 = hcur;
+      dir_begin(d, Q + qm, S + sm, 1, lq - qm, ls - sm, INT32_MAX, M, ring, mask,
+                nlog + nbase + ncur, hlog + hbase + hcur, int64_t(nlog_words - ncur) * 8,
+                hlog_rows - hcur);
+      phase = 1;
     }
-    if (over) {  // redo the whole pair with big rings
-      for (int32_t k = g0; k < g1; ++k) {
-        status[k] = 0;
-        need[2 * k] = need[2 * k + 1] = 0;
-      }
-      const unsigned long long slot = atomicAdd(&counters[kNumOver], 1ull);
-      over_list[slot] = g;
-    }
+    if (finished) break;
   }
 }
 
-// pass 2: per reported direction whose store starts in [base, base + window)
+// pass 2: per reported direction (work counter): a logged one is traced back
+// from pass 1's logs; one that was not, if its store starts in [base, base +
+// window), is re-run to its best row into that store and traced back.  One
+// DP cell or one traceback move per loop turn.
 __global__ void __launch_bounds__(128) gapped_trace_kernel(
     GappedArgs a, Matrix32 mat, const uint32_t *perm, blastp_gapped *rec, const DirInfo *dinfo,
-    const int64_t *need, const int64_t *off, int64_t base, int64_t window, uint8_t *store) {
+    const int64_t *need, const int64_t *off, int64_t base, int64_t window, uint8_t *store,
+    const uint32_t *nlog, const int2 *hlog, unsigned long long *cursor) {
   __shared__ int8_t M[32][32];
   load_matrix(M, mat);
-  for (int64_t t = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < 2 * a.n;
-       t += int64_t(gridDim.x) * blockDim.x) {
-    if (need[t] == 0 || off[t] < base || off[t] >= base + window) continue;
-    const int64_t k = t >> 1;
-    const bool right = (t & 1) == 0;
-    const blastp_hsp h = a.hsps[perm[k]];
-    const uint8_t *Q = a.qcodes[h.query_id];
-    const int32_t lq = a.qlens[h.query_id];
-    const Subject sub = subject_of(a, int64_t(h.subject_id) - a.subject_base);
-    const int32_t qm = h.q_start + h.length / 2, sm = h.s_start + h.length / 2;
-    const DirInfo di = dinfo[t];
-    uint8_t *slab = store + (off[t] - base);
-    int2 *hdr = reinterpret_cast<int2 *>(slab);
-    const int32_t rows = di.bi + 1;
-    const int64_t nib_bytes = need[t] - slab_hdr_bytes(rows) - int64_t(pow2_at_least(di.maxspan)) * 8;
-    uint8_t *nib = slab + slab_hdr_bytes(rows);
-    int2 *ring = reinterpret_cast<int2 *>(nib + nib_bytes);
-    const uint8_t *A = right ? Q + qm : Q + qm - 1;
-    const uint8_t *B = right ? sub.S + sm : sub.S + sm - 1;
-    const int step = right ? 1 : -1;
-    const int32_t la = right ? lq - qm : qm, lb = right ? sub.ls - sm : sm;
-    gapped_dir(A, B, step, la, lb, M, a.gap_open, a.gap_extend, a.xdrop, ring,
-               pow2_at_least(di.maxspan) - 1, nib, hdr, di.bi);
-    int32_t idn, gop, gl;
-    traceback(A, B, step, di.bi, di.bj, nib, hdr, &idn, &gop, &gl);
-    atomicAdd(&rec[k].ident, idn);
-    atomicAdd(&rec[k].gap_opens, gop);
-    atomicAdd(&rec[k].gap_len, gl);
+  const int32_t ge = a.gap_extend, goe = a.gap_open + a.gap_extend;
+  Dir d;
+  d.done = true;
+  Trace tr{0, 0, 0, 0, 0, 0};
+  int phase = 0;  // 0 fetch, 1 DP, 2 traceback
+  int64_t item = 0;
+  const uint32_t *nibw = nullptr;
+  const int2 *hdr = nullptr;
+  const uint8_t *A = nullptr, *B = nullptr;
+  int step = 1;
+  int2 *ring = nullptr;
+  int32_t mask = 0;
+  for (;;) {
+    if (phase == 0) {
+      bool got = false, logged = false;
+      while (!got) {
+        const unsigned long long t = atomicAdd(cursor, 1ull);
+        if (t >= static_cast<unsigned long long>(2 * a.n)) break;
+        item = int64_t(t);
+        if (need[item] > 0) {
+          got = off[item] >= base && off[item] < base + window;
+        } else if (base == 0) {
+          logged = got = dinfo[item].logged != 0;
+        }
+      }
+      if (!got) break;
+      const int64_t k = item >> 1;
+      const bool right = (item & 1) == 0;
+      const blastp_hsp h = a.hsps[perm[k]];
+      const uint8_t *Q = a.qcodes[h.query_id];
+      const int32_t lq = a.qlens[h.query_id];
+      const Subject sub = subject_of(a, int64_t(h.subject_id) - a.subject_base);
+      const int32_t qm = h.q_start + h.length / 2, sm = h.s_start + h.length / 2;
+      const DirInfo di = dinfo[item];
+      A = right ? Q + qm : Q + qm - 1;
+      B = right ? sub.S + sm : sub.S + sm - 1;
+      step = right ? 1 : -1;
+      tr = Trace{di.bi, di.bj, 0, 0, 0, 0};
+      if (logged) {
+        nibw = nlog + di.nib_off;
+        hdr = hlog + di.hdr_off;
+        phase = 2;
+        continue;
+      }
+      uint8_t *slab = store + (off[item] - base);
+      const int32_t rows = di.bi + 1, rcols = slab_ring_cols(di.maxspan);
+      int2 *shdr = reinterpret_cast<int2 *>(slab);
+      uint32_t *snib = reinterpret_cast<uint32_t *>(slab + slab_hdr_bytes(rows));
+      ring = reinterpret_cast<int2 *>(slab + need[item] - int64_t(rcols) * 8);
+      mask = rcols - 1;
+      dir_begin(d, A, B, step, right ? lq - qm : qm, right ? sub.ls - sm : sm, di.bi, M, ring,
+                mask, snib, shdr, INT64_MAX, INT32_MAX);
+      nibw = snib;
+      hdr = shdr;
+      phase = d.done ? 2 : 1;
+      continue;
+    }
+    if (phase == 1) {
+      dir_step(d, M, ring, mask, ge, goe, a.xdrop);
+      if (d.done) phase = 2;
+    } else if (trace_step(tr, A, B, step, nibw, hdr)) {
+      blastp_gapped *r = rec + (item >> 1);
+      atomicAdd(&r->ident, tr.ident);
+      atomicAdd(&r->gap_opens, tr.gopen);
+      atomicAdd(&r->gap_len, tr.glen);
+      phase = 0;
+    }
   }
 }
 
@@ -469,12 +629,21 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   if (a.n > int64_t(0x7ffffff0)) return cudaErrorInvalidValue;
   const int64_t n = a.n;
   const Matrix32 mat = host_matrix();
-  int32_t ring_small = 512;
+  int32_t ring_small = 256;
   if (const char *v = std::getenv("BLASTP_GAPPED_RING"))  // tests: force the big-ring pass
     ring_small = pow2_at_least(std::max(2, std::min(1 << 16, std::atoi(v))));
   const int32_t ring_big = pow2_at_least(int32_t(std::min<int64_t>(a.max_subject_len + 2, 1 << 30)));
   const int threads = 128;
-  const int blocks1 = num_sms * 4;
+  int bps = 4;  // pass-1 blocks of 128 per SM
+  if (const char *v = std::getenv("BLASTP_GAPPED_BPS")) bps = std::max(1, std::min(16, std::atoi(v)));
+  const int blocks1 = num_sms * bps;
+  // per-thread logs of pass 1's codes: nibble words and row headers (the
+  // nibble log in bytes; BLASTP_GAPPED_TBBUF=0: every direction re-run by pass 2)
+  int32_t tb_bytes = 16384;
+  if (const char *v = std::getenv("BLASTP_GAPPED_TBBUF"))
+    tb_bytes = std::max(0, std::min(1 << 20, std::atoi(v))) / 16 * 16;
+  const int32_t nlog_words = tb_bytes / 4, hlog_rows = tb_bytes / 16;
+  const bool verbose = std::getenv("BLASTP_GAPPED_VERBOSE") != nullptr;
   const int64_t t1 = int64_t(blocks1) * threads;
   const int64_t big_budget = int64_t(256) << 20;
   int64_t t2 = std::max<int64_t>(32, std::min<int64_t>(int64_t(num_sms) * 32,
@@ -485,7 +654,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   unsigned long long *key = nullptr, *key2 = nullptr, *counters = nullptr;
   uint32_t *val = nullptr, *perm = nullptr;
   blastp_gapped *rec = nullptr;
-  uint8_t *status = nullptr, *store = nullptr;
+  uint8_t *status = nullptr, *store = nullptr, *tbuf = nullptr;
   DirInfo *dinfo = nullptr;
   int64_t *need = nullptr, *off = nullptr, *goff = nullptr, *dmax = nullptr;
   int2 *scratch = nullptr, *scratch_big = nullptr;
@@ -494,7 +663,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   cudaError_t e = cudaSuccess;
   auto cleanup = [&]() {
     void *ptrs[] = {flag, gid, gstart, over, cnt, key, key2, counters, val, perm, rec, status,
-                    store, dinfo, need, off, goff, dmax, scratch, scratch_big, temp};
+                    store, tbuf, dinfo, need, off, goff, dmax, scratch, scratch_big, temp};
     for (void *p : ptrs)
       if (p) cudaFreeAsync(p, s);
   };
@@ -536,9 +705,14 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   GTRY(alloc(&goff, n, s));
   GTRY(alloc(&dmax, 1, s));
   GTRY(alloc(&scratch, size_t(t1) * ring_small, s));
+  GTRY(alloc(&tbuf, size_t(t1) * (size_t(nlog_words) * 4 + size_t(hlog_rows) * 8), s));
+  uint32_t *nlog = reinterpret_cast<uint32_t *>(tbuf);
+  int2 *hlog = reinterpret_cast<int2 *>(tbuf + size_t(t1) * size_t(nlog_words) * 4);
   GTRY(alloc(&temp, temp_bytes, s));
   GTRY(cudaMemsetAsync(counters, 0, kNumCounters * sizeof(unsigned long long), s));
   GTRY(cudaMemsetAsync(cnt, 0, size_t(n) * sizeof(int32_t), s));
+  GTRY(cudaMemsetAsync(dinfo, 0, size_t(2 * n) * sizeof(DirInfo), s));
+  GTRY(cudaMemsetAsync(need, 0, size_t(2 * n) * sizeof(int64_t), s));
 
   const int gb = int(std::min<int64_t>((n + 255) / 256, int64_t(num_sms) * 16));
   gapped_flags_kernel<<<gb, 256, 0, s>>>(a, flag, counters);
@@ -559,14 +733,17 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   }
   // pass 1, then the pairs that overflowed the small rings
   gapped_score_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, gstart, rec, status, dinfo, need,
-                                                  scratch, ring_small, over, false, counters);
+                                                  scratch, ring_small, nlog, nlog_words, hlog,
+                                                  hlog_rows, over, false,
+                                                  counters);
   GTRY(cudaGetLastError());
   GTRY(cudaMemcpyAsync(hc, counters, sizeof(hc), cudaMemcpyDeviceToHost, s));
   GTRY(cudaStreamSynchronize(s));
   if (hc[kNumOver] > 0) {
     GTRY(alloc(&scratch_big, size_t(t2) * size_t(ring_big), s));
     gapped_score_kernel<<<int(t2 / 32), 32, 0, s>>>(a, mat, perm, gstart, rec, status, dinfo, need,
-                                                    scratch_big, ring_big, over, true, counters);
+                                                    scratch_big, ring_big, nlog, 0, hlog, 0, over,
+                                                    true, counters);
     GTRY(cudaGetLastError());
   }
   // traceback stores: exclusive scan of the needs, total and largest one
@@ -586,16 +763,23 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
     return cudaSuccess;
   }
   const int64_t total = last[0] + last[1], maxneed = last[2];
-  if (total > 0) {
+  if (verbose)
+    fprintf(stderr, "gapped: %lld HSPs, %llu pairs, %llu pairs redone with %d-column rings "
+            "(small %d), traceback store %.1f MB (largest %lld B)\n", (long long)n,
+            hc[kNumGroups], hc[kNumOver], ring_big, ring_small, total / 1e6, (long long)maxneed);
+  {  // pass 2: the logged directions (first window) and the re-runs, window by window
     int64_t window = std::max<int64_t>(std::min<int64_t>(total, int64_t(2) << 30), maxneed);
     if (const char *v = std::getenv("BLASTP_GAPPED_STORE"))  // tests: force several windows
       window = std::max<int64_t>(maxneed, std::atoll(v));
-    GTRY(alloc(&store, size_t(window + maxneed), s));
+    window = std::max<int64_t>(window, 1);
+    if (total > 0) GTRY(alloc(&store, size_t(window + maxneed), s));
     const int64_t items = 2 * n;
     const int tblocks = int(std::min<int64_t>((items + threads - 1) / threads, int64_t(num_sms) * 8));
-    for (int64_t base = 0; base < total; base += window) {
+    for (int64_t base = 0; base == 0 || base < total; base += window) {
+      GTRY(cudaMemsetAsync(counters + kCurTrace, 0, sizeof(unsigned long long), s));
       gapped_trace_kernel<<<tblocks, threads, 0, s>>>(a, mat, perm, rec, dinfo, need, off, base,
-                                                       window, store);
+                                                       window, store, nlog, hlog,
+                                                       counters + kCurTrace);
       GTRY(cudaGetLastError());
     }
   }

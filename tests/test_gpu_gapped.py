@@ -92,11 +92,14 @@ def test_config3_gapped_full(bp, orc):
 
 
 @pytest.mark.parametrize("knobs", [{"BLASTP_GAPPED_RING": "16"}, {"BLASTP_GAPPED_RING": "64"},
-                                   {"BLASTP_GAPPED_STORE": "4096"}],
-                         ids=["ring16", "ring64", "store4k"])
+                                   {"BLASTP_GAPPED_TBBUF": "0", "BLASTP_GAPPED_STORE": "4096"},
+                                   {"BLASTP_GAPPED_TBBUF": "256"},
+                                   {"BLASTP_GAPPED_TBBUF": "1024", "BLASTP_GAPPED_RING": "32"}],
+                         ids=["ring16", "ring64", "pass2-store4k", "tbuf256", "tbuf1k-ring32"])
 def test_ring_overflow_and_store_windows(bp, orc, monkeypatch, knobs):
     """Pairs whose DP rows outgrow the per-thread ring are redone with
-    subject-sized rings; traceback stores split into several windows: same
+    subject-sized rings; directions whose codes outgrow the per-thread store
+    are traced by pass 2, whose stores split into several windows: same
     results."""
     for k, v in knobs.items():
         monkeypatch.setenv(k, v)
