@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cstdarg>
+#include <cstdint>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -783,37 +784,48 @@ static int check_pair(const blastp_query_table *q, const blastp_db *db, const bl
   return BLASTP_OK;
 }
 
-// Enqueue the search of every query of `q` against `db`: HSPs appended to
+// The search launches of a table ("units"): a batch's query groups (one scan
+// per group) when the two-hit window fits the sentinel gap they were built
+// with, and the queries left alone; traced runs search query by query.
+// ids[u] = the query id of a single-query unit, -1 for a group.
+static void launch_units(const blastp_query_table *q, const blastp_params *p, bool traced,
+                         std::vector<const QueryDev *> *list, std::vector<int32_t> *ids) {
+  list->clear();
+  ids->clear();
+  if (!q->groups.empty() && !traced && p->window + 8 <= q->group_gap) {
+    for (const QueryDev &g : q->groups) {
+      list->push_back(&g);
+      ids->push_back(-1);
+    }
+    for (int32_t i : q->alone) {
+      list->push_back(&q->q[static_cast<size_t>(i)]);
+      ids->push_back(i);
+    }
+  } else {
+    for (size_t i = 0; i < q->q.size(); ++i) {
+      list->push_back(&q->q[i]);
+      ids->push_back(static_cast<int32_t>(i));
+    }
+  }
+}
+
+// Enqueue the search of every query of `q` against `db` (or of the launch
+// units [unit_begin, unit_end) only): HSPs appended to
 // out (capacity cap) with the count in *count (device).  trace: optional.
 static int enqueue_search(const blastp_query_table *q, const blastp_db *db,
                           const blastp_params *p, cudaStream_t s, blastp_hsp *out, int64_t cap,
                           unsigned long long *count, TraceRec *const trace[3],
                           const int64_t trace_cap[3], unsigned long long *trace_count,
-                          bool reset_count = true, bool out_fence = false) {
+                          bool reset_count = true, bool out_fence = false,
+                          size_t unit_begin = 0, size_t unit_end = SIZE_MAX) {
   if (reset_count) CUDA_TRY(cudaMemsetAsync(count, 0, sizeof(unsigned long long), s));
   if (trace_count)  // [0..3): trace record counts, [3..3+kNumStats): event counters
     CUDA_TRY(cudaMemsetAsync(trace_count, 0, (3 + kNumStats) * sizeof(unsigned long long), s));
   if (db->nchunks == 0) return BLASTP_OK;
-  // a batch's query groups (one scan per group) when the two-hit window fits
-  // the sentinel gap they were built with; traced runs search query by query
   std::vector<const QueryDev *> list;
   std::vector<int32_t> ids;
-  if (!q->groups.empty() && trace == nullptr && p->window + 8 <= q->group_gap) {
-    for (const QueryDev &g : q->groups) {
-      list.push_back(&g);
-      ids.push_back(-1);
-    }
-    for (int32_t i : q->alone) {
-      list.push_back(&q->q[static_cast<size_t>(i)]);
-      ids.push_back(i);
-    }
-  } else {
-    for (size_t i = 0; i < q->q.size(); ++i) {
-      list.push_back(&q->q[i]);
-      ids.push_back(static_cast<int32_t>(i));
-    }
-  }
-  for (size_t li = 0; li < list.size(); ++li) {
+  launch_units(q, p, trace != nullptr, &list, &ids);
+  for (size_t li = unit_begin; li < list.size() && li < unit_end; ++li) {
     const QueryDev &qd = *list[li];
     SearchArgs a{};
     a.stream = db->stream;
@@ -1625,6 +1637,157 @@ int blastp_gapped_extend_device(const blastp_query_table *q, const blastp_db *db
                        capacity, out_count);
 }
 
+// Fig. 12's overlap on one GPU: the search of launch unit
+// u + 1 (a query group or a lone query) runs on stream s while the gapped
+// stage of unit u runs on a second stream; two unit buffers alternate.
+// Results are gathered on the host and put in canonical order.  Synchronous.
+static int search_gapped_pipelined(const blastp_query_table *q, const blastp_db *db,
+                                   const blastp_params *p, const blastp_gapped_params *gp,
+                                   cudaStream_t s, std::vector<blastp_gapped> *gout,
+                                   std::vector<blastp_hsp> *uout, bool want_ungapped) {
+  std::vector<const QueryDev *> list;
+  std::vector<int32_t> ids;
+  launch_units(q, p, false, &list, &ids);
+  const size_t U = list.size();
+  int32_t max_members = 1;
+  for (const QueryDev *u : list) max_members = std::max(max_members, std::max(u->nsub, 1));
+  int64_t cap = std::max<int64_t>(4096, (db->residues / 1000 + 1) * max_members);
+  if (const char *v = std::getenv("BLASTP_PIPE_CAP"))  // tests: force the overflow re-run
+    cap = std::max<int64_t>(1, std::atoll(v));
+  cudaStream_t s2 = nullptr;
+  CUDA_TRY(cudaStreamCreateWithFlags(&s2, cudaStreamNonBlocking));
+  blastp_hsp *buf[2] = {nullptr, nullptr};
+  int64_t bcap[2] = {0, 0};
+  unsigned long long *cnt = nullptr;
+  blastp_gapped *gbuf = nullptr;
+  int64_t gcap = 0;
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+  int rc = BLASTP_OK;
+  auto cleanup = [&]() {
+    cudaStreamSynchronize(s);
+    cudaStreamSynchronize(s2);
+    for (int k = 0; k < 2; ++k) {
+      if (buf[k]) cudaFree(buf[k]);
+      if (ev[k]) cudaEventDestroy(ev[k]);
+    }
+    if (cnt) cudaFree(cnt);
+    if (gbuf) cudaFree(gbuf);
+    cudaStreamDestroy(s2);
+  };
+  auto grow = [&](int k, int64_t want) -> bool {
+    if (bcap[k] >= want) return true;
+    if (buf[k]) cudaFree(buf[k]);
+    buf[k] = nullptr;
+    bcap[k] = 0;
+    if (cudaMalloc(&buf[k], sizeof(blastp_hsp) * static_cast<size_t>(want)) != cudaSuccess) return false;
+    bcap[k] = want;
+    return true;
+  };
+  if (!grow(0, cap) || !grow(1, cap) ||
+      cudaMalloc(&cnt, 2 * sizeof(unsigned long long)) != cudaSuccess ||
+      cudaEventCreateWithFlags(&ev[0], cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&ev[1], cudaEventDisableTiming) != cudaSuccess) {
+    cleanup();
+    return fail(BLASTP_E_NOMEM, "pipeline buffers");
+  }
+  auto enqueue_unit = [&](size_t u, cudaStream_t st) -> int {
+    const int k = int(u & 1);
+    int r = enqueue_search(q, db, p, st, buf[k], bcap[k], cnt + k, nullptr, nullptr, nullptr,
+                           true, false, u, u + 1);
+    if (!r && cudaEventRecord(ev[k], st) != cudaSuccess) r = fail(BLASTP_E_CUDA, "event record");
+    return r;
+  };
+  rc = enqueue_unit(0, s);
+  for (size_t u = 0; u < U && rc == BLASTP_OK; ++u) {
+    const int k = int(u & 1);
+    // the next unit's search goes ahead on s while this one is extended on s2
+    if (u + 1 < U && (rc = enqueue_unit(u + 1, s))) break;
+    unsigned long long n = 0;
+    cudaError_t e = cudaStreamWaitEvent(s2, ev[k], 0);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&n, cnt + k, sizeof(n), cudaMemcpyDeviceToHost, s2);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s2);
+    if (e != cudaSuccess) {
+      rc = fail(BLASTP_E_CUDA, "pipeline unit %zu: %s", u, cudaGetErrorString(e));
+      break;
+    }
+    if (static_cast<int64_t>(n) > bcap[k]) {
+      // overflow: drain s (the next unit's search shares the db's chunk
+      // cursor), grow and re-run this unit on s2
+      if ((e = cudaStreamSynchronize(s)) != cudaSuccess) {
+        rc = fail(BLASTP_E_CUDA, "pipeline drain: %s", cudaGetErrorString(e));
+        break;
+      }
+      if (!grow(k, static_cast<int64_t>(n) + static_cast<int64_t>(n) / 4 + 1024)) {
+        rc = fail(BLASTP_E_NOMEM, "pipeline unit buffer (%llu HSPs)", n);
+        break;
+      }
+      if ((rc = enqueue_search(q, db, p, s2, buf[k], bcap[k], cnt + k, nullptr, nullptr, nullptr,
+                               true, false, u, u + 1)))
+        break;
+      e = cudaMemcpyAsync(&n, cnt + k, sizeof(n), cudaMemcpyDeviceToHost, s2);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s2);
+      if (e != cudaSuccess) {
+        rc = fail(BLASTP_E_CUDA, "pipeline re-run: %s", cudaGetErrorString(e));
+        break;
+      }
+    }
+    int64_t m = static_cast<int64_t>(n);
+    if (p->ext_mode == BLASTP_EXT_HIT_DEDUP) {
+      e = dedup_covered(buf[k], m, p->cutoff, reinterpret_cast<int64_t *>(cnt + k), s2);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&m, cnt + k, sizeof(m), cudaMemcpyDeviceToHost, s2);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s2);
+    } else {
+      e = sort_hsps(buf[k], m, s2);
+    }
+    if (e != cudaSuccess) {
+      rc = e == cudaErrorMemoryAllocation ? fail(BLASTP_E_NOMEM, "sort scratch")
+                                          : fail(BLASTP_E_CUDA, "sort: %s", cudaGetErrorString(e));
+      break;
+    }
+    if (gcap < std::max<int64_t>(m, 1)) {
+      if (gbuf) cudaFree(gbuf);
+      gbuf = nullptr;
+      gcap = 0;
+      if (cudaMalloc(&gbuf, sizeof(blastp_gapped) * static_cast<size_t>(std::max<int64_t>(m, 1))) != cudaSuccess) {
+        rc = fail(BLASTP_E_NOMEM, "gapped output");
+        break;
+      }
+      gcap = std::max<int64_t>(m, 1);
+    }
+    int64_t g = 0;
+    if ((rc = gapped_device(q, db, buf[k], m, gp, s2, gbuf, gcap, &g))) break;
+    const size_t g0 = gout->size(), u0 = uout->size();
+    gout->resize(g0 + static_cast<size_t>(g));
+    if (want_ungapped) uout->resize(u0 + static_cast<size_t>(m));
+    e = cudaSuccess;
+    if (g > 0) e = cudaMemcpyAsync(gout->data() + g0, gbuf, sizeof(blastp_gapped) * size_t(g), cudaMemcpyDeviceToHost, s2);
+    if (e == cudaSuccess && want_ungapped && m > 0)
+      e = cudaMemcpyAsync(uout->data() + u0, buf[k], sizeof(blastp_hsp) * size_t(m), cudaMemcpyDeviceToHost, s2);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s2);
+    if (e != cudaSuccess) {
+      rc = fail(BLASTP_E_CUDA, "pipeline results: %s", cudaGetErrorString(e));
+      break;
+    }
+  }
+  cleanup();
+  if (rc) return rc;
+  // units partition the queries and each unit's list is canonical: a stable
+  // counting sort by query id gives the canonical order of the whole
+  const size_t nq = q->q.size();
+  auto by_query = [nq](auto &v) {
+    using T = typename std::decay<decltype(v)>::type::value_type;
+    std::vector<size_t> start(nq + 1, 0);
+    for (const T &r : v) ++start[static_cast<size_t>(r.query_id) + 1];
+    for (size_t i = 0; i < nq; ++i) start[i + 1] += start[i];
+    std::vector<T> out(v.size());
+    for (const T &r : v) out[start[static_cast<size_t>(r.query_id)]++] = r;
+    v.swap(out);
+  };
+  by_query(*gout);
+  if (want_ungapped) by_query(*uout);
+  return BLASTP_OK;
+}
+
 int blastp_search_gapped(const blastp_query_table *q, const blastp_db *db,
                          const blastp_params *p, const blastp_gapped_params *gp,
                          void *cuda_stream, blastp_gapped **out_host, int64_t *out_count,
@@ -1639,6 +1802,33 @@ int blastp_search_gapped(const blastp_query_table *q, const blastp_db *db,
   if ((rc = validate_gapped(gp))) return rc;
   DeviceGuard g(db->device);
   cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+  std::vector<const QueryDev *> list;
+  std::vector<int32_t> ids;
+  launch_units(q, p, false, &list, &ids);
+  // BLASTP_GAPPED_PIPE=1: Fig. 12's overlap across launch units (measured
+  // slower on one B200 -- both stages fill every SM, DESIGN.md 5.11 -- so the
+  // default runs the two stages one after the other)
+  const char *pipe = std::getenv("BLASTP_GAPPED_PIPE");
+  if (list.size() > 1 && db->nchunks > 0 && pipe && std::atoi(pipe) == 1) {
+    std::vector<blastp_gapped> gv;
+    std::vector<blastp_hsp> uv;
+    if ((rc = search_gapped_pipelined(q, db, p, gp, s, &gv, &uv, ungapped_host != nullptr))) return rc;
+    auto *h = static_cast<blastp_gapped *>(malloc(sizeof(blastp_gapped) * std::max<size_t>(gv.size(), 1)));
+    blastp_hsp *u = nullptr;
+    if (ungapped_host) u = static_cast<blastp_hsp *>(malloc(sizeof(blastp_hsp) * std::max<size_t>(uv.size(), 1)));
+    if (!h || (ungapped_host && !u)) {
+      free(h);
+      free(u);
+      return fail(BLASTP_E_NOMEM, "host result arrays");
+    }
+    std::copy(gv.begin(), gv.end(), h);
+    if (u) std::copy(uv.begin(), uv.end(), u);
+    *out_host = h;
+    *out_count = static_cast<int64_t>(gv.size());
+    if (ungapped_host) *ungapped_host = u;
+    if (ungapped_count) *ungapped_count = static_cast<int64_t>(uv.size());
+    return BLASTP_OK;
+  }
   int64_t n = 0;
   if ((rc = search_sorted_device(q, db, p, s, &n))) return rc;
   blastp_gapped *d_out = nullptr;

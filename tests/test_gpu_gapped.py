@@ -215,3 +215,28 @@ def test_errors_and_capacity(bp, orc):
         bp.gapped_extend_device(t, d, dev.data_ptr(), len(u), out.data_ptr(), len(u),
                                 bp.GappedParams(gap_extend=0))
     assert bp.gapped_extend_device(t, d, dev.data_ptr(), 0, out.data_ptr(), len(u)) == 0
+
+
+@pytest.mark.parametrize("knobs", [{}, {"BLASTP_PIPE_CAP": "7"}], ids=["pipe", "pipe-overflow"])
+def test_batch_pipeline_equals_sequential_and_oracle(bp, orc, monkeypatch, knobs):
+    """Fig. 12's overlap: a batch whose launch units (query groups, lone
+    queries) are searched on one stream while the previous unit is gapped on
+    another gives the oracle's result, as the sequential two-stage run does;
+    unit buffers that overflow are regrown and the unit re-run."""
+    from synth import gen_queries
+    queries = gen_queries(77, 12, 100, 900)
+    db = gen_db(78, 79, n_subjects=2500, mean_len=300.0, queries=queries, plant_frac=0.2)
+    t = bp.build_query_batch(queries)
+    assert t.groups[0] >= 1
+    d = bp.pack_db(db.ascii, db.offsets)
+    for k, v in knobs.items():
+        monkeypatch.setenv(k, v)
+    monkeypatch.setenv("BLASTP_GAPPED_PIPE", "1")
+    got, ung = bp.search_gapped(t, d, want_ungapped=True)
+    monkeypatch.setenv("BLASTP_GAPPED_PIPE", "0")
+    seq, sung = bp.search_gapped(t, d, want_ungapped=True)
+    assert_same(got, seq, "pipelined vs sequential")
+    assert (ung == sung).all()
+    u, exp = oracle_gapped(orc, queries, db.ascii, db.offsets, bp.GappedParams())
+    assert_same(got, exp, "pipelined vs oracle")
+    assert len(exp) > 100
