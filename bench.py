@@ -60,6 +60,8 @@ def parse_args():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-gapped", action="store_true",
+                    help="skip the gapped-stage measurement (SURVEY 8(f) rank 4)")
     ap.add_argument("--gather", choices=["p2p", "nccl"], default="p2p",
                     help="N > 1: HSPs appended by the search kernels into rank 0's buffer over "
                          "NVLink (CUDA IPC), or per-rank lists gathered with NCCL")
@@ -563,6 +565,38 @@ def main():
                            "blastp_search_ungapped_device on the HBM-resident shard + "
                            + ("NCCL gather + " if world > 1 else "") + "D2H of the HSP list"}
 
+    # ---- the gapped consumer of this step's HSP list,
+    # outside the headline: the rank's own list sorted (R11), then
+    # blastp_gapped_extend_device timed with CUDA events on the stream
+    gapped = None
+    if not args.no_gapped and hasattr(bp.lib, "blastp_gapped_extend_device") and peer is None:
+        try:
+            search()
+            torch.cuda.synchronize()
+            ng = int(cnt.item())
+            hs = out[:ng].clone()
+            bp.sort_hsps_device(hs.data_ptr(), ng, stream)
+            gout = torch.empty((max(ng, 1), 10), dtype=torch.int32, device=dev)
+            gms = []
+            for k in range(4):
+                g0 = torch.cuda.Event(enable_timing=True)
+                g1 = torch.cuda.Event(enable_timing=True)
+                g0.record(stream)
+                m = bp.gapped_extend_device(table, gdb, hs.data_ptr(), ng, gout.data_ptr(), ng,
+                                            stream=stream)
+                g1.record(stream)
+                torch.cuda.synchronize()
+                if k > 0:
+                    gms.append(g0.elapsed_time(g1))
+            gmean = statistics.mean(gms)
+            gapped = {"hsps_in": ng, "alignments_out": int(m), "ms": gmean,
+                      "hsps_per_s": ng / (gmean / 1e3),
+                      "path": "blastp_gapped_extend_device on the rank's canonical device HSP "
+                              "list (affine Gotoh X-drop, R18-R22; 3 timed calls after 1 warm-up)"}
+            del hs, gout
+        except Exception as ex:  # noqa: BLE001 -- a report beside the headline
+            gapped = {"error": str(ex)}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = oracle_rate(queries, db, steps=3, warmup=1)
@@ -604,6 +638,7 @@ def main():
             "gpu_launches": args.steps * (table.launches(params)
                                           if hasattr(table, "launches") else nq),
             "cpu_baseline": cpu,
+            "gapped_stage": gapped,
         }
         print(json.dumps(line), flush=True)
     if peer is not None:
