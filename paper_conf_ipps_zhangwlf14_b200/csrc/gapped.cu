@@ -234,6 +234,8 @@ __device__ __forceinline__ void dir_step(Dir &d, const int8_t (*M)[32], int2 *ri
   } else if (j > d.phi && j > 0) {
     row_end = true;  // dead and beyond the previous row's live cells: the row ends
   }
+  // (the row end as selects for every lane plus a small branch for its loads
+  // and stores measured the same: 51.6 vs 51.2 ms)
   if (row_end) dir_end_row(d, M, ring, mask);
   else d.j = j + 1;
 }
