@@ -38,6 +38,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cassert>
 #include <cstdio>
 #include <cstdlib>
 
@@ -48,6 +49,14 @@ namespace blastp {
 namespace {
 
 constexpr int32_t kNeg = INT32_MIN / 4;  // -infinity that survives a few subtractions
+
+// -DGAPPED_CHECK: device asserts on every sequence read and store index (the
+// bounds-checked build the tests run besides the product build)
+#ifdef GAPPED_CHECK
+#define GCHECK(c) assert(c)
+#else
+#define GCHECK(c) ((void)0)
+#endif
 
 // counters[]
 enum { kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kNumCounters = 8 };
@@ -111,7 +120,10 @@ struct Dir {
 };
 
 __device__ __forceinline__ void dir_finish(Dir &d) {
-  if (d.nibw && (d.nc & 7)) d.nibw[d.nc >> 3] = d.nword;
+  if (d.nibw && (d.nc & 7)) {
+    GCHECK(d.nc - 1 < d.cap_cells);
+    d.nibw[d.nc >> 3] = d.nword;
+  }
   d.done = true;
 }
 
@@ -137,11 +149,13 @@ __device__ __forceinline__ void dir_end_row(Dir &d, const int8_t (*M)[32], const
   }
   d.lo = d.hi = -1;
   d.lh = d.le = d.dh = kNeg;
+  GCHECK(d.i - 1 < d.la);
   d.mrow = M[d.A[int64_t(d.i - 1) * d.step]];
   if (d.nibw) {
     if (d.cum + mask + 1 > d.cap_cells || d.i >= d.cap_rows) {
       d.nibw = nullptr;  // this row might not fit: no traceback store for this direction
     } else {
+      GCHECK(d.i < d.cap_rows);
       d.hdr[d.i] = make_int2(d.start, int32_t(d.cum));
     }
   }
@@ -193,6 +207,7 @@ __device__ __forceinline__ void dir_step(Dir &d, const int8_t (*M)[32], int2 *ri
   // (loading the next cell's ring entry and residue one step ahead, carried
   // in registers, measured 5x slower: 300 vs 62 ms at config 3)
   const int2 up = (j <= d.phi) ? ring[j & mask] : make_int2(kNeg, kNeg);
+  GCHECK(j <= d.lb && j >= d.start && (j <= d.phi || j > 0 || d.i == 0));
   const int32_t bres = j > 0 ? d.B[int64_t(j - 1) * d.step] : 0;
   const int32_t e = j > 0 ? imax(d.le - ge, d.lh - goe) : kNeg;
   const int32_t f = imax(up.y - ge, up.x - goe);
@@ -220,6 +235,7 @@ __device__ __forceinline__ void dir_step(Dir &d, const int8_t (*M)[32], int2 *ri
                                    (e == d.lh - goe ? 4 : 0) | (f == up.x - goe ? 8 : 0));
     d.nword |= code << ((d.nc & 7) * 4);
     if ((d.nc & 7) == 7) {
+      GCHECK(d.nc < d.cap_cells);
       d.nibw[d.nc >> 3] = d.nword;
       d.nword = 0;
     }
@@ -550,8 +566,11 @@ __global__ void __launch_bounds__(128) gapped_trace_kernel(
       uint32_t *snib = reinterpret_cast<uint32_t *>(slab + slab_hdr_bytes(rows));
       ring = reinterpret_cast<int2 *>(slab + need[item] - int64_t(rcols) * 8);
       mask = rcols - 1;
+      // the store's capacities: rows 0..bi and their cells fit by construction
+      // (+ one ring width: the per-row check is conservative by a row's span)
+      const int64_t scells = (need[item] - slab_hdr_bytes(rows) - int64_t(rcols) * 8) * 2;
       dir_begin(d, A, B, step, right ? lq - qm : qm, right ? sub.ls - sm : sm, di.bi, M, ring,
-                mask, snib, shdr, INT64_MAX, INT32_MAX);
+                mask, snib, shdr, scells + mask + 1, rows);
       nibw = snib;
       hdr = shdr;
       phase = d.done ? 2 : 1;
