@@ -25,6 +25,7 @@ from typing import Callable
 import numpy as np
 
 HSP_FIELDS = 7
+GAPPED_FIELDS = 10  # blastp_gapped records (the gapped consumer)
 
 
 def shard_subjects(offsets: np.ndarray, rank: int, world: int) -> tuple[int, int]:
@@ -44,8 +45,9 @@ def shard_subjects(offsets: np.ndarray, rank: int, world: int) -> tuple[int, int
     return lo, max(lo, hi)
 
 
-def gather_hsps(local, group=None, dst: int = 0):
-    """Gather [n_r, 7] int32 HSP tensors of every rank onto rank `dst`.
+def gather_hsps(local, group=None, dst: int = 0, fields: int = HSP_FIELDS):
+    """Gather [n_r, fields] int32 record tensors of every rank onto rank `dst`
+    (HSPs: 7 fields; gapped alignments: 10, gather_gapped).
 
     Returns the concatenation in rank order on rank dst (None elsewhere).
     One collective for the counts (all_gather_into_tensor of one int64 per
@@ -64,7 +66,7 @@ def gather_hsps(local, group=None, dst: int = 0):
         return local
     if local.is_cuda and dist.get_backend(group) != "nccl":
         # gloo (functional multi-rank checks on one device): collectives on host
-        out = gather_hsps(local.cpu(), group, dst)
+        out = gather_hsps(local.cpu(), group, dst, fields)
         return None if out is None else out.to(local.device)
     dev = local.device
     n = torch.tensor([local.shape[0]], dtype=torch.int64, device=dev)
@@ -75,7 +77,7 @@ def gather_hsps(local, group=None, dst: int = 0):
     ops = []
     out = None
     if rank == dst:
-        out = local.new_empty((sum(counts), HSP_FIELDS))
+        out = local.new_empty((sum(counts), fields))
         offs = np.concatenate([[0], np.cumsum(counts)]).astype(np.int64)
         for r in range(world):
             if counts[r] == 0:
@@ -91,6 +93,26 @@ def gather_hsps(local, group=None, dst: int = 0):
         for req in dist.batch_isend_irecv(ops):
             req.wait()
     return out
+
+
+def gather_gapped(local, group=None, dst: int = 0):
+    """gather_hsps for [n_r, 10] int32 gapped alignments.  Shards partition
+    the subjects and a (query, subject) pair's alignments are made on the
+    shard holding the subject, so the rank-order concatenation is the whole
+    database's gapped list (canonical for one query; batches re-sort by
+    query id)."""
+    return gather_hsps(local, group, dst, GAPPED_FIELDS)
+
+
+def gapped_sharded(gapped_fn: Callable[[int, int], "object"], offsets: np.ndarray, group=None,
+                   dst: int = 0):
+    """Run `gapped_fn(lo, hi)` (search + gapped stage of this rank's shard,
+    a [n, 10] int32 tensor with GLOBAL subject ids) and gather to rank dst."""
+    import torch.distributed as dist
+    rank = dist.get_rank(group)
+    world = dist.get_world_size(group)
+    lo, hi = shard_subjects(offsets, rank, world)
+    return gather_gapped(gapped_fn(lo, hi), group=group, dst=dst)
 
 
 def search_sharded(search_fn: Callable[[int, int], "object"], offsets: np.ndarray, group=None,

@@ -79,3 +79,45 @@ def test_shard_subjects_matches_c_abi():
     for world in (1, 2, 4, 8, 16):
         for k in range(world):
             assert shard_subjects(off, k, world) == bp.shard_range(off, k, world)
+
+
+def _gapped_worker(rank, world, port, q, ascii, offsets, result_path):
+    sys.path.insert(0, ROOT)
+    from oracle import oracle as o
+    from paper_conf_ipps_zhangwlf14_b200.dist import gapped_sharded
+
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank,
+                            world_size=world)
+    try:
+        def gapped_fn(lo, hi):
+            sub = offsets[lo:hi + 1]
+            codes = o.encode(ascii[sub[0]:sub[-1]].tobytes())
+            r = o.search(o.encode(q), codes, sub - sub[0], subject_base=lo)
+            g = o.gapped_hsps([o.encode(q)], codes, sub - sub[0], r.hsps, subject_base=lo)
+            return torch.from_numpy(g.view(np.int32).reshape(-1, 10).copy())
+
+        out = gapped_sharded(gapped_fn, offsets)
+        if rank == 0:
+            np.save(result_path, out.numpy())
+        else:
+            assert out is None
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_gapped_gather_equals_whole_db(orc, tmp_path, world):
+    """The gapped consumer per shard (the oracle standing in for each rank's
+    GPU stage) gathered to rank 0 equals the gapped stage over the whole
+    database: (query, subject) pairs never span shards."""
+    from synth import config_workload
+    (q,), db = config_workload(1)
+    codes = orc.encode(db.ascii.tobytes())
+    u = orc.search(orc.encode(q), codes, db.offsets).hsps
+    whole = orc.gapped_hsps([orc.encode(q)], codes, db.offsets, u)
+    path = str(tmp_path / "gapped.npy")
+    mp.spawn(_gapped_worker, args=(world, _free_port(), q, db.ascii, db.offsets, path),
+             nprocs=world, join=True)
+    got = np.load(path)
+    exp = whole.view(np.int32).reshape(-1, 10)
+    assert len(got) == len(exp) > 10 and (got == exp).all()
