@@ -59,7 +59,9 @@ constexpr int32_t kNeg = INT32_MIN / 4;  // -infinity that survives a few subtra
 #endif
 
 // counters[]
-enum { kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kNumCounters = 8 };
+enum {
+  kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kCurFirst, kNumCounters = 9
+};
 
 // a reported direction for pass 2: its best cell, widest span, and whether
 // pass 1 logged its codes (then at nib_off / hdr_off of the logs)
@@ -360,8 +362,135 @@ __global__ void gapped_keys_kernel(GappedArgs a, const int32_t *flag, const int3
   }
 }
 
-// pass 1: one thread per pair (work counter), or per pair of the overflow
-// list (big rings).  The thread's pairs, their HSPs (R21 order) and both
+// One direction of a pair's first HSP (R21: the top-scored one, never
+// inside an earlier box), pass 1a.
+struct FirstDir {
+  int32_t score, bi, bj, maxspan, logged, overflow;
+  int64_t cells, nib_off, hdr_off;
+};
+
+// pass 1a: every HSP's two directions as independent work items (item 2k:
+// right, 2k + 1: left of the k-th HSP in R21 order), one DP cell per loop
+// turn, codes appended to the thread's logs.  An alignment depends only on
+// its own HSP; whether it is used (R21: its seed outside the boxes of the
+// pair's earlier alignments) is decided afterwards by gapped_resolve_kernel,
+// so a pair's HSPs run in parallel instead of as one thread's chain (the
+// chain form left a 25 ms tail of pairs with many HSPs at config 3).  A
+// direction outgrowing the ring sends its pair to the big-ring pass.
+__global__ void __launch_bounds__(128) gapped_first_kernel(
+    GappedArgs a, Matrix32 mat, const uint32_t *perm, const int32_t *gstart, FirstDir *fd,
+    int2 *scratch, int32_t ring_cols, uint32_t *nlog, int32_t nlog_words, int2 *hlog,
+    int32_t hlog_rows, unsigned long long *counters) {
+  __shared__ int8_t M[32][32];
+  load_matrix(M, mat);
+  const int64_t tid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+  int2 *ring = scratch + tid * ring_cols;
+  const int64_t nbase = tid * nlog_words, hbase = tid * hlog_rows;
+  int32_t ncur = 0, hcur = 0;
+  const int32_t mask = ring_cols - 1, ge = a.gap_extend, goe = a.gap_open + a.gap_extend;
+  const unsigned long long nitems = 2 * static_cast<unsigned long long>(a.n);
+  Dir d;
+  d.done = true;
+  bool active = false;
+  unsigned long long item = 0;
+  for (;;) {
+    if (active && !d.done) {  // the common turn: one cell, straight back to the top
+      dir_step(d, M, ring, mask, ge, goe, a.xdrop);
+      if (!d.done) continue;
+    }
+    if (active) {
+      FirstDir f;
+      f.score = d.best;
+      f.bi = d.bi;
+      f.bj = d.bj;
+      f.maxspan = d.r_maxspan;
+      f.cells = d.r_cells;
+      f.overflow = d.overflow ? 1 : 0;
+      f.logged = d.nibw != nullptr && !d.overflow ? 1 : 0;
+      f.nib_off = nbase + ncur;
+      f.hdr_off = hbase + hcur;
+      if (f.logged) {
+        ncur += int32_t((d.nc + 7) >> 3);
+        hcur += d.i + 1;
+      }
+      fd[item] = f;
+      active = false;
+    }
+    item = atomicAdd(&counters[kCurFirst], 1ull);
+    if (item >= nitems) break;
+    const blastp_hsp h = a.hsps[perm[item >> 1]];
+    const uint8_t *Q = a.qcodes[h.query_id];
+    const int32_t lq = a.qlens[h.query_id];
+    const Subject sub = subject_of(a, int64_t(h.subject_id) - a.subject_base);
+    const int32_t qm = h.q_start + h.length / 2, sm = h.s_start + h.length / 2;  // R20
+    if (qm > lq || sm > sub.ls) {
+      atomicOr(&counters[kErr], 2ull);
+      continue;
+    }
+    if ((item & 1) == 0)
+      dir_begin(d, Q + qm, sub.S + sm, 1, lq - qm, sub.ls - sm, INT32_MAX, M, ring, mask,
+                nlog + nbase + ncur, hlog + hbase + hcur, int64_t(nlog_words - ncur) * 8,
+                hlog_rows - hcur);
+    else
+      dir_begin(d, Q + qm - 1, sub.S + sm - 1, -1, qm, sm, INT32_MAX, M, ring, mask,
+                nlog + nbase + ncur, hlog + hbase + hcur, int64_t(nlog_words - ncur) * 8,
+                hlog_rows - hcur);
+    active = true;
+  }
+}
+
+// pass 1b: per pair, R21 over the alignments of pass 1a in the pair's order:
+// an HSP whose seed lies in the box of an earlier kept alignment is skipped;
+// pairs with an overflowing direction go to the big-ring pass.
+__global__ void gapped_resolve_kernel(GappedArgs a, const uint32_t *perm, const int32_t *gstart,
+                                      const FirstDir *fd, blastp_gapped *rec, uint8_t *status,
+                                      DirInfo *dinfo, int64_t *need, int32_t *over_list,
+                                      unsigned long long *counters) {
+  const int64_t ng = int64_t(counters[kNumGroups]);
+  for (int64_t g = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; g < ng;
+       g += int64_t(gridDim.x) * blockDim.x) {
+    const int32_t g0 = gstart[g], g1 = gstart[g + 1];
+    bool over = false;
+    for (int32_t k = g0; k < g1 && !over; ++k) over = fd[2 * k].overflow || fd[2 * k + 1].overflow;
+    if (over) {
+      over_list[atomicAdd(&counters[kNumOver], 1ull)] = int32_t(g);
+      continue;
+    }
+    for (int32_t k = g0; k < g1; ++k) {
+      const blastp_hsp h = a.hsps[perm[k]];
+      const int32_t qm = h.q_start + h.length / 2, sm = h.s_start + h.length / 2;  // R20
+      bool inside = false;
+      for (int32_t t = g0; t < k && !inside; ++t)
+        if (status[t]) {
+          const blastp_gapped &b = rec[t];
+          inside = b.q_start <= qm && qm < b.q_end && b.s_start <= sm && sm < b.s_end;
+        }
+      status[k] = inside ? 0 : 1;
+      if (inside) continue;
+      const FirstDir R = fd[2 * k], L = fd[2 * k + 1];
+      blastp_gapped o;
+      o.query_id = h.query_id;
+      o.subject_id = h.subject_id;
+      o.q_start = qm - L.bi;
+      o.q_end = qm + R.bi;
+      o.s_start = sm - L.bj;
+      o.s_end = sm + R.bj;
+      o.score = L.score + R.score;
+      o.ident = o.gap_opens = o.gap_len = 0;
+      rec[k] = o;
+      if (o.score >= a.cutoff) {  // reported: traced by pass 2 from the logs or re-run
+        dinfo[2 * k] = DirInfo{R.bi, R.bj, R.maxspan, R.logged, R.nib_off, R.hdr_off};
+        dinfo[2 * k + 1] = DirInfo{L.bi, L.bj, L.maxspan, L.logged, L.nib_off, L.hdr_off};
+        if (!R.logged) need[2 * k] = slab_bytes(R.bi + 1, R.cells, R.maxspan);
+        if (!L.logged) need[2 * k + 1] = slab_bytes(L.bi + 1, L.cells, L.maxspan);
+      }
+    }
+  }
+}
+
+// pass 1, general form (the big-ring pass): one thread per pair of a work
+// list (work counter), the pair's HSPs in R21 order with the box test as it
+// goes (or, from_second, from the pair's second HSP on).  The thread's pairs, their HSPs (R21 order) and both
 // directions of each run as one flat loop, one DP cell per turn.  The codes
 // of each direction are appended to the thread's logs (nibbles: nlog_words
 // 32-bit words; row headers: hlog_rows) and kept if the alignment is
@@ -372,7 +501,8 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
     GappedArgs a, Matrix32 mat, const uint32_t *perm, const int32_t *gstart, blastp_gapped *rec,
     uint8_t *status, DirInfo *dinfo, int64_t *need, int2 *scratch, int32_t ring_cols,
     uint32_t *nlog, int32_t nlog_words, int2 *hlog, int32_t hlog_rows, int32_t *over_list,
-    bool big, unsigned long long *counters) {
+    const int32_t *list, int list_count, int list_cursor, bool from_second, int64_t nib_base,
+    int64_t hdr_base, unsigned long long *counters) {
   __shared__ int8_t M[32][32];
   load_matrix(M, mat);
   const int64_t tid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -380,7 +510,7 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
   const int64_t nbase = tid * nlog_words, hbase = tid * hlog_rows;
   int32_t ncur = 0, hcur = 0;  // the logs' fill
   const int32_t mask = ring_cols - 1, ge = a.gap_extend, goe = a.gap_open + a.gap_extend;
-  const unsigned long long ngroups = big ? counters[kNumOver] : counters[kNumGroups];
+  const unsigned long long ngroups = counters[list_count];
   Dir d;
   d.done = true;
   int phase = 0;  // 0 fetch, 1 DP
@@ -439,9 +569,11 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
         rec[cur] = o;
         status[cur] = 1;
         if (o.score >= a.cutoff) {  // reported: traced by pass 2 from the logs or re-run
-          dinfo[2 * cur] = DirInfo{r_bi, r_bj, r_span, r_logged ? 1 : 0, nbase + r_n, hbase + r_h};
-          dinfo[2 * cur + 1] = DirInfo{d.bi, d.bj, d.r_maxspan, logged ? 1 : 0, nbase + ncur,
-                                       hbase + hcur};
+          // log offsets relative to pass 1a's logs (what pass 2 indexes)
+          dinfo[2 * cur] = DirInfo{r_bi, r_bj, r_span, r_logged ? 1 : 0, nib_base + nbase + r_n,
+                                   hdr_base + hbase + r_h};
+          dinfo[2 * cur + 1] = DirInfo{d.bi, d.bj, d.r_maxspan, logged ? 1 : 0,
+                                       nib_base + nbase + ncur, hdr_base + hbase + hcur};
           if (!r_logged) need[2 * cur] = slab_bytes(r_bi + 1, r_cells, r_span);
           if (!logged) need[2 * cur + 1] = slab_bytes(d.bi + 1, d.r_cells, d.r_maxspan);
           ncur += used_n;
@@ -457,14 +589,15 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
     bool finished = false;
     while (phase == 0) {  // the next HSP to extend
       if (k >= g1) {
-        const unsigned long long w = atomicAdd(&counters[big ? kCurBig : kCurPass1], 1ull);
+        const unsigned long long w = atomicAdd(&counters[list_cursor], 1ull);
         if (w >= ngroups) {
           finished = true;
           break;
         }
-        g = big ? over_list[w] : int32_t(w);
+        g = list ? list[w] : int32_t(w);
         g0 = k = gstart[g];
         g1 = gstart[g + 1];
+        if (from_second) ++k;  // the pair's first HSP was extended by gapped_first_kernel
         n0 = ncur;  // the pair's first log position (a redo rewinds to it)
         h0 = hcur;
         continue;
@@ -676,6 +809,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   t2 = (t2 + 31) / 32 * 32;
 
   int32_t *flag = nullptr, *gid = nullptr, *gstart = nullptr, *over = nullptr, *cnt = nullptr;
+  FirstDir *fd = nullptr;
   unsigned long long *key = nullptr, *key2 = nullptr, *counters = nullptr;
   uint32_t *val = nullptr, *perm = nullptr;
   blastp_gapped *rec = nullptr;
@@ -688,7 +822,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   cudaError_t e = cudaSuccess;
   auto cleanup = [&]() {
     void *ptrs[] = {flag, gid, gstart, over, cnt, key, key2, counters, val, perm, rec, status,
-                    store, tbuf, dinfo, need, off, goff, dmax, scratch, scratch_big, temp};
+                    store, tbuf, dinfo, need, off, goff, dmax, scratch, scratch_big, temp, fd};
     for (void *p : ptrs)
       if (p) cudaFreeAsync(p, s);
   };
@@ -733,6 +867,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   GTRY(alloc(&tbuf, size_t(t1) * (size_t(nlog_words) * 4 + size_t(hlog_rows) * 8), s));
   uint32_t *nlog = reinterpret_cast<uint32_t *>(tbuf);
   int2 *hlog = reinterpret_cast<int2 *>(tbuf + size_t(t1) * size_t(nlog_words) * 4);
+  GTRY(alloc(&fd, 2 * n, s));
   GTRY(alloc(&temp, temp_bytes, s));
   GTRY(cudaMemsetAsync(counters, 0, kNumCounters * sizeof(unsigned long long), s));
   GTRY(cudaMemsetAsync(cnt, 0, size_t(n) * sizeof(int32_t), s));
@@ -756,11 +891,14 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
     cleanup();
     return cudaSuccess;
   }
-  // pass 1, then the pairs that overflowed the small rings
-  gapped_score_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, gstart, rec, status, dinfo, need,
-                                                  scratch, ring_small, nlog, nlog_words, hlog,
-                                                  hlog_rows, over, false,
-                                                  counters);
+  // pass 1: every HSP's two directions as independent items, R21 per pair,
+  // then the pairs that overflowed the small rings (general kernel, big
+  // rings, no logs)
+  gapped_first_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, gstart, fd, scratch, ring_small,
+                                                  nlog, nlog_words, hlog, hlog_rows, counters);
+  GTRY(cudaGetLastError());
+  gapped_resolve_kernel<<<gb, 128, 0, s>>>(a, perm, gstart, fd, rec, status, dinfo, need, over,
+                                           counters);
   GTRY(cudaGetLastError());
   GTRY(cudaMemcpyAsync(hc, counters, sizeof(hc), cudaMemcpyDeviceToHost, s));
   GTRY(cudaStreamSynchronize(s));
@@ -768,7 +906,8 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
     GTRY(alloc(&scratch_big, size_t(t2) * size_t(ring_big), s));
     gapped_score_kernel<<<int(t2 / 32), 32, 0, s>>>(a, mat, perm, gstart, rec, status, dinfo, need,
                                                     scratch_big, ring_big, nlog, 0, hlog, 0, over,
-                                                    true, counters);
+                                                    over, kNumOver, kCurBig, false, 0, 0,
+                                                    counters);
     GTRY(cudaGetLastError());
   }
   // traceback stores: exclusive scan of the needs, total and largest one
