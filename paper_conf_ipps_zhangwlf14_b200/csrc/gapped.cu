@@ -362,6 +362,17 @@ __global__ void gapped_keys_kernel(GappedArgs a, const int32_t *flag, const int3
   }
 }
 
+// pass 1a's work order: HSPs by descending ungapped score (high scores are
+// the long homologous alignments; starting them first shortens the tail)
+__global__ void gapped_order_keys_kernel(GappedArgs a, const uint32_t *perm, uint32_t *okey,
+                                         uint32_t *oval) {
+  for (int64_t k = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; k < a.n;
+       k += int64_t(gridDim.x) * blockDim.x) {
+    okey[k] = ~(uint32_t(a.hsps[perm[k]].score) ^ 0x80000000u);
+    oval[k] = uint32_t(k);
+  }
+}
+
 // One direction of a pair's first HSP (R21: the top-scored one, never
 // inside an earlier box), pass 1a.
 struct FirstDir {
@@ -378,7 +389,7 @@ struct FirstDir {
 // chain form left a 25 ms tail of pairs with many HSPs at config 3).  A
 // direction outgrowing the ring sends its pair to the big-ring pass.
 __global__ void __launch_bounds__(128) gapped_first_kernel(
-    GappedArgs a, Matrix32 mat, const uint32_t *perm, const int32_t *gstart, FirstDir *fd,
+    GappedArgs a, Matrix32 mat, const uint32_t *perm, const uint32_t *order, FirstDir *fd,
     int2 *scratch, int32_t ring_cols, uint32_t *nlog, int32_t nlog_words, int2 *hlog,
     int32_t hlog_rows, unsigned long long *counters) {
   __shared__ int8_t M[32][32];
@@ -413,12 +424,12 @@ __global__ void __launch_bounds__(128) gapped_first_kernel(
         ncur += int32_t((d.nc + 7) >> 3);
         hcur += d.i + 1;
       }
-      fd[item] = f;
+      fd[2 * int64_t(order[item >> 1]) + (item & 1)] = f;
       active = false;
     }
     item = atomicAdd(&counters[kCurFirst], 1ull);
     if (item >= nitems) break;
-    const blastp_hsp h = a.hsps[perm[item >> 1]];
+    const blastp_hsp h = a.hsps[perm[order[item >> 1]]];
     const uint8_t *Q = a.qcodes[h.query_id];
     const int32_t lq = a.qlens[h.query_id];
     const Subject sub = subject_of(a, int64_t(h.subject_id) - a.subject_base);
@@ -792,12 +803,14 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
     ring_small = pow2_at_least(std::max(2, std::min(1 << 16, std::atoi(v))));
   const int32_t ring_big = pow2_at_least(int32_t(std::min<int64_t>(a.max_subject_len + 2, 1 << 30)));
   const int threads = 128;
-  int bps = 4;  // pass-1 blocks of 128 per SM
+  // pass-1 blocks of 128 per SM: 4 (32.5 ms at config 3; 8: 31.0 ms but twice the logs'
+  // memory, 3.6 GB, or half the log per thread and 38 MB of re-runs: 35.4 ms)
+  int bps = 4;
   if (const char *v = std::getenv("BLASTP_GAPPED_BPS")) bps = std::max(1, std::min(16, std::atoi(v)));
   const int blocks1 = num_sms * bps;
   // per-thread logs of pass 1's codes: nibble words and row headers (the
   // nibble log in bytes; BLASTP_GAPPED_TBBUF=0: every direction re-run by pass 2)
-  int32_t tb_bytes = 16384;
+  int32_t tb_bytes = 16384;  // + half as much for row headers: 24 KB per thread, 1.8 GB
   if (const char *v = std::getenv("BLASTP_GAPPED_TBBUF"))
     tb_bytes = std::max(0, std::min(1 << 20, std::atoi(v))) / 16 * 16;
   const int32_t nlog_words = tb_bytes / 4, hlog_rows = tb_bytes / 16;
@@ -811,7 +824,8 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   int32_t *flag = nullptr, *gid = nullptr, *gstart = nullptr, *over = nullptr, *cnt = nullptr;
   FirstDir *fd = nullptr;
   unsigned long long *key = nullptr, *key2 = nullptr, *counters = nullptr;
-  uint32_t *val = nullptr, *perm = nullptr;
+  uint32_t *val = nullptr, *perm = nullptr, *okey = nullptr, *okey2 = nullptr, *oval = nullptr,
+           *order = nullptr;
   blastp_gapped *rec = nullptr;
   uint8_t *status = nullptr, *store = nullptr, *tbuf = nullptr;
   DirInfo *dinfo = nullptr;
@@ -822,7 +836,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   cudaError_t e = cudaSuccess;
   auto cleanup = [&]() {
     void *ptrs[] = {flag, gid, gstart, over, cnt, key, key2, counters, val, perm, rec, status,
-                    store, tbuf, dinfo, need, off, goff, dmax, scratch, scratch_big, temp, fd};
+                    store, tbuf, dinfo, need, off, goff, dmax, scratch, scratch_big, temp, fd, okey, okey2, oval, order};
     for (void *p : ptrs)
       if (p) cudaFreeAsync(p, s);
   };
@@ -844,6 +858,8 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   GTRY(cub::DeviceReduce::Max(nullptr, tb, need, dmax, int(2 * n), s));
   temp_bytes = std::max(temp_bytes, tb);
   GTRY(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, goff, int(n), s));
+  temp_bytes = std::max(temp_bytes, tb);
+  GTRY(cub::DeviceRadixSort::SortPairs(nullptr, tb, okey, okey2, oval, order, int(n), 0, 32, s));
   temp_bytes = std::max(temp_bytes, tb);
 
   GTRY(alloc(&flag, n, s));
@@ -868,6 +884,10 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   uint32_t *nlog = reinterpret_cast<uint32_t *>(tbuf);
   int2 *hlog = reinterpret_cast<int2 *>(tbuf + size_t(t1) * size_t(nlog_words) * 4);
   GTRY(alloc(&fd, 2 * n, s));
+  GTRY(alloc(&okey, n, s));
+  GTRY(alloc(&okey2, n, s));
+  GTRY(alloc(&oval, n, s));
+  GTRY(alloc(&order, n, s));
   GTRY(alloc(&temp, temp_bytes, s));
   GTRY(cudaMemsetAsync(counters, 0, kNumCounters * sizeof(unsigned long long), s));
   GTRY(cudaMemsetAsync(cnt, 0, size_t(n) * sizeof(int32_t), s));
@@ -894,7 +914,13 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   // pass 1: every HSP's two directions as independent items, R21 per pair,
   // then the pairs that overflowed the small rings (general kernel, big
   // rings, no logs)
-  gapped_first_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, gstart, fd, scratch, ring_small,
+  gapped_order_keys_kernel<<<gb, 256, 0, s>>>(a, perm, okey, oval);
+  if (const char *v = std::getenv("BLASTP_GAPPED_ORDER"))  // A/B: 0 = the pairs' order
+    if (std::atoi(v) == 0) GTRY(cudaMemsetAsync(okey, 0, size_t(n) * 4, s));
+  GTRY(cudaGetLastError());
+  tb = temp_bytes;
+  GTRY(cub::DeviceRadixSort::SortPairs(temp, tb, okey, okey2, oval, order, int(n), 0, 32, s));
+  gapped_first_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, order, fd, scratch, ring_small,
                                                   nlog, nlog_words, hlog, hlog_rows, counters);
   GTRY(cudaGetLastError());
   gapped_resolve_kernel<<<gb, 128, 0, s>>>(a, perm, gstart, fd, rec, status, dinfo, need, over,
