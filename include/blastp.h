@@ -367,7 +367,9 @@ void blastp_gapped_params_default(blastp_gapped_params *gp);
  * (NULL pointers, bad params, an id outside the table / shard, pairs not
  * contiguous, a seed outside its sequences), CAPACITY (count > capacity:
  * the first `capacity` records are written, *out_count is the full count),
- * NOMEM, CUDA. */
+ * NOMEM, CUDA.  At most 2^30 - 1 HSPs per call; device scratch ~300 bytes
+ * per HSP plus ~1.8 GB of per-thread code logs (library pool, returned to
+ * the pool after the call). */
 int blastp_gapped_extend_device(const blastp_query_table *q, const blastp_db *db,
                                 const blastp_hsp *d_hsps, int64_t n,
                                 const blastp_gapped_params *gp, void *cuda_stream,

@@ -1566,6 +1566,9 @@ static int gapped_device(const blastp_query_table *q, const blastp_db *db, const
                          blastp_gapped *d_out, int64_t capacity, int64_t *count) {
   *count = 0;
   if (n == 0) return BLASTP_OK;
+  if (n > (int64_t(1) << 30) - 1)
+    return fail(BLASTP_E_INVALID_ARG, "%lld HSPs in one gapped call (at most 2^30 - 1)",
+                static_cast<long long>(n));
   const int32_t nq = static_cast<int32_t>(q->q.size());
   std::vector<const uint8_t *> qp(static_cast<size_t>(nq));
   std::vector<int32_t> ql(static_cast<size_t>(nq));

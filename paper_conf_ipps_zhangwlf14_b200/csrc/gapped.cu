@@ -795,7 +795,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   *h_count = 0;
   *h_err = 0;
   if (a.n == 0) return cudaSuccess;
-  if (a.n > int64_t(0x7ffffff0)) return cudaErrorInvalidValue;
+  if (a.n > (int64_t(1) << 30) - 1) return cudaErrorInvalidValue;  // 2n work items in an int
   const int64_t n = a.n;
   const Matrix32 mat = host_matrix();
   int32_t ring_small = 256;
