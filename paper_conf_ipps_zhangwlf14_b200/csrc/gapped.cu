@@ -60,7 +60,7 @@ constexpr int32_t kNeg = INT32_MIN / 4;  // -infinity that survives a few subtra
 
 // counters[]
 enum {
-  kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kCurFirst, kNumCounters = 9
+  kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kCurFirst, kCells, kNumCounters = 10
 };
 
 // a reported direction for pass 2: its best cell, widest span, and whether
@@ -425,6 +425,7 @@ __global__ void __launch_bounds__(128) gapped_first_kernel(
         hcur += d.i + 1;
       }
       fd[2 * int64_t(order[item >> 1]) + (item & 1)] = f;
+      atomicAdd(&counters[kCells], static_cast<unsigned long long>(d.cum + (d.lo < 0 ? d.j - d.start + 1 : 0)));
       active = false;
     }
     item = atomicAdd(&counters[kCurFirst], 1ull);
@@ -955,8 +956,9 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   const int64_t total = last[0] + last[1], maxneed = last[2];
   if (verbose)
     fprintf(stderr, "gapped: %lld HSPs, %llu pairs, %llu pairs redone with %d-column rings "
-            "(small %d), traceback store %.1f MB (largest %lld B)\n", (long long)n,
-            hc[kNumGroups], hc[kNumOver], ring_big, ring_small, total / 1e6, (long long)maxneed);
+            "(small %d), traceback store %.1f MB (largest %lld B), pass-1a cells %llu\n",
+            (long long)n, hc[kNumGroups], hc[kNumOver], ring_big, ring_small, total / 1e6,
+            (long long)maxneed, hc[kCells]);
   {  // pass 2: the logged directions (first window) and the re-runs, window by window
     int64_t window = std::max<int64_t>(std::min<int64_t>(total, int64_t(2) << 30), maxneed);
     if (const char *v = std::getenv("BLASTP_GAPPED_STORE"))  // tests: force several windows
