@@ -41,6 +41,7 @@
 #include <cassert>
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
 
 #include "common.cuh"
 
@@ -378,6 +379,7 @@ __global__ void gapped_order_keys_kernel(GappedArgs a, const uint32_t *perm, uin
 struct FirstDir {
   int32_t score, bi, bj, maxspan, logged, overflow;
   int64_t cells, nib_off, hdr_off;
+  int32_t traced, ident, gopen, glen;  // traced: the traceback's counts are final
 };
 
 // pass 1a: every HSP's two directions as independent work items (item 2k:
@@ -418,6 +420,7 @@ __global__ void __launch_bounds__(128) gapped_first_kernel(
       f.cells = d.r_cells;
       f.overflow = d.overflow ? 1 : 0;
       f.logged = d.nibw != nullptr && !d.overflow ? 1 : 0;
+      f.traced = f.ident = f.gopen = f.glen = 0;
       f.nib_off = nbase + ncur;
       f.hdr_off = hbase + hcur;
       if (f.logged) {
@@ -448,6 +451,242 @@ __global__ void __launch_bounds__(128) gapped_first_kernel(
                 nlog + nbase + ncur, hlog + hbase + hcur, int64_t(nlog_words - ncur) * 8,
                 hlog_rows - hcur);
     active = true;
+  }
+}
+
+// pass 1a, warp form (BLASTP_GAPPED_KERNEL=warp): one direction per warp,
+// each row computed by the 32 lanes over 32 columns at a time.  R19 is
+// sequential along a row only through E and the running best, and both are
+// prefix maxima once the kills are taken out: with u_k = max(D_k, F_k) +
+// ge * k, E_j = max_{k<j} u_k - go - ge * j (a gap never follows a gap), and
+// the running best before cell j is the largest H of the row's earlier
+// cells (a killed cell's H is below best - X, so neither it nor an E term
+// from before it -- each below best - X for good -- can make a later cell
+// live or move the best; the live cells' values, the best and the traceback
+// codes are therefore R19's exactly).  The row ends at its first dead cell
+// beyond the previous row's last live one (a ballot); the previous row is in
+// a per-warp shared-memory ring; each 32-cell chunk's codes go to shared
+// memory as 4 bit-planes (ballots), and lane 0 traces the direction back
+// right away.  A direction whose rows outgrow the ring sends its pair to the
+// big-ring pass; one whose codes outgrow the warp's log is traced by pass 2.
+constexpr int kWRing = 256;       // ring columns (power of two)
+constexpr int kWChunks = 256;     // 32-cell code chunks per warp
+constexpr int kWRows = 768;       // row headers per warp: start column | first chunk << 16
+constexpr int kWWarps = 4;        // warps per block
+struct WarpArea {
+  int2 ring[kWRing];
+  uint4 planes[kWChunks];
+  uint32_t hdr[kWRows];
+};
+
+__global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
+    GappedArgs a, Matrix32 mat, const uint32_t *perm, const uint32_t *order, FirstDir *fd,
+    unsigned long long *counters) {
+  __shared__ int8_t M[32][32];
+  __shared__ WarpArea areas[kWWarps];
+  load_matrix(M, mat);
+  const int lane = threadIdx.x & 31;
+  WarpArea &W = areas[threadIdx.x >> 5];
+  const int32_t ge = a.gap_extend, goe = a.gap_open + a.gap_extend, X = a.xdrop;
+  const unsigned long long nitems = 2ull * static_cast<unsigned long long>(a.n);
+  const unsigned FULL = 0xffffffffu;
+  for (;;) {
+    unsigned long long item = 0;
+    if (lane == 0) item = atomicAdd(&counters[kCurFirst], 1ull);
+    item = __shfl_sync(FULL, item, 0);
+    if (item >= nitems) break;
+    const int64_t k = order[item >> 1];
+    const bool right = (item & 1) == 0;
+    const blastp_hsp h = a.hsps[perm[k]];
+    const uint8_t *Q = a.qcodes[h.query_id];
+    const int32_t lq = a.qlens[h.query_id];
+    const Subject sub = subject_of(a, int64_t(h.subject_id) - a.subject_base);
+    const int32_t qm = h.q_start + h.length / 2, sm = h.s_start + h.length / 2;  // R20
+    if (qm > lq || sm > sub.ls) {
+      if (lane == 0) atomicOr(&counters[kErr], 2ull);
+      continue;
+    }
+    const uint8_t *A = right ? Q + qm : Q + qm - 1;
+    const uint8_t *B = right ? sub.S + sm : sub.S + sm - 1;
+    const int step = right ? 1 : -1;
+    const int32_t la = right ? lq - qm : qm, lb = right ? sub.ls - sm : sm;
+    int32_t best = 0, bi = 0, bj = 0, best_row = 0, i = 0, plo = 0, phi = -1;
+    int64_t cum = 0, r_cells = 0;
+    int32_t maxspan_all = 0, r_maxspan = 0, nch = 0;
+    bool tb_ok = true, overflow = false, truncated = false;
+    const int8_t *mrow = M[0];
+    for (;;) {  // rows
+      const int32_t start = plo;
+      if (tb_ok) {
+        // room for a full row of chunks; when the log is full, the rows after
+        // the best row so far are dropped (the X-drop tail) -- a later move of
+        // the best past them leaves the direction to pass 2
+        if (nch + kWRing / 32 > kWChunks) {
+          if (best_row < i - 1) {
+            nch = int32_t(W.hdr[best_row + 1] >> 16);
+            truncated = true;
+          } else {
+            tb_ok = false;
+          }
+        }
+        if (i >= kWRows || start > 0xffff) tb_ok = false;
+        if (tb_ok && lane == 0) W.hdr[i] = uint32_t(start) | (uint32_t(nch) << 16);
+      }
+      int32_t ucarry = kNeg, up_last = kNeg, h_last = kNeg;
+      int32_t lo = -1, hi = -1, stop = -1;
+      for (int32_t c0 = start;; c0 += 32) {
+        const int32_t j = c0 + lane;
+        const bool inr = j <= lb;
+        int2 up = make_int2(kNeg, kNeg);
+        if (inr && j <= phi) up = W.ring[j & (kWRing - 1)];
+        int32_t dh = __shfl_up_sync(FULL, up.x, 1);
+        if (lane == 0) dh = up_last;  // the previous chunk's last column (row start: dead)
+        up_last = __shfl_sync(FULL, up.x, 31);
+        int32_t d = kNeg;
+        if (inr && j > 0 && dh > kNeg) d = dh + mrow[B[int64_t(j - 1) * step]];
+        if (i == 0 && j == 0) d = 0;  // the origin
+        const int32_t f = imax(up.y - ge, up.x - goe);
+        const int32_t u = inr ? imax(d, f) + ge * j : kNeg;
+        int32_t U = u;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const int32_t t = __shfl_up_sync(FULL, U, o);
+          if (lane >= o) U = imax(U, t);
+        }
+        int32_t Ux = __shfl_up_sync(FULL, U, 1);
+        Ux = imax(lane == 0 ? kNeg : Ux, ucarry);
+        const int32_t e = j > 0 ? Ux - goe - ge * (j - 1) : kNeg;
+        const int32_t hraw = imax(d, imax(e, f));
+        // running best before j: the carry, unless a cell of this chunk rises
+        // above it (rare past the first rows) -- then a prefix maximum
+        int32_t bprev = best;
+        if (__reduce_max_sync(FULL, inr ? hraw : kNeg) > best) {
+          int32_t Hm = inr ? hraw : kNeg;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const int32_t t = __shfl_up_sync(FULL, Hm, o);
+            if (lane >= o) Hm = imax(Hm, t);
+          }
+          const int32_t Hx = __shfl_up_sync(FULL, Hm, 1);
+          bprev = imax(lane == 0 ? kNeg : Hx, best);
+        }
+        const bool live = inr && hraw >= bprev - X;
+        const bool stopper = inr && ((!live && j > phi && j > 0) || j == lb);
+        const unsigned sb = __ballot_sync(FULL, stopper);
+        const int last = sb ? __ffs(sb) - 1 : 31;
+        const bool valid = inr && lane <= last;
+        // the best: the first live cell reaching the chunk's maximum, if above
+        const int32_t cand = (valid && live) ? hraw : kNeg;
+        const int32_t cm = __reduce_max_sync(FULL, cand);
+        if (cm > best) {
+          const unsigned at = __ballot_sync(FULL, cand == cm);
+          if (truncated) tb_ok = false;  // rows between were dropped
+          best = cm;
+          bi = i;
+          bj = c0 + __ffs(at) - 1;
+          best_row = i;
+        }
+        const int32_t hs = live ? hraw : kNeg;
+        if (valid) W.ring[j & (kWRing - 1)] = live ? make_int2(hraw, f) : make_int2(kNeg, kNeg);
+        if (tb_ok) {
+          int32_t lh = __shfl_up_sync(FULL, hs, 1);
+          if (lane == 0) lh = h_last;
+          const int src = hraw == d ? 0 : (hraw == e ? 1 : 2);
+          const unsigned p0 = __ballot_sync(FULL, valid && (src & 1));
+          const unsigned p1 = __ballot_sync(FULL, valid && (src & 2));
+          const unsigned p2 = __ballot_sync(FULL, valid && e == lh - goe);
+          const unsigned p3 = __ballot_sync(FULL, valid && f == up.x - goe);
+          if (nch >= kWChunks) {
+            tb_ok = false;
+          } else {
+            if (lane == 0) W.planes[nch] = make_uint4(p0, p1, p2, p3);
+            ++nch;
+          }
+        }
+        h_last = __shfl_sync(FULL, hs, 31);
+        const unsigned lv = __ballot_sync(FULL, valid && live);
+        if (lv) {
+          if (lo < 0) lo = c0 + __ffs(lv) - 1;
+          hi = c0 + 31 - __clz(lv);
+        }
+        if (sb) {
+          stop = c0 + last;
+          break;
+        }
+        ucarry = imax(ucarry, __shfl_sync(FULL, U, 31));
+        if (c0 + 64 - start > kWRing) {  // the next chunk would not fit the ring
+          overflow = true;
+          break;
+        }
+      }
+      __syncwarp();  // the row's ring stores before the next row's loads
+      if (overflow || lo < 0) break;  // a row without live cells ends the extension
+      const int32_t span = stop - start + 1;
+      cum += span;
+      maxspan_all = imax(maxspan_all, span);
+      if (best_row == i) {
+        r_cells = cum;
+        r_maxspan = maxspan_all;
+      }
+      plo = lo;
+      phi = hi;
+      ++i;
+      if (i > la) break;
+      mrow = M[A[int64_t(i - 1) * step]];
+    }
+    __syncwarp();
+    FirstDir out;
+    out.score = best;
+    out.bi = bi;
+    out.bj = bj;
+    out.maxspan = r_maxspan;
+    out.cells = r_cells;
+    out.overflow = overflow ? 1 : 0;
+    out.logged = 0;
+    out.nib_off = out.hdr_off = 0;
+    out.traced = 0;
+    out.ident = out.gopen = out.glen = 0;
+    if (!overflow && tb_ok && lane == 0) {  // R22 traceback over the bit-planes
+      int32_t ti = bi, tj = bj, state = 0, idn = 0, gop = 0, gl = 0;
+      while (ti > 0 || tj > 0) {
+        const uint32_t hd = W.hdr[ti];
+        const int32_t c = tj - int32_t(hd & 0xffffu);
+        const uint4 pl = W.planes[(hd >> 16) + (c >> 5)];
+        const int bit = c & 31;
+        const int code = int((pl.x >> bit) & 1u) | (int((pl.y >> bit) & 1u) << 1) |
+                         (int((pl.z >> bit) & 1u) << 2) | (int((pl.w >> bit) & 1u) << 3);
+        if (state == 0) {
+          const int src = code & 3;
+          if (src == 0) {
+            idn += A[int64_t(ti - 1) * step] == B[int64_t(tj - 1) * step];
+            --ti;
+            --tj;
+          } else {
+            state = src;
+          }
+        } else if (state == 1) {
+          ++gl;
+          if (code & 4) {
+            ++gop;
+            state = 0;
+          }
+          --tj;
+        } else {
+          ++gl;
+          if (code & 8) {
+            ++gop;
+            state = 0;
+          }
+          --ti;
+        }
+      }
+      out.traced = 1;
+      out.ident = idn;
+      out.gopen = gop;
+      out.glen = gl;
+    }
+    if (lane == 0) fd[2 * k + (right ? 0 : 1)] = out;
+    __syncwarp();
   }
 }
 
@@ -488,13 +727,21 @@ __global__ void gapped_resolve_kernel(GappedArgs a, const uint32_t *perm, const 
       o.s_start = sm - L.bj;
       o.s_end = sm + R.bj;
       o.score = L.score + R.score;
-      o.ident = o.gap_opens = o.gap_len = 0;
+      // directions traced in pass 1a (warp kernel) count now; the others are
+      // traced by pass 2 from the logs or re-run
+      o.ident = (R.traced ? R.ident : 0) + (L.traced ? L.ident : 0);
+      o.gap_opens = (R.traced ? R.gopen : 0) + (L.traced ? L.gopen : 0);
+      o.gap_len = (R.traced ? R.glen : 0) + (L.traced ? L.glen : 0);
       rec[k] = o;
-      if (o.score >= a.cutoff) {  // reported: traced by pass 2 from the logs or re-run
-        dinfo[2 * k] = DirInfo{R.bi, R.bj, R.maxspan, R.logged, R.nib_off, R.hdr_off};
-        dinfo[2 * k + 1] = DirInfo{L.bi, L.bj, L.maxspan, L.logged, L.nib_off, L.hdr_off};
-        if (!R.logged) need[2 * k] = slab_bytes(R.bi + 1, R.cells, R.maxspan);
-        if (!L.logged) need[2 * k + 1] = slab_bytes(L.bi + 1, L.cells, L.maxspan);
+      if (o.score >= a.cutoff) {
+        if (!R.traced) {
+          dinfo[2 * k] = DirInfo{R.bi, R.bj, R.maxspan, R.logged, R.nib_off, R.hdr_off};
+          if (!R.logged) need[2 * k] = slab_bytes(R.bi + 1, R.cells, R.maxspan);
+        }
+        if (!L.traced) {
+          dinfo[2 * k + 1] = DirInfo{L.bi, L.bj, L.maxspan, L.logged, L.nib_off, L.hdr_off};
+          if (!L.logged) need[2 * k + 1] = slab_bytes(L.bi + 1, L.cells, L.maxspan);
+        }
       }
     }
   }
@@ -921,8 +1168,13 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   GTRY(cudaGetLastError());
   tb = temp_bytes;
   GTRY(cub::DeviceRadixSort::SortPairs(temp, tb, okey, okey2, oval, order, int(n), 0, 32, s));
-  gapped_first_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, order, fd, scratch, ring_small,
-                                                  nlog, nlog_words, hlog, hlog_rows, counters);
+  const char *kv = std::getenv("BLASTP_GAPPED_KERNEL");
+  if (kv && std::strcmp(kv, "warp") == 0) {
+    gapped_warp_kernel<<<num_sms * 8, kWWarps * 32, 0, s>>>(a, mat, perm, order, fd, counters);
+  } else {
+    gapped_first_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, order, fd, scratch, ring_small,
+                                                    nlog, nlog_words, hlog, hlog_rows, counters);
+  }
   GTRY(cudaGetLastError());
   gapped_resolve_kernel<<<gb, 128, 0, s>>>(a, perm, gstart, fd, rec, status, dinfo, need, over,
                                            counters);

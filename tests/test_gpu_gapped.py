@@ -23,6 +23,15 @@ def bp():
     return blastp
 
 
+@pytest.fixture(params=["thread", "warp"], autouse=True)
+def gapped_kernel(request, monkeypatch):
+    """Every gapped test runs on both pass-1a forms (BLASTP_GAPPED_KERNEL):
+    a thread per direction, and a warp per direction with its rows computed
+    32 columns at a time."""
+    monkeypatch.setenv("BLASTP_GAPPED_KERNEL", request.param)
+    return request.param
+
+
 def assert_same(got, exp, what):
     got, exp = np.asarray(got), np.asarray(exp)
     if len(got) == len(exp) and (got.view(np.int32).reshape(-1, 10) ==
