@@ -454,7 +454,8 @@ __global__ void __launch_bounds__(128) gapped_first_kernel(
   }
 }
 
-// pass 1a, warp form (BLASTP_GAPPED_KERNEL=warp): one direction per warp,
+// pass 1a, warp form (the default; BLASTP_GAPPED_KERNEL=thread selects the
+// thread form above): one direction per warp,
 // each row computed by the 32 lanes over 32 columns at a time.  R19 is
 // sequential along a row only through E and the running best, and both are
 // prefix maxima once the kills are taken out: with u_k = max(D_k, F_k) +
@@ -547,6 +548,8 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
         if (i == 0 && j == 0) d = 0;  // the origin
         const int32_t f = imax(up.y - ge, up.x - goe);
         const int32_t u = inr ? imax(d, f) + ge * j : kNeg;
+        // (skipping this prefix maximum for chunks whose E bound is below best -
+        // X measured 4% slower: the extra reduction costs more than it saves)
         int32_t U = u;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -1168,8 +1171,10 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   GTRY(cudaGetLastError());
   tb = temp_bytes;
   GTRY(cub::DeviceRadixSort::SortPairs(temp, tb, okey, okey2, oval, order, int(n), 0, 32, s));
+  // pass 1a's form: the warp per direction (default; 28 vs 31 ms at config 3)
+  // or BLASTP_GAPPED_KERNEL=thread
   const char *kv = std::getenv("BLASTP_GAPPED_KERNEL");
-  if (kv && std::strcmp(kv, "warp") == 0) {
+  if (!(kv && std::strcmp(kv, "thread") == 0)) {
     gapped_warp_kernel<<<num_sms * 8, kWWarps * 32, 0, s>>>(a, mat, perm, order, fd, counters);
   } else {
     gapped_first_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, order, fd, scratch, ring_small,
