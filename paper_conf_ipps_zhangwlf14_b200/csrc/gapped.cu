@@ -550,12 +550,11 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
         const int32_t u = inr ? imax(d, f) + ge * j : kNeg;
         // (skipping this prefix maximum for chunks whose E bound is below best -
         // X measured 4% slower: the extra reduction costs more than it saves)
+        // (a lane below the shuffle distance gets its own value back, which a
+        // maximum ignores: no lane test)
         int32_t U = u;
 #pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-          const int32_t t = __shfl_up_sync(FULL, U, o);
-          if (lane >= o) U = imax(U, t);
-        }
+        for (int o = 1; o < 32; o <<= 1) U = imax(U, __shfl_up_sync(FULL, U, o));
         int32_t Ux = __shfl_up_sync(FULL, U, 1);
         Ux = imax(lane == 0 ? kNeg : Ux, ucarry);
         const int32_t e = j > 0 ? Ux - goe - ge * (j - 1) : kNeg;
@@ -566,10 +565,7 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
         if (__reduce_max_sync(FULL, inr ? hraw : kNeg) > best) {
           int32_t Hm = inr ? hraw : kNeg;
 #pragma unroll
-          for (int o = 1; o < 32; o <<= 1) {
-            const int32_t t = __shfl_up_sync(FULL, Hm, o);
-            if (lane >= o) Hm = imax(Hm, t);
-          }
+          for (int o = 1; o < 32; o <<= 1) Hm = imax(Hm, __shfl_up_sync(FULL, Hm, o));
           const int32_t Hx = __shfl_up_sync(FULL, Hm, 1);
           bprev = imax(lane == 0 ? kNeg : Hx, best);
         }
