@@ -145,6 +145,7 @@ struct blastp_db {
   unsigned seq = 0;  // search launches on this db (segment publication epoch)
   bool carved = false;  // stream/sstart/chunks/counters live in a caller's arena
   std::vector<int64_t> h_sstart;
+  int64_t max_len = -1;  // longest subject (the gapped stage's big-ring width), computed once
   unsigned long long *counters = nullptr;  // [0] hsp count, [1] chunk cursor, [6] long chunks
   blastp_hsp *out = nullptr;               // scratch for the host-array search
   int64_t out_cap = 0;
@@ -1576,12 +1577,17 @@ static int gapped_device(const blastp_query_table *q, const blastp_db *db, const
     qp[k] = q->q[k].qcodes;
     ql[k] = q->q[k].lq;
   }
-  int64_t maxlen = 0;
-  const std::vector<int64_t> &st = host_sstart(db);
-  for (int64_t i = 0; i < db->nseq; ++i) {
-    const int64_t en = i + 1 < db->nseq ? st[i + 1] - 1 : kStreamPadFront + db->residues + db->nseq - 1;
-    maxlen = std::max(maxlen, en - st[i]);
+  if (db->max_len < 0) {  // once per shard (a pass over the host copy of the subject starts)
+    int64_t maxlen = 0;
+    const std::vector<int64_t> &st = host_sstart(db);
+    for (int64_t i = 0; i < db->nseq; ++i) {
+      const int64_t en =
+          i + 1 < db->nseq ? st[i + 1] - 1 : kStreamPadFront + db->residues + db->nseq - 1;
+      maxlen = std::max(maxlen, en - st[i]);
+    }
+    const_cast<blastp_db *>(db)->max_len = maxlen;
   }
+  const int64_t maxlen = db->max_len;
   const uint8_t **d_qp = nullptr;
   int32_t *d_ql = nullptr;
   if (pool_malloc_async(&d_qp, sizeof(void *) * static_cast<size_t>(nq), s) != cudaSuccess ||

@@ -61,7 +61,8 @@ constexpr int32_t kNeg = INT32_MIN / 4;  // -infinity that survives a few subtra
 
 // counters[]
 enum {
-  kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kCurFirst, kCells, kNumCounters = 10
+  kCurPass1 = 0, kCurBig, kNumOver, kErr, kNumGroups, kTotal, kCurTrace, kCurFirst, kCells, kNumWork,
+  kNumCounters = 11
 };
 
 // a reported direction for pass 2: its best cell, widest span, and whether
@@ -471,32 +472,47 @@ __global__ void __launch_bounds__(128) gapped_first_kernel(
 // right away.  A direction whose rows outgrow the ring sends its pair to the
 // big-ring pass; one whose codes outgrow the warp's log is traced by pass 2.
 constexpr int kWRing = 256;       // ring columns (power of two)
-constexpr int kWChunks = 256;     // 32-cell code chunks per warp
+constexpr int kWChunks = 256;     // 32-cell code chunks per warp (first launch)
 constexpr int kWRows = 768;       // row headers per warp: start column | first chunk << 16
-constexpr int kWWarps = 4;        // warps per block
-struct WarpArea {
-  int2 ring[kWRing];
-  uint4 planes[kWChunks];
-  uint32_t hdr[kWRows];
-};
+constexpr int kWWarps = 4;        // warps per block (first launch)
+constexpr int kW2Chunks = 8192;   // second launch, one warp per block: 128 KB of chunks
+constexpr int kW2Rows = 16384;    // + 64 KB of row headers
+__host__ __device__ inline size_t warp_area_bytes(int chunks, int rows) {
+  return size_t(kWRing) * 8 + size_t(chunks) * 16 + size_t(rows) * 4;
+}
 
+// kSecond: the directions pass 1b left over (work list, need > 0: a log that
+// did not fit), one warp per block with a log as large as shared memory
+// allows -- traced here, their counts added to the alignment, need cleared;
+// any still too long stay for pass 2.
+template <bool kSecond>
 __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
     GappedArgs a, Matrix32 mat, const uint32_t *perm, const uint32_t *order, FirstDir *fd,
+    const int32_t *work, int64_t *need, blastp_gapped *rec, int32_t cap_chunks, int32_t cap_rows,
     unsigned long long *counters) {
   __shared__ int8_t M[32][32];
-  __shared__ WarpArea areas[kWWarps];
+  extern __shared__ __align__(16) uint8_t warp_smem[];
   load_matrix(M, mat);
   const int lane = threadIdx.x & 31;
-  WarpArea &W = areas[threadIdx.x >> 5];
+  const size_t area = size_t(kWRing) * 8 + size_t(cap_chunks) * 16 + size_t(cap_rows) * 4;
+  uint8_t *wbase = warp_smem + size_t(threadIdx.x >> 5) * area;
+  int2 *ring = reinterpret_cast<int2 *>(wbase);
+  uint4 *planes = reinterpret_cast<uint4 *>(wbase + size_t(kWRing) * 8);
+  uint32_t *hdr = reinterpret_cast<uint32_t *>(wbase + size_t(kWRing) * 8 + size_t(cap_chunks) * 16);
   const int32_t ge = a.gap_extend, goe = a.gap_open + a.gap_extend, X = a.xdrop;
-  const unsigned long long nitems = 2ull * static_cast<unsigned long long>(a.n);
+  const unsigned long long nitems =
+      kSecond ? counters[kNumWork] : 2ull * static_cast<unsigned long long>(a.n);
   const unsigned FULL = 0xffffffffu;
   for (;;) {
     unsigned long long item = 0;
-    if (lane == 0) item = atomicAdd(&counters[kCurFirst], 1ull);
+    if (lane == 0) item = atomicAdd(&counters[kSecond ? kCurBig : kCurFirst], 1ull);
     item = __shfl_sync(FULL, item, 0);
     if (item >= nitems) break;
-    const int64_t k = order[item >> 1];
+    if (kSecond) {
+      item = static_cast<unsigned long long>(work[item]);
+      if (need[item] == 0) continue;  // a thread-form log: pass 2 traces it
+    }
+    const int64_t k = kSecond ? int64_t(item >> 1) : int64_t(order[item >> 1]);
     const bool right = (item & 1) == 0;
     const blastp_hsp h = a.hsps[perm[k]];
     const uint8_t *Q = a.qcodes[h.query_id];
@@ -522,16 +538,16 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
         // room for a full row of chunks; when the log is full, the rows after
         // the best row so far are dropped (the X-drop tail) -- a later move of
         // the best past them leaves the direction to pass 2
-        if (nch + kWRing / 32 > kWChunks) {
+        if (nch + kWRing / 32 > cap_chunks) {
           if (best_row < i - 1) {
-            nch = int32_t(W.hdr[best_row + 1] >> 16);
+            nch = int32_t(hdr[best_row + 1] >> 16);
             truncated = true;
           } else {
             tb_ok = false;
           }
         }
-        if (i >= kWRows || start > 0xffff) tb_ok = false;
-        if (tb_ok && lane == 0) W.hdr[i] = uint32_t(start) | (uint32_t(nch) << 16);
+        if (i >= cap_rows || start > 0xffff || nch + kWRing / 32 > 0xffff) tb_ok = false;
+        if (tb_ok && lane == 0) hdr[i] = uint32_t(start) | (uint32_t(nch) << 16);
       }
       int32_t ucarry = kNeg, up_last = kNeg, h_last = kNeg;
       int32_t lo = -1, hi = -1, stop = -1;
@@ -539,7 +555,7 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
         const int32_t j = c0 + lane;
         const bool inr = j <= lb;
         int2 up = make_int2(kNeg, kNeg);
-        if (inr && j <= phi) up = W.ring[j & (kWRing - 1)];
+        if (inr && j <= phi) up = ring[j & (kWRing - 1)];
         int32_t dh = __shfl_up_sync(FULL, up.x, 1);
         if (lane == 0) dh = up_last;  // the previous chunk's last column (row start: dead)
         up_last = __shfl_sync(FULL, up.x, 31);
@@ -586,7 +602,7 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
           best_row = i;
         }
         const int32_t hs = live ? hraw : kNeg;
-        if (valid) W.ring[j & (kWRing - 1)] = live ? make_int2(hraw, f) : make_int2(kNeg, kNeg);
+        if (valid) ring[j & (kWRing - 1)] = live ? make_int2(hraw, f) : make_int2(kNeg, kNeg);
         if (tb_ok) {
           int32_t lh = __shfl_up_sync(FULL, hs, 1);
           if (lane == 0) lh = h_last;
@@ -595,10 +611,10 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
           const unsigned p1 = __ballot_sync(FULL, valid && (src & 2));
           const unsigned p2 = __ballot_sync(FULL, valid && e == lh - goe);
           const unsigned p3 = __ballot_sync(FULL, valid && f == up.x - goe);
-          if (nch >= kWChunks) {
+          if (nch >= cap_chunks) {
             tb_ok = false;
           } else {
-            if (lane == 0) W.planes[nch] = make_uint4(p0, p1, p2, p3);
+            if (lane == 0) planes[nch] = make_uint4(p0, p1, p2, p3);
             ++nch;
           }
         }
@@ -648,9 +664,9 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
     if (!overflow && tb_ok && lane == 0) {  // R22 traceback over the bit-planes
       int32_t ti = bi, tj = bj, state = 0, idn = 0, gop = 0, gl = 0;
       while (ti > 0 || tj > 0) {
-        const uint32_t hd = W.hdr[ti];
+        const uint32_t hd = hdr[ti];
         const int32_t c = tj - int32_t(hd & 0xffffu);
-        const uint4 pl = W.planes[(hd >> 16) + (c >> 5)];
+        const uint4 pl = planes[(hd >> 16) + (c >> 5)];
         const int bit = c & 31;
         const int code = int((pl.x >> bit) & 1u) | (int((pl.y >> bit) & 1u) << 1) |
                          (int((pl.z >> bit) & 1u) << 2) | (int((pl.w >> bit) & 1u) << 3);
@@ -684,7 +700,16 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
       out.gopen = gop;
       out.glen = gl;
     }
-    if (lane == 0) fd[2 * k + (right ? 0 : 1)] = out;
+    if (kSecond) {
+      if (out.traced && lane == 0) {
+        atomicAdd(&rec[k].ident, out.ident);
+        atomicAdd(&rec[k].gap_opens, out.gopen);
+        atomicAdd(&rec[k].gap_len, out.glen);
+        need[item] = 0;
+      }
+    } else if (lane == 0) {
+      fd[2 * k + (right ? 0 : 1)] = out;
+    }
     __syncwarp();
   }
 }
@@ -695,7 +720,7 @@ __global__ void __launch_bounds__(kWWarps * 32) gapped_warp_kernel(
 __global__ void gapped_resolve_kernel(GappedArgs a, const uint32_t *perm, const int32_t *gstart,
                                       const FirstDir *fd, blastp_gapped *rec, uint8_t *status,
                                       DirInfo *dinfo, int64_t *need, int32_t *over_list,
-                                      unsigned long long *counters) {
+                                      int32_t *work, unsigned long long *counters) {
   const int64_t ng = int64_t(counters[kNumGroups]);
   for (int64_t g = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; g < ng;
        g += int64_t(gridDim.x) * blockDim.x) {
@@ -736,10 +761,12 @@ __global__ void gapped_resolve_kernel(GappedArgs a, const uint32_t *perm, const 
         if (!R.traced) {
           dinfo[2 * k] = DirInfo{R.bi, R.bj, R.maxspan, R.logged, R.nib_off, R.hdr_off};
           if (!R.logged) need[2 * k] = slab_bytes(R.bi + 1, R.cells, R.maxspan);
+          work[atomicAdd(&counters[kNumWork], 1ull)] = int32_t(2 * k);
         }
         if (!L.traced) {
           dinfo[2 * k + 1] = DirInfo{L.bi, L.bj, L.maxspan, L.logged, L.nib_off, L.hdr_off};
           if (!L.logged) need[2 * k + 1] = slab_bytes(L.bi + 1, L.cells, L.maxspan);
+          work[atomicAdd(&counters[kNumWork], 1ull)] = int32_t(2 * k + 1);
         }
       }
     }
@@ -760,7 +787,7 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
     uint8_t *status, DirInfo *dinfo, int64_t *need, int2 *scratch, int32_t ring_cols,
     uint32_t *nlog, int32_t nlog_words, int2 *hlog, int32_t hlog_rows, int32_t *over_list,
     const int32_t *list, int list_count, int list_cursor, bool from_second, int64_t nib_base,
-    int64_t hdr_base, unsigned long long *counters) {
+    int64_t hdr_base, int32_t *work, unsigned long long *counters) {
   __shared__ int8_t M[32][32];
   load_matrix(M, mat);
   const int64_t tid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -834,6 +861,9 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
                                        nib_base + nbase + ncur, hdr_base + hbase + hcur};
           if (!r_logged) need[2 * cur] = slab_bytes(r_bi + 1, r_cells, r_span);
           if (!logged) need[2 * cur + 1] = slab_bytes(d.bi + 1, d.r_cells, d.r_maxspan);
+          const unsigned long long wslot = atomicAdd(&counters[kNumWork], 2ull);
+          work[wslot] = 2 * cur;
+          work[wslot + 1] = 2 * cur + 1;
           ncur += used_n;
           hcur += used_h;
         } else {  // not reported: the logs forget both directions
@@ -904,7 +934,7 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
 __global__ void __launch_bounds__(128) gapped_trace_kernel(
     GappedArgs a, Matrix32 mat, const uint32_t *perm, blastp_gapped *rec, const DirInfo *dinfo,
     const int64_t *need, const int64_t *off, int64_t base, int64_t window, uint8_t *store,
-    const uint32_t *nlog, const int2 *hlog, unsigned long long *cursor) {
+    const uint32_t *nlog, const int2 *hlog, const int32_t *work, unsigned long long *counters) {
   __shared__ int8_t M[32][32];
   load_matrix(M, mat);
   const int32_t ge = a.gap_extend, goe = a.gap_open + a.gap_extend;
@@ -913,6 +943,7 @@ __global__ void __launch_bounds__(128) gapped_trace_kernel(
   Trace tr{0, 0, 0, 0, 0, 0};
   int phase = 0;  // 0 fetch, 1 DP, 2 traceback
   int64_t item = 0;
+  const unsigned long long nwork = counters[kNumWork];
   const uint32_t *nibw = nullptr;
   const int2 *hdr = nullptr;
   const uint8_t *A = nullptr, *B = nullptr;
@@ -922,10 +953,10 @@ __global__ void __launch_bounds__(128) gapped_trace_kernel(
   for (;;) {
     if (phase == 0) {
       bool got = false, logged = false;
-      while (!got) {
-        const unsigned long long t = atomicAdd(cursor, 1ull);
-        if (t >= static_cast<unsigned long long>(2 * a.n)) break;
-        item = int64_t(t);
+      while (!got) {  // the directions resolve (or the big-ring pass) left to this pass
+        const unsigned long long t = atomicAdd(&counters[kCurTrace], 1ull);
+        if (t >= nwork) break;
+        item = int64_t(work[t]);
         if (need[item] > 0) {
           got = off[item] >= base && off[item] < base + window;
         } else if (base == 0) {
@@ -1068,7 +1099,8 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
                                                       big_budget / (int64_t(ring_big) * 8)));
   t2 = (t2 + 31) / 32 * 32;
 
-  int32_t *flag = nullptr, *gid = nullptr, *gstart = nullptr, *over = nullptr, *cnt = nullptr;
+  int32_t *flag = nullptr, *gid = nullptr, *gstart = nullptr, *over = nullptr, *cnt = nullptr,
+          *work = nullptr;
   FirstDir *fd = nullptr;
   unsigned long long *key = nullptr, *key2 = nullptr, *counters = nullptr;
   uint32_t *val = nullptr, *perm = nullptr, *okey = nullptr, *okey2 = nullptr, *oval = nullptr,
@@ -1083,7 +1115,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   cudaError_t e = cudaSuccess;
   auto cleanup = [&]() {
     void *ptrs[] = {flag, gid, gstart, over, cnt, key, key2, counters, val, perm, rec, status,
-                    store, tbuf, dinfo, need, off, goff, dmax, scratch, scratch_big, temp, fd, okey, okey2, oval, order};
+                    store, tbuf, dinfo, need, off, goff, dmax, scratch, scratch_big, temp, fd, okey, okey2, oval, order, work};
     for (void *p : ptrs)
       if (p) cudaFreeAsync(p, s);
   };
@@ -1131,6 +1163,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   uint32_t *nlog = reinterpret_cast<uint32_t *>(tbuf);
   int2 *hlog = reinterpret_cast<int2 *>(tbuf + size_t(t1) * size_t(nlog_words) * 4);
   GTRY(alloc(&fd, 2 * n, s));
+  GTRY(alloc(&work, 2 * n, s));
   GTRY(alloc(&okey, n, s));
   GTRY(alloc(&okey2, n, s));
   GTRY(alloc(&oval, n, s));
@@ -1170,15 +1203,20 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   // pass 1a's form: the warp per direction (default; 28 vs 31 ms at config 3)
   // or BLASTP_GAPPED_KERNEL=thread
   const char *kv = std::getenv("BLASTP_GAPPED_KERNEL");
-  if (!(kv && std::strcmp(kv, "thread") == 0)) {
-    gapped_warp_kernel<<<num_sms * 8, kWWarps * 32, 0, s>>>(a, mat, perm, order, fd, counters);
+  const bool warp_form = !(kv && std::strcmp(kv, "thread") == 0);
+  if (warp_form) {
+    const size_t sm1 = size_t(kWWarps) * warp_area_bytes(kWChunks, kWRows);
+    GTRY(cudaFuncSetAttribute(gapped_warp_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              int(sm1)));
+    gapped_warp_kernel<false><<<num_sms * 8, kWWarps * 32, sm1, s>>>(
+        a, mat, perm, order, fd, nullptr, nullptr, nullptr, kWChunks, kWRows, counters);
   } else {
     gapped_first_kernel<<<blocks1, threads, 0, s>>>(a, mat, perm, order, fd, scratch, ring_small,
                                                     nlog, nlog_words, hlog, hlog_rows, counters);
   }
   GTRY(cudaGetLastError());
   gapped_resolve_kernel<<<gb, 128, 0, s>>>(a, perm, gstart, fd, rec, status, dinfo, need, over,
-                                           counters);
+                                           work, counters);
   GTRY(cudaGetLastError());
   GTRY(cudaMemcpyAsync(hc, counters, sizeof(hc), cudaMemcpyDeviceToHost, s));
   GTRY(cudaStreamSynchronize(s));
@@ -1186,8 +1224,20 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
     GTRY(alloc(&scratch_big, size_t(t2) * size_t(ring_big), s));
     gapped_score_kernel<<<int(t2 / 32), 32, 0, s>>>(a, mat, perm, gstart, rec, status, dinfo, need,
                                                     scratch_big, ring_big, nlog, 0, hlog, 0, over,
-                                                    over, kNumOver, kCurBig, false, 0, 0,
+                                                    over, kNumOver, kCurBig, false, 0, 0, work,
                                                     counters);
+    GTRY(cudaGetLastError());
+  }
+  // the directions left over by the warp form, again by warps with large
+  // shared-memory logs (a handful of long alignments: their thread-form re-runs
+  // in pass 2 were a tail of single threads)
+  if (warp_form && hc[kNumWork] > 0) {
+    const size_t sm2 = warp_area_bytes(kW2Chunks, kW2Rows);
+    GTRY(cudaFuncSetAttribute(gapped_warp_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              int(sm2)));
+    GTRY(cudaMemsetAsync(counters + kCurBig, 0, sizeof(unsigned long long), s));
+    gapped_warp_kernel<true><<<num_sms, 32, sm2, s>>>(a, mat, perm, order, fd, work, need, rec,
+                                                      kW2Chunks, kW2Rows, counters);
     GTRY(cudaGetLastError());
   }
   // traceback stores: exclusive scan of the needs, total and largest one
@@ -1209,22 +1259,23 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   const int64_t total = last[0] + last[1], maxneed = last[2];
   if (verbose)
     fprintf(stderr, "gapped: %lld HSPs, %llu pairs, %llu pairs redone with %d-column rings "
-            "(small %d), traceback store %.1f MB (largest %lld B), pass-1a cells %llu\n",
+            "(small %d), traceback store %.1f MB (largest %lld B), pass-1a cells %llu, "
+            "directions left to pass 2 %llu\n",
             (long long)n, hc[kNumGroups], hc[kNumOver], ring_big, ring_small, total / 1e6,
-            (long long)maxneed, hc[kCells]);
+            (long long)maxneed, hc[kCells], hc[kNumWork]);
   {  // pass 2: the logged directions (first window) and the re-runs, window by window
     int64_t window = std::max<int64_t>(std::min<int64_t>(total, int64_t(2) << 30), maxneed);
     if (const char *v = std::getenv("BLASTP_GAPPED_STORE"))  // tests: force several windows
       window = std::max<int64_t>(maxneed, std::atoll(v));
     window = std::max<int64_t>(window, 1);
     if (total > 0) GTRY(alloc(&store, size_t(window + maxneed), s));
-    const int64_t items = 2 * n;
+    const int64_t items = int64_t(hc[kNumWork]);  // the directions left to this pass
     const int tblocks = int(std::min<int64_t>((items + threads - 1) / threads, int64_t(num_sms) * 8));
-    for (int64_t base = 0; base == 0 || base < total; base += window) {
+    for (int64_t base = 0; items > 0 && (base == 0 || base < total); base += window) {
       GTRY(cudaMemsetAsync(counters + kCurTrace, 0, sizeof(unsigned long long), s));
       gapped_trace_kernel<<<tblocks, threads, 0, s>>>(a, mat, perm, rec, dinfo, need, off, base,
-                                                       window, store, nlog, hlog,
-                                                       counters + kCurTrace);
+                                                       window, store, nlog, hlog, work,
+                                                       counters);
       GTRY(cudaGetLastError());
     }
   }
