@@ -775,7 +775,7 @@ __global__ void gapped_resolve_kernel(GappedArgs a, const uint32_t *perm, const 
 
 // pass 1, general form (the big-ring pass): one thread per pair of a work
 // list (work counter), the pair's HSPs in R21 order with the box test as it
-// goes (or, from_second, from the pair's second HSP on).  The thread's pairs, their HSPs (R21 order) and both
+// goes.  The thread's pairs, their HSPs (R21 order) and both
 // directions of each run as one flat loop, one DP cell per turn.  The codes
 // of each direction are appended to the thread's logs (nibbles: nlog_words
 // 32-bit words; row headers: hlog_rows) and kept if the alignment is
@@ -786,8 +786,8 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
     GappedArgs a, Matrix32 mat, const uint32_t *perm, const int32_t *gstart, blastp_gapped *rec,
     uint8_t *status, DirInfo *dinfo, int64_t *need, int2 *scratch, int32_t ring_cols,
     uint32_t *nlog, int32_t nlog_words, int2 *hlog, int32_t hlog_rows, int32_t *over_list,
-    const int32_t *list, int list_count, int list_cursor, bool from_second, int64_t nib_base,
-    int64_t hdr_base, int32_t *work, unsigned long long *counters) {
+    const int32_t *list, int list_count, int list_cursor, int32_t *work,
+    unsigned long long *counters) {
   __shared__ int8_t M[32][32];
   load_matrix(M, mat);
   const int64_t tid = int64_t(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -854,11 +854,9 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
         rec[cur] = o;
         status[cur] = 1;
         if (o.score >= a.cutoff) {  // reported: traced by pass 2 from the logs or re-run
-          // log offsets relative to pass 1a's logs (what pass 2 indexes)
-          dinfo[2 * cur] = DirInfo{r_bi, r_bj, r_span, r_logged ? 1 : 0, nib_base + nbase + r_n,
-                                   hdr_base + hbase + r_h};
-          dinfo[2 * cur + 1] = DirInfo{d.bi, d.bj, d.r_maxspan, logged ? 1 : 0,
-                                       nib_base + nbase + ncur, hdr_base + hbase + hcur};
+          dinfo[2 * cur] = DirInfo{r_bi, r_bj, r_span, r_logged ? 1 : 0, nbase + r_n, hbase + r_h};
+          dinfo[2 * cur + 1] = DirInfo{d.bi, d.bj, d.r_maxspan, logged ? 1 : 0, nbase + ncur,
+                                       hbase + hcur};
           if (!r_logged) need[2 * cur] = slab_bytes(r_bi + 1, r_cells, r_span);
           if (!logged) need[2 * cur + 1] = slab_bytes(d.bi + 1, d.r_cells, d.r_maxspan);
           const unsigned long long wslot = atomicAdd(&counters[kNumWork], 2ull);
@@ -885,7 +883,6 @@ __global__ void __launch_bounds__(128) gapped_score_kernel(
         g = list ? list[w] : int32_t(w);
         g0 = k = gstart[g];
         g1 = gstart[g + 1];
-        if (from_second) ++k;  // the pair's first HSP was extended by gapped_first_kernel
         n0 = ncur;  // the pair's first log position (a redo rewinds to it)
         h0 = hcur;
         continue;
@@ -1224,8 +1221,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
     GTRY(alloc(&scratch_big, size_t(t2) * size_t(ring_big), s));
     gapped_score_kernel<<<int(t2 / 32), 32, 0, s>>>(a, mat, perm, gstart, rec, status, dinfo, need,
                                                     scratch_big, ring_big, nlog, 0, hlog, 0, over,
-                                                    over, kNumOver, kCurBig, false, 0, 0, work,
-                                                    counters);
+                                                    over, kNumOver, kCurBig, work, counters);
     GTRY(cudaGetLastError());
   }
   // the directions left over by the warp form, again by warps with large
