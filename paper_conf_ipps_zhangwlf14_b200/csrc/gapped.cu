@@ -11,27 +11,32 @@
 // lies in the box of an alignment already made (R21), traceback preferring the
 // diagonal, then E, then F, a gap opening over its extension (R22).
 //
-// B200 form.  The recurrences are sequential inside a row (E and the running
-// best), and R21 is sequential inside a (query, subject) pair, so a pair is
-// one thread's work; pairs are independent (~286K at config 3), which fills
-// the GPU several times over.  Per thread one DP row lives in a ring of
-// (H, F) int32 pairs indexed by subject column (global scratch, L1/L2
-// resident): the live band of a row only drifts right (a cell left of the
-// previous row's first live cell is dead), so a ring of C columns suffices
-// while no row's computed span exceeds C; a pair whose span does is re-run by
-// a second launch with rings the size of the longest subject.
-//   order   : pairs = runs of equal (query, subject) in the canonical list;
-//             a stable radix sort by (pair, descending score) gives R21's
-//             order inside each pair;
-//   pass 1  : (gapped_score_kernel) per pair: scores, boxes, containment,
-//             and per reported direction the traceback store it needs (rows
-//             and cells up to the best cell);
-//   pass 2  : (gapped_trace_kernel) per reported direction: the DP re-run up
-//             to the best row into its store (4 bits per cell: H source,
-//             E opened, F opened), then the traceback (identities, gap
-//             opens, gap residues);
-//   emit    : (gapped_emit_kernel) per pair: its reported alignments in
-//             canonical order at the pair's offset of an exclusive scan.
+// B200 form.  An alignment depends only on its own HSP --
+// R21 only decides whether it is used -- so every HSP's two directions are
+// independent work items and R21 runs afterwards, per pair.  Along a row R19
+// is sequential only through E and the running best, both prefix maxima once
+// the kills are taken out (a killed cell cannot make a later one live), so a
+// warp computes a row 32 columns at a time.
+//   order    : pairs = runs of equal (query, subject) in the canonical list; a
+//              stable radix sort by (pair, descending score) gives R21's order
+//              inside each pair; pass 1a takes HSPs by descending score;
+//   pass 1a  : gapped_warp_kernel<false> (default): a warp per direction, the
+//              previous row in a shared-memory ring, codes (H from diagonal /
+//              E / F, E opened, F opened) as ballot bit-planes in shared
+//              memory, traced back at once by lane 0;  gapped_first_kernel
+//              (BLASTP_GAPPED_KERNEL=thread): a thread per direction, one DP
+//              cell per loop turn, codes to per-thread nibble logs;
+//   pass 1b  : gapped_resolve_kernel: R21 per pair over the boxes; the
+//              directions not traced yet go to a work list;
+//   big ring : gapped_score_kernel: pairs with a row wider than the ring,
+//              redone by a thread per pair with subject-sized rings;
+//   leftover : gapped_warp_kernel<true>: the work list's directions whose codes
+//              did not fit, a warp per block with a 194 KB shared-memory log;
+//   pass 2   : gapped_trace_kernel: whatever is still left -- the thread
+//              form's logs, or a re-run up to the best row into an exactly
+//              sized store -- traced back;
+//   emit     : gapped_emit_kernel: per pair, its reported alignments in
+//              canonical order at the pair's offset of an exclusive scan.
 #include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_reduce.cuh>
 #include <cub/device/device_scan.cuh>
@@ -375,15 +380,14 @@ __global__ void gapped_order_keys_kernel(GappedArgs a, const uint32_t *perm, uin
   }
 }
 
-// One direction of a pair's first HSP (R21: the top-scored one, never
-// inside an earlier box), pass 1a.
+// Pass 1a's result for one direction of one HSP.
 struct FirstDir {
   int32_t score, bi, bj, maxspan, logged, overflow;
   int64_t cells, nib_off, hdr_off;
   int32_t traced, ident, gopen, glen;  // traced: the traceback's counts are final
 };
 
-// pass 1a: every HSP's two directions as independent work items (item 2k:
+// pass 1a, thread form: every HSP's two directions as independent work items (item 2k:
 // right, 2k + 1: left of the k-th HSP in R21 order), one DP cell per loop
 // turn, codes appended to the thread's logs.  An alignment depends only on
 // its own HSP; whether it is used (R21: its seed outside the boxes of the
