@@ -368,8 +368,8 @@ void blastp_gapped_params_default(blastp_gapped_params *gp);
  * contiguous, a seed outside its sequences), CAPACITY (count > capacity:
  * the first `capacity` records are written, *out_count is the full count),
  * NOMEM, CUDA.  At most 2^30 - 1 HSPs per call; device scratch ~300 bytes
- * per HSP plus ~1.8 GB of per-thread code logs (library pool, returned to
- * the pool after the call). */
+ * per HSP from the library's pool (returned to it after the call; plus ~2 GB
+ * of per-thread rings and code logs with BLASTP_GAPPED_KERNEL=thread). */
 int blastp_gapped_extend_device(const blastp_query_table *q, const blastp_db *db,
                                 const blastp_hsp *d_hsps, int64_t n,
                                 const blastp_gapped_params *gp, void *cuda_stream,

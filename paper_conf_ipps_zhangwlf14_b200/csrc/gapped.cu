@@ -1159,8 +1159,14 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   GTRY(alloc(&off, 2 * n, s));
   GTRY(alloc(&goff, n, s));
   GTRY(alloc(&dmax, 1, s));
-  GTRY(alloc(&scratch, size_t(t1) * ring_small, s));
-  GTRY(alloc(&tbuf, size_t(t1) * (size_t(nlog_words) * 4 + size_t(hlog_rows) * 8), s));
+  // pass 1a's form: the warp per direction (default) or BLASTP_GAPPED_KERNEL=thread,
+  // whose per-thread rings and code logs (~1.8 GB) only it allocates
+  const char *kv = std::getenv("BLASTP_GAPPED_KERNEL");
+  const bool warp_form = !(kv && std::strcmp(kv, "thread") == 0);
+  if (!warp_form) {
+    GTRY(alloc(&scratch, size_t(t1) * ring_small, s));
+    GTRY(alloc(&tbuf, size_t(t1) * (size_t(nlog_words) * 4 + size_t(hlog_rows) * 8), s));
+  }
   uint32_t *nlog = reinterpret_cast<uint32_t *>(tbuf);
   int2 *hlog = reinterpret_cast<int2 *>(tbuf + size_t(t1) * size_t(nlog_words) * 4);
   GTRY(alloc(&fd, 2 * n, s));
@@ -1201,10 +1207,7 @@ cudaError_t launch_gapped(const GappedArgs &a, int num_sms, blastp_gapped *d_out
   GTRY(cudaGetLastError());
   tb = temp_bytes;
   GTRY(cub::DeviceRadixSort::SortPairs(temp, tb, okey, okey2, oval, order, int(n), 0, 32, s));
-  // pass 1a's form: the warp per direction (default; 28 vs 31 ms at config 3)
-  // or BLASTP_GAPPED_KERNEL=thread
-  const char *kv = std::getenv("BLASTP_GAPPED_KERNEL");
-  const bool warp_form = !(kv && std::strcmp(kv, "thread") == 0);
+  // (warp form: 28 vs 31 ms for the thread form at config 3, same box)
   if (warp_form) {
     const size_t sm1 = size_t(kWWarps) * warp_area_bytes(kWChunks, kWRows);
     GTRY(cudaFuncSetAttribute(gapped_warp_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
