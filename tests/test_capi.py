@@ -92,3 +92,19 @@ def test_invalid_params_rejected_before_any_gpu_work(bp):
         with pytest.raises(bp.BlastpError) as e:
             bp.build_query_table("MKVLAAGIVALLA", bp.Params(**bad))
         assert e.value.status == bp.E_INVALID_ARG, bad
+
+
+def test_gapped_defaults_and_validation_without_gpu(bp, orc):
+    """The gapped stage's defaults equal the oracle's (R18-R21: 11 + 1 per
+    residue, X-drop 38, cutoff 41), the record is 40 bytes with the oracle's
+    field order, and bad arguments fail before any device work."""
+    g = bp._CGappedParams()
+    bp.lib.blastp_gapped_params_default(ctypes.byref(g))
+    o = orc.GappedParams()
+    assert (g.gap_open, g.gap_extend, g.xdrop, g.cutoff) == (o.gap_open, o.gap_extend, o.xdrop,
+                                                             o.cutoff)
+    assert bp.GAPPED_DTYPE.itemsize == 40 and bp.GAPPED_DTYPE.names == orc.GAPPED_DTYPE.names
+    cnt = ctypes.c_int64()
+    rc = bp.lib.blastp_gapped_extend_device(None, None, None, 0, ctypes.byref(g), None, None, 0,
+                                            ctypes.byref(cnt))
+    assert rc == bp.E_INVALID_ARG
