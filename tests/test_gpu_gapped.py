@@ -249,3 +249,27 @@ def test_batch_pipeline_equals_sequential_and_oracle(bp, orc, monkeypatch, knobs
     u, exp = oracle_gapped(orc, queries, db.ascii, db.offsets, bp.GappedParams())
     assert_same(got, exp, "pipelined vs oracle")
     assert len(exp) > 100
+
+
+def test_config4_gapped_sharded_full(bp, orc, gapped_kernel):
+    """Config 4 at full size: queries 127/517/1054 (one batch) against config
+    3's database cut into 4 shards; each shard's gapped stage on the GPU
+    (blastp_search_gapped), concatenated and sorted, equals the oracle's gapped
+    stage over the oracle's whole-database list (pairs never span shards)."""
+    if gapped_kernel != "warp":
+        pytest.skip("the thread form is covered by config 3; one form at this size")
+    from synth import CONFIGS
+    (_,), db = config_workload(3)
+    queries = [gen_query(CONFIGS[1]["query_seed"], 127), gen_query(CONFIGS[2]["query_seed"], 517),
+               gen_query(CONFIGS[3]["query_seed"], 1054)]
+    t = bp.build_query_batch(queries)
+    parts = []
+    for k in range(4):
+        d = bp.pack_db(db.ascii, db.offsets, k, 4)
+        parts.append(bp.search_gapped(t, d))
+        d.free()
+    got = np.concatenate(parts)
+    got = np.sort(got, order=list(got.dtype.names))
+    _, exp = oracle_gapped(orc, queries, db.ascii, db.offsets, bp.GappedParams())
+    assert_same(got, exp, "config 4, 4 shards")
+    assert len(exp) > 100000
