@@ -273,3 +273,58 @@ def test_config4_gapped_sharded_full(bp, orc, gapped_kernel):
     _, exp = oracle_gapped(orc, queries, db.ascii, db.offsets, bp.GappedParams())
     assert_same(got, exp, "config 4, 4 shards")
     assert len(exp) > 100000
+
+
+def test_constructed_hsp_lists_edges(bp, orc, gapped_kernel):
+    """HSP lists built by hand rather than by the search: seeds at both ends
+    of the query and the subject (empty directions), length-0 and length-1
+    HSPs, exact duplicates, 150 HSPs on one (query, subject) pair (R21's box
+    test over a long chain, equal scores keeping canonical order), poly-W
+    rows wide enough for the big-ring pass, the last subject of the shard --
+    all against the oracle, on both pass-1a forms."""
+    import torch
+    rng = np.random.default_rng(2024)
+    q = gen_query(606, 400)
+    qc = orc.encode(q)
+    alpha = np.frombuffer(b"ARNDCQEGHILKMFPSTWYV", dtype=np.uint8)
+    subs = [alpha[rng.integers(0, 20, size=int(rng.integers(50, 900)))].copy() for _ in range(40)]
+    subs[3][100:300] = np.frombuffer(q[50:250], dtype=np.uint8)      # a long copy
+    subs[7] = np.frombuffer(b"W" * 700, dtype=np.uint8).copy()        # poly-W: wide rows
+    subs[-1][:120] = np.frombuffer(q[-120:], dtype=np.uint8)          # last subject, query end
+    ascii = np.concatenate(subs)
+    off = np.concatenate([[0], np.cumsum([len(s) for s in subs])]).astype(np.int64)
+    lens = [len(s) for s in subs]
+    recs = []
+
+    def add(sid, qs, ss, ln, score):
+        recs.append((0, sid, ss - qs, qs, ss, ln, score))
+    add(0, 0, 0, 0, 50)                      # seed at both starts: left directions empty
+    add(1, 399, lens[1] - 1, 1, 45)          # seed at both ends (middle pair = the last pair)
+    add(2, 399, 0, 0, 44)                    # qm = lq: right direction has no rows
+    add(5, 10, 20, 6, 60)
+    add(5, 10, 20, 6, 60)                    # an exact duplicate: inside the first box
+    for k in range(150):                     # one long chain on the pair (0, 3)
+        qs = int(rng.integers(0, 390))
+        ss = int(rng.integers(0, lens[3] - 10))
+        add(3, qs, ss, int(rng.integers(0, 10)), int(rng.integers(41, 90)) if k % 7 else 55)
+    add(7, 0, 0, 3, 41)                      # poly-W subject vs the query's W's
+    add(7, 200, 600, 3, 41)
+    add(39, 280, 0, 120, 300)                # the last subject: the copy of the query's end
+    h = np.array(sorted(recs), dtype=np.int32)
+    d = bp.pack_db(ascii, off)
+    t = bp.build_query_table(q)
+    dev = torch.from_numpy(h.copy()).cuda()
+    out = torch.zeros((len(h), 10), dtype=torch.int32, device="cuda")
+    for knobs in ({}, {"BLASTP_GAPPED_RING": "16"}):
+        for k_, v in knobs.items():
+            os.environ[k_] = v
+        try:
+            n = bp.gapped_extend_device(t, d, dev.data_ptr(), len(h), out.data_ptr(), len(h))
+        finally:
+            for k_ in knobs:
+                os.environ.pop(k_, None)
+        got = out[:n].cpu().numpy().view(bp.GAPPED_DTYPE).ravel()
+        exp = orc.gapped_hsps([qc], orc.encode(ascii.tobytes()), off,
+                              h.view(orc.HSP_DTYPE).ravel(), orc.GappedParams())
+        assert_same(got, exp, f"constructed list {knobs}")
+        assert len(exp) >= 4  # the copies, poly-W; most chain seeds fall inside the copy's box
