@@ -589,10 +589,23 @@ def main():
                 if k > 0:
                     gms.append(g0.elapsed_time(g1))
             gmean = statistics.mean(gms)
+            # the two stages through the public host-result call (search +
+            # canonical order + gapped stage + D2H of the alignments)
+            ems = []
+            for k in range(3):
+                torch.cuda.synchronize()
+                t0 = time.perf_counter()
+                al = bp.search_gapped(table, gdb, params, stream=stream)
+                ems.append(1e3 * (time.perf_counter() - t0))
             gapped = {"hsps_in": ng, "alignments_out": int(m), "ms": gmean,
                       "hsps_per_s": ng / (gmean / 1e3),
                       "path": "blastp_gapped_extend_device on the rank's canonical device HSP "
-                              "list (affine Gotoh X-drop, R18-R22; 3 timed calls after 1 warm-up)"}
+                              "list (affine Gotoh X-drop, R18-R22; 3 timed calls after 1 warm-up)",
+                      "search_plus_gapped_host_ms": statistics.median(ems[1:]),
+                      "search_plus_gapped_path": "blastp_search_gapped (search, canonical sort, "
+                                                 "gapped stage, alignments copied to the host; "
+                                                 f"{len(al)} alignments), wall clock, median of 2 "
+                                                 "after 1 warm-up"}
             del hs, gout
         except Exception as ex:  # noqa: BLE001 -- a report beside the headline
             gapped = {"error": str(ex)}
