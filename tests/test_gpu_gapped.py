@@ -328,3 +328,64 @@ def test_constructed_hsp_lists_edges(bp, orc, gapped_kernel):
                               h.view(orc.HSP_DTYPE).ravel(), orc.GappedParams())
         assert_same(got, exp, f"constructed list {knobs}")
         assert len(exp) >= 4  # the copies, poly-W; most chain seeds fall inside the copy's box
+
+
+_C5 = {}
+
+
+def _c5_gapped_chunk(bounds):
+    a, b = bounds
+    o = _C5["orc"]
+    return o.gapped_hsps(_C5["qcodes"], _C5["codes"], _C5["off"], _C5["u"][a:b])
+
+
+@pytest.mark.skipif(os.environ.get("BLASTP_FULL_CONFIG5") != "1",
+                    reason="~12 min of oracle time on 16 cores: run once per round with "
+                           "BLASTP_FULL_CONFIG5=1 (log in profiles/)")
+def test_config5_shard_gapped_full(bp, orc, gapped_kernel):
+    """Config 5, one full shard: the 64 queries against shard 0 of 8 (~1.9G
+    residues); the GPU's gapped alignments equal the oracle's gapped stage run
+    over the oracle's own complete ungapped list (split at pair boundaries
+    over the host's cores; ~21.5M HSPs)."""
+    if gapped_kernel != "warp":
+        pytest.skip("the default form at this size")
+    import multiprocessing as mp
+    import time
+    from paper_conf_ipps_zhangwlf14_b200.dist import shard_subjects
+    from synth import config_offsets
+    off = config_offsets(5)
+    lo, hi = shard_subjects(off, 0, 8)
+    queries, db = config_workload(5, subject_range=(lo, hi))
+    loc = (db.offsets - db.offsets[0]).astype(np.int64)
+    t0 = time.perf_counter()
+    got = bp.search_gapped(bp.build_query_batch(queries), bp.pack_db(db.ascii, loc))
+    t_gpu = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    codes = orc.encode(db.ascii.tobytes())
+    lists = [orc.search(orc.encode(q), codes, loc, orc.Params(), nthreads=os.cpu_count() or 8,
+                        want_extensions=False, query_id=k, cap_hint=int(loc[-1]) // 500).hsps
+             for k, q in enumerate(queries)]
+    u = np.concatenate(lists)
+    u = np.sort(u, order=list(u.dtype.names))
+    t_search = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    # chunks of the canonical list split at (query, subject) boundaries
+    nproc = os.cpu_count() or 8
+    cuts = [0]
+    for c in range(1, nproc):
+        i = len(u) * c // nproc
+        while 0 < i < len(u) and (u["query_id"][i], u["subject_id"][i]) == \
+                (u["query_id"][i - 1], u["subject_id"][i - 1]):
+            i += 1
+        cuts.append(max(i, cuts[-1]))
+    cuts.append(len(u))
+    _C5.update(orc=orc, qcodes=[orc.encode(q) for q in queries], codes=codes, off=loc, u=u)
+    with mp.get_context("fork").Pool(nproc) as pool:
+        parts = pool.map(_c5_gapped_chunk, list(zip(cuts[:-1], cuts[1:])))
+    exp = np.concatenate(parts)
+    t_gapped = time.perf_counter() - t0
+    _C5.clear()
+    assert_same(got, exp, "config 5 shard 0 of 8, gapped")
+    print(f"config5 shard 0/8 gapped parity: {len(u)} HSPs -> {len(exp)} alignments; GPU search + "
+          f"gapped {t_gpu:.1f} s (incl. table build + pack); oracle search {t_search:.0f} s, "
+          f"oracle gapped {t_gapped:.0f} s on {nproc} processes")
