@@ -389,3 +389,21 @@ def test_config5_shard_gapped_full(bp, orc, gapped_kernel):
     print(f"config5 shard 0/8 gapped parity: {len(u)} HSPs -> {len(exp)} alignments; GPU search + "
           f"gapped {t_gpu:.1f} s (incl. table build + pack); oracle search {t_search:.0f} s, "
           f"oracle gapped {t_gapped:.0f} s on {nproc} processes")
+
+
+@pytest.mark.parametrize("mode,ext_mode", [(0, 1), (1, 0), (2, 0), (3, 0)],
+                         ids=["HIT", "EITHER", "STATEFUL", "STATEFUL_RB"])
+def test_gapped_over_other_readings(bp, orc, mode, ext_mode):
+    """The gapped stage consumes whatever list a search reading hands off --
+    ext_mode HIT's one record per seed (duplicates inside each other's boxes,
+    R21), EITHER, STATEFUL, STATEFUL_RB -- identically to the oracle's gapped
+    stage over the oracle's list of the same reading (config 1)."""
+    (q,), db = config_workload(1)
+    p = bp.Params(filter_mode=mode, ext_mode=ext_mode)
+    t = bp.build_query_table(q, p)
+    d = bp.pack_db(db.ascii, db.offsets)
+    got = bp.search_gapped(t, d, p)
+    P = orc.Params(filter_mode=mode, ext_mode=ext_mode)
+    _, exp = oracle_gapped(orc, [q], db.ascii, db.offsets, bp.GappedParams(), p=P)
+    assert_same(got, exp, f"config 1 {p}")
+    assert len(exp) > 5
