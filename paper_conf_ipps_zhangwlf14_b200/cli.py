@@ -9,7 +9,13 @@ HSP in canonical order (R11):
 
     query  subject  q_start  s_start  length  score  diagonal
 
-with FASTA identifiers (first word of the header) and 0-based starts.  All of
+with FASTA identifiers (first word of the header) and 0-based starts; with
+--gapped, the gapped consumer of those HSPs (R18-R22) instead, one
+line per gapped alignment:
+
+    query  subject  q_start  q_end  s_start  s_end  score  identities  gap_opens  gap_residues
+
+(ends exclusive).  All of
 the search runs in libblastp.so (include/blastp.h); this module only parses
 FASTA and formats the result.  Options map to blastp_params (P:L143-144 T,
 P:L1344-1351 A, Fig. 8 X; R3-R15).
@@ -65,6 +71,13 @@ def main(argv: list[str] | None = None) -> int:
                     help="keep the database in pinned host memory (formatted image) and stream it "
                          "(each part's copy overlaps the previous part's search; the shard's "
                          "device image must fit in HBM)")
+    ap.add_argument("--gapped", action="store_true",
+                    help="run the gapped stage on the HSPs (blastp_search_gapped) and print the "
+                         "gapped alignments (resident database, one GPU)")
+    ap.add_argument("--gap-open", type=int, default=11)
+    ap.add_argument("--gap-extend", type=int, default=1)
+    ap.add_argument("--gapped-xdrop", type=int, default=38)
+    ap.add_argument("--gapped-cutoff", type=int, default=41)
     ap.add_argument("--device", type=int, default=0)
     ap.add_argument("--distributed", action="store_true",
                     help="one process per GPU under torchrun: each rank searches a residue-"
@@ -73,6 +86,8 @@ def main(argv: list[str] | None = None) -> int:
                     help="--distributed: the search kernels append into rank 0's buffer over "
                          "NVLink (CUDA IPC), or per-rank lists gathered with NCCL")
     args = ap.parse_args(argv)
+    if args.gapped and (args.stream or args.distributed):
+        ap.error("--gapped runs on a resident database on one GPU (no --stream / --distributed)")
 
     import os
 
@@ -177,6 +192,15 @@ def main(argv: list[str] | None = None) -> int:
         bp.sort_hsps_device(out.data_ptr(), n)
         hsps = out[: n * 7].view(n, 7).cpu().numpy()
         h.free()
+    elif args.gapped:
+        db = bp.pack_db(residues, soff, device=args.device)
+        gp = bp.GappedParams(args.gap_open, args.gap_extend, args.gapped_xdrop, args.gapped_cutoff)
+        al = bp.search_gapped(table, db, p, gp)
+        db.free()
+        w = sys.stdout.write
+        for qi, si, q0, q1, s0, s1, sc, idn, gop, gl in al.view(np.int32).reshape(-1, 10).tolist():
+            w(f"{qids[qi]}\t{sids[si]}\t{q0}\t{q1}\t{s0}\t{s1}\t{sc}\t{idn}\t{gop}\t{gl}\n")
+        return 0
     else:
         db = bp.pack_db(residues, soff, device=args.device)
         hsps = bp.search_ungapped(table, db, p).view(np.int32).reshape(-1, 7)

@@ -58,6 +58,13 @@ def test_cli_matches_oracle(tmp_path, capsys, orc):
         assert out == exp_lines, extra
     assert cli.main([str(tmp_path / "q.fa"), str(tmp_path / "d.fa"), "--filter", "stateful"]) == 0
     assert len(capsys.readouterr().out.strip().split("\n")) > 20
+    # --gapped: the gapped stage over the same HSPs vs the oracle's gapped stage
+    u = np.array(tuples, dtype=np.int32).view(orc.HSP_DTYPE).ravel()
+    g = orc.gapped_hsps([orc.encode(q) for q in qs], codes, db.offsets, u)
+    exp_g = [f"{qids[r[0]]}\t{sids[r[1]]}\t" + "\t".join(str(int(x)) for x in list(r)[2:])
+             for r in g.tolist()]
+    assert cli.main([str(tmp_path / "q.fa"), str(tmp_path / "d.fa"), "--gapped"]) == 0
+    assert capsys.readouterr().out.strip().split("\n") == exp_g and len(exp_g) > 20
 
 
 @pytest.mark.gpu
